@@ -1,0 +1,57 @@
+// Fused HBM-bound kernels of the block / embedding / head (K5-K8, K10 of
+// SURVEY §2.2).  T is the path type (__nv_bfloat16 or float); reductions
+// and statistics are fp32.  All launchers are asynchronous on `s` and
+// return a mobius_status.
+#pragma once
+
+#include <cstdint>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+
+namespace mobius {
+
+// x0[r, :] = wte[tok(r)] + wpe[r % s],  r = b*s + i,  tok(r) = tok[b*(s+1) + i]
+template <typename T>
+int embed_fwd(const int32_t* tok, const T* wte, const T* wpe, T* x, int mbs, int s, int h, cudaStream_t st);
+// dwte[tok(r)] += dx[r];  dwpe[i] += sum_b dx[b*s + i]   (fp32 accumulators)
+template <typename T>
+int embed_bwd(const int32_t* tok, const T* dx, float* dwte, float* dwpe, int mbs, int s, int h, cudaStream_t st);
+
+// y = g (x - mu) rstd + b over rows of length h; saves mu, rstd (fp32)
+template <typename T>
+int layernorm_fwd(const T* x, const T* g, const T* b, T* y, float* mu, float* rstd, int rows, int h, cudaStream_t st);
+// dx = rstd (g dy - mean(g dy) - xhat mean(g dy xhat)) [+ dres];  dg += sum dy xhat; db += sum dy
+template <typename T>
+int layernorm_bwd(const T* dy, const T* x, const T* g, const float* mu, const float* rstd, const T* dres, T* dx,
+                  float* dg, float* db, int rows, int h, cudaStream_t st);
+
+// Causal row softmax of S (fp32, [B][s][s], row stride s) scaled by `scale`:
+// P[i, j] = softmax_j<=i(scale S[i, :]) and 0 for i < j < roundup(i+1, 128).
+template <typename T>
+int softmax_causal_fwd(const float* S, T* P, int B, int s, float scale, cudaStream_t st);
+// dS = scale * P (dP - sum_j P dP) on j <= i, 0 for i < j < roundup(i+1,128)
+template <typename T>
+int softmax_causal_bwd(const T* P, const float* dP, T* dS, int B, int s, float scale, cudaStream_t st);
+
+// Row-wise cross entropy on logits [rows][V] (in place -> dlogits):
+// loss_rows[r] = logsumexp(z_r) - z_r[t_r];  dz = (softmax(z) - onehot) * inv_ntok.
+// t_r = tok[b*(s+1) + i + 1] for r = b*s + i.
+template <typename T>
+int cross_entropy_fwd_bwd(T* logits, const int32_t* tok, float* loss_rows, int rows, int V, int s, float inv_ntok,
+                          cudaStream_t st);
+// acc[0] += sum(loss_rows)  (double, single block: deterministic)
+int loss_accumulate(const float* loss_rows, int rows, double* acc, cudaStream_t st);
+
+// out[n] += sum_r X[r, n] (fp32 out), X row stride ld
+template <typename T>
+int colsum_accum(const T* X, int64_t ld, int rows, int n, float* out, cudaStream_t st);
+
+// dst = (T) src
+template <typename T>
+int cast_from_f32(const float* src, T* dst, int64_t n, cudaStream_t st);
+
+// device-side flag wait / set (inter-rank arrival flags, release/acquire at system scope)
+int flag_wait(const volatile int* flag, int value, cudaStream_t st);
+int flag_set(int* flag, int value, cudaStream_t st);
+
+}  // namespace mobius

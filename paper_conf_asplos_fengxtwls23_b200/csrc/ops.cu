@@ -1,0 +1,475 @@
+// GPT layer forward/backward composed from the tcgen05 GEMM (bf16 path) or
+// the SIMT GEMM (fp32 debug path) and the fused HBM-bound kernels.
+// Equations: SURVEY §8(c) O-2 (reading #1 of the paper's "GPT-like"
+// blocks).
+#include <cmath>
+
+#include "common.h"
+#include "elem.h"
+#include "gemm.h"
+#include "ops.h"
+
+namespace mobius {
+
+thread_local int64_t g_kernel_launches = 0;
+static KernelTimer* g_timer = nullptr;
+void set_kernel_timer(KernelTimer* t) { g_timer = t; }
+KernelTimer* kernel_timer() { return g_timer; }
+
+BlockLayout::BlockLayout(int64_t h) {
+  int64_t p = 0;
+  ln1_g = p; p += h;
+  ln1_b = p; p += h;
+  w_qkv = p; p += h * 3 * h;
+  b_qkv = p; p += 3 * h;
+  w_o = p; p += h * h;
+  b_o = p; p += h;
+  ln2_g = p; p += h;
+  ln2_b = p; p += h;
+  w_1 = p; p += h * 4 * h;
+  b_1 = p; p += 4 * h;
+  w_2 = p; p += 4 * h * h;
+  b_2 = p; p += h;
+  total = p;
+}
+EmbedLayout::EmbedLayout(int64_t h, int64_t V, int64_t s) {
+  wte = 0;
+  wpe = V * h;
+  total = V * h + s * h;
+}
+HeadLayout::HeadLayout(int64_t h, int64_t V) {
+  lnf_g = 0;
+  lnf_b = h;
+  w_head = 2 * h;
+  total = 2 * h + h * V;
+}
+
+template <>
+int gemm<__nv_bfloat16>(const GemmDesc& d, cudaStream_t st) {
+  return gemm_bf16(d, st);
+}
+template <>
+int gemm<float>(const GemmDesc& d, cudaStream_t st) {
+  return gemm_f32(d, st);
+}
+
+namespace {
+
+inline int64_t align256(int64_t x) { return (x + 255) & ~int64_t(255); }
+
+struct Carver {
+  uint8_t* base;
+  int64_t off = 0;
+  template <typename P>
+  P* take(int64_t bytes) {
+    P* p = base ? reinterpret_cast<P*>(base + off) : nullptr;
+    off += align256(bytes);
+    return p;
+  }
+};
+
+MatView mv(const void* p, int64_t ld, int64_t bs1 = 0, int64_t bs2 = 0) {
+  MatView v;
+  v.ptr = p;
+  v.ld = ld;
+  v.bs1 = bs1;
+  v.bs2 = bs2;
+  return v;
+}
+
+template <typename T>
+int run_gemm(GemmDesc& d, cudaStream_t st, int cls) {
+  KernelTimer* t = g_timer;
+  int64_t flops = 2LL * d.M * d.N * d.K * d.nb1 * d.nb2;
+  if (d.causal != CAUSAL_NONE) flops /= 2;  // algorithmic work of a causal product
+  if (t) t->begin(cls, st);
+  int rc = gemm<T>(d, st);
+  if (t) t->end(cls, st, flops);
+  ++g_kernel_launches;
+  return rc;
+}
+
+#define RC(x)              \
+  do {                     \
+    int _rc = (x);         \
+    if (_rc) return _rc;   \
+  } while (0)
+
+struct ElemScope {
+  cudaStream_t st;
+  int n;
+  ElemScope(cudaStream_t s, int n_) : st(s), n(n_) {
+    if (g_timer) g_timer->begin(KCLS_ELEM, st);
+  }
+  ~ElemScope() {
+    if (g_timer) g_timer->end(KCLS_ELEM, st, 0);
+    g_kernel_launches += n;
+  }
+};
+
+}  // namespace
+
+int64_t block_acts_bytes(const Shape& sh, int e) {
+  Carver c{nullptr};
+  const int64_t T = sh.T(), h = sh.h, B = (int64_t)sh.mbs * sh.nh, s = sh.s;
+  c.take<char>(T * h * e);      // a
+  c.take<char>(T * 4);          // mu1
+  c.take<char>(T * 4);          // rs1
+  c.take<char>(T * 3 * h * e);  // qkv
+  c.take<char>(B * s * s * e);  // P
+  c.take<char>(T * h * e);      // o
+  c.take<char>(T * h * e);      // x1
+  c.take<char>(T * h * e);      // a2
+  c.take<char>(T * 4);
+  c.take<char>(T * 4);
+  c.take<char>(T * 4 * h * e);  // u
+  c.take<char>(T * 4 * h * e);  // g
+  return c.off;
+}
+
+template <typename T>
+void carve_block_acts(const Shape& sh, uint8_t* base, BlockActs<T>& a) {
+  Carver c{base};
+  const int64_t Tn = sh.T(), h = sh.h, B = (int64_t)sh.mbs * sh.nh, s = sh.s, e = sizeof(T);
+  a.a = c.take<T>(Tn * h * e);
+  a.mu1 = c.take<float>(Tn * 4);
+  a.rs1 = c.take<float>(Tn * 4);
+  a.qkv = c.take<T>(Tn * 3 * h * e);
+  a.P = c.take<T>(B * s * s * e);
+  a.o = c.take<T>(Tn * h * e);
+  a.x1 = c.take<T>(Tn * h * e);
+  a.a2 = c.take<T>(Tn * h * e);
+  a.mu2 = c.take<float>(Tn * 4);
+  a.rs2 = c.take<float>(Tn * 4);
+  a.u = c.take<T>(Tn * 4 * h * e);
+  a.g = c.take<T>(Tn * 4 * h * e);
+}
+
+int64_t scratch_bytes(const Shape& sh, int e, bool with_head) {
+  const int64_t T = sh.T(), h = sh.h, B = (int64_t)sh.mbs * sh.nh, s = sh.s;
+  Carver c{nullptr};
+  c.take<char>(B * s * s * 4);
+  c.take<char>(B * s * s * e);
+  c.take<char>(T * 4 * h * e);
+  c.take<char>(T * h * e);
+  c.take<char>(T * h * e);
+  c.take<char>(T * h * e);
+  c.take<char>(T * 3 * h * e);
+  c.take<char>(with_head ? T * (int64_t)sh.V * e : 0);
+  c.take<char>(T * 4);
+  c.take<char>(T * 4);
+  c.take<char>(T * 4);
+  return c.off;
+}
+
+template <typename T>
+void carve_scratch(const Shape& sh, uint8_t* base, bool with_head, Scratch<T>& sc) {
+  const int64_t Tn = sh.T(), h = sh.h, B = (int64_t)sh.mbs * sh.nh, s = sh.s, e = sizeof(T);
+  Carver c{base};
+  sc.S = c.take<float>(B * s * s * 4);
+  sc.dS = c.take<T>(B * s * s * e);
+  sc.big1 = c.take<T>(Tn * 4 * h * e);
+  sc.t1 = c.take<T>(Tn * h * e);
+  sc.t2 = c.take<T>(Tn * h * e);
+  sc.t3 = c.take<T>(Tn * h * e);
+  sc.qkv_g = c.take<T>(Tn * 3 * h * e);
+  sc.logits = c.take<T>(with_head ? Tn * (int64_t)sh.V * e : 0);
+  sc.loss_rows = c.take<float>(Tn * 4);
+  sc.mu = c.take<float>(Tn * 4);
+  sc.rs = c.take<float>(Tn * 4);
+}
+
+// ------------------------------------------------------------------ block
+template <typename T>
+int block_fwd(const Shape& sh, const T* w, BlockActs<T>& A, T* y, Scratch<T>& sc, cudaStream_t st) {
+  const BlockLayout L(sh.h);
+  const int Tn = sh.T(), h = sh.h, nh = sh.nh, s = sh.s, dh = sh.dh(), mbs = sh.mbs;
+  const int64_t Sbs2 = (int64_t)s * s, Sbs1 = nh * Sbs2;
+  {
+    ElemScope es(st, 1);
+    RC(layernorm_fwd<T>(A.x, w + L.ln1_g, w + L.ln1_b, A.a, A.mu1, A.rs1, Tn, h, st));
+  }
+  {  // qkv = a Wqkv + bqkv
+    GemmDesc d;
+    d.M = Tn; d.N = 3 * h; d.K = h;
+    d.A = mv(A.a, h);
+    d.B = mv(w + L.w_qkv, 3 * h); d.b_mn = true;
+    d.C = mv(A.qkv, 3 * h);
+    d.epi = EPI_BIAS; d.bias = w + L.b_qkv;
+    RC(run_gemm<T>(d, st, KCLS_GEMM));
+  }
+  {  // S = q k^T (fp32), causal tiles only
+    GemmDesc d;
+    d.M = s; d.N = s; d.K = dh; d.nb1 = mbs; d.nb2 = nh;
+    d.A = mv(A.qkv, 3 * h, (int64_t)s * 3 * h, dh);
+    d.B = mv(A.qkv + h, 3 * h, (int64_t)s * 3 * h, dh);
+    d.C = mv(sc.S, s, Sbs1, Sbs2); d.c_f32 = true;
+    d.causal = CAUSAL_SKIP_UPPER;
+    RC(run_gemm<T>(d, st, KCLS_ATTN));
+  }
+  {
+    ElemScope es(st, 1);
+    RC(softmax_causal_fwd<T>(sc.S, A.P, mbs * nh, s, 1.0f / sqrtf((float)dh), st));
+  }
+  {  // o = P v
+    GemmDesc d;
+    d.M = s; d.N = dh; d.K = s; d.nb1 = mbs; d.nb2 = nh;
+    d.A = mv(A.P, s, Sbs1, Sbs2);
+    d.B = mv(A.qkv + 2 * h, 3 * h, (int64_t)s * 3 * h, dh); d.b_mn = true;
+    d.C = mv(A.o, h, (int64_t)s * h, dh);
+    d.causal = CAUSAL_K_LT_MEND;
+    RC(run_gemm<T>(d, st, KCLS_ATTN));
+  }
+  {  // x1 = x + o Wo + bo
+    GemmDesc d;
+    d.M = Tn; d.N = h; d.K = h;
+    d.A = mv(A.o, h);
+    d.B = mv(w + L.w_o, h); d.b_mn = true;
+    d.C = mv(A.x1, h);
+    d.epi = EPI_BIAS_RESID; d.bias = w + L.b_o; d.R = mv(A.x, h);
+    RC(run_gemm<T>(d, st, KCLS_GEMM));
+  }
+  {
+    ElemScope es(st, 1);
+    RC(layernorm_fwd<T>(A.x1, w + L.ln2_g, w + L.ln2_b, A.a2, A.mu2, A.rs2, Tn, h, st));
+  }
+  {  // u = a2 W1 + b1 ; g = gelu(u)
+    GemmDesc d;
+    d.M = Tn; d.N = 4 * h; d.K = h;
+    d.A = mv(A.a2, h);
+    d.B = mv(w + L.w_1, 4 * h); d.b_mn = true;
+    d.C = mv(A.g, 4 * h);
+    d.epi = EPI_BIAS_GELU; d.bias = w + L.b_1; d.AUX = mv(A.u, 4 * h);
+    RC(run_gemm<T>(d, st, KCLS_GEMM));
+  }
+  {  // y = x1 + g W2 + b2
+    GemmDesc d;
+    d.M = Tn; d.N = h; d.K = 4 * h;
+    d.A = mv(A.g, 4 * h);
+    d.B = mv(w + L.w_2, h); d.b_mn = true;
+    d.C = mv(y, h);
+    d.epi = EPI_BIAS_RESID; d.bias = w + L.b_2; d.R = mv(A.x1, h);
+    RC(run_gemm<T>(d, st, KCLS_GEMM));
+  }
+  return MOBIUS_OK;
+}
+
+template <typename T>
+int block_bwd(const Shape& sh, const T* w, const BlockActs<T>& A, const T* dy, T* dx, float* G, Scratch<T>& sc,
+              cudaStream_t st) {
+  const BlockLayout L(sh.h);
+  const int Tn = sh.T(), h = sh.h, nh = sh.nh, s = sh.s, dh = sh.dh(), mbs = sh.mbs;
+  const int64_t Sbs2 = (int64_t)s * s, Sbs1 = nh * Sbs2;
+  const float scale = 1.0f / sqrtf((float)dh);
+  T* du = sc.big1;
+  {  // du = (dy W2^T) * gelu'(u)
+    GemmDesc d;
+    d.M = Tn; d.N = 4 * h; d.K = h;
+    d.A = mv(dy, h);
+    d.B = mv(w + L.w_2, h);
+    d.C = mv(du, 4 * h);
+    d.epi = EPI_GELU_BWD; d.R = mv(A.u, 4 * h);
+    RC(run_gemm<T>(d, st, KCLS_GEMM));
+  }
+  {  // dW2 += g^T dy
+    GemmDesc d;
+    d.M = 4 * h; d.N = h; d.K = Tn;
+    d.A = mv(A.g, 4 * h); d.a_mn = true;
+    d.B = mv(dy, h); d.b_mn = true;
+    d.C = mv(G + L.w_2, h); d.c_f32 = true;
+    d.epi = EPI_ACCUM; d.accumulate = true;
+    RC(run_gemm<T>(d, st, KCLS_GEMM));
+  }
+  {
+    ElemScope es(st, 2);
+    RC(colsum_accum<T>(dy, h, Tn, h, G + L.b_2, st));
+    RC(colsum_accum<T>(du, 4 * h, Tn, 4 * h, G + L.b_1, st));
+  }
+  {  // dW1 += a2^T du
+    GemmDesc d;
+    d.M = h; d.N = 4 * h; d.K = Tn;
+    d.A = mv(A.a2, h); d.a_mn = true;
+    d.B = mv(du, 4 * h); d.b_mn = true;
+    d.C = mv(G + L.w_1, 4 * h); d.c_f32 = true;
+    d.epi = EPI_ACCUM; d.accumulate = true;
+    RC(run_gemm<T>(d, st, KCLS_GEMM));
+  }
+  {  // da2 = du W1^T
+    GemmDesc d;
+    d.M = Tn; d.N = h; d.K = 4 * h;
+    d.A = mv(du, 4 * h);
+    d.B = mv(w + L.w_1, 4 * h);
+    d.C = mv(sc.t1, h);
+    RC(run_gemm<T>(d, st, KCLS_GEMM));
+  }
+  T* dx1 = sc.t2;
+  {
+    ElemScope es(st, 1);
+    RC(layernorm_bwd<T>(sc.t1, A.x1, w + L.ln2_g, A.mu2, A.rs2, dy, dx1, G + L.ln2_g, G + L.ln2_b, Tn, h, st));
+  }
+  {  // dWo += o^T dx1
+    GemmDesc d;
+    d.M = h; d.N = h; d.K = Tn;
+    d.A = mv(A.o, h); d.a_mn = true;
+    d.B = mv(dx1, h); d.b_mn = true;
+    d.C = mv(G + L.w_o, h); d.c_f32 = true;
+    d.epi = EPI_ACCUM; d.accumulate = true;
+    RC(run_gemm<T>(d, st, KCLS_GEMM));
+  }
+  {
+    ElemScope es(st, 1);
+    RC(colsum_accum<T>(dx1, h, Tn, h, G + L.b_o, st));
+  }
+  T* dO = sc.t3;
+  {  // do = dx1 Wo^T
+    GemmDesc d;
+    d.M = Tn; d.N = h; d.K = h;
+    d.A = mv(dx1, h);
+    d.B = mv(w + L.w_o, h);
+    d.C = mv(dO, h);
+    RC(run_gemm<T>(d, st, KCLS_GEMM));
+  }
+  {  // dP = do v^T (fp32)
+    GemmDesc d;
+    d.M = s; d.N = s; d.K = dh; d.nb1 = mbs; d.nb2 = nh;
+    d.A = mv(dO, h, (int64_t)s * h, dh);
+    d.B = mv(A.qkv + 2 * h, 3 * h, (int64_t)s * 3 * h, dh);
+    d.C = mv(sc.S, s, Sbs1, Sbs2); d.c_f32 = true;
+    d.causal = CAUSAL_SKIP_UPPER;
+    RC(run_gemm<T>(d, st, KCLS_ATTN));
+  }
+  {
+    ElemScope es(st, 1);
+    RC(softmax_causal_bwd<T>(A.P, sc.S, sc.dS, mbs * nh, s, scale, st));
+  }
+  T* dqkv = sc.qkv_g;
+  {  // dV = P^T do
+    GemmDesc d;
+    d.M = s; d.N = dh; d.K = s; d.nb1 = mbs; d.nb2 = nh;
+    d.A = mv(A.P, s, Sbs1, Sbs2); d.a_mn = true;
+    d.B = mv(dO, h, (int64_t)s * h, dh); d.b_mn = true;
+    d.C = mv(dqkv + 2 * h, 3 * h, (int64_t)s * 3 * h, dh);
+    d.causal = CAUSAL_K_GE_M0;
+    RC(run_gemm<T>(d, st, KCLS_ATTN));
+  }
+  {  // dQ = dS K
+    GemmDesc d;
+    d.M = s; d.N = dh; d.K = s; d.nb1 = mbs; d.nb2 = nh;
+    d.A = mv(sc.dS, s, Sbs1, Sbs2);
+    d.B = mv(A.qkv + h, 3 * h, (int64_t)s * 3 * h, dh); d.b_mn = true;
+    d.C = mv(dqkv, 3 * h, (int64_t)s * 3 * h, dh);
+    d.causal = CAUSAL_K_LT_MEND;
+    RC(run_gemm<T>(d, st, KCLS_ATTN));
+  }
+  {  // dK = dS^T Q
+    GemmDesc d;
+    d.M = s; d.N = dh; d.K = s; d.nb1 = mbs; d.nb2 = nh;
+    d.A = mv(sc.dS, s, Sbs1, Sbs2); d.a_mn = true;
+    d.B = mv(A.qkv, 3 * h, (int64_t)s * 3 * h, dh); d.b_mn = true;
+    d.C = mv(dqkv + h, 3 * h, (int64_t)s * 3 * h, dh);
+    d.causal = CAUSAL_K_GE_M0;
+    RC(run_gemm<T>(d, st, KCLS_ATTN));
+  }
+  {  // dWqkv += a^T dqkv
+    GemmDesc d;
+    d.M = h; d.N = 3 * h; d.K = Tn;
+    d.A = mv(A.a, h); d.a_mn = true;
+    d.B = mv(dqkv, 3 * h); d.b_mn = true;
+    d.C = mv(G + L.w_qkv, 3 * h); d.c_f32 = true;
+    d.epi = EPI_ACCUM; d.accumulate = true;
+    RC(run_gemm<T>(d, st, KCLS_GEMM));
+  }
+  {
+    ElemScope es(st, 1);
+    RC(colsum_accum<T>(dqkv, 3 * h, Tn, 3 * h, G + L.b_qkv, st));
+  }
+  {  // da = dqkv Wqkv^T
+    GemmDesc d;
+    d.M = Tn; d.N = h; d.K = 3 * h;
+    d.A = mv(dqkv, 3 * h);
+    d.B = mv(w + L.w_qkv, 3 * h);
+    d.C = mv(sc.t1, h);
+    RC(run_gemm<T>(d, st, KCLS_GEMM));
+  }
+  {
+    ElemScope es(st, 1);
+    RC(layernorm_bwd<T>(sc.t1, A.x, w + L.ln1_g, A.mu1, A.rs1, dx1, dx, G + L.ln1_g, G + L.ln1_b, Tn, h, st));
+  }
+  return MOBIUS_OK;
+}
+
+template <typename T>
+int embed_layer_fwd(const Shape& sh, const T* w, const int32_t* tok, T* x, cudaStream_t st) {
+  const EmbedLayout L(sh.h, sh.V, sh.s);
+  ElemScope es(st, 1);
+  return embed_fwd<T>(tok, w + L.wte, w + L.wpe, x, sh.mbs, sh.s, sh.h, st);
+}
+
+template <typename T>
+int embed_layer_bwd(const Shape& sh, const T* w, const int32_t* tok, const T* dx, float* G, cudaStream_t st) {
+  const EmbedLayout L(sh.h, sh.V, sh.s);
+  ElemScope es(st, 2);
+  return embed_bwd<T>(tok, dx, G + L.wte, G + L.wpe, sh.mbs, sh.s, sh.h, st);
+}
+
+template <typename T>
+int head_layer_fwd_bwd(const Shape& sh, const T* w, const T* x, const int32_t* tok, float inv_ntok, T* dx, float* G,
+                       double* loss_acc, Scratch<T>& sc, cudaStream_t st) {
+  const HeadLayout L(sh.h, sh.V);
+  const int Tn = sh.T(), h = sh.h, V = sh.V;
+  {
+    ElemScope es(st, 1);
+    RC(layernorm_fwd<T>(x, w + L.lnf_g, w + L.lnf_b, sc.t1, sc.mu, sc.rs, Tn, h, st));
+  }
+  {  // logits = a Whead
+    GemmDesc d;
+    d.M = Tn; d.N = V; d.K = h;
+    d.A = mv(sc.t1, h);
+    d.B = mv(w + L.w_head, V); d.b_mn = true;
+    d.C = mv(sc.logits, V);
+    RC(run_gemm<T>(d, st, KCLS_GEMM));
+  }
+  {
+    ElemScope es(st, 2);
+    RC(cross_entropy_fwd_bwd<T>(sc.logits, tok, sc.loss_rows, Tn, V, sh.s, inv_ntok, st));
+    RC(loss_accumulate(sc.loss_rows, Tn, loss_acc, st));
+  }
+  {  // dWhead += a^T dlogits
+    GemmDesc d;
+    d.M = h; d.N = V; d.K = Tn;
+    d.A = mv(sc.t1, h); d.a_mn = true;
+    d.B = mv(sc.logits, V); d.b_mn = true;
+    d.C = mv(G + L.w_head, V); d.c_f32 = true;
+    d.epi = EPI_ACCUM; d.accumulate = true;
+    RC(run_gemm<T>(d, st, KCLS_GEMM));
+  }
+  {  // da = dlogits Whead^T
+    GemmDesc d;
+    d.M = Tn; d.N = h; d.K = V;
+    d.A = mv(sc.logits, V);
+    d.B = mv(w + L.w_head, V);
+    d.C = mv(sc.t2, h);
+    RC(run_gemm<T>(d, st, KCLS_GEMM));
+  }
+  {
+    ElemScope es(st, 1);
+    RC(layernorm_bwd<T>(sc.t2, x, w + L.lnf_g, sc.mu, sc.rs, (const T*)nullptr, dx, G + L.lnf_g, G + L.lnf_b, Tn,
+                        h, st));
+  }
+  return MOBIUS_OK;
+}
+
+#define INST(T)                                                                                                   \
+  template void carve_block_acts<T>(const Shape&, uint8_t*, BlockActs<T>&);                                      \
+  template void carve_scratch<T>(const Shape&, uint8_t*, bool, Scratch<T>&);                                     \
+  template int block_fwd<T>(const Shape&, const T*, BlockActs<T>&, T*, Scratch<T>&, cudaStream_t);               \
+  template int block_bwd<T>(const Shape&, const T*, const BlockActs<T>&, const T*, T*, float*, Scratch<T>&,      \
+                            cudaStream_t);                                                                       \
+  template int embed_layer_fwd<T>(const Shape&, const T*, const int32_t*, T*, cudaStream_t);                      \
+  template int embed_layer_bwd<T>(const Shape&, const T*, const int32_t*, const T*, float*, cudaStream_t);        \
+  template int head_layer_fwd_bwd<T>(const Shape&, const T*, const T*, const int32_t*, float, T*, float*, double*, \
+                                     Scratch<T>&, cudaStream_t);
+INST(float)
+INST(__nv_bfloat16)
+
+}  // namespace mobius

@@ -1,0 +1,106 @@
+// Layer-level operations of the GPT stage compute (rows a4, a6, a7 of
+// SURVEY §8(a)).  Weights are the packed oracle-layout tensors of one
+// profile layer in the path type T; gradients are fp32 accumulators of the
+// same layout.  Everything is launched on one stream.
+#pragma once
+
+#include <cstdint>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+
+#include "../../include/mobius.h"
+
+namespace mobius {
+
+struct Shape {
+  int h, nh, s, mbs, V;
+  int T() const { return mbs * s; }
+  int dh() const { return h / nh; }
+};
+
+// element offsets of the block tensors inside one packed block (oracle order)
+struct BlockLayout {
+  int64_t ln1_g, ln1_b, w_qkv, b_qkv, w_o, b_o, ln2_g, ln2_b, w_1, b_1, w_2, b_2, total;
+  explicit BlockLayout(int64_t h);
+};
+struct EmbedLayout {
+  int64_t wte, wpe, total;
+  EmbedLayout(int64_t h, int64_t V, int64_t s);
+};
+struct HeadLayout {
+  int64_t lnf_g, lnf_b, w_head, total;
+  HeadLayout(int64_t h, int64_t V);
+};
+
+// Saved activations of one block for one microbatch (all device pointers).
+template <typename T>
+struct BlockActs {
+  const T* x;      // input [T, h]
+  T* a;            // LN1(x)
+  float *mu1, *rs1;
+  T* qkv;          // [T, 3h]
+  T* P;            // [mbs*nh, s, s] causal softmax probabilities
+  T* o;            // attention output [T, h]
+  T* x1;           // x + o Wo + bo
+  T* a2;           // LN2(x1)
+  float *mu2, *rs2;
+  T* u;            // a2 W1 + b1  [T, 4h]
+  T* g;            // gelu(u)     [T, 4h]
+};
+
+template <typename T>
+struct Scratch {
+  float* S;        // [mbs*nh, s, s] fp32 scores / dP
+  T* dS;           // [mbs*nh, s, s]
+  T* big1;         // [T, 4h]
+  T* t1;           // [T, h]
+  T* t2;           // [T, h]
+  T* t3;           // [T, h]
+  T* qkv_g;        // [T, 3h]
+  T* logits;       // [T, V]
+  float* loss_rows;  // [T]
+  float *mu, *rs;  // [T] (head LN)
+};
+
+// bytes of one BlockActs set / of the Scratch (for arena planning)
+int64_t block_acts_bytes(const Shape& sh, int elem);
+int64_t scratch_bytes(const Shape& sh, int elem, bool with_head);
+template <typename T>
+void carve_block_acts(const Shape& sh, uint8_t* base, BlockActs<T>& a);
+template <typename T>
+void carve_scratch(const Shape& sh, uint8_t* base, bool with_head, Scratch<T>& s);
+
+// y = block(x); fills acts (acts.x must be set)
+template <typename T>
+int block_fwd(const Shape& sh, const T* w, BlockActs<T>& acts, T* y, Scratch<T>& sc, cudaStream_t st);
+// dx = d block / dx (dy); grads (fp32, block layout) +=
+template <typename T>
+int block_bwd(const Shape& sh, const T* w, const BlockActs<T>& acts, const T* dy, T* dx, float* grads,
+              Scratch<T>& sc, cudaStream_t st);
+// x0 = wte[tok] + wpe; tok = microbatch tokens [mbs][s+1]
+template <typename T>
+int embed_layer_fwd(const Shape& sh, const T* w, const int32_t* tok, T* x, cudaStream_t st);
+template <typename T>
+int embed_layer_bwd(const Shape& sh, const T* w, const int32_t* tok, const T* dx, float* grads, cudaStream_t st);
+// LN_f + LM head + CE fwd+bwd: loss accumulated into loss_acc (sum of token
+// losses, double); dx = d/dx of (sum loss) * inv_ntok; grads +=
+template <typename T>
+int head_layer_fwd_bwd(const Shape& sh, const T* w, const T* x, const int32_t* tok, float inv_ntok, T* dx,
+                       float* grads, double* loss_acc, Scratch<T>& sc, cudaStream_t st);
+
+// GEMM dispatch on the path type
+template <typename T>
+int gemm(const struct GemmDesc& d, cudaStream_t st);
+
+// per-kernel-class timing hooks (set by the runtime when MOBIUS_FLAG_TIMING)
+struct KernelTimer {
+  virtual ~KernelTimer() {}
+  virtual void begin(int cls, cudaStream_t st) = 0;
+  virtual void end(int cls, cudaStream_t st, int64_t flops) = 0;
+};
+enum { KCLS_GEMM = 0, KCLS_ATTN = 1, KCLS_ELEM = 2 };
+void set_kernel_timer(KernelTimer* t);
+KernelTimer* kernel_timer();
+extern thread_local int64_t g_kernel_launches;
+
+}  // namespace mobius

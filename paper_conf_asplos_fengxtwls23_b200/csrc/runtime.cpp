@@ -1,0 +1,1087 @@
+// Mobius per-rank runtime (rows a1-a11 of SURVEY §8(a)).
+//
+//  * Stage store: this rank's stages live in pinned host DRAM in the
+//    transfer precision; fp32 master / m / v in host memory (P:L428-434,
+//    P:L150-152).
+//  * HBM ring of G bytes (the cap of Eq 4/5) with two-ended placement:
+//    residence r sits at the bottom (r even) or the top (r odd) of the ring.
+//    Loading residence r+1 starts when residence r starts computing and
+//    writes only bytes that do not overlap residence r (the Eq 5/6 prefetch
+//    P <= G - S); the remainder waits for residence r's release (Eq 9).
+//  * Per-GPU schedule (Fig 4): F_{j,1..M} for my stages
+//    ascending, then B_{j,1..M} descending; the last stage stays resident.
+//  * Stage-input checkpoints are the activation receive slots;
+//    backward recomputes the stage forward from them.
+//  * Activations / activation-gradients go straight from the producing
+//    kernel's epilogue into the consumer rank's slot (CUDA IPC mapping over
+//    NVLink), followed by a system-scope release flag (Eq 8).
+//  * After B_{j,M}: fp32 dW -> transfer precision, D2H on a side stream,
+//    host AdamW on worker threads, overlapping the remaining
+//    backward.  The step returns when every update has landed (synchronous
+//    update).
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <cmath>
+#include <condition_variable>
+#include <cstring>
+#include <deque>
+#include <memory>
+#include <mutex>
+#include <random>
+#include <thread>
+#include <vector>
+
+#include "common.h"
+#include "elem.h"
+#include "host.h"
+#include "ops.h"
+
+namespace mobius {
+
+typedef __nv_bfloat16 bf16;
+
+namespace {
+
+inline int64_t al256(int64_t x) { return (x + 255) & ~int64_t(255); }
+
+int64_t now_ns() {
+  return std::chrono::duration_cast<std::chrono::nanoseconds>(std::chrono::steady_clock::now().time_since_epoch())
+      .count();
+}
+
+struct StageDesc {
+  int j = 0;                      // global 0-based stage index
+  int first = 0, last = 0;        // profile layers [first, last)
+  int64_t n_params = 0;           // elements
+  int64_t param_off = 0;          // offset in the oracle flat vector
+  std::vector<int64_t> layer_off; // element offset of each layer inside the stage blob
+  bool has_embed = false, has_head = false;
+  int n_blocks = 0;
+  int owner = 0;                  // rank (GPU) running the stage
+  int ord = 0;                    // index among the owner's stages (ascending)
+};
+
+struct PeerInfo {
+  int rank;
+  cudaIpcMemHandle_t handle;
+  int64_t off_ckpt, off_gslot, off_fflag, off_bflag, slot_bytes;
+  int n_local, M;
+};
+
+struct Load {           // one residence of a stage in the ring
+  int stage_local;      // index into mine
+  int end;              // 0 bottom, 1 top
+  int64_t base;         // byte offset in the ring
+  int64_t bytes;
+};
+
+struct EventTimer : KernelTimer {
+  struct Rec {
+    cudaEvent_t a, b;
+    int cls;
+    int64_t flops;
+  };
+  std::vector<Rec> recs;
+  std::vector<cudaEvent_t> pool;
+  size_t used = 0;
+  cudaEvent_t get() {
+    if (used == pool.size()) {
+      cudaEvent_t e;
+      cudaEventCreate(&e);
+      pool.push_back(e);
+    }
+    return pool[used++];
+  }
+  void begin(int cls, cudaStream_t st) override {
+    Rec r;
+    r.a = get();
+    r.b = nullptr;
+    r.cls = cls;
+    r.flops = 0;
+    cudaEventRecord(r.a, st);
+    recs.push_back(r);
+  }
+  void end(int cls, cudaStream_t st, int64_t flops) override {
+    Rec& r = recs.back();
+    r.b = get();
+    r.flops = flops;
+    cudaEventRecord(r.b, st);
+  }
+  void reset() {
+    recs.clear();
+    used = 0;
+  }
+  ~EventTimer() {
+    for (auto e : pool) cudaEventDestroy(e);
+  }
+};
+
+}  // namespace
+
+}  // namespace mobius
+
+using namespace mobius;
+
+struct mobius_ctx {
+  mobius_model_cfg cfg;
+  mobius_plan_t plan;
+  mobius_dist dist;
+  Shape sh;
+  int esz = 2;
+  bool poisoned = false;
+  int64_t step_count = 0;
+
+  std::vector<StageDesc> all;   // every stage of the plan
+  std::vector<int> mine;        // global indices of my stages (ascending)
+  std::vector<int> rank_of;     // stage -> rank
+  std::vector<Load> loads;      // residences in load order
+  std::vector<int> res_f, res_b;  // local stage -> residence index (fwd / bwd)
+
+  // host
+  std::vector<void*> h_weights;   // pinned, per local stage, transfer precision
+  std::vector<void*> h_grads;     // pinned, per local stage
+  std::vector<float*> h_master, h_m, h_v;
+  int32_t* h_tokens = nullptr;    // pinned staging of the step's tokens
+  int64_t h_tokens_cap = 0;
+  double* h_loss = nullptr;
+  std::unique_ptr<ThreadPool> pool;
+
+  // device
+  uint8_t* arena = nullptr;
+  int64_t arena_bytes = 0, ring_bytes = 0;
+  uint8_t* ring = nullptr;
+  float* grad_acc = nullptr;      // fp32, max local stage params
+  uint8_t* grad_stage = nullptr;  // transfer precision, max local stage params
+  uint8_t* ckpt = nullptr;        // [n_local][M] act slots (stage inputs)
+  uint8_t* gslot = nullptr;       // [n_local][M] act-grad slots
+  int* fflag = nullptr;           // [n_local][M]
+  int* bflag = nullptr;           // [n_local][M]
+  int64_t slot_bytes = 0;
+  int max_M = 0;
+  uint8_t* acts_base = nullptr;   // per-block saved activations (recompute)
+  int64_t acts_bytes = 0;
+  int max_blocks = 0;
+  uint8_t* xs_base = nullptr;     // [max_blocks+1] x buffers [T,h]
+  uint8_t* scratch_base = nullptr;
+  uint8_t* tok_dev = nullptr;
+  double* loss_dev = nullptr;
+  int64_t off_ckpt = 0, off_gslot = 0, off_fflag = 0, off_bflag = 0;
+
+  // peers
+  std::vector<uint8_t*> peer_base;  // opened IPC bases (nullptr for me)
+  std::vector<PeerInfo> peers;
+  bool connected = false;
+
+  // streams / events
+  cudaStream_t s_comp = nullptr, s_h2d = nullptr, s_d2h = nullptr;
+  std::vector<cudaEvent_t> ev_release, ev_loaded;
+  std::vector<cudaEvent_t> ev_part_a, ev_part_b;   // per-copy timing (2 parts per load)
+  std::vector<int64_t> part_bytes;
+  std::vector<cudaEvent_t> ev_gready, ev_d2h;      // per local stage
+  cudaEvent_t ev_step0 = nullptr, ev_step1 = nullptr;
+  std::vector<cudaEvent_t> ev_wait_a, ev_wait_b;   // exposed load waits
+
+  // update worker
+  std::thread upd_thread;
+  std::mutex upd_mu;
+  std::condition_variable upd_cv, upd_done_cv;
+  std::deque<int> upd_queue;
+  int upd_pending = 0;
+  bool upd_stop = false;
+  int64_t upd_ns = 0;
+  int64_t last_bwd_host_ns = 0, last_update_end_ns = 0;
+
+  // stats / trace
+  std::vector<int32_t> trace;
+  EventTimer timer;
+  mobius_step_stats stats;
+  int64_t launches_step = 0;
+};
+
+namespace {
+
+#define CU(x)                                                                               \
+  do {                                                                                      \
+    cudaError_t _e = (x);                                                                   \
+    if (_e != cudaSuccess) {                                                                \
+      ctx->poisoned = true;                                                                 \
+      MOBIUS_FAIL(MOBIUS_ECUDA, "%s failed: %s (%s:%d)", #x, cudaGetErrorString(_e), __FILE__, __LINE__); \
+    }                                                                                       \
+  } while (0)
+
+#define RC(x)                       \
+  do {                              \
+    int _rc = (x);                  \
+    if (_rc) {                      \
+      ctx->poisoned = true;         \
+      return _rc;                   \
+    }                               \
+  } while (0)
+
+int64_t layer_numel(const mobius_model_cfg& c, int i) {
+  const int64_t h = c.hidden, V = c.vocab, s = c.seq_len;
+  if (i == 0) return V * h + s * h;
+  if (i == c.n_layers + 1) return 2 * h + h * V;
+  return 12 * h * h + 13 * h;
+}
+
+void update_worker(mobius_ctx* ctx) {
+  for (;;) {
+    int ls;
+    {
+      std::unique_lock<std::mutex> lk(ctx->upd_mu);
+      ctx->upd_cv.wait(lk, [&] { return ctx->upd_stop || !ctx->upd_queue.empty(); });
+      if (ctx->upd_stop && ctx->upd_queue.empty()) return;
+      ls = ctx->upd_queue.front();
+      ctx->upd_queue.pop_front();
+    }
+    cudaEventSynchronize(ctx->ev_d2h[ls]);
+    int64_t t0 = now_ns();
+    const StageDesc& st = ctx->all[ctx->mine[ls]];
+    AdamWArgs a{ctx->cfg.lr, ctx->cfg.beta1, ctx->cfg.beta2, ctx->cfg.eps, ctx->cfg.weight_decay,
+                ctx->step_count + 1};
+    const int kind = ctx->cfg.dtype == MOBIUS_F32 ? 1 : 0;
+    adamw_update(ctx->h_master[ls], ctx->h_m[ls], ctx->h_v[ls], ctx->h_grads[ls], kind, ctx->h_weights[ls], kind,
+                 st.n_params, a, *ctx->pool);
+    int64_t t1 = now_ns();
+    {
+      std::lock_guard<std::mutex> g(ctx->upd_mu);
+      ctx->upd_ns += t1 - t0;
+      ctx->last_update_end_ns = t1;
+      if (--ctx->upd_pending == 0) ctx->upd_done_cv.notify_all();
+    }
+  }
+}
+
+void fill_seeded(float* dst, int64_t n, uint64_t seed, int64_t stream_off, float std_) {
+  // counter-based N(0, std^2): splitmix64 -> Box-Muller (deterministic per element index)
+  for (int64_t i = 0; i < n; ++i) {
+    uint64_t z = seed * 0x9E3779B97F4A7C15ull + (uint64_t)(stream_off + i) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    z ^= z >> 31;
+    double u1 = ((z >> 11) + 1) * (1.0 / 9007199254740993.0);
+    double u2 = ((z & 0x7FF) + 0.5) / 2048.0;
+    dst[i] = (float)(std::sqrt(-2.0 * std::log(u1)) * std::cos(6.283185307179586 * u2) * std_);
+  }
+}
+
+// initialise the fp32 master of one local stage (oracle init recipe O-1 when
+// init_params is NULL: N(0,0.02) weights, N(0,0.02/sqrt(2L)) for w_o/w_2,
+// zero biases, unit LN gains)
+void seeded_stage_init(const mobius_model_cfg& c, const StageDesc& st, float* out, uint64_t seed) {
+  const int64_t h = c.hidden;
+  const float proj = 0.02f / std::sqrt(2.0f * c.n_layers);
+  for (int li = st.first; li < st.last; ++li) {
+    float* p = out + st.layer_off[li - st.first];
+    int64_t base = st.param_off + st.layer_off[li - st.first];
+    if (li == 0) {
+      fill_seeded(p, layer_numel(c, 0), seed, base, 0.02f);
+    } else if (li == c.n_layers + 1) {
+      for (int64_t i = 0; i < h; ++i) p[i] = 1.f, p[h + i] = 0.f;
+      fill_seeded(p + 2 * h, h * (int64_t)c.vocab, seed, base + 2 * h, 0.02f);
+    } else {
+      BlockLayout L(h);
+      for (int64_t i = 0; i < h; ++i) {
+        p[L.ln1_g + i] = 1.f;
+        p[L.ln1_b + i] = 0.f;
+        p[L.ln2_g + i] = 1.f;
+        p[L.ln2_b + i] = 0.f;
+        p[L.b_o + i] = 0.f;
+        p[L.b_2 + i] = 0.f;
+      }
+      for (int64_t i = 0; i < 3 * h; ++i) p[L.b_qkv + i] = 0.f;
+      for (int64_t i = 0; i < 4 * h; ++i) p[L.b_1 + i] = 0.f;
+      fill_seeded(p + L.w_qkv, 3 * h * h, seed, base + L.w_qkv, 0.02f);
+      fill_seeded(p + L.w_o, h * h, seed, base + L.w_o, proj);
+      fill_seeded(p + L.w_1, 4 * h * h, seed, base + L.w_1, 0.02f);
+      fill_seeded(p + L.w_2, 4 * h * h, seed, base + L.w_2, proj);
+    }
+  }
+}
+
+template <typename T>
+T* tptr(uint8_t* p) {
+  return reinterpret_cast<T*>(p);
+}
+
+// ---------------------------------------------------------------- step
+template <typename T>
+struct StepRunner {
+  mobius_ctx* ctx;
+  const int32_t* tok_dev;
+  int M;
+  int64_t seq;  // flag value for this step
+  float inv_ntok;
+  Scratch<T> sc;
+  std::vector<BlockActs<T>> acts;
+  int64_t h2d_bytes = 0;
+  int n_parts = 0;
+
+  T* xbuf(int i) { return tptr<T>(ctx->xs_base + (int64_t)i * ctx->slot_bytes); }
+  T* ckpt_slot(int ls, int m) { return tptr<T>(ctx->ckpt + ((int64_t)ls * M + m) * ctx->slot_bytes); }
+  T* grad_slot(int ls, int m) { return tptr<T>(ctx->gslot + ((int64_t)ls * M + m) * ctx->slot_bytes); }
+  const int32_t* tok(int m) { return tok_dev + (int64_t)m * ctx->sh.mbs * (ctx->sh.s + 1); }
+
+  // destination slot of stage j's output for microbatch m (the input of j+1)
+  T* fwd_dest(int j, int m, int** flag) {
+    const StageDesc& nx = ctx->all[j + 1];
+    int r = nx.owner;
+    if (r == ctx->dist.rank) {
+      *flag = nullptr;
+      return ckpt_slot(nx.ord, m);
+    }
+    const PeerInfo& pi = ctx->peers[r];
+    uint8_t* b = ctx->peer_base[r];
+    *flag = reinterpret_cast<int*>(b + pi.off_fflag) + (int64_t)nx.ord * pi.M + m;
+    return tptr<T>(b + pi.off_ckpt + ((int64_t)nx.ord * pi.M + m) * pi.slot_bytes);
+  }
+  T* bwd_dest(int j, int m, int** flag) {
+    const StageDesc& pv = ctx->all[j - 1];
+    int r = pv.owner;
+    if (r == ctx->dist.rank) {
+      *flag = nullptr;
+      return grad_slot(pv.ord, m);
+    }
+    const PeerInfo& pi = ctx->peers[r];
+    uint8_t* b = ctx->peer_base[r];
+    *flag = reinterpret_cast<int*>(b + pi.off_bflag) + (int64_t)pv.ord * pi.M + m;
+    return tptr<T>(b + pi.off_gslot + ((int64_t)pv.ord * pi.M + m) * pi.slot_bytes);
+  }
+
+  const T* stage_w(int res, const StageDesc& st, int layer) {
+    return tptr<T>(ctx->ring + ctx->loads[res].base) + st.layer_off[layer - st.first];
+  }
+
+  int issue_part(int r, int64_t b0, int64_t b1) {
+    if (b1 <= b0) return MOBIUS_OK;
+    const Load& L = ctx->loads[r];
+    const StageDesc& st = ctx->all[ctx->mine[L.stage_local]];
+    (void)st;
+    uint8_t* dst = ctx->ring + L.base + b0;
+    const uint8_t* src = (const uint8_t*)ctx->h_weights[L.stage_local] + b0;
+    cudaEvent_t a = ctx->ev_part_a[n_parts], b = ctx->ev_part_b[n_parts];
+    CU(cudaEventRecord(a, ctx->s_h2d));
+    CU(cudaMemcpyAsync(dst, src, b1 - b0, cudaMemcpyHostToDevice, ctx->s_h2d));
+    CU(cudaEventRecord(b, ctx->s_h2d));
+    ctx->part_bytes[n_parts] = b1 - b0;
+    ++n_parts;
+    h2d_bytes += b1 - b0;
+    return MOBIUS_OK;
+  }
+
+  // byte split of residence r: [0, split) does not overlap residence r-1 for a
+  // bottom load; for a top load the non-overlapping bytes are [split, S)
+  void split_of(int r, int64_t& first0, int64_t& first1, int64_t& second0, int64_t& second1) {
+    const Load& L = ctx->loads[r];
+    const int64_t S = L.bytes, G = ctx->ring_bytes;
+    if (r == 0) {
+      first0 = 0, first1 = S, second0 = second1 = 0;
+      return;
+    }
+    const Load& P = ctx->loads[r - 1];
+    if (L.end == 0) {  // bottom [0,S) vs top [P.base, G)
+      int64_t a = std::min(S, P.base);
+      first0 = 0, first1 = a, second0 = a, second1 = S;
+    } else {           // top [L.base, G) vs bottom [0, P.bytes)
+      int64_t ov = std::max<int64_t>(0, std::min(S, P.bytes - L.base));
+      first0 = ov, first1 = S, second0 = 0, second1 = ov;
+    }
+    (void)G;
+  }
+
+  int load_first_part(int r) {  // issued when residence r-1 starts computing
+    if (r >= (int)ctx->loads.size()) return MOBIUS_OK;
+    if (r >= 2) CU(cudaStreamWaitEvent(ctx->s_h2d, ctx->ev_release[r - 2], 0));
+    int64_t a0, a1, b0, b1;
+    split_of(r, a0, a1, b0, b1);
+    return issue_part(r, a0, a1);
+  }
+  int load_second_part(int r) {  // issued right after residence r-1's release
+    if (r >= (int)ctx->loads.size()) return MOBIUS_OK;
+    int64_t a0, a1, b0, b1;
+    split_of(r, a0, a1, b0, b1);
+    if (r >= 1 && b1 > b0) CU(cudaStreamWaitEvent(ctx->s_h2d, ctx->ev_release[r - 1], 0));
+    RC(issue_part(r, b0, b1));
+    CU(cudaEventRecord(ctx->ev_loaded[r], ctx->s_h2d));
+    return MOBIUS_OK;
+  }
+
+  int wait_loaded(int r) {
+    CU(cudaEventRecord(ctx->ev_wait_a[r], ctx->s_comp));
+    CU(cudaStreamWaitEvent(ctx->s_comp, ctx->ev_loaded[r], 0));
+    CU(cudaEventRecord(ctx->ev_wait_b[r], ctx->s_comp));
+    return MOBIUS_OK;
+  }
+
+  void tr(int op, int j, int m) {
+    ctx->trace.push_back(op);
+    ctx->trace.push_back(j + 1);
+    ctx->trace.push_back(m + 1);
+  }
+
+  // ---------------- F_{j,m}
+  int forward(int ls, int res, int m) {
+    const StageDesc& st = ctx->all[ctx->mine[ls]];
+    const Shape& sh = ctx->sh;
+    cudaStream_t s = ctx->s_comp;
+    tr(0, st.j, m);
+    const bool last_stage = st.j == ctx->plan.n_stages - 1;
+    const T* x = nullptr;
+    if (st.has_embed) {
+      T* out;
+      int* flag = nullptr;
+      if (st.n_blocks == 0 && !last_stage)
+        out = fwd_dest(st.j, m, &flag);
+      else
+        out = xbuf(0);
+      RC(embed_layer_fwd<T>(sh, stage_w(res, st, 0), tok(m), out, s));
+      if (flag) { RC(flag_set(flag, (int)seq, s)); ++ctx->launches_step; }
+      x = out;
+    } else {
+      if (ctx->all[st.j - 1].owner != ctx->dist.rank)
+        { RC(flag_wait(ctx->fflag + (int64_t)st.ord * M + m, (int)seq, s)); ++ctx->launches_step; }
+      x = ckpt_slot(ls, m);
+    }
+    if (last_stage) return MOBIUS_OK;  // head runs fused with backward (B_{K,m} recomputes it)
+    int bi = 0;
+    for (int li = st.first; li < st.last; ++li) {
+      if (li == 0) continue;
+      const bool last_block = (bi == st.n_blocks - 1);
+      int* flag = nullptr;
+      T* y = last_block ? fwd_dest(st.j, m, &flag) : xbuf(1 + (bi % 2));
+      acts[0].x = x;
+      RC(block_fwd<T>(sh, stage_w(res, st, li), acts[0], y, sc, s));
+      if (flag) { RC(flag_set(flag, (int)seq, s)); ++ctx->launches_step; }
+      x = y;
+      ++bi;
+    }
+    return MOBIUS_OK;
+  }
+
+  // ---------------- B_{j,m}
+  int backward(int ls, int res, int m) {
+    const StageDesc& st = ctx->all[ctx->mine[ls]];
+    const Shape& sh = ctx->sh;
+    cudaStream_t s = ctx->s_comp;
+    tr(1, st.j, m);
+    // recompute the stage forward from the checkpoint (a5/a7)
+    const T* x;
+    if (st.has_embed) {
+      RC(embed_layer_fwd<T>(sh, stage_w(res, st, 0), tok(m), xbuf(0), s));
+      x = xbuf(0);
+    } else {
+      x = ckpt_slot(ls, m);
+    }
+    int bi = 0;
+    for (int li = st.first; li < st.last; ++li) {
+      if (li == 0 || li == ctx->cfg.n_layers + 1) continue;
+      T* y = xbuf(bi + 1);
+      acts[bi].x = x;
+      RC(block_fwd<T>(sh, stage_w(res, st, li), acts[bi], y, sc, s));
+      x = y;
+      ++bi;
+    }
+    // gradient w.r.t. the stage output
+    const T* dy;
+    T* pingpong[2] = {xbuf(ctx->max_blocks + 1), xbuf(ctx->max_blocks + 2)};
+    int pp = 0;
+    if (st.has_head) {
+      const int hl = ctx->cfg.n_layers + 1;
+      float* G = ctx->grad_acc + st.layer_off[hl - st.first];
+      T* dx = pingpong[pp];
+      pp ^= 1;
+      RC(head_layer_fwd_bwd<T>(sh, stage_w(res, st, hl), x, tok(m), inv_ntok, dx, G, ctx->loss_dev, sc, s));
+      dy = dx;
+    } else {
+      if (ctx->all[st.j + 1].owner != ctx->dist.rank)
+        { RC(flag_wait(ctx->bflag + (int64_t)st.ord * M + m, (int)seq, s)); ++ctx->launches_step; }
+      dy = grad_slot(ls, m);
+    }
+    // blocks in reverse
+    for (int li = st.last - 1; li >= st.first; --li) {
+      if (li == 0 || li == ctx->cfg.n_layers + 1) continue;
+      --bi;
+      const bool first_block = (bi == 0);
+      int* flag = nullptr;
+      T* dx;
+      if (first_block && !st.has_embed)
+        dx = bwd_dest(st.j, m, &flag);
+      else {
+        dx = pingpong[pp];
+        pp ^= 1;
+      }
+      float* G = ctx->grad_acc + st.layer_off[li - st.first];
+      RC(block_bwd<T>(sh, stage_w(res, st, li), acts[bi], dy, dx, G, sc, s));
+      if (flag) { RC(flag_set(flag, (int)seq, s)); ++ctx->launches_step; }
+      dy = dx;
+    }
+    if (st.has_embed) {
+      RC(embed_layer_bwd<T>(sh, stage_w(res, st, 0), tok(m), dy, ctx->grad_acc, s));
+    } else if (st.n_blocks == 0) {
+      // head-only stage: pass the head's input gradient upstream
+      int* flag = nullptr;
+      T* dst = bwd_dest(st.j, m, &flag);
+      CU(cudaMemcpyAsync(dst, dy, (int64_t)sh.T() * sh.h * sizeof(T), cudaMemcpyDeviceToDevice, s));
+      if (flag) { RC(flag_set(flag, (int)seq, s)); ++ctx->launches_step; }
+    }
+    return MOBIUS_OK;
+  }
+
+  int finish_stage_grads(int ls) {
+    const StageDesc& st = ctx->all[ctx->mine[ls]];
+    cudaStream_t s = ctx->s_comp;
+    // staging buffer reuse: previous offload must have drained
+    if (ls + 1 < (int)ctx->mine.size()) CU(cudaStreamWaitEvent(s, ctx->ev_d2h[ls + 1], 0));
+    RC(cast_from_f32<T>(ctx->grad_acc, tptr<T>(ctx->grad_stage), st.n_params, s));
+    ++ctx->launches_step;
+    CU(cudaEventRecord(ctx->ev_gready[ls], s));
+    CU(cudaStreamWaitEvent(ctx->s_d2h, ctx->ev_gready[ls], 0));
+    CU(cudaMemcpyAsync(ctx->h_grads[ls], ctx->grad_stage, st.n_params * sizeof(T), cudaMemcpyDeviceToHost,
+                       ctx->s_d2h));
+    CU(cudaEventRecord(ctx->ev_d2h[ls], ctx->s_d2h));
+    ctx->stats.d2h_bytes += st.n_params * sizeof(T);
+    {
+      std::lock_guard<std::mutex> g(ctx->upd_mu);
+      ctx->upd_queue.push_back(ls);
+      ++ctx->upd_pending;
+    }
+    ctx->upd_cv.notify_one();
+    return MOBIUS_OK;
+  }
+
+  int run() {
+    const int n = (int)ctx->mine.size();
+    cudaStream_t s = ctx->s_comp;
+    // exec list: F of my stages ascending, then B descending (Fig 4)
+    struct Exec {
+      int fwd, ls, res;
+      bool first_of_res, last_of_res;
+    };
+    std::vector<Exec> ex;
+    for (int k = 0; k < n; ++k) ex.push_back({1, k, ctx->res_f[k], true, k != n - 1});
+    for (int k = n - 1; k >= 0; --k) ex.push_back({0, k, ctx->res_b[k], k != n - 1, true});
+    RC(load_first_part(0));
+    RC(load_second_part(0));
+    for (const Exec& e : ex) {
+      if (e.first_of_res) {
+        RC(wait_loaded(e.res));
+        RC(load_first_part(e.res + 1));  // prefetch of the next residence starts with this one
+      }
+      if (!e.fwd) CU(cudaMemsetAsync(ctx->grad_acc, 0, ctx->all[ctx->mine[e.ls]].n_params * 4, s));
+      for (int m = 0; m < M; ++m) {
+        if (e.fwd)
+          RC(forward(e.ls, e.res, m));
+        else
+          RC(backward(e.ls, e.res, m));
+      }
+      if (e.last_of_res) {
+        CU(cudaEventRecord(ctx->ev_release[e.res], s));
+        RC(load_second_part(e.res + 1));
+      }
+      if (!e.fwd) RC(finish_stage_grads(e.ls));
+    }
+    ctx->last_bwd_host_ns = 0;
+    return MOBIUS_OK;
+  }
+};
+
+int check_ctx(mobius_ctx* ctx) {
+  if (!ctx) MOBIUS_FAIL(MOBIUS_EINVAL, "null context");
+  if (ctx->poisoned) MOBIUS_FAIL(MOBIUS_ESTATE, "context poisoned by an earlier failure");
+  return MOBIUS_OK;
+}
+
+template <typename T>
+int do_step(mobius_ctx* ctx, const int32_t* tok_dev, int M, float* loss_out) {
+  const Shape& sh = ctx->sh;
+  StepRunner<T> R;
+  R.ctx = ctx;
+  R.tok_dev = tok_dev;
+  R.M = M;
+  R.seq = ctx->step_count + 1;
+  R.inv_ntok = 1.0f / ((float)M * sh.mbs * sh.s);
+  carve_scratch<T>(sh, ctx->scratch_base, true, R.sc);
+  R.acts.resize(std::max(1, ctx->max_blocks));
+  for (int i = 0; i < (int)R.acts.size(); ++i) carve_block_acts<T>(sh, ctx->acts_base + i * ctx->acts_bytes, R.acts[i]);
+  ctx->trace.clear();
+  ctx->timer.reset();
+  ctx->launches_step = 0;
+  g_kernel_launches = 0;
+  std::memset(&ctx->stats, 0, sizeof(ctx->stats));
+  set_kernel_timer((ctx->dist.flags & MOBIUS_FLAG_TIMING) ? &ctx->timer : nullptr);
+  int64_t t0 = now_ns();
+  CU(cudaEventRecord(ctx->ev_step0, ctx->s_comp));
+  CU(cudaMemsetAsync(ctx->loss_dev, 0, sizeof(double), ctx->s_comp));
+  int rc = R.run();
+  set_kernel_timer(nullptr);
+  if (rc) {
+    ctx->poisoned = true;
+    return rc;
+  }
+  CU(cudaStreamWaitEvent(ctx->s_comp, ctx->ev_d2h[0], 0));
+  CU(cudaEventRecord(ctx->ev_step1, ctx->s_comp));
+  CU(cudaMemcpyAsync(ctx->h_loss, ctx->loss_dev, sizeof(double), cudaMemcpyDeviceToHost, ctx->s_comp));
+  CU(cudaStreamSynchronize(ctx->s_comp));
+  CU(cudaStreamSynchronize(ctx->s_h2d));
+  CU(cudaStreamSynchronize(ctx->s_d2h));
+  int64_t t_gpu_done = now_ns();
+  {  // synchronous update: every stage's AdamW has landed
+    std::unique_lock<std::mutex> lk(ctx->upd_mu);
+    ctx->upd_done_cv.wait(lk, [&] { return ctx->upd_pending == 0; });
+  }
+  int64_t t1 = now_ns();
+  const bool has_last = ctx->all.back().owner == ctx->dist.rank;
+  *loss_out = has_last ? (float)(*ctx->h_loss * R.inv_ntok) : NAN;
+  // stats
+  mobius_step_stats& S = ctx->stats;
+  S.step_ns = t1 - t0;
+  float ms = 0.f;
+  cudaEventElapsedTime(&ms, ctx->ev_step0, ctx->ev_step1);
+  S.device_step_ns = (int64_t)(ms * 1e6);
+  S.h2d_bytes = R.h2d_bytes;
+  S.n_h2d_copies = R.n_parts;
+  std::vector<double> gbps;
+  for (int i = 0; i < R.n_parts; ++i) {
+    float pm = 0.f;
+    if (cudaEventElapsedTime(&pm, ctx->ev_part_a[i], ctx->ev_part_b[i]) == cudaSuccess && pm > 0)
+      gbps.push_back(ctx->part_bytes[i] / (pm * 1e-3) / 1e9);
+  }
+  if (!gbps.empty()) {
+    std::sort(gbps.begin(), gbps.end());
+    S.h2d_GBps_median = gbps[gbps.size() / 2];
+    S.h2d_GBps_max = gbps.back();
+  }
+  int64_t exposed = 0;
+  for (size_t r = 0; r < ctx->loads.size(); ++r) {
+    float wm = 0.f;
+    if (cudaEventElapsedTime(&wm, ctx->ev_wait_a[r], ctx->ev_wait_b[r]) == cudaSuccess) exposed += (int64_t)(wm * 1e6);
+  }
+  S.exposed_load_ns = exposed;
+  for (auto& rec : ctx->timer.recs) {
+    float km = 0.f;
+    if (cudaEventElapsedTime(&km, rec.a, rec.b) != cudaSuccess) continue;
+    int64_t ns = (int64_t)(km * 1e6);
+    if (rec.cls == KCLS_GEMM) {
+      S.gemm_ns += ns;
+      S.gemm_flops += rec.flops;
+      S.gemm_launches++;
+    } else if (rec.cls == KCLS_ATTN) {
+      S.attn_ns += ns;
+    } else {
+      S.elem_ns += ns;
+    }
+  }
+  S.kernel_launches = ctx->launches_step + g_kernel_launches;
+  S.arena_bytes = ctx->arena_bytes;
+  S.ring_bytes = ctx->ring_bytes;
+  int64_t pinned = 0;
+  for (int ls = 0; ls < (int)ctx->mine.size(); ++ls) pinned += 2 * ctx->all[ctx->mine[ls]].n_params * ctx->esz;
+  S.pinned_bytes = pinned;
+  S.host_update_ns = ctx->upd_ns;
+  S.update_tail_ns = t1 - t_gpu_done;
+  S.n_local_stages = (int)ctx->mine.size();
+  S.recompute = 1;
+  ctx->upd_ns = 0;
+  ctx->step_count++;
+  return MOBIUS_OK;
+}
+
+}  // namespace
+
+// ======================================================================
+extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* plan, const mobius_dist* dist,
+                             const float* init_params, uint64_t seed, mobius_ctx** out) {
+  MOBIUS_CHECK_ARG(cfg && plan && dist && out, "null argument");
+  *out = nullptr;
+  const mobius_model_cfg& c = *cfg;
+  MOBIUS_CHECK_ARG(c.dtype == MOBIUS_BF16 || c.dtype == MOBIUS_F32, "bad dtype");
+  MOBIUS_CHECK_ARG(c.n_layers >= 1 && c.hidden % 64 == 0 && c.n_heads > 0 && c.hidden % c.n_heads == 0,
+                   "hidden must be a multiple of 64 and of n_heads");
+  const int dh = c.hidden / c.n_heads;
+  if (c.dtype == MOBIUS_BF16) {
+    MOBIUS_CHECK_ARG(dh == 64 || dh == 128, "bf16 path needs head_dim 64 or 128 (got %d)", dh);
+    MOBIUS_CHECK_ARG(c.seq_len % 8 == 0 && c.vocab % 8 == 0, "seq_len and vocab must be multiples of 8");
+  }
+  const int Lp = c.n_layers + 2;
+  MOBIUS_CHECK_ARG(plan->n_layers == Lp || plan->n_layers == 0, "plan has %d layers, model %d", plan->n_layers, Lp);
+  MOBIUS_CHECK_ARG(plan->n_stages >= 1 && plan->n_stages <= Lp, "bad stage count");
+  MOBIUS_CHECK_ARG(plan->n_gpus == dist->world && dist->world >= 1 && dist->rank >= 0 && dist->rank < dist->world,
+                   "plan n_gpus %d != world %d", plan->n_gpus, dist->world);
+  MOBIUS_CHECK_ARG(plan->stage_first_layer[0] == 0 && plan->stage_first_layer[plan->n_stages] == Lp,
+                   "stage boundaries must cover all %d profile layers", Lp);
+  for (int j = 0; j < plan->n_stages; ++j) {
+    MOBIUS_CHECK_ARG(plan->stage_first_layer[j + 1] > plan->stage_first_layer[j], "empty stage %d", j);
+    MOBIUS_CHECK_ARG(plan->stage_gpu[j] >= 0 && plan->stage_gpu[j] < dist->world, "bad stage_gpu");
+    MOBIUS_CHECK_ARG(plan->stage_gpu[j] == plan->stage_gpu[j % plan->n_gpus], "stage_gpu must be round-robin");
+  }
+
+  std::unique_ptr<mobius_ctx> ctx(new mobius_ctx());
+  ctx->cfg = c;
+  ctx->plan = *plan;
+  ctx->plan.n_layers = Lp;
+  ctx->dist = *dist;
+  ctx->sh = Shape{c.hidden, c.n_heads, c.seq_len, c.micro_batch, c.vocab};
+  ctx->esz = c.dtype == MOBIUS_F32 ? 4 : 2;
+  const int esz = ctx->esz;
+  mobius_ctx* raw = ctx.get();
+  (void)raw;
+
+  // stages
+  const int K = plan->n_stages;
+  ctx->all.resize(K);
+  std::vector<int> count(dist->world, 0);
+  int64_t poff = 0;
+  for (int j = 0; j < K; ++j) {
+    StageDesc& st = ctx->all[j];
+    st.j = j;
+    st.first = plan->stage_first_layer[j];
+    st.last = plan->stage_first_layer[j + 1];
+    st.param_off = poff;
+    int64_t o = 0;
+    for (int li = st.first; li < st.last; ++li) {
+      st.layer_off.push_back(o);
+      o += layer_numel(c, li);
+      if (li == 0) st.has_embed = true;
+      else if (li == Lp - 1) st.has_head = true;
+      else st.n_blocks++;
+    }
+    st.n_params = o;
+    poff += o;
+    st.owner = plan->stage_gpu[j];
+    st.ord = count[st.owner]++;
+    if (st.owner == dist->rank) ctx->mine.push_back(j);
+  }
+  MOBIUS_CHECK_ARG(!ctx->mine.empty(), "rank %d owns no stage", dist->rank);
+  const int n = (int)ctx->mine.size();
+
+  // ring: cap G (plan) or double-buffer default
+  int64_t max_stage = 0, max_params = 0;
+  for (int ls = 0; ls < n; ++ls) {
+    const StageDesc& st = ctx->all[ctx->mine[ls]];
+    max_stage = std::max(max_stage, st.n_params * esz);
+    max_params = std::max(max_params, st.n_params);
+    ctx->max_blocks = std::max(ctx->max_blocks, st.n_blocks);
+  }
+  int64_t G = plan->hbm_cap_bytes > 0 ? (plan->hbm_cap_bytes & ~int64_t(255)) : 2 * al256(max_stage);
+  if (c.dtype == MOBIUS_F32 && plan->hbm_cap_bytes > 0) G = G;  // cap given in the path precision by the caller
+  if (max_stage > G) MOBIUS_FAIL(MOBIUS_EINFEASIBLE, "stage of %lld bytes exceeds the cap %lld", (long long)max_stage, (long long)G);
+  ctx->ring_bytes = G;
+
+  // residences: fwd loads ascending, bwd reloads descending except the last
+  ctx->res_f.assign(n, -1);
+  ctx->res_b.assign(n, -1);
+  for (int k = 0; k < n; ++k) {
+    ctx->res_f[k] = (int)ctx->loads.size();
+    ctx->loads.push_back({k, 0, 0, ctx->all[ctx->mine[k]].n_params * esz});
+  }
+  ctx->res_b[n - 1] = ctx->res_f[n - 1];
+  for (int k = n - 2; k >= 0; --k) {
+    ctx->res_b[k] = (int)ctx->loads.size();
+    ctx->loads.push_back({k, 0, 0, ctx->all[ctx->mine[k]].n_params * esz});
+  }
+  for (size_t r = 0; r < ctx->loads.size(); ++r) {
+    Load& L = ctx->loads[r];
+    L.end = (int)(r % 2);
+    L.base = L.end == 0 ? 0 : ((G - L.bytes) & ~int64_t(255));
+  }
+
+  // arena layout
+  const Shape& sh = ctx->sh;
+  const int M = plan->n_microbatches > 0 ? plan->n_microbatches : dist->world;
+  ctx->max_M = M;
+  ctx->slot_bytes = al256((int64_t)sh.T() * sh.h * esz);
+  ctx->acts_bytes = al256(block_acts_bytes(sh, esz));
+  int64_t off = al256(G);
+  auto take = [&](int64_t bytes) {
+    int64_t o = off;
+    off += al256(bytes);
+    return o;
+  };
+  int64_t o_gacc = take(max_params * 4);
+  int64_t o_gstage = take(max_params * esz);
+  ctx->off_ckpt = take((int64_t)n * M * ctx->slot_bytes);
+  ctx->off_gslot = take((int64_t)n * M * ctx->slot_bytes);
+  ctx->off_fflag = take((int64_t)n * M * 4);
+  ctx->off_bflag = take((int64_t)n * M * 4);
+  int64_t o_acts = take(ctx->acts_bytes * std::max(1, ctx->max_blocks));
+  int64_t o_xs = take(ctx->slot_bytes * (ctx->max_blocks + 3));
+  int64_t o_scr = take(scratch_bytes(sh, esz, true));
+  int64_t o_tok = take((int64_t)M * sh.mbs * (sh.s + 1) * 4);
+  int64_t o_loss = take(8);
+  ctx->arena_bytes = off;
+
+  int cu_dev = dist->device;
+  {
+    mobius_ctx* ctxp = ctx.get();
+    mobius_ctx* ctx = ctxp;  // for CU()
+    CU(cudaSetDevice(cu_dev));
+    CU(cudaMalloc(&ctx->arena, ctx->arena_bytes));
+    CU(cudaMemset(ctx->arena + o_gacc, 0, max_params * 4));
+    ctx->ring = ctx->arena;
+    ctx->grad_acc = reinterpret_cast<float*>(ctx->arena + o_gacc);
+    ctx->grad_stage = ctx->arena + o_gstage;
+    ctx->ckpt = ctx->arena + ctx->off_ckpt;
+    ctx->gslot = ctx->arena + ctx->off_gslot;
+    ctx->fflag = reinterpret_cast<int*>(ctx->arena + ctx->off_fflag);
+    ctx->bflag = reinterpret_cast<int*>(ctx->arena + ctx->off_bflag);
+    ctx->acts_base = ctx->arena + o_acts;
+    ctx->xs_base = ctx->arena + o_xs;
+    ctx->scratch_base = ctx->arena + o_scr;
+    ctx->tok_dev = ctx->arena + o_tok;
+    ctx->loss_dev = reinterpret_cast<double*>(ctx->arena + o_loss);
+    CU(cudaMemset(ctx->fflag, 0, (int64_t)n * M * 4));
+    CU(cudaMemset(ctx->bflag, 0, (int64_t)n * M * 4));
+
+    // streams: H2D prefetch gets the highest priority
+    int lo = 0, hi = 0;
+    CU(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+    CU(cudaStreamCreateWithPriority(&ctx->s_comp, cudaStreamNonBlocking, lo));
+    CU(cudaStreamCreateWithPriority(&ctx->s_h2d, cudaStreamNonBlocking, hi));
+    CU(cudaStreamCreateWithPriority(&ctx->s_d2h, cudaStreamNonBlocking, lo));
+    const int R = (int)ctx->loads.size();
+    auto mk = [&](std::vector<cudaEvent_t>& v, int cnt, unsigned flags) -> int {
+      v.resize(cnt);
+      for (auto& e : v) CU(cudaEventCreateWithFlags(&e, flags));
+      return MOBIUS_OK;
+    };
+    RC(mk(ctx->ev_release, R, cudaEventDisableTiming));
+    RC(mk(ctx->ev_loaded, R, cudaEventDisableTiming));
+    RC(mk(ctx->ev_part_a, 2 * R + 2, cudaEventDefault));
+    RC(mk(ctx->ev_part_b, 2 * R + 2, cudaEventDefault));
+    ctx->part_bytes.assign(2 * R + 2, 0);
+    RC(mk(ctx->ev_gready, n, cudaEventDisableTiming));
+    RC(mk(ctx->ev_d2h, n, cudaEventDisableTiming));
+    RC(mk(ctx->ev_wait_a, R, cudaEventDefault));
+    RC(mk(ctx->ev_wait_b, R, cudaEventDefault));
+    CU(cudaEventCreate(&ctx->ev_step0));
+    CU(cudaEventCreate(&ctx->ev_step1));
+    for (int k = 0; k < n; ++k) CU(cudaEventRecord(ctx->ev_d2h[k], ctx->s_d2h));
+
+    // host stage store
+    unsigned hw = std::thread::hardware_concurrency();
+    int nthreads = std::max(1, (int)(hw ? hw : 4) / dist->world);
+    ctx->pool.reset(new ThreadPool(nthreads));
+    ctx->h_weights.resize(n);
+    ctx->h_grads.resize(n);
+    ctx->h_master.resize(n);
+    ctx->h_m.resize(n);
+    ctx->h_v.resize(n);
+    for (int k = 0; k < n; ++k) {
+      const StageDesc& st = ctx->all[ctx->mine[k]];
+      const int64_t np = st.n_params;
+      CU(cudaHostAlloc(&ctx->h_weights[k], al256(np * esz), cudaHostAllocDefault));
+      CU(cudaHostAlloc(&ctx->h_grads[k], al256(np * esz), cudaHostAllocDefault));
+      float* mst = (float*)std::malloc(np * 4);
+      float* mm = (float*)std::malloc(np * 4);
+      float* vv = (float*)std::malloc(np * 4);
+      if (!mst || !mm || !vv) MOBIUS_FAIL(MOBIUS_ENOMEM, "host optimizer state (%lld params)", (long long)np);
+      ctx->h_master[k] = mst;
+      ctx->h_m[k] = mm;
+      ctx->h_v[k] = vv;
+      // first touch from the pool threads (NUMA-local pages)
+      const int64_t chunk = 1 << 20;
+      const int tasks = (int)((np + chunk - 1) / chunk);
+      ctx->pool->parallel_for(tasks, [&](int t) {
+        int64_t b = (int64_t)t * chunk, e = std::min(np, b + chunk);
+        if (init_params)
+          std::memcpy(mst + b, init_params + st.param_off + b, (e - b) * 4);
+        std::memset(mm + b, 0, (e - b) * 4);
+        std::memset(vv + b, 0, (e - b) * 4);
+      });
+      if (!init_params) seeded_stage_init(c, st, mst, seed);
+      ctx->pool->parallel_for(tasks, [&](int t) {
+        int64_t b = (int64_t)t * chunk, e = std::min(np, b + chunk);
+        if (esz == 2) {
+          uint16_t* w = (uint16_t*)ctx->h_weights[k];
+          for (int64_t i = b; i < e; ++i) w[i] = f32_to_bf16_rne(mst[i]);
+        } else {
+          std::memcpy((float*)ctx->h_weights[k] + b, mst + b, (e - b) * 4);
+        }
+      });
+    }
+    CU(cudaHostAlloc(&ctx->h_loss, sizeof(double), cudaHostAllocDefault));
+    ctx->h_tokens_cap = (int64_t)M * sh.mbs * (sh.s + 1);
+    CU(cudaHostAlloc(&ctx->h_tokens, ctx->h_tokens_cap * 4, cudaHostAllocDefault));
+    ctx->peer_base.assign(dist->world, nullptr);
+    ctx->connected = dist->world == 1;
+    ctx->upd_thread = std::thread(update_worker, ctxp);
+    CU(cudaDeviceSynchronize());
+  }
+  *out = ctx.release();
+  return MOBIUS_OK;
+}
+
+struct ExportBlob {
+  uint32_t magic;
+  int32_t rank;
+  cudaIpcMemHandle_t handle;
+  int64_t off_ckpt, off_gslot, off_fflag, off_bflag, slot_bytes;
+  int32_t n_local, M;
+};
+
+extern "C" int mobius_dist_export(mobius_ctx* ctx, void* buf, size_t cap, size_t* len) {
+  int rc = check_ctx(ctx);
+  if (rc) return rc;
+  MOBIUS_CHECK_ARG(buf && len && cap >= sizeof(ExportBlob), "export buffer too small");
+  ExportBlob b;
+  std::memset(&b, 0, sizeof(b));
+  b.magic = 0x4d4f4249;
+  b.rank = ctx->dist.rank;
+  CU(cudaSetDevice(ctx->dist.device));
+  CU(cudaIpcGetMemHandle(&b.handle, ctx->arena));
+  b.off_ckpt = ctx->off_ckpt;
+  b.off_gslot = ctx->off_gslot;
+  b.off_fflag = ctx->off_fflag;
+  b.off_bflag = ctx->off_bflag;
+  b.slot_bytes = ctx->slot_bytes;
+  b.n_local = (int)ctx->mine.size();
+  b.M = ctx->max_M;
+  std::memcpy(buf, &b, sizeof(b));
+  *len = sizeof(b);
+  return MOBIUS_OK;
+}
+
+extern "C" int mobius_dist_connect(mobius_ctx* ctx, const void* all, size_t blob_len) {
+  int rc = check_ctx(ctx);
+  if (rc) return rc;
+  MOBIUS_CHECK_ARG(all && blob_len >= sizeof(ExportBlob), "bad blobs");
+  const int W = ctx->dist.world;
+  ctx->peers.resize(W);
+  CU(cudaSetDevice(ctx->dist.device));
+  for (int r = 0; r < W; ++r) {
+    ExportBlob b;
+    std::memcpy(&b, (const char*)all + r * blob_len, sizeof(b));
+    MOBIUS_CHECK_ARG(b.magic == 0x4d4f4249 && b.rank == r, "blob %d is not a mobius export", r);
+    PeerInfo& p = ctx->peers[r];
+    p.rank = r;
+    p.handle = b.handle;
+    p.off_ckpt = b.off_ckpt;
+    p.off_gslot = b.off_gslot;
+    p.off_fflag = b.off_fflag;
+    p.off_bflag = b.off_bflag;
+    p.slot_bytes = b.slot_bytes;
+    p.n_local = b.n_local;
+    p.M = b.M;
+    if (r == ctx->dist.rank) continue;
+    // only neighbours in the stage chain need a mapping
+    bool neighbour = false;
+    for (int j = 0; j + 1 < ctx->plan.n_stages; ++j) {
+      int a = ctx->all[j].owner, c = ctx->all[j + 1].owner;
+      if ((a == ctx->dist.rank && c == r) || (c == ctx->dist.rank && a == r)) neighbour = true;
+    }
+    if (!neighbour) continue;
+    void* ptr = nullptr;
+    CU(cudaIpcOpenMemHandle(&ptr, b.handle, cudaIpcMemLazyEnablePeerAccess));
+    ctx->peer_base[r] = (uint8_t*)ptr;
+  }
+  ctx->connected = true;
+  return MOBIUS_OK;
+}
+
+static int step_common(mobius_ctx* ctx, const int32_t* tok_dev, int M, float* loss_out) {
+  if (ctx->cfg.dtype == MOBIUS_F32) return do_step<float>(ctx, tok_dev, M, loss_out);
+  return do_step<bf16>(ctx, tok_dev, M, loss_out);
+}
+
+extern "C" int mobius_step(mobius_ctx* ctx, const int32_t* tokens, int M, float* loss_out) {
+  int rc = check_ctx(ctx);
+  if (rc) return rc;
+  MOBIUS_CHECK_ARG(tokens && loss_out && M >= 1, "bad arguments");
+  MOBIUS_CHECK_ARG(M == ctx->max_M, "n_microbatches %d != plan's %d", M, ctx->max_M);
+  if (!ctx->connected) MOBIUS_FAIL(MOBIUS_ESTATE, "world > 1: call mobius_dist_connect first");
+  CU(cudaSetDevice(ctx->dist.device));
+  const int64_t n = (int64_t)M * ctx->sh.mbs * (ctx->sh.s + 1);
+  std::memcpy(ctx->h_tokens, tokens, n * 4);
+  CU(cudaMemcpyAsync(ctx->tok_dev, ctx->h_tokens, n * 4, cudaMemcpyHostToDevice, ctx->s_comp));
+  return step_common(ctx, reinterpret_cast<const int32_t*>(ctx->tok_dev), M, loss_out);
+}
+
+extern "C" int mobius_step_device(mobius_ctx* ctx, const int32_t* tokens_dev, int M, float* loss_out) {
+  int rc = check_ctx(ctx);
+  if (rc) return rc;
+  MOBIUS_CHECK_ARG(tokens_dev && loss_out && M == ctx->max_M, "bad arguments");
+  if (!ctx->connected) MOBIUS_FAIL(MOBIUS_ESTATE, "world > 1: call mobius_dist_connect first");
+  CU(cudaSetDevice(ctx->dist.device));
+  return step_common(ctx, tokens_dev, M, loss_out);
+}
+
+extern "C" int mobius_read_grads(mobius_ctx* ctx, float* out, size_t n) {
+  int rc = check_ctx(ctx);
+  if (rc) return rc;
+  MOBIUS_CHECK_ARG(out, "null out");
+  for (int ls = 0; ls < (int)ctx->mine.size(); ++ls) {
+    const StageDesc& st = ctx->all[ctx->mine[ls]];
+    MOBIUS_CHECK_ARG((size_t)(st.param_off + st.n_params) <= n, "output too small");
+    if (ctx->esz == 2) {
+      const uint16_t* g = (const uint16_t*)ctx->h_grads[ls];
+      for (int64_t i = 0; i < st.n_params; ++i) out[st.param_off + i] = bf16_to_f32(g[i]);
+    } else {
+      std::memcpy(out + st.param_off, ctx->h_grads[ls], st.n_params * 4);
+    }
+  }
+  return MOBIUS_OK;
+}
+
+extern "C" int mobius_read_params(mobius_ctx* ctx, float* out, size_t n) {
+  int rc = check_ctx(ctx);
+  if (rc) return rc;
+  MOBIUS_CHECK_ARG(out, "null out");
+  for (int ls = 0; ls < (int)ctx->mine.size(); ++ls) {
+    const StageDesc& st = ctx->all[ctx->mine[ls]];
+    MOBIUS_CHECK_ARG((size_t)(st.param_off + st.n_params) <= n, "output too small");
+    std::memcpy(out + st.param_off, ctx->h_master[ls], st.n_params * 4);
+  }
+  return MOBIUS_OK;
+}
+
+extern "C" int mobius_read_trace(mobius_ctx* ctx, int32_t* out, size_t cap, size_t* n) {
+  MOBIUS_CHECK_ARG(ctx && out && n, "null argument");
+  size_t t = ctx->trace.size() / 3;
+  *n = t;
+  std::memcpy(out, ctx->trace.data(), std::min(t, cap) * 3 * sizeof(int32_t));
+  return MOBIUS_OK;
+}
+
+extern "C" int mobius_stats(mobius_ctx* ctx, mobius_step_stats* out) {
+  MOBIUS_CHECK_ARG(ctx && out, "null argument");
+  *out = ctx->stats;
+  return MOBIUS_OK;
+}
+
+extern "C" void mobius_destroy(mobius_ctx* ctx) {
+  if (!ctx) return;
+  cudaSetDevice(ctx->dist.device);
+  {
+    std::lock_guard<std::mutex> g(ctx->upd_mu);
+    ctx->upd_stop = true;
+  }
+  ctx->upd_cv.notify_all();
+  if (ctx->upd_thread.joinable()) ctx->upd_thread.join();
+  if (ctx->s_comp) cudaStreamSynchronize(ctx->s_comp);
+  if (ctx->s_h2d) cudaStreamSynchronize(ctx->s_h2d);
+  if (ctx->s_d2h) cudaStreamSynchronize(ctx->s_d2h);
+  for (auto p : ctx->peer_base)
+    if (p) cudaIpcCloseMemHandle(p);
+  for (auto* v : {&ctx->ev_release, &ctx->ev_loaded, &ctx->ev_part_a, &ctx->ev_part_b, &ctx->ev_gready,
+                  &ctx->ev_d2h, &ctx->ev_wait_a, &ctx->ev_wait_b})
+    for (auto e : *v) cudaEventDestroy(e);
+  if (ctx->ev_step0) cudaEventDestroy(ctx->ev_step0);
+  if (ctx->ev_step1) cudaEventDestroy(ctx->ev_step1);
+  for (auto p : ctx->h_weights) cudaFreeHost(p);
+  for (auto p : ctx->h_grads) cudaFreeHost(p);
+  for (auto p : ctx->h_master) std::free(p);
+  for (auto p : ctx->h_m) std::free(p);
+  for (auto p : ctx->h_v) std::free(p);
+  if (ctx->h_loss) cudaFreeHost(ctx->h_loss);
+  if (ctx->h_tokens) cudaFreeHost(ctx->h_tokens);
+  if (ctx->arena) cudaFree(ctx->arena);
+  if (ctx->s_comp) cudaStreamDestroy(ctx->s_comp);
+  if (ctx->s_h2d) cudaStreamDestroy(ctx->s_h2d);
+  if (ctx->s_d2h) cudaStreamDestroy(ctx->s_d2h);
+  delete ctx;
+}

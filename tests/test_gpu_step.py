@@ -1,0 +1,136 @@
+"""GPU parity of the whole Mobius step (rows a1-a11) through the C ABI
+against the CPU oracle: loss, every gradient, the per-GPU schedule trace
+(Fig 4 order), the H2D / D2H byte counters (O-10, reading #11) and the
+post-AdamW parameters, on BASELINE configs[0] (tiny GPT, 4 MiB cap forcing
+DRAM stage swaps with a partial prefetch).
+
+Tolerances: north_star - rel 2e-2 (bf16 path, fp32 accumulate), rel 1e-4
+(fp32 debug path), norm-wise per tensor group (reading #20)."""
+import os
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+if not torch.cuda.is_available():  # pragma: no cover
+    pytest.skip("needs a GPU", allow_module_level=True)
+
+import synth  # noqa: E402
+from oracle import adamw as oa  # noqa: E402
+from oracle import model as om  # noqa: E402
+from oracle import planner as op  # noqa: E402
+from oracle import schedule as osch  # noqa: E402
+from paper_conf_asplos_fengxtwls23_b200 import (BF16, F32, MobiusContext, mobius_layer_sizes,  # noqa: E402
+                                                model_cfg, plan_from_sizes)
+
+MiB = 1 << 20
+
+
+def rel(a, b):
+    return float(np.linalg.norm(np.asarray(a, np.float64) - b) / max(np.linalg.norm(b), 1e-30))
+
+
+def mk_cfg(c, dtype):
+    return model_cfg(c.n_layers, c.hidden, c.n_heads, c.seq_len, c.vocab, c.micro_batch, dtype=dtype)
+
+
+def tensor_errs(cfg, g, ref):
+    errs = {}
+    offs = cfg.layer_offsets()
+    for i in range(cfg.n_profile_layers):
+        pos = offs[i]
+        for name, shape, _ in cfg.layer_specs(i):
+            n = int(np.prod(shape))
+            errs[f"L{i}.{name}"] = rel(g[pos:pos + n], ref[pos:pos + n])
+            pos += n
+    return errs
+
+
+def bounds(sizes):
+    b = [0]
+    for s in sizes:
+        b.append(b[-1] + s)
+    return b
+
+
+@pytest.mark.parametrize("dtype,tol,cap", [(BF16, 2e-2, 4 * MiB), (F32, 1e-4, 8 * MiB)])
+@pytest.mark.parametrize("sizes", [(3, 3), (1, 2, 1, 2), (6,)])
+def test_tiny_step_parity(dtype, tol, cap, sizes):
+    c = synth.TINY
+    M = 2
+    w = synth.perturb_norm_params(c, synth.gen_params(c), scale=0.1)
+    if dtype == BF16:
+        w = synth.round_bf16(w)
+    tok = synth.gen_tokens(c, M)
+    if sizes == (6,):
+        cap = 16 * MiB if dtype == BF16 else 32 * MiB  # a single stage must fit
+    plan = plan_from_sizes(sizes, 1, M, hbm_cap_bytes=cap)
+    ctx = MobiusContext(mk_cfg(c, dtype), plan, init_params=w)
+    loss = ctx.step(tok)
+    g = ctx.read_grads(c.n_params)
+    trace = ctx.read_trace()
+    st = ctx.stats()
+    p1 = ctx.read_params(c.n_params)
+    ctx.close()
+
+    ref_loss, ref_g = om.reference_loss_and_grads(c, w, tok)
+    assert abs(loss - ref_loss) / abs(ref_loss) < tol
+    errs = tensor_errs(c, g, ref_g)
+    assert rel(g, ref_g) < tol and max(errs.values()) < tol, errs
+    # schedule trace == the oracle's per-GPU queue (Fig 4 rule)
+    sg = op.sequential_stage_gpu(len(sizes), 1)
+    assert trace == osch.per_gpu_ops(sg, M)[0]
+    # byte counters (O-10): xfer = stage weight bytes in the transfer precision
+    prof = mobius_layer_sizes(mk_cfg(c, dtype))
+    layers = [op.LayerProfile(0, 0, p.mem_fwd, p.mem_bwd, p.xfer_fwd, p.xfer_bwd, p.act_out) for p in prof]
+    ss = op.stage_sums(layers, sizes)
+    h2d, d2h, _ = osch.byte_counts(ss, sg, M, [s["Xf"] for s in ss])
+    assert st.h2d_bytes == h2d[0]
+    assert st.d2h_bytes == d2h[0]
+    # AdamW on host (a11): the oracle's AdamW applied to the offloaded
+    # gradients must reproduce the updated master (Adam's first step is
+    # ~lr*sign(g), so the delta itself is compared on identical gradients;
+    # gradient parity is asserted above)
+    w1, _, _ = oa.adamw_step(w, np.zeros_like(w), np.zeros_like(w), g, 1)
+    assert rel(p1 - w, w1 - w) < 1e-5
+    assert np.max(np.abs(p1 - w1)) < 1e-6
+
+
+def test_tiny_two_steps_bf16():
+    """Second step runs on the host-updated stages (swap-in of the new
+    weights) and matches the oracle's second step."""
+    c = synth.TINY
+    M = 2
+    w = synth.round_bf16(synth.gen_params(c))
+    tok1 = synth.gen_tokens(c, M, seed=11)
+    tok2 = synth.gen_tokens(c, M, seed=12)
+    ctx = MobiusContext(mk_cfg(c, BF16), plan_from_sizes((3, 3), 1, M, hbm_cap_bytes=4 * MiB), init_params=w)
+    l1 = ctx.step(tok1)
+    l2 = ctx.step(tok2)
+    g2 = ctx.read_grads(c.n_params)
+    ctx.close()
+    r1, g1 = om.reference_loss_and_grads(c, w, tok1)
+    w1, m1, v1 = oa.adamw_step(w, np.zeros_like(w), np.zeros_like(w), g1.astype(np.float32), 1)
+    # the GPU consumes bf16 weights (RNE of the fp32 master)
+    r2, rg2 = om.reference_loss_and_grads(c, synth.round_bf16(w1), tok2)
+    assert abs(l1 - r1) / r1 < 2e-2
+    assert abs(l2 - r2) / r2 < 2e-2
+    assert rel(g2, rg2) < 2e-2
+    assert l2 < l1 + 0.05  # training signal sanity
+
+
+def test_infeasible_cap_rejected():
+    c = synth.TINY
+    from paper_conf_asplos_fengxtwls23_b200 import MobiusError
+    with pytest.raises(MobiusError) as e:
+        MobiusContext(mk_cfg(c, BF16), plan_from_sizes((3, 3), 1, 2, hbm_cap_bytes=2 * MiB), init_params=None)
+    assert e.value.code == -2
+
+
+def test_seeded_init_runs():
+    c = synth.TINY
+    ctx = MobiusContext(mk_cfg(c, BF16), plan_from_sizes((2, 2, 2), 1, 2, hbm_cap_bytes=4 * MiB), seed=7)
+    loss = ctx.step(synth.gen_tokens(c, 2))
+    ctx.close()
+    assert abs(loss - np.log(c.vocab)) < 0.5
