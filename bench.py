@@ -1,0 +1,338 @@
+#!/usr/bin/env python
+"""Mobius fine-tuning step benchmark (BASELINE.json metric: fine-tune tokens/s
+at 1/2/4/8 B200; stage swap-in GB/s vs host-link peak).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config 1.5b] [--impl reference]
+
+N=1 workload = BASELINE configs[1]: GPT 1.5B (48 layers, h=1600, s=1024,
+mbs=8) on one B200 with the stage ring capped (default 1 GiB) so every stage
+swaps from pinned DRAM each step.  N>1 (torchrun, one rank per GPU): the same
+model pipelined over N GPUs with M = M1*N microbatches (weak scaling).
+
+Timing: W untimed warm-up steps; K timed steps between a barrier +
+torch.cuda.synchronize() on both sides, CUDA events on the current stream
+(mobius_step returns only after its GPU work and the host AdamW update have
+completed, so the events bracket complete steps), max over ranks.  Each step
+streams every stage's weights (3.1 GB bf16 > 126 MB L2) from host DRAM, so
+inputs are larger than L2.  The reference arm (--impl reference) times the
+CPU oracle (oracle/, test infrastructure) on a bounded sample; it is a
+deliberately slow baseline, not a target.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import synth  # noqa: E402
+
+GiB = 1 << 30
+METRIC = "fine-tune tokens/s at 1/2/4/8 B200; stage swap-in GB/s vs host-link peak"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=3)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="1.5b")
+    ap.add_argument("--microbatches", type=int, default=0, help="M per GPU (default 16 for 1.5b)")
+    ap.add_argument("--cap-gib", type=float, default=1.0, help="HBM stage-ring cap G per GPU")
+    ap.add_argument("--impl", default="mobius", choices=["mobius", "reference"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    return ap.parse_args()
+
+
+def dist_env():
+    return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return d, "measured"
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons during the timed region."""
+
+    def __init__(self, index=0):
+        self.index = index
+        self.samples = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def _run(self):
+        q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+             "clocks_event_reasons.sw_power_cap")
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={q}",
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True,
+                                     timeout=5).stdout.strip()
+                if out:
+                    self.samples.append([x.strip() for x in out.split(",")])
+            except Exception:
+                pass
+            self._stop.wait(0.2)
+
+    def start(self):
+        self._t = threading.Thread(target=self._run, daemon=True)
+        self._t.start()
+
+    def stop(self):
+        self._stop.set()
+        if self._t:
+            self._t.join(timeout=10)
+        sm = [float(s[0]) for s in self.samples if s[0].replace(".", "").isdigit()]
+        mx = [float(s[1]) for s in self.samples if s[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for s in self.samples for i in range(4) if len(s) > 3 + i and "Active" in s[3 + i]
+                          and not s[3 + i].startswith("Not")})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.samples)}
+
+
+def model_flops_per_token(c: synth.GPTConfig) -> float:
+    """Algorithmic FLOPs per token, fwd + bwd, causal attention, LM head
+    (SURVEY §8(d)): L (72 h^2 + 6 s h) + 6 h V.  Recompute excluded."""
+    h = c.hidden
+    return c.n_layers * (72 * h * h + 6 * c.seq_len * h) + 6 * h * c.vocab
+
+
+# --------------------------------------------------------------- reference
+def cpu_oracle_sample(c: synth.GPTConfig, tokens_per_step: int, budget_s: float = 20.0):
+    """Time the oracle (numpy fp32) on one block fwd+bwd and the head at
+    mbs=1, extrapolate to tokens/s:  T_step ~ (L t_block + t_head + t_embed)
+    * tokens_per_step / s."""
+    from oracle import model as om
+    cores = len(os.sched_getaffinity(0))
+    s, h, V = c.seq_len, c.hidden, c.vocab
+    c1 = synth.GPTConfig(n_layers=c.n_layers, hidden=h, n_heads=c.n_heads, seq_len=s, vocab=V, micro_batch=1)
+    rng = np.random.default_rng(0)
+    blk = {name: (rng.standard_normal(shape) * 0.02).astype(np.float32) if init.startswith("normal")
+           else (np.ones(shape, np.float32) if init == "ones" else np.zeros(shape, np.float32))
+           for name, shape, init in c1.layer_specs(1)}
+    head = {name: (rng.standard_normal(shape) * 0.02).astype(np.float32) if init.startswith("normal")
+            else (np.ones(shape, np.float32) if init == "ones" else np.zeros(shape, np.float32))
+            for name, shape, init in c1.layer_specs(c1.n_layers + 1)}
+    x = rng.standard_normal((s, h)).astype(np.float32)
+    tok = rng.integers(0, V, size=(1, s + 1))
+    t0 = time.perf_counter()
+    y, cache = om.block_fwd(c1, blk, x, 1)
+    om.block_bwd(c1, blk, y, cache, 1)
+    t_block = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    om.head_fwd_bwd(c1, head, x, tok[:, 1:], s)
+    t_head = time.perf_counter() - t0
+    t_step = (c.n_layers * t_block + t_head) * tokens_per_step / s
+    return {"value": tokens_per_step / t_step, "unit": "tokens/s", "cores": cores, "kind": "oracle",
+            "sample": f"numpy fp32 oracle: 1 block fwd+bwd ({t_block:.2f}s) + LM head fwd+bwd ({t_head:.2f}s) "
+                      f"at mbs=1 s={s} h={h} V={V}, extrapolated x{c.n_layers} blocks to the step's "
+                      f"{tokens_per_step} tokens (host AdamW and transfers not included)"}
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    c = synth.CONFIGS[args.config]
+    M = (args.microbatches or 16) * args.gpus
+    tps = M * c.micro_batch * c.seq_len
+    vals = []
+    for _ in range(args.warmup):
+        cpu_oracle_sample(c, tps)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        vals.append(cpu_oracle_sample(c, tps))
+    wall = time.perf_counter() - t0
+    v = float(np.median([x["value"] for x in vals]))
+    cb = dict(vals[-1])
+    cb["value"] = v
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "tokens/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000.0 * tps / v,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": f"GPT {args.config} CPU oracle sample", "model": f"gpt-{args.config}",
+                       "global_batch": M * c.micro_batch, "seq_len": c.seq_len, "microbatches": M},
+            "cpu_baseline": cb,
+            "e2e": {"value": v, "unit": "tokens/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+            "wall_s": wall}
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------ mobius
+def measure_h2d_GBps(torch, nbytes=512 << 20):
+    h = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    d = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    d.copy_(h, non_blocking=True)
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record()
+    for _ in range(3):
+        d.copy_(h, non_blocking=True)
+    b.record()
+    torch.cuda.synchronize()
+    return 3 * nbytes / (a.elapsed_time(b) * 1e-3) / 1e9
+
+
+def run_mobius(args, rank, world, local):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_asplos_fengxtwls23_b200 import (BF16, FLAG_TIMING, MobiusContext, make_topology,
+                                                    mobius_discover_topology, mobius_plan, mobius_profile,
+                                                    model_cfg)
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    c = synth.CONFIGS[args.config]
+    M = (args.microbatches or 16) * world
+    cfg = model_cfg(c.n_layers, c.hidden, c.n_heads, c.seq_len, c.vocab, c.micro_batch, dtype=BF16)
+    G = int(args.cap_gib * GiB)
+    # profile (layer similarity) and plan (MIP + cross mapping)
+    prof = mobius_profile(cfg, local)
+    h2d_gbps = measure_h2d_GBps(torch)
+    topo = mobius_discover_topology()
+    groups = [topo.group[i] for i in range(topo.n_gpus)][:world]
+    if len(groups) < world:
+        groups = list(range(world))
+    t = make_topology(groups, host_bw_Bps=int(h2d_gbps * 1e9), p2p_bw_Bps=int(700e9))
+    t0 = time.perf_counter()
+    plan = mobius_plan(prof, world, G, M, t)
+    plan_s = time.perf_counter() - t0
+    ctx = MobiusContext(cfg, plan, rank=rank, world=world, device=local, seed=1234, flags=FLAG_TIMING)
+    if world > 1:
+        blobs = [None] * world
+        dist.all_gather_object(blobs, ctx.dist_export())
+        ctx.dist_connect(blobs)
+        dist.barrier()
+    tokens = synth.gen_tokens(c, M)
+    tok_dev = torch.from_numpy(tokens).cuda()
+
+    def barrier():
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+            torch.cuda.synchronize()
+
+    def max_over_ranks(x):
+        if world == 1:
+            return x
+        tt = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        return float(tt.item())
+
+    loss = float("nan")
+    for _ in range(args.warmup):
+        loss = ctx.step_device(tok_dev, M)
+    sampler = ClockSampler(local)
+    sampler.start()
+    barrier()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev0.record()
+    stats = []
+    for _ in range(args.steps):
+        loss = ctx.step_device(tok_dev, M)
+        stats.append(ctx.stats())
+    ev1.record()
+    barrier()
+    clocks = sampler.stop()
+    ms = max_over_ranks(ev0.elapsed_time(ev1) / args.steps)
+    tokens_per_step = M * c.micro_batch * c.seq_len
+    value = tokens_per_step / (ms * 1e-3)
+
+    # e2e: same step through the public API with HOST tokens (H2D inside the
+    # timed region) and the loss read back (D2H)
+    e2e = None
+    if not args.no_e2e:
+        barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(args.steps):
+            ctx.step(tokens)
+        e1.record()
+        barrier()
+        ems = max_over_ranks(e0.elapsed_time(e1) / args.steps)
+        e2e = {"value": tokens_per_step / (ems * 1e-3), "unit": "tokens/s", "h2d_bytes_per_step": int(tokens.nbytes),
+               "d2h_bytes_per_step": 8, "ms_per_step": ems}
+
+    st = stats[-1]
+    peaks, peak_src = load_peaks()
+    gemm_ns = sum(s.gemm_ns for s in stats)
+    gemm_flops = sum(s.gemm_flops for s in stats)
+    achieved_tf = gemm_flops / (gemm_ns * 1e-9) / 1e12 if gemm_ns else 0.0
+    peak_tf = peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops"))
+    # step roofline (north_star): max(FLOP / P_tc, H2D bytes / host link), per GPU
+    flop_step = model_flops_per_token(c) * tokens_per_step / world
+    t_tc = flop_step / (peak_tf * 1e12)
+    t_link = max(st.h2d_bytes, st.d2h_bytes) / (h2d_gbps * 1e9)
+    t_roof = max(t_tc, t_link)
+    line = None
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "tokens/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "bf16", "data": "synthetic (seeded GPT-shaped tokens, random-init weights)",
+            "config": {"workload": f"GPT {args.config} (configs[1]): L={c.n_layers} h={c.hidden} heads={c.n_heads} "
+                                   f"s={c.seq_len} V={c.vocab}, stage ring capped at {args.cap_gib} GiB per GPU",
+                       "model": f"gpt-{args.config}", "global_batch": M * c.micro_batch, "seq_len": c.seq_len,
+                       "microbatches": M, "micro_batch": c.micro_batch, "parallelism": f"mobius-pp{world}",
+                       "n_stages": plan.n_stages, "stage_layers": [plan.stage_first_layer[j + 1] - plan.stage_first_layer[j]
+                                                                   for j in range(plan.n_stages)],
+                       "gpu_perm": [plan.gpu_perm[g] for g in range(world)], "plan_s": plan_s,
+                       "l2": "inputs larger than L2: every stage (3.1 GB bf16 total) streams from host DRAM each step"},
+            "loss": loss,
+            "e2e": e2e,
+            "roofline": {"bound": "tensor", "kernel": "gemm_tc (tcgen05 bf16, all block/head GEMMs)",
+                         "achieved": achieved_tf, "peak": peak_tf, "unit": "TFLOP/s",
+                         "frac": achieved_tf / peak_tf if peak_tf else None, "traffic": None,
+                         "peak_source": f"MEASURED_PEAKS.json bf16_tflops_sustained ({peak_src})"},
+            "step_roofline": {"t_tensor_ms": t_tc * 1e3, "t_link_ms": t_link * 1e3, "t_roofline_ms": t_roof * 1e3,
+                              "frac": t_roof / (ms * 1e-3), "h2d_GBps_link": h2d_gbps,
+                              "note": "north_star step roofline = max(algorithmic FLOPs / tensor peak, stage bytes / "
+                                      "measured pinned H2D); recompute, bubble and host update excluded"},
+            "swap_in": {"h2d_bytes_per_step": st.h2d_bytes, "d2h_bytes_per_step": st.d2h_bytes,
+                        "copies": st.n_h2d_copies, "GBps_median": st.h2d_GBps_median, "GBps_max": st.h2d_GBps_max,
+                        "link_peak_GBps": h2d_gbps, "exposed_load_ms": st.exposed_load_ns / 1e6},
+            "breakdown_ms": {"gemm": st.gemm_ns / 1e6, "attention": st.attn_ns / 1e6, "elementwise": st.elem_ns / 1e6,
+                             "device_step": st.device_step_ns / 1e6, "host_update_total": st.host_update_ns / 1e6,
+                             "update_tail": st.update_tail_ns / 1e6},
+            "gpu_launches": int(sum(s.kernel_launches for s in stats)),
+            "clocks": clocks,
+        }
+    ctx.close()
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_oracle_sample(c, tokens_per_step)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def main():
+    args = parse()
+    rank, world, local = dist_env()
+    if world != args.gpus and world > 1:
+        print(f"warning: WORLD_SIZE={world} != --gpus {args.gpus}", file=sys.stderr)
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    run_mobius(args, rank, world, local)
+
+
+if __name__ == "__main__":
+    main()

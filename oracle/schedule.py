@@ -26,10 +26,10 @@ import numpy as np
 from . import model as om
 
 
-def per_gpu_ops(stage_gpu, M):
+def per_gpu_ops(stage_gpu, M, n_gpus=None):
     """Per-GPU op lists [(op, j, m)], j and m 1-based (row a1)."""
     K = len(stage_gpu)
-    N = max(stage_gpu) + 1
+    N = max(stage_gpu) + 1 if n_gpus is None else n_gpus
     q = {g: [] for g in range(N)}
     for g in range(N):
         mine = [j for j in range(1, K + 1) if stage_gpu[j - 1] == g]
@@ -181,13 +181,13 @@ def execute(cfg, flat_params, tokens, boundaries, stage_gpu, dtype=np.float32):
     return loss_sum / n_tok, om.pack_layers(cfg, G, dtype=dtype), trace
 
 
-def byte_counts(stage_sums_list, stage_gpu, M, grad_bytes):
+def byte_counts(stage_sums_list, stage_gpu, M, grad_bytes, n_gpus=None):
     """O-10 byte accounting per GPU.  stage_sums_list[j-1] has Xf, Xb, A;
     grad_bytes[j-1] = offloaded gradient bytes of stage j.  Loads: every
     stage once in forward, stage j again in backward iff j + N <= K
     (reading #11 -> 2K - N loads per step)."""
     K = len(stage_gpu)
-    N = max(stage_gpu) + 1
+    N = max(stage_gpu) + 1 if n_gpus is None else n_gpus
     h2d = [0] * N
     d2h = [0] * N
     p2p = [0] * N

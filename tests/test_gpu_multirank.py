@@ -1,0 +1,92 @@
+"""Multi-rank Mobius step (rows a3 / a8: activation and activation-gradient
+P2P over CUDA-IPC mappings with release/acquire flags) with N = 2 ranks as
+two processes on ONE GPU (the IPC path is the same one NVLink peers use;
+gpurun gives one GPU).  Gradients of both ranks together must match the
+unpartitioned oracle step; each rank's trace must equal its Fig-4 queue."""
+import os
+import socket
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+if not torch.cuda.is_available():  # pragma: no cover
+    pytest.skip("needs a GPU", allow_module_level=True)
+
+import torch.multiprocessing as mp  # noqa: E402
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _rank_main(rank, world, port, sizes, perm, dtype, M, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    import torch.distributed as dist
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import synth
+        from paper_conf_asplos_fengxtwls23_b200 import MobiusContext, model_cfg, plan_from_sizes
+        from paper_conf_asplos_fengxtwls23_b200 import dist as mdist
+        c = synth.TINY
+        w = synth.perturb_norm_params(c, synth.gen_params(c), scale=0.1)
+        if dtype == 0:
+            w = synth.round_bf16(w)
+        tok = synth.gen_tokens(c, M)
+        cfg = model_cfg(c.n_layers, c.hidden, c.n_heads, c.seq_len, c.vocab, c.micro_batch, dtype=dtype)
+        plan = plan_from_sizes(sizes, world, M, perm=perm, hbm_cap_bytes=(4 << 20) * (2 if dtype else 1))
+        ctx = MobiusContext(cfg, plan, rank=rank, world=world, device=0, init_params=w)
+        mdist.connect(ctx)
+        losses = [ctx.step(tok) for _ in range(1)]
+        g = ctx.read_grads(c.n_params)
+        tr = ctx.read_trace()
+        st = ctx.stats()
+        ctx.close()
+        q.put((rank, losses, g, tr, st.h2d_bytes))
+    except Exception as e:  # pragma: no cover
+        q.put((rank, "ERR", repr(e), None, None))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("dtype,tol", [(0, 2e-2), (1, 1e-4)])
+@pytest.mark.parametrize("sizes,perm", [((2, 1, 1, 2), [0, 1]), ((1, 2, 2, 1), [1, 0]), ((3, 3), [0, 1])])
+def test_two_ranks_one_gpu(dtype, tol, sizes, perm):
+    import synth
+    from oracle import model as om
+    from oracle import schedule as osch
+    world, M = 2, 2
+    port = _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_rank_main, args=(r, world, port, sizes, perm, dtype, M, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = sorted([q.get(timeout=600) for _ in range(world)], key=lambda r: r[0])
+    for p in procs:
+        p.join(timeout=120)
+    for r in res:
+        assert r[1] != "ERR", r[2]
+    c = synth.TINY
+    w = synth.perturb_norm_params(c, synth.gen_params(c), scale=0.1)
+    if dtype == 0:
+        w = synth.round_bf16(w)
+    tok = synth.gen_tokens(c, M)
+    ref_loss, ref_g = om.reference_loss_and_grads(c, w, tok)
+    K = len(sizes)
+    sg = [perm[j % world] for j in range(K)]
+    last_rank = sg[-1]
+    loss = res[last_rank][1][0]
+    assert abs(loss - ref_loss) / ref_loss < tol
+    g = np.where(np.isnan(res[0][2]), res[1][2], res[0][2])
+    assert not np.isnan(g).any()
+    assert np.linalg.norm(g - ref_g) / np.linalg.norm(ref_g) < tol
+    queues = osch.per_gpu_ops(sg, M, n_gpus=world)
+    for r in range(world):
+        assert res[r][3] == queues[r]
