@@ -47,6 +47,12 @@ int mobius_kt_embed_fwd(int dtype, const int32_t* tok, const void* wte, const vo
 int mobius_kt_embed_bwd(int dtype, const int32_t* tok, const void* dx, float* dwte, float* dwpe, int mbs, int s,
                         int h);
 int mobius_kt_colsum(int dtype, const void* X, int64_t ld, int rows, int n, float* out);
+/* Causal attention core of a block (the path the block uses: fused tcgen05
+ * flash kernels on the bf16 path when head_dim in {64,128} and s % 128 == 0,
+ * else GEMM + softmax).  qkv [mbs*s, 3h] -> o [mbs*s, h]; if dout != NULL,
+ * dqkv [mbs*s, 3h] = d(sum o*dout)/d qkv. */
+int mobius_kt_attention(int dtype, int mbs, int s, int n_heads, int head_dim, const void* qkv, void* o,
+                        const void* dout, void* dqkv);
 /* One transformer block forward + backward through the runtime's block ops
  * (weights in oracle layout, path dtype, on device).  x [T,h] -> y [T,h];
  * dy [T,h] -> dx [T,h], grads (fp32, oracle layout of one block) +=. */

@@ -110,6 +110,7 @@ SIGNATURES = {
     "mobius_kt_embed_bwd": (I, [I, P, P, P, P, I, I, I]),
     "mobius_kt_colsum": (I, [I, P, I64, I, I, P]),
     "mobius_kt_block": (I, [I, I, I, I, I, P, P, P, P, P, P]),
+    "mobius_kt_attention": (I, [I, I, I, I, I, P, P, P, P]),
 }
 
 

@@ -251,6 +251,9 @@ class _KT:
     def colsum(self, dtype, X, ld, rows, n, out):
         check(lib.mobius_kt_colsum(dtype, self._p(X), ld, rows, n, self._p(out)))
 
+    def attention(self, dtype, mbs, s, nh, dh, qkv, o, dout=None, dqkv=None):
+        check(lib.mobius_kt_attention(dtype, mbs, s, nh, dh, *map(self._p, (qkv, o, dout, dqkv))))
+
     def block(self, dtype, h, nh, s, mbs, w, x, y, dy=None, dx=None, grads=None):
         check(lib.mobius_kt_block(dtype, h, nh, s, mbs, *map(self._p, (w, x, y, dy, dx, grads))))
 

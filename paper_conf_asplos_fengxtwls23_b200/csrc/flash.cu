@@ -1,0 +1,795 @@
+// Fused causal attention (flash-style) on tcgen05 for sm_100a (SURVEY
+// §8(f) f1; replaces the materialised S / P of K3/K4).
+//
+// Forward, one CTA per (batch, head, 128-query tile):
+//   warp 0     TMA producer: Q once, then K_j / V_j tiles (2-stage ring)
+//   warp 1     MMA issuer:   S_j = Q K_j^T  -> TMEM (double buffered)
+//                            O_j = P_j V_j  -> TMEM (double buffered, fresh per tile)
+//   warps 2-5  softmax:      thread = query row; online max / sum in the log2
+//                            domain, P_j (bf16) -> smem (UMMA K-major SW128
+//                            layout), O_reg = O_reg * 2^(a_{j-2}-a_{j-1}) + O_{j-1}
+//                            merged from TMEM; writes O (bf16) and lse (log2).
+// Backward, one CTA per (batch, head, 128-key tile), loop over query tiles
+// i >= j:  S^T = K Q_i^T, dP^T = V dO_i^T (TMEM); thread = key row computes
+// P^T = 2^(S^T*c - lse_q), dS^T = P^T (dP^T - D_q) * scale into smem; then
+// dV += P^T dO_i, dK += dS^T Q_i (TMEM accumulators), dQ_i = dS K_j (TMEM,
+// red.global.add.f32 into an fp32 dQ buffer).  The same smem tiles serve as
+// K-major and MN-major UMMA operands, so no transposes are materialised.
+#include <cuda.h>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+
+#include <cstring>
+
+#include "common.h"
+#include "flash.h"
+#include "ptx.cuh"
+
+namespace mobius {
+
+namespace {
+
+constexpr int BQ = 128;
+constexpr int BKV = 128;
+constexpr int NT = 192;
+
+__device__ __forceinline__ void named_bar(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
+
+// byte offset of 16-byte chunk `c` (8 bf16) of row `r` in a K-major SW128
+// tile of 128 rows whose K extent is split in 64-element atoms of 16 KiB
+__device__ __forceinline__ uint32_t sw128_off(int r, int c) {
+  return (uint32_t)((c >> 3) * 16384 + (r >> 3) * 1024 + (r & 7) * 128 + (((c & 7) ^ (r & 7)) << 4));
+}
+
+__device__ __forceinline__ uint32_t pack_bf16(float a, float b) {
+  __nv_bfloat162 h = __floats2bfloat162_rn(a, b);
+  return *reinterpret_cast<uint32_t*>(&h);
+}
+
+__device__ __forceinline__ void st_shared_v4(uint32_t addr, uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
+  asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(a), "r"(b), "r"(c), "r"(d) : "memory");
+}
+
+__device__ __forceinline__ void sts_f32(uint32_t addr, float v) {
+  asm volatile("st.shared.f32 [%0], %1;" ::"r"(addr), "f"(v) : "memory");
+}
+__device__ __forceinline__ float lds_f32(uint32_t addr) {
+  float v;
+  asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(addr) : "memory");
+  return v;
+}
+__device__ __forceinline__ float2 lds_f32x2(uint32_t addr) {
+  float2 v;
+  asm volatile("ld.shared.v2.f32 {%0, %1}, [%2];" : "=f"(v.x), "=f"(v.y) : "r"(addr) : "memory");
+  return v;
+}
+
+__device__ __forceinline__ float ex2(float x) {
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+
+constexpr int NT_FWD = 320;  // 10 warps: TMA, MMA, 8 softmax warps (4 lane quadrants x 2 column halves)
+
+template <int DH>
+struct FwdCfg {
+  static constexpr int Q_BYTES = BQ * DH * 2;
+  static constexpr int KV_BYTES = BKV * DH * 2;
+  static constexpr int P_BYTES = BQ * BKV * 2;
+  static constexpr int KVS = DH == 64 ? 2 : 1;  // K/V ring depth (smem budget)
+  static constexpr int SMEM = 1024 + 2 * Q_BYTES + 2 * KVS * KV_BYTES + 2 * P_BYTES + 4096;
+};
+
+struct FwdParams {
+  __nv_bfloat16* O;  // [mbs*s, h] (head view)
+  float* lse;        // [mbs, nh, s], log2 domain
+  int s, nh, h, mbs;
+  float scale_log2;  // log2(e) / sqrt(dh)
+};
+
+__device__ __forceinline__ void fwd_item(const FwdParams& p, int i, int& qt, int& hd, int& b) {
+  const int n_qt = p.s / BQ, nb = p.nh * p.mbs;
+  qt = n_qt - 1 - i / nb;  // heaviest (most kv tiles) first
+  const int r = i % nb;
+  hd = r % p.nh;
+  b = r / p.nh;
+}
+
+// Persistent: one CTA per SM loops over (batch, head, 128-query tile) items.
+// The TMA warp runs ahead into the next item (Q and O double-buffered), S_j
+// is double-buffered in TMEM so the tensor core computes S_{j+1} while the
+// softmax warps process S_j, P_j is double-buffered in smem, O accumulates in
+// TMEM with lazy rescaling.  Each query row is handled by two softmax warps
+// (column halves) that exchange only the row max.  All barrier phases run on
+// global step counters across items.
+template <int DH>
+__global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_constant__ CUtensorMap tm, const FwdParams p) {
+  using C = FwdCfg<DH>;
+  constexpr int KVS = C::KVS;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sQ = smem;                     // [2]
+  uint8_t* sK = sQ + 2 * C::Q_BYTES;      // [KVS]
+  uint8_t* sV = sK + KVS * C::KV_BYTES;   // [KVS]
+  uint8_t* sP = sV + KVS * C::KV_BYTES;   // [2]
+  float* sMax = reinterpret_cast<float*>(sP + 2 * C::P_BYTES);  // [2 iters][2 halves][128]
+  float* sSum = sMax + 512;                                       // [2 halves][128]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sSum + 256);
+  uint64_t* q_full = bars;          // [2]
+  uint64_t* q_empty = bars + 2;     // [2]
+  uint64_t* k_full = bars + 4;      // [2]
+  uint64_t* k_empty = bars + 6;     // [2]
+  uint64_t* v_full = bars + 8;      // [2]
+  uint64_t* v_empty = bars + 10;    // [2]
+  uint64_t* s_full = bars + 12;     // [2]
+  uint64_t* s_empty = bars + 14;    // [2] (count 8)
+  uint64_t* p_full = bars + 16;     // [2] (count 8)
+  uint64_t* pv_done = bars + 18;    // [2] PV of global step g commits pv_done[g & 1]
+  uint64_t* o_ready = bars + 20;    // [2] all PVs of an item done
+  uint64_t* o_empty = bars + 22;    // [2] (count 8) O read out
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 24);
+
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int n_items = (p.s / BQ) * p.nh * p.mbs;
+
+  if (threadIdx.x == 0) {
+    ptx::tma_prefetch_desc(&tm);
+    for (int i = 0; i < 2; ++i) {
+      ptx::mbar_init(&q_full[i], 1);
+      ptx::mbar_init(&q_empty[i], 1);
+      ptx::mbar_init(&k_full[i], 1);
+      ptx::mbar_init(&k_empty[i], 1);
+      ptx::mbar_init(&v_full[i], 1);
+      ptx::mbar_init(&v_empty[i], 1);
+      ptx::mbar_init(&s_full[i], 1);
+      ptx::mbar_init(&s_empty[i], 8);
+      ptx::mbar_init(&p_full[i], 8);
+      ptx::mbar_init(&pv_done[i], 1);
+      ptx::mbar_init(&o_ready[i], 1);
+      ptx::mbar_init(&o_empty[i], 8);
+    }
+    ptx::fence_mbar_init();
+  }
+  if (warp == 1) ptx::tmem_alloc<512>(tmem_slot);
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  // TMEM: S[2] at 0 / 128, O[2] at 256 / 256 + DH
+  if (warp == 0) {
+    if (lane == 0) {
+      int g = 0, it = 0;
+      for (int i = blockIdx.x; i < n_items; i += gridDim.x, ++it) {
+        int qt, hd, b;
+        fwd_item(p, i, qt, hd, b);
+        const int qb = it & 1;
+        ptx::mbar_wait(&q_empty[qb], ((it >> 1) & 1) ^ 1);
+        ptx::mbar_arrive_expect_tx(&q_full[qb], C::Q_BYTES);
+#pragma unroll
+        for (int c = 0; c < DH / 64; ++c)
+          ptx::tma_load_4d(sQ + qb * C::Q_BYTES + c * 16384, &tm, &q_full[qb], 64 * c, qt * BQ, hd, b);
+        for (int j = 0; j <= qt; ++j, ++g) {
+          const int st = g % KVS, kph = (g / KVS) & 1;
+          ptx::mbar_wait(&k_empty[st], kph ^ 1);
+          ptx::mbar_arrive_expect_tx(&k_full[st], C::KV_BYTES);
+#pragma unroll
+          for (int c = 0; c < DH / 64; ++c)
+            ptx::tma_load_4d(sK + st * C::KV_BYTES + c * 16384, &tm, &k_full[st], 64 * c, j * BKV, p.nh + hd, b);
+          ptx::mbar_wait(&v_empty[st], kph ^ 1);
+          ptx::mbar_arrive_expect_tx(&v_full[st], C::KV_BYTES);
+#pragma unroll
+          for (int c = 0; c < DH / 64; ++c)
+            ptx::tma_load_4d(sV + st * C::KV_BYTES + c * 16384, &tm, &v_full[st], 64 * c, j * BKV, 2 * p.nh + hd, b);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {
+      constexpr uint32_t ID_S = ptx::idesc_bf16(BQ, BKV, 0, 0);
+      constexpr uint32_t ID_O = ptx::idesc_bf16(BQ, DH, 0, 1);
+      int gs = 0, gp = 0, it = 0;  // global S-issue step, global PV step, local item count
+      for (int i = blockIdx.x; i < n_items; i += gridDim.x, ++it) {
+        int qt, hd, b;
+        fwd_item(p, i, qt, hd, b);
+        const int nkv = qt + 1, ob = it & 1;
+        ptx::mbar_wait(&q_full[ob], (it >> 1) & 1);
+        const uint32_t aq = ptx::smem_u32(sQ + ob * C::Q_BYTES);
+        auto issue_s = [&](int last) {
+          const int st = gs % KVS, kph = (gs / KVS) & 1, sb = gs & 1;
+          ptx::mbar_wait(&k_full[st], kph);
+          ptx::mbar_wait(&s_empty[sb], ((gs >> 1) & 1) ^ 1);
+          ptx::tc_fence_after();
+          const uint32_t ak = ptx::smem_u32(sK + st * C::KV_BYTES);
+#pragma unroll
+          for (int k = 0; k < DH / 16; ++k) {
+            const uint32_t off = (k >> 2) * 16384 + (k & 3) * 32;
+            ptx::mma_bf16(tmem + sb * 128, ptx::sdesc_sw128(aq + off, 16, 1024), ptx::sdesc_sw128(ak + off, 16, 1024),
+                          ID_S, k > 0);
+          }
+          ptx::mma_commit(&s_full[sb]);
+          ptx::mma_commit(&k_empty[st]);
+          if (last) ptx::mma_commit(&q_empty[ob]);
+          ++gs;
+        };
+        issue_s(nkv == 1);
+        ptx::mbar_wait(&o_empty[ob], ((it >> 1) & 1) ^ 1);  // O[ob] read out (item it-2)
+        for (int j = 0; j < nkv; ++j) {
+          if (j + 1 < nkv) issue_s(j + 2 == nkv);
+          const int st = gp % KVS, kph = (gp / KVS) & 1, pb = gp & 1;
+          ptx::mbar_wait(&p_full[pb], (gp >> 1) & 1);
+          ptx::mbar_wait(&v_full[st], kph);
+          ptx::tc_fence_after();
+          const uint32_t ap = ptx::smem_u32(sP + pb * C::P_BYTES), av = ptx::smem_u32(sV + st * C::KV_BYTES);
+#pragma unroll
+          for (int k = 0; k < BKV / 16; ++k) {
+            const uint32_t offp = (k >> 2) * 16384 + (k & 3) * 32;
+            ptx::mma_bf16(tmem + 256 + ob * DH, ptx::sdesc_sw128(ap + offp, 16, 1024),
+                          ptx::sdesc_sw128(av + k * 2048, 16384, 1024), ID_O, (j > 0 || k > 0) ? 1u : 0u);
+          }
+          ptx::mma_commit(&pv_done[pb]);
+          ptx::mma_commit(&v_empty[st]);
+          ++gp;
+        }
+        ptx::mma_commit(&o_ready[ob]);
+      }
+    }
+  } else {
+    // ------------------------------------------------ softmax warps
+    const int q4 = warp & 3;          // TMEM lane quadrant
+    const int hf = (warp - 2) >> 2;   // column half of S (and of O)
+    const int row = q4 * 32 + lane;
+    const uint32_t lb = (uint32_t)(q4 * 32) << 16;
+    const float sc = p.scale_log2;
+    int g = 0, it = 0;
+    for (int i = blockIdx.x; i < n_items; i += gridDim.x, ++it) {
+      int qt, hd, b;
+      fwd_item(p, i, qt, hd, b);
+      const int nkv = qt + 1, ob = it & 1;
+      const int qrow = qt * BQ + row;
+      float m_run = -INFINITY, l_run = 0.f;
+      for (int j = 0; j < nkv; ++j, ++g) {
+        const int sb = g & 1;
+        const bool diag = (j == qt);
+        const uint32_t TS = tmem + sb * 128 + hf * 64 + lb;
+        ptx::mbar_wait(&s_full[sb], (g >> 1) & 1);
+        ptx::tc_fence_after();
+        uint32_t v0[32], v1[32];
+        __syncwarp();
+        ptx::tmem_ld32(TS, v0);
+        ptx::tmem_ld32(TS + 32, v1);
+        ptx::tmem_ld_wait();
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(&s_empty[sb]);  // S values are in registers
+        const int cbase = hf * 64;  // first key column of this half
+        if (diag) {  // mask keys > query (only on the diagonal tile)
+#pragma unroll
+          for (int e = 0; e < 32; ++e) {
+            if (cbase + e > row) v0[e] = __float_as_uint(-INFINITY);
+            if (cbase + 32 + e > row) v1[e] = __float_as_uint(-INFINITY);
+          }
+        }
+        // pass A: half-row max of raw scores, combined across the warp pair
+        float mx = -INFINITY;
+#pragma unroll
+        for (int e = 0; e < 32; e += 2) mx = fmaxf(mx, fmaxf(__uint_as_float(v0[e]), __uint_as_float(v0[e + 1])));
+#pragma unroll
+        for (int e = 0; e < 32; e += 2) mx = fmaxf(mx, fmaxf(__uint_as_float(v1[e]), __uint_as_float(v1[e + 1])));
+        sts_f32(ptx::smem_u32(sMax + (g & 1) * 256 + hf * 128 + row), mx);
+        named_bar(2 + q4, 64);
+        mx = fmaxf(mx, lds_f32(ptx::smem_u32(sMax + (g & 1) * 256 + (1 - hf) * 128 + row)));
+        // lazy rescaling: keep the running max unless it grows by > 8 (log2)
+        const float m_cand = fmaxf(m_run, mx * sc);
+        const bool grow = m_cand > m_run + 8.f;
+        const float m_new = grow ? m_cand : m_run;
+        const float alpha = ex2(m_run - m_new);  // 1 when not growing; 0 at j = 0
+        if (j >= 1 && __any_sync(0xffffffffu, grow)) {  // rescale this half of O (PV of step g-1 done)
+          ptx::mbar_wait(&pv_done[(g - 1) & 1], ((g - 1) >> 1) & 1);
+          ptx::tc_fence_after();
+#pragma unroll
+          for (int c = 0; c < DH / 64; ++c) {
+            uint32_t o[32];
+            const uint32_t TO = tmem + 256 + ob * DH + hf * (DH / 2) + c * 32 + lb;
+            ptx::tmem_ld32(TO, o);
+            ptx::tmem_ld_wait();
+#pragma unroll
+            for (int e = 0; e < 32; ++e) o[e] = __float_as_uint(__uint_as_float(o[e]) * alpha);
+            ptx::tmem_st32(TO, o);
+          }
+          ptx::tmem_st_wait();
+        }
+        // P buffer sb is free once the PV of global step g-2 completed
+        if (g >= 2) ptx::mbar_wait(&pv_done[sb], ((g - 2) >> 1) & 1);
+        // pass B: P = 2^(x*sc - m_new) -> smem (bf16), half-row sum
+        const uint32_t sp = ptx::smem_u32(sP + sb * C::P_BYTES);
+        float rs = 0.f;
+        {
+          uint32_t pk[16];
+#pragma unroll
+          for (int e = 0; e < 32; e += 2) {
+            const float p0 = ex2(fmaf(__uint_as_float(v0[e]), sc, -m_new));
+            const float p1 = ex2(fmaf(__uint_as_float(v0[e + 1]), sc, -m_new));
+            rs += p0 + p1;
+            pk[e >> 1] = pack_bf16(p0, p1);
+          }
+#pragma unroll
+          for (int k = 0; k < 4; ++k)
+            st_shared_v4(sp + sw128_off(row, hf * 8 + k), pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
+#pragma unroll
+          for (int e = 0; e < 32; e += 2) {
+            const float p0 = ex2(fmaf(__uint_as_float(v1[e]), sc, -m_new));
+            const float p1 = ex2(fmaf(__uint_as_float(v1[e + 1]), sc, -m_new));
+            rs += p0 + p1;
+            pk[e >> 1] = pack_bf16(p0, p1);
+          }
+#pragma unroll
+          for (int k = 0; k < 4; ++k)
+            st_shared_v4(sp + sw128_off(row, hf * 8 + 4 + k), pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
+        }
+        l_run = l_run * alpha + rs;
+        m_run = m_new;
+        ptx::tc_fence_before();
+        ptx::fence_proxy_async();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(&p_full[sb]);
+      }
+      // output: O / l  (l = sum of both halves)
+      sts_f32(ptx::smem_u32(sSum + hf * 128 + row), l_run);
+      named_bar(2 + q4, 64);
+      const float l_tot = l_run + lds_f32(ptx::smem_u32(sSum + (1 - hf) * 128 + row));
+      ptx::mbar_wait(&o_ready[ob], (it >> 1) & 1);
+      ptx::tc_fence_after();
+      const float inv_l = 1.f / l_tot;
+      __nv_bfloat16* orow = p.O + ((int64_t)b * p.s + qrow) * p.h + hd * DH + hf * (DH / 2);
+#pragma unroll
+      for (int c = 0; c < DH / 64; ++c) {
+        uint32_t v[32];
+        __syncwarp();
+        ptx::tmem_ld32(tmem + 256 + ob * DH + hf * (DH / 2) + c * 32 + lb, v);
+        ptx::tmem_ld_wait();
+        uint32_t pk[16];
+#pragma unroll
+        for (int e = 0; e < 32; e += 2)
+          pk[e / 2] = pack_bf16(__uint_as_float(v[e]) * inv_l, __uint_as_float(v[e + 1]) * inv_l);
+#pragma unroll
+        for (int k = 0; k < 4; ++k)
+          *reinterpret_cast<uint4*>(orow + c * 32 + k * 8) =
+              make_uint4(pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
+      }
+      if (hf == 0) p.lse[((int64_t)b * p.nh + hd) * p.s + qrow] = m_run + __log2f(l_tot);
+      ptx::tc_fence_before();
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(&o_empty[ob]);
+      named_bar(2 + q4, 64);  // partner read sSum before the next item overwrites it
+    }
+  }
+  __syncthreads();
+  if (warp == 1) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc<512>(tmem);
+  }
+}
+
+// ====================================================================== bwd
+template <int DH>
+struct BwdCfg {
+  static constexpr int T_BYTES = 128 * DH * 2;       // one K / V / Q / dO tile
+  static constexpr int QS = DH == 64 ? 2 : 1;        // Q/dO pipeline depth
+  static constexpr int PT_BYTES = 128 * 128 * 2;     // P^T or dS^T tile
+  static constexpr int SMEM = 1024 + 2 * T_BYTES + QS * 2 * T_BYTES + 2 * PT_BYTES + 2 * 2 * 128 * 4 + 256;
+};
+
+struct BwdParams {
+  const float* lse;     // [mbs, nh, s] log2 domain
+  const float* Dsum;    // [mbs, nh, s] rowsum(dO * O)
+  float* dQacc;         // [mbs*s, h] fp32 (head view), accumulated with red.add
+  __nv_bfloat16* dK;    // head view into dqkv (k part)
+  __nv_bfloat16* dV;    // head view into dqkv (v part)
+  int64_t ldd;          // row stride of dK/dV (3h)
+  int s, nh, h;
+  float scale_log2, scale;
+};
+
+__device__ __forceinline__ void red_add_v4(float* addr, float a, float b, float c, float d) {
+  asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(addr), "f"(a), "f"(b), "f"(c), "f"(d)
+               : "memory");
+}
+
+template <int DH>
+__global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_constant__ CUtensorMap tm,
+                                                          const __grid_constant__ CUtensorMap tdo, const BwdParams p) {
+  using C = BwdCfg<DH>;
+  constexpr int QS = C::QS;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sK = smem;
+  uint8_t* sV = sK + C::T_BYTES;
+  uint8_t* sQ = sV + C::T_BYTES;             // [QS]
+  uint8_t* sdO = sQ + QS * C::T_BYTES;       // [QS]
+  uint8_t* sPT = sdO + QS * C::T_BYTES;
+  uint8_t* sdST = sPT + C::PT_BYTES;
+  float* sLse = reinterpret_cast<float*>(sdST + C::PT_BYTES);  // [2][128]
+  float* sD = sLse + 2 * 128;                                  // [2][128]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sD + 2 * 128);
+  uint64_t* kv_full = bars;          // 1
+  uint64_t* q_full = bars + 1;       // [QS] (Q, dO, lse, D)
+  uint64_t* q_empty = bars + 3;      // [QS]
+  uint64_t* s_full = bars + 5;       // S^T and dP^T ready
+  uint64_t* p_full = bars + 6;       // P^T / dS^T in smem (count 4)
+  uint64_t* mm_done = bars + 7;      // dV/dK/dQ MMAs of this tile done (P^T/dS^T smem free, dQ ready)
+  uint64_t* dq_empty = bars + 8;     // dQ read out (count 4) -> TMEM S/dQ region free
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 9);
+
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int n_t = p.s / 128;
+  const int kt = (int)blockIdx.x;  // key tile (tile kt has n_t - kt query tiles; light-first is fine)
+  const int hd = blockIdx.y, b = blockIdx.z;
+  const int i0 = kt, nq = n_t - kt;
+
+  if (threadIdx.x == 0) {
+    ptx::tma_prefetch_desc(&tm);
+    ptx::tma_prefetch_desc(&tdo);
+    ptx::mbar_init(kv_full, 1);
+    for (int i = 0; i < 2; ++i) {
+      ptx::mbar_init(&q_full[i], 1);
+      ptx::mbar_init(&q_empty[i], 1);
+    }
+    ptx::mbar_init(s_full, 1);
+    ptx::mbar_init(p_full, 8);
+    ptx::mbar_init(mm_done, 1);
+    ptx::mbar_init(dq_empty, 8);
+    ptx::fence_mbar_init();
+  }
+  if (warp == 1) ptx::tmem_alloc<512>(tmem_slot);
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  const uint32_t T_S = tmem, T_DP = tmem + 128, T_DV = tmem + 256, T_DK = tmem + 256 + DH;
+  (void)T_DK;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      ptx::mbar_arrive_expect_tx(kv_full, 2 * C::T_BYTES);
+#pragma unroll
+      for (int c = 0; c < DH / 64; ++c) {
+        ptx::tma_load_4d(sK + c * 16384, &tm, kv_full, 64 * c, kt * 128, p.nh + hd, b);
+        ptx::tma_load_4d(sV + c * 16384, &tm, kv_full, 64 * c, kt * 128, 2 * p.nh + hd, b);
+      }
+      for (int it = 0; it < nq; ++it) {
+        const int st = it % QS;
+        const int ph = (it / QS) & 1;
+        const int qi = i0 + it;
+        ptx::mbar_wait(&q_empty[st], ph ^ 1);
+        ptx::mbar_arrive_expect_tx(&q_full[st], 2 * C::T_BYTES);
+#pragma unroll
+        for (int c = 0; c < DH / 64; ++c) {
+          ptx::tma_load_4d(sQ + st * C::T_BYTES + c * 16384, &tm, &q_full[st], 64 * c, qi * 128, hd, b);
+          ptx::tma_load_4d(sdO + st * C::T_BYTES + c * 16384, &tdo, &q_full[st], 64 * c, qi * 128, hd, b);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {
+      // S^T (M=kv, N=q, K=d): A = K tile (K-major), B = Q tile (K-major)
+      constexpr uint32_t ID_ST = ptx::idesc_bf16(128, 128, 0, 0);
+      // dV (M=kv, N=d, K=q): A = P^T (K-major), B = dO (MN-major)
+      constexpr uint32_t ID_DV = ptx::idesc_bf16(128, DH, 0, 1);
+      // dQ (M=q, N=d, K=kv): A = dS (MN-major view of dS^T), B = K (MN-major)
+      constexpr uint32_t ID_DQ = ptx::idesc_bf16(128, DH, 1, 1);
+      const uint32_t ak = ptx::smem_u32(sK), av = ptx::smem_u32(sV);
+      const uint32_t apt = ptx::smem_u32(sPT), adst = ptx::smem_u32(sdST);
+      ptx::mbar_wait(kv_full, 0);
+      for (int it = 0; it < nq; ++it) {
+        const int st = it % QS;
+        const int ph = (it / QS) & 1;
+        const uint32_t aq = ptx::smem_u32(sQ + st * C::T_BYTES), ado = ptx::smem_u32(sdO + st * C::T_BYTES);
+        ptx::mbar_wait(&q_full[st], ph);
+        ptx::mbar_wait(dq_empty, (it & 1) ^ 1);  // S/dQ TMEM region free (dQ_{it-1} read)
+        ptx::tc_fence_after();
+#pragma unroll
+        for (int t = 0; t < DH / 16; ++t) {
+          const uint32_t off = (t >> 2) * 16384 + (t & 3) * 32;
+          ptx::mma_bf16(T_S, ptx::sdesc_sw128(ak + off, 16, 1024), ptx::sdesc_sw128(aq + off, 16, 1024), ID_ST, t > 0);
+        }
+#pragma unroll
+        for (int t = 0; t < DH / 16; ++t) {
+          const uint32_t off = (t >> 2) * 16384 + (t & 3) * 32;
+          ptx::mma_bf16(T_DP, ptx::sdesc_sw128(av + off, 16, 1024), ptx::sdesc_sw128(ado + off, 16, 1024), ID_ST,
+                        t > 0);
+        }
+        ptx::mma_commit(s_full);
+        // wait for P^T / dS^T in smem
+        ptx::mbar_wait(p_full, it & 1);
+        ptx::tc_fence_after();
+#pragma unroll
+        for (int t = 0; t < 128 / 16; ++t) {  // K = 128 queries
+          const uint32_t offa = (t >> 2) * 16384 + (t & 3) * 32;
+          // dV += P^T dO
+          ptx::mma_bf16(T_DV, ptx::sdesc_sw128(apt + offa, 16, 1024), ptx::sdesc_sw128(ado + t * 2048, 16384, 1024),
+                        ID_DV, (it > 0 || t > 0) ? 1u : 0u);
+          // dK += dS^T Q
+          ptx::mma_bf16(T_DV + DH, ptx::sdesc_sw128(adst + offa, 16, 1024),
+                        ptx::sdesc_sw128(aq + t * 2048, 16384, 1024), ID_DV, (it > 0 || t > 0) ? 1u : 0u);
+        }
+#pragma unroll
+        for (int t = 0; t < 128 / 16; ++t) {  // K = 128 keys: dQ = dS K
+          ptx::mma_bf16(T_S, ptx::sdesc_sw128(adst + t * 2048, 16384, 1024),
+                        ptx::sdesc_sw128(ak + t * 2048, 16384, 1024), ID_DQ, t > 0);
+        }
+        ptx::mma_commit(mm_done);
+        ptx::mma_commit(&q_empty[st]);
+      }
+    }
+  } else {
+    // ---------------------------------------- softmax-gradient warps
+    // 8 warps: (lane quadrant q4, column half hf); thread = key row r,
+    // query columns [64 hf, 64 hf + 64)
+    const int q4 = warp & 3;
+    const int hf = (warp - 2) >> 2;
+    const int r = q4 * 32 + lane;     // key row of this thread (TMEM lane)
+    const int t8 = threadIdx.x - 64;  // 0..255
+    const uint32_t lane_base = (uint32_t)(q4 * 32) << 16;
+    const uint32_t spt = ptx::smem_u32(sPT), sdst = ptx::smem_u32(sdST);
+    for (int it = 0; it < nq; ++it) {
+      const int st = it & 1;  // lse / D double buffer (independent of QS)
+      const int qi = i0 + it;
+      const bool diag = (qi == kt);
+      {  // stage lse / D of this query tile in smem
+        const int64_t base = ((int64_t)b * p.nh + hd) * p.s + qi * 128;
+        if (t8 < 128)
+          sts_f32(ptx::smem_u32(sLse + st * 128 + t8), p.lse[base + t8]);
+        else
+          sts_f32(ptx::smem_u32(sD + st * 128 + t8 - 128), p.Dsum[base + t8 - 128]);
+      }
+      named_bar(1, 256);
+      ptx::mbar_wait(s_full, it & 1);
+      ptx::tc_fence_after();
+      // P^T / dS^T smem must be free: previous tile's MMAs done
+      if (it >= 1) ptx::mbar_wait(mm_done, (it - 1) & 1);
+#pragma unroll
+      for (int cc = 0; cc < 2; ++cc) {
+        const int c = hf * 2 + cc;
+        uint32_t vs[32], vd[32];
+        __syncwarp();
+        ptx::tmem_ld32(T_S + c * 32 + lane_base, vs);
+        ptx::tmem_ld32(T_DP + c * 32 + lane_base, vd);
+        ptx::tmem_ld_wait();
+        uint32_t ppk[16], dpk[16];
+        const uint32_t aL = ptx::smem_u32(sLse + st * 128 + c * 32), aD = ptx::smem_u32(sD + st * 128 + c * 32);
+#pragma unroll
+        for (int e = 0; e < 32; e += 2) {
+          const int q = c * 32 + e;
+          const float2 L = lds_f32x2(aL + e * 4), Dd = lds_f32x2(aD + e * 4);  // broadcast reads
+          float p0 = ex2(fmaf(__uint_as_float(vs[e]), p.scale_log2, -L.x));
+          float p1 = ex2(fmaf(__uint_as_float(vs[e + 1]), p.scale_log2, -L.y));
+          if (diag) {  // key r attends only from queries >= r
+            if (q < r) p0 = 0.f;
+            if (q + 1 < r) p1 = 0.f;
+          }
+          const float d0 = p0 * (__uint_as_float(vd[e]) - Dd.x) * p.scale;
+          const float d1 = p1 * (__uint_as_float(vd[e + 1]) - Dd.y) * p.scale;
+          ppk[e >> 1] = pack_bf16(p0, p1);
+          dpk[e >> 1] = pack_bf16(d0, d1);
+        }
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const uint32_t o = sw128_off(r, c * 4 + k);
+          st_shared_v4(spt + o, ppk[4 * k], ppk[4 * k + 1], ppk[4 * k + 2], ppk[4 * k + 3]);
+          st_shared_v4(sdst + o, dpk[4 * k], dpk[4 * k + 1], dpk[4 * k + 2], dpk[4 * k + 3]);
+        }
+      }
+      ptx::tc_fence_before();
+      ptx::fence_proxy_async();
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(p_full);
+      // dQ of this query tile: TMEM lane = query row; this warp's column half
+      ptx::mbar_wait(mm_done, it & 1);
+      ptx::tc_fence_after();
+      float* dq = p.dQacc + ((int64_t)b * p.s + qi * 128 + r) * p.h + hd * DH;
+#pragma unroll
+      for (int cc = 0; cc < DH / 64; ++cc) {
+        const int c = hf * (DH / 64) + cc;
+        uint32_t v[32];
+        __syncwarp();
+        ptx::tmem_ld32(T_S + c * 32 + lane_base, v);
+        ptx::tmem_ld_wait();
+#pragma unroll
+        for (int e = 0; e < 32; e += 4)
+          red_add_v4(dq + c * 32 + e, __uint_as_float(v[e]), __uint_as_float(v[e + 1]), __uint_as_float(v[e + 2]),
+                     __uint_as_float(v[e + 3]));
+      }
+      ptx::tc_fence_before();
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(dq_empty);
+    }
+    // dV (half 0) / dK (half 1) of this key tile (rows = keys)
+    ptx::mbar_wait(mm_done, (nq - 1) & 1);
+    ptx::tc_fence_after();
+    __nv_bfloat16* out = (hf == 0 ? p.dV : p.dK) + ((int64_t)b * p.s + kt * 128 + r) * p.ldd + hd * DH;
+#pragma unroll
+    for (int c = 0; c < DH / 32; ++c) {
+      uint32_t v[32];
+      __syncwarp();
+      ptx::tmem_ld32(T_DV + hf * DH + c * 32 + lane_base, v);
+      ptx::tmem_ld_wait();
+      uint32_t pk[16];
+#pragma unroll
+      for (int e = 0; e < 32; e += 2) pk[e / 2] = pack_bf16(__uint_as_float(v[e]), __uint_as_float(v[e + 1]));
+#pragma unroll
+      for (int k = 0; k < 4; ++k)
+        *reinterpret_cast<uint4*>(out + c * 32 + k * 8) = make_uint4(pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
+    }
+    ptx::tc_fence_before();
+  }
+  __syncthreads();
+  if (warp == 1) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc<512>(tmem);
+  }
+}
+
+// D[b, h, q] = sum_d dO[q, d] * O[q, d]  (one warp per (row, head))
+__global__ void flash_dsum_kernel(const __nv_bfloat16* dO, const __nv_bfloat16* O, float* D, int rows, int nh, int dh,
+                                  int h, int s) {
+  const int64_t w = (int64_t)blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32;
+  const int lane = threadIdx.x % 32;
+  if (w >= (int64_t)rows * nh) return;
+  const int row = (int)(w / nh), hd = (int)(w % nh);
+  const __nv_bfloat16* a = dO + (int64_t)row * h + hd * dh;
+  const __nv_bfloat16* o = O + (int64_t)row * h + hd * dh;
+  float acc = 0.f;
+  for (int d = lane * 2; d < dh; d += 64) {
+    float2 x = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(a + d));
+    float2 y = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(o + d));
+    acc += x.x * y.x + x.y * y.y;
+  }
+#pragma unroll
+  for (int k = 16; k; k >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, k);
+  if (lane == 0) {
+    const int b = row / s, q = row % s;
+    D[((int64_t)b * nh + hd) * s + q] = acc;
+  }
+}
+
+// dqkv q-part (bf16, row stride 3h) = dQacc (fp32, row stride h)
+__global__ void flash_dq_cast_kernel(const float* dQacc, __nv_bfloat16* dq, int64_t rows, int h, int64_t ldd) {
+  const int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 4;
+  if (i >= rows * h) return;
+  const int64_t r = i / h, c = i % h;
+  float4 v = *reinterpret_cast<const float4*>(dQacc + i);
+  __nv_bfloat162* o = reinterpret_cast<__nv_bfloat162*>(dq + r * ldd + c);
+  o[0] = __floats2bfloat162_rn(v.x, v.y);
+  o[1] = __floats2bfloat162_rn(v.z, v.w);
+}
+
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeTiledFn encode_fn() {
+  static EncodeTiledFn fn = nullptr;
+  if (!fn) {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<EncodeTiledFn>(p);
+  }
+  return fn;
+}
+
+// {d, token, head-slot, batch} map over a [mbs*s, ld] bf16 buffer whose head
+// slots are dh apart; box {64, 128, 1, 1}
+int head_map(CUtensorMap* m, const void* base, int64_t ld, int dh, int s, int n_slots, int mbs) {
+  EncodeTiledFn enc = encode_fn();
+  if (!enc) MOBIUS_FAIL(MOBIUS_ECUDA, "cuTensorMapEncodeTiled unavailable");
+  cuuint64_t dims[4] = {(cuuint64_t)dh, (cuuint64_t)s, (cuuint64_t)n_slots, (cuuint64_t)mbs};
+  cuuint64_t strides[3] = {(cuuint64_t)(ld * 2), (cuuint64_t)(dh * 2), (cuuint64_t)(s * ld * 2)};
+  cuuint32_t box[4] = {64, 128, 1, 1};
+  cuuint32_t es[4] = {1, 1, 1, 1};
+  CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void*>(base), dims, strides, box, es,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) MOBIUS_FAIL(MOBIUS_ECUDA, "flash tensor map (%d)", (int)r);
+  return MOBIUS_OK;
+}
+
+template <typename K>
+int set_smem(K k, int bytes) {
+  if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, bytes) != cudaSuccess)
+    MOBIUS_FAIL(MOBIUS_ECUDA, "flash smem attribute");
+  return MOBIUS_OK;
+}
+
+}  // namespace
+
+int flash_supported(int dh, int s) { return (dh == 64 || dh == 128) && s % 128 == 0; }
+
+int flash_attn_fwd(const __nv_bfloat16* qkv, __nv_bfloat16* o, float* lse, int mbs, int s, int nh, int dh,
+                   cudaStream_t st) {
+  MOBIUS_CHECK_ARG(flash_supported(dh, s), "flash: dh %d / s %d unsupported", dh, s);
+  const int h = nh * dh;
+  CUtensorMap tm;
+  int rc = head_map(&tm, qkv, 3 * h, dh, s, 3 * nh, mbs);
+  if (rc) return rc;
+  FwdParams p;
+  p.O = o;
+  p.lse = lse;
+  p.s = s;
+  p.nh = nh;
+  p.h = h;
+  p.mbs = mbs;
+  p.scale_log2 = 1.4426950408889634f / sqrtf((float)dh);
+  int n_items = (s / BQ) * nh * mbs;
+  int sms = 148;
+  {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  }
+  dim3 grid(n_items < sms ? n_items : sms);
+  if (dh == 64) {
+    static bool once = false;
+    if (!once) { rc = set_smem(flash_fwd_kernel<64>, FwdCfg<64>::SMEM); if (rc) return rc; once = true; }
+    flash_fwd_kernel<64><<<grid, NT_FWD, FwdCfg<64>::SMEM, st>>>(tm, p);
+  } else {
+    static bool once = false;
+    if (!once) { rc = set_smem(flash_fwd_kernel<128>, FwdCfg<128>::SMEM); if (rc) return rc; once = true; }
+    flash_fwd_kernel<128><<<grid, NT_FWD, FwdCfg<128>::SMEM, st>>>(tm, p);
+  }
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) MOBIUS_FAIL(MOBIUS_ECUDA, "flash_fwd launch: %s", cudaGetErrorString(e));
+  return MOBIUS_OK;
+}
+
+int flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* o, const __nv_bfloat16* dout, const float* lse,
+                   float* dsum_ws, float* dq_ws, __nv_bfloat16* dqkv, int mbs, int s, int nh, int dh,
+                   cudaStream_t st) {
+  MOBIUS_CHECK_ARG(flash_supported(dh, s), "flash: dh %d / s %d unsupported", dh, s);
+  const int h = nh * dh;
+  const int64_t rows = (int64_t)mbs * s;
+  CUtensorMap tm, tdo;
+  int rc = head_map(&tm, qkv, 3 * h, dh, s, 3 * nh, mbs);
+  if (rc) return rc;
+  rc = head_map(&tdo, dout, h, dh, s, nh, mbs);
+  if (rc) return rc;
+  {
+    const int64_t warps = rows * nh;
+    flash_dsum_kernel<<<(unsigned)((warps + 7) / 8), 256, 0, st>>>(dout, o, dsum_ws, (int)rows, nh, dh, h, s);
+  }
+  cudaError_t e = cudaMemsetAsync(dq_ws, 0, rows * h * sizeof(float), st);
+  if (e != cudaSuccess) MOBIUS_FAIL(MOBIUS_ECUDA, "flash dq memset");
+  BwdParams p;
+  p.lse = lse;
+  p.Dsum = dsum_ws;
+  p.dQacc = dq_ws;
+  p.dK = dqkv + h;
+  p.dV = dqkv + 2 * h;
+  p.ldd = 3 * h;
+  p.s = s;
+  p.nh = nh;
+  p.h = h;
+  p.scale_log2 = 1.4426950408889634f / sqrtf((float)dh);
+  p.scale = 1.0f / sqrtf((float)dh);
+  dim3 grid(s / 128, nh, mbs);
+  if (dh == 64) {
+    static bool once = false;
+    if (!once) { rc = set_smem(flash_bwd_kernel<64>, BwdCfg<64>::SMEM); if (rc) return rc; once = true; }
+    flash_bwd_kernel<64><<<grid, NT_FWD, BwdCfg<64>::SMEM, st>>>(tm, tdo, p);
+  } else {
+    static bool once = false;
+    if (!once) { rc = set_smem(flash_bwd_kernel<128>, BwdCfg<128>::SMEM); if (rc) return rc; once = true; }
+    flash_bwd_kernel<128><<<grid, NT_FWD, BwdCfg<128>::SMEM, st>>>(tm, tdo, p);
+  }
+  {
+    const int64_t n = rows * h / 4;
+    flash_dq_cast_kernel<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(dq_ws, dqkv, rows, h, 3 * h);
+  }
+  e = cudaGetLastError();
+  if (e != cudaSuccess) MOBIUS_FAIL(MOBIUS_ECUDA, "flash_bwd launch: %s", cudaGetErrorString(e));
+  return MOBIUS_OK;
+}
+
+}  // namespace mobius

@@ -10,12 +10,29 @@
 #include "common.h"
 #include "elem.h"
 #include "gemm.h"
+#include "flash.h"
 #include "ops.h"
 
 using namespace mobius;
 typedef __nv_bfloat16 bf16;
 
 namespace {
+// grow-only device workspace reused across kernel-test calls (no cudaMalloc
+// inside timed loops)
+uint8_t* ws_get(int64_t bytes) {
+  static uint8_t* buf = nullptr;
+  static int64_t cap = 0;
+  if (bytes > cap) {
+    if (buf) cudaFree(buf);
+    buf = nullptr;
+    if (cudaMalloc(&buf, bytes) != cudaSuccess) {
+      cap = 0;
+      return nullptr;
+    }
+    cap = bytes;
+  }
+  return buf;
+}
 int sync_rc(int rc) {
   if (rc) return rc;
   cudaError_t e = cudaDeviceSynchronize();
@@ -106,9 +123,10 @@ int kt_block(int hidden, int nh, int s, int mbs, const void* w, const void* x, v
              float* grads) {
   Shape sh{hidden, nh, s, mbs, 0};
   const int e = sizeof(T);
-  int64_t ab = block_acts_bytes(sh, e), sb = scratch_bytes(sh, e, false);
-  uint8_t* buf = nullptr;
-  if (cudaMalloc(&buf, ab + sb) != cudaSuccess) MOBIUS_FAIL(MOBIUS_ENOMEM, "kt_block alloc");
+  const bool fl = use_flash<T>(sh);
+  int64_t ab = block_acts_bytes(sh, e, fl), sb = scratch_bytes(sh, e, false, fl);
+  uint8_t* buf = ws_get(ab + sb);
+  if (!buf) MOBIUS_FAIL(MOBIUS_ENOMEM, "kt_block alloc");
   BlockActs<T> acts;
   Scratch<T> sc;
   carve_block_acts<T>(sh, buf, acts);
@@ -116,9 +134,7 @@ int kt_block(int hidden, int nh, int s, int mbs, const void* w, const void* x, v
   acts.x = (const T*)x;
   int rc = block_fwd<T>(sh, (const T*)w, acts, (T*)y, sc, 0);
   if (!rc && dy) rc = block_bwd<T>(sh, (const T*)w, acts, (const T*)dy, (T*)dx, grads, sc, 0);
-  rc = sync_rc(rc);
-  cudaFree(buf);
-  return rc;
+  return sync_rc(rc);
 }
 }  // namespace
 
@@ -126,4 +142,29 @@ extern "C" int mobius_kt_block(int dtype, int hidden, int n_heads, int seq_len, 
                                void* y, const void* dy, void* dx, float* grads) {
   if (dtype == MOBIUS_BF16) return kt_block<bf16>(hidden, n_heads, seq_len, mbs, w, x, y, dy, dx, grads);
   return kt_block<float>(hidden, n_heads, seq_len, mbs, w, x, y, dy, dx, grads);
+}
+
+namespace {
+template <typename T>
+int kt_attn(int mbs, int s, int nh, int dh, const void* qkv, void* o, const void* dout, void* dqkv) {
+  Shape sh{nh * dh, nh, s, mbs, 0};
+  const int e = sizeof(T);
+  const bool fl = use_flash<T>(sh);
+  int64_t ab = block_acts_bytes(sh, e, fl), sb = scratch_bytes(sh, e, false, fl);
+  uint8_t* buf = ws_get(ab + sb);
+  if (!buf) MOBIUS_FAIL(MOBIUS_ENOMEM, "kt_attn alloc");
+  BlockActs<T> acts;
+  Scratch<T> sc;
+  carve_block_acts<T>(sh, buf, acts);
+  carve_scratch<T>(sh, buf + ab, false, sc);
+  int rc = attention_fwd<T>(sh, (const T*)qkv, (T*)o, acts.P, acts.lse, sc, 0);
+  if (!rc && dout) rc = attention_bwd<T>(sh, (const T*)qkv, (const T*)o, acts.P, acts.lse, (const T*)dout, (T*)dqkv, sc, 0);
+  return sync_rc(rc);
+}
+}  // namespace
+
+extern "C" int mobius_kt_attention(int dtype, int mbs, int s, int n_heads, int head_dim, const void* qkv, void* o,
+                                   const void* dout, void* dqkv) {
+  if (dtype == MOBIUS_BF16) return kt_attn<bf16>(mbs, s, n_heads, head_dim, qkv, o, dout, dqkv);
+  return kt_attn<float>(mbs, s, n_heads, head_dim, qkv, o, dout, dqkv);
 }

@@ -6,6 +6,7 @@
 
 #include "common.h"
 #include "elem.h"
+#include "flash.h"
 #include "gemm.h"
 #include "ops.h"
 
@@ -109,14 +110,24 @@ struct ElemScope {
 
 }  // namespace
 
-int64_t block_acts_bytes(const Shape& sh, int e) {
+template <>
+bool use_flash<float>(const Shape&) {
+  return false;
+}
+template <>
+bool use_flash<__nv_bfloat16>(const Shape& sh) {
+  return flash_supported(sh.dh(), sh.s) != 0;
+}
+
+int64_t block_acts_bytes(const Shape& sh, int e, bool flash) {
   Carver c{nullptr};
   const int64_t T = sh.T(), h = sh.h, B = (int64_t)sh.mbs * sh.nh, s = sh.s;
   c.take<char>(T * h * e);      // a
   c.take<char>(T * 4);          // mu1
   c.take<char>(T * 4);          // rs1
   c.take<char>(T * 3 * h * e);  // qkv
-  c.take<char>(B * s * s * e);  // P
+  c.take<char>(flash ? 0 : B * s * s * e);  // P
+  c.take<char>(flash ? B * s * 4 : 0);      // lse
   c.take<char>(T * h * e);      // o
   c.take<char>(T * h * e);      // x1
   c.take<char>(T * h * e);      // a2
@@ -134,8 +145,10 @@ void carve_block_acts(const Shape& sh, uint8_t* base, BlockActs<T>& a) {
   a.a = c.take<T>(Tn * h * e);
   a.mu1 = c.take<float>(Tn * 4);
   a.rs1 = c.take<float>(Tn * 4);
+  const bool fl = use_flash<T>(sh);
   a.qkv = c.take<T>(Tn * 3 * h * e);
-  a.P = c.take<T>(B * s * s * e);
+  a.P = c.take<T>(fl ? 0 : B * s * s * e);
+  a.lse = c.take<float>(fl ? B * s * 4 : 0);
   a.o = c.take<T>(Tn * h * e);
   a.x1 = c.take<T>(Tn * h * e);
   a.a2 = c.take<T>(Tn * h * e);
@@ -145,11 +158,13 @@ void carve_block_acts(const Shape& sh, uint8_t* base, BlockActs<T>& a) {
   a.g = c.take<T>(Tn * 4 * h * e);
 }
 
-int64_t scratch_bytes(const Shape& sh, int e, bool with_head) {
+int64_t scratch_bytes(const Shape& sh, int e, bool with_head, bool flash) {
   const int64_t T = sh.T(), h = sh.h, B = (int64_t)sh.mbs * sh.nh, s = sh.s;
   Carver c{nullptr};
-  c.take<char>(B * s * s * 4);
-  c.take<char>(B * s * s * e);
+  c.take<char>(flash ? 0 : B * s * s * 4);
+  c.take<char>(flash ? 0 : B * s * s * e);
+  c.take<char>(flash ? T * h * 4 : 0);
+  c.take<char>(flash ? B * s * 4 : 0);
   c.take<char>(T * 4 * h * e);
   c.take<char>(T * h * e);
   c.take<char>(T * h * e);
@@ -166,8 +181,11 @@ template <typename T>
 void carve_scratch(const Shape& sh, uint8_t* base, bool with_head, Scratch<T>& sc) {
   const int64_t Tn = sh.T(), h = sh.h, B = (int64_t)sh.mbs * sh.nh, s = sh.s, e = sizeof(T);
   Carver c{base};
-  sc.S = c.take<float>(B * s * s * 4);
-  sc.dS = c.take<T>(B * s * s * e);
+  const bool fl = use_flash<T>(sh);
+  sc.S = c.take<float>(fl ? 0 : B * s * s * 4);
+  sc.dS = c.take<T>(fl ? 0 : B * s * s * e);
+  sc.dq = c.take<float>(fl ? Tn * h * 4 : 0);
+  sc.dsum = c.take<float>(fl ? B * s * 4 : 0);
   sc.big1 = c.take<T>(Tn * 4 * h * e);
   sc.t1 = c.take<T>(Tn * h * e);
   sc.t2 = c.take<T>(Tn * h * e);
@@ -177,6 +195,104 @@ void carve_scratch(const Shape& sh, uint8_t* base, bool with_head, Scratch<T>& s
   sc.loss_rows = c.take<float>(Tn * 4);
   sc.mu = c.take<float>(Tn * 4);
   sc.rs = c.take<float>(Tn * 4);
+}
+
+// ------------------------------------------------------------ attention
+template <typename T>
+int attention_fwd(const Shape& sh, const T* qkv, T* o, T* P, float* lse, Scratch<T>& sc, cudaStream_t st) {
+  const int h = sh.h, nh = sh.nh, s = sh.s, dh = sh.dh(), mbs = sh.mbs;
+  const int64_t Sbs2 = (int64_t)s * s, Sbs1 = nh * Sbs2;
+  if (use_flash<T>(sh)) {
+    KernelTimer* t = g_timer;
+    if (t) t->begin(KCLS_ATTN, st);
+    int rc = flash_attn_fwd(reinterpret_cast<const __nv_bfloat16*>(qkv), reinterpret_cast<__nv_bfloat16*>(o), lse,
+                            mbs, s, nh, dh, st);
+    if (t) t->end(KCLS_ATTN, st, 2LL * mbs * nh * s * s * dh);
+    ++g_kernel_launches;
+    return rc;
+  }
+  {  // S = q k^T (fp32), causal tiles only
+    GemmDesc d;
+    d.M = s; d.N = s; d.K = dh; d.nb1 = mbs; d.nb2 = nh;
+    d.A = mv(qkv, 3 * h, (int64_t)s * 3 * h, dh);
+    d.B = mv(qkv + h, 3 * h, (int64_t)s * 3 * h, dh);
+    d.C = mv(sc.S, s, Sbs1, Sbs2); d.c_f32 = true;
+    d.causal = CAUSAL_SKIP_UPPER;
+    RC(run_gemm<T>(d, st, KCLS_ATTN));
+  }
+  {
+    ElemScope es(st, 1);
+    RC(softmax_causal_fwd<T>(sc.S, P, mbs * nh, s, 1.0f / sqrtf((float)dh), st));
+  }
+  {  // o = P v
+    GemmDesc d;
+    d.M = s; d.N = dh; d.K = s; d.nb1 = mbs; d.nb2 = nh;
+    d.A = mv(P, s, Sbs1, Sbs2);
+    d.B = mv(qkv + 2 * h, 3 * h, (int64_t)s * 3 * h, dh); d.b_mn = true;
+    d.C = mv(o, h, (int64_t)s * h, dh);
+    d.causal = CAUSAL_K_LT_MEND;
+    RC(run_gemm<T>(d, st, KCLS_ATTN));
+  }
+  return MOBIUS_OK;
+}
+
+template <typename T>
+int attention_bwd(const Shape& sh, const T* qkv, const T* o, const T* P, const float* lse, const T* dO, T* dqkv,
+                  Scratch<T>& sc, cudaStream_t st) {
+  const int h = sh.h, nh = sh.nh, s = sh.s, dh = sh.dh(), mbs = sh.mbs;
+  const int64_t Sbs2 = (int64_t)s * s, Sbs1 = nh * Sbs2;
+  const float scale = 1.0f / sqrtf((float)dh);
+  if (use_flash<T>(sh)) {
+    KernelTimer* t = g_timer;
+    if (t) t->begin(KCLS_ATTN, st);
+    int rc = flash_attn_bwd(reinterpret_cast<const __nv_bfloat16*>(qkv), reinterpret_cast<const __nv_bfloat16*>(o),
+                            reinterpret_cast<const __nv_bfloat16*>(dO), lse, sc.dsum, sc.dq,
+                            reinterpret_cast<__nv_bfloat16*>(dqkv), mbs, s, nh, dh, st);
+    if (t) t->end(KCLS_ATTN, st, 4LL * mbs * nh * s * s * dh);
+    g_kernel_launches += 3;
+    return rc;
+  }
+  {  // dP = do v^T (fp32)
+    GemmDesc d;
+    d.M = s; d.N = s; d.K = dh; d.nb1 = mbs; d.nb2 = nh;
+    d.A = mv(dO, h, (int64_t)s * h, dh);
+    d.B = mv(qkv + 2 * h, 3 * h, (int64_t)s * 3 * h, dh);
+    d.C = mv(sc.S, s, Sbs1, Sbs2); d.c_f32 = true;
+    d.causal = CAUSAL_SKIP_UPPER;
+    RC(run_gemm<T>(d, st, KCLS_ATTN));
+  }
+  {
+    ElemScope es(st, 1);
+    RC(softmax_causal_bwd<T>(P, sc.S, sc.dS, mbs * nh, s, scale, st));
+  }
+  {  // dV = P^T do
+    GemmDesc d;
+    d.M = s; d.N = dh; d.K = s; d.nb1 = mbs; d.nb2 = nh;
+    d.A = mv(P, s, Sbs1, Sbs2); d.a_mn = true;
+    d.B = mv(dO, h, (int64_t)s * h, dh); d.b_mn = true;
+    d.C = mv(dqkv + 2 * h, 3 * h, (int64_t)s * 3 * h, dh);
+    d.causal = CAUSAL_K_GE_M0;
+    RC(run_gemm<T>(d, st, KCLS_ATTN));
+  }
+  {  // dQ = dS K
+    GemmDesc d;
+    d.M = s; d.N = dh; d.K = s; d.nb1 = mbs; d.nb2 = nh;
+    d.A = mv(sc.dS, s, Sbs1, Sbs2);
+    d.B = mv(qkv + h, 3 * h, (int64_t)s * 3 * h, dh); d.b_mn = true;
+    d.C = mv(dqkv, 3 * h, (int64_t)s * 3 * h, dh);
+    d.causal = CAUSAL_K_LT_MEND;
+    RC(run_gemm<T>(d, st, KCLS_ATTN));
+  }
+  {  // dK = dS^T Q
+    GemmDesc d;
+    d.M = s; d.N = dh; d.K = s; d.nb1 = mbs; d.nb2 = nh;
+    d.A = mv(sc.dS, s, Sbs1, Sbs2); d.a_mn = true;
+    d.B = mv(qkv, 3 * h, (int64_t)s * 3 * h, dh); d.b_mn = true;
+    d.C = mv(dqkv + h, 3 * h, (int64_t)s * 3 * h, dh);
+    d.causal = CAUSAL_K_GE_M0;
+    RC(run_gemm<T>(d, st, KCLS_ATTN));
+  }
+  return MOBIUS_OK;
 }
 
 // ------------------------------------------------------------------ block
@@ -198,28 +314,7 @@ int block_fwd(const Shape& sh, const T* w, BlockActs<T>& A, T* y, Scratch<T>& sc
     d.epi = EPI_BIAS; d.bias = w + L.b_qkv;
     RC(run_gemm<T>(d, st, KCLS_GEMM));
   }
-  {  // S = q k^T (fp32), causal tiles only
-    GemmDesc d;
-    d.M = s; d.N = s; d.K = dh; d.nb1 = mbs; d.nb2 = nh;
-    d.A = mv(A.qkv, 3 * h, (int64_t)s * 3 * h, dh);
-    d.B = mv(A.qkv + h, 3 * h, (int64_t)s * 3 * h, dh);
-    d.C = mv(sc.S, s, Sbs1, Sbs2); d.c_f32 = true;
-    d.causal = CAUSAL_SKIP_UPPER;
-    RC(run_gemm<T>(d, st, KCLS_ATTN));
-  }
-  {
-    ElemScope es(st, 1);
-    RC(softmax_causal_fwd<T>(sc.S, A.P, mbs * nh, s, 1.0f / sqrtf((float)dh), st));
-  }
-  {  // o = P v
-    GemmDesc d;
-    d.M = s; d.N = dh; d.K = s; d.nb1 = mbs; d.nb2 = nh;
-    d.A = mv(A.P, s, Sbs1, Sbs2);
-    d.B = mv(A.qkv + 2 * h, 3 * h, (int64_t)s * 3 * h, dh); d.b_mn = true;
-    d.C = mv(A.o, h, (int64_t)s * h, dh);
-    d.causal = CAUSAL_K_LT_MEND;
-    RC(run_gemm<T>(d, st, KCLS_ATTN));
-  }
+  RC(attention_fwd<T>(sh, A.qkv, A.o, A.P, A.lse, sc, st));
   {  // x1 = x + o Wo + bo
     GemmDesc d;
     d.M = Tn; d.N = h; d.K = h;
@@ -329,47 +424,8 @@ int block_bwd(const Shape& sh, const T* w, const BlockActs<T>& A, const T* dy, T
     d.C = mv(dO, h);
     RC(run_gemm<T>(d, st, KCLS_GEMM));
   }
-  {  // dP = do v^T (fp32)
-    GemmDesc d;
-    d.M = s; d.N = s; d.K = dh; d.nb1 = mbs; d.nb2 = nh;
-    d.A = mv(dO, h, (int64_t)s * h, dh);
-    d.B = mv(A.qkv + 2 * h, 3 * h, (int64_t)s * 3 * h, dh);
-    d.C = mv(sc.S, s, Sbs1, Sbs2); d.c_f32 = true;
-    d.causal = CAUSAL_SKIP_UPPER;
-    RC(run_gemm<T>(d, st, KCLS_ATTN));
-  }
-  {
-    ElemScope es(st, 1);
-    RC(softmax_causal_bwd<T>(A.P, sc.S, sc.dS, mbs * nh, s, scale, st));
-  }
   T* dqkv = sc.qkv_g;
-  {  // dV = P^T do
-    GemmDesc d;
-    d.M = s; d.N = dh; d.K = s; d.nb1 = mbs; d.nb2 = nh;
-    d.A = mv(A.P, s, Sbs1, Sbs2); d.a_mn = true;
-    d.B = mv(dO, h, (int64_t)s * h, dh); d.b_mn = true;
-    d.C = mv(dqkv + 2 * h, 3 * h, (int64_t)s * 3 * h, dh);
-    d.causal = CAUSAL_K_GE_M0;
-    RC(run_gemm<T>(d, st, KCLS_ATTN));
-  }
-  {  // dQ = dS K
-    GemmDesc d;
-    d.M = s; d.N = dh; d.K = s; d.nb1 = mbs; d.nb2 = nh;
-    d.A = mv(sc.dS, s, Sbs1, Sbs2);
-    d.B = mv(A.qkv + h, 3 * h, (int64_t)s * 3 * h, dh); d.b_mn = true;
-    d.C = mv(dqkv, 3 * h, (int64_t)s * 3 * h, dh);
-    d.causal = CAUSAL_K_LT_MEND;
-    RC(run_gemm<T>(d, st, KCLS_ATTN));
-  }
-  {  // dK = dS^T Q
-    GemmDesc d;
-    d.M = s; d.N = dh; d.K = s; d.nb1 = mbs; d.nb2 = nh;
-    d.A = mv(sc.dS, s, Sbs1, Sbs2); d.a_mn = true;
-    d.B = mv(A.qkv, 3 * h, (int64_t)s * 3 * h, dh); d.b_mn = true;
-    d.C = mv(dqkv + h, 3 * h, (int64_t)s * 3 * h, dh);
-    d.causal = CAUSAL_K_GE_M0;
-    RC(run_gemm<T>(d, st, KCLS_ATTN));
-  }
+  RC(attention_bwd<T>(sh, A.qkv, A.o, A.P, A.lse, dO, dqkv, sc, st));
   {  // dWqkv += a^T dqkv
     GemmDesc d;
     d.M = h; d.N = 3 * h; d.K = Tn;
@@ -468,7 +524,10 @@ int head_layer_fwd_bwd(const Shape& sh, const T* w, const T* x, const int32_t* t
   template int embed_layer_fwd<T>(const Shape&, const T*, const int32_t*, T*, cudaStream_t);                      \
   template int embed_layer_bwd<T>(const Shape&, const T*, const int32_t*, const T*, float*, cudaStream_t);        \
   template int head_layer_fwd_bwd<T>(const Shape&, const T*, const T*, const int32_t*, float, T*, float*, double*, \
-                                     Scratch<T>&, cudaStream_t);
+                                     Scratch<T>&, cudaStream_t);                                                  \
+  template int attention_fwd<T>(const Shape&, const T*, T*, T*, float*, Scratch<T>&, cudaStream_t);                \
+  template int attention_bwd<T>(const Shape&, const T*, const T*, const T*, const float*, const T*, T*, Scratch<T>&, \
+                                cudaStream_t);
 INST(float)
 INST(__nv_bfloat16)
 

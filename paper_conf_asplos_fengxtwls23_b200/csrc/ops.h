@@ -39,7 +39,8 @@ struct BlockActs {
   T* a;            // LN1(x)
   float *mu1, *rs1;
   T* qkv;          // [T, 3h]
-  T* P;            // [mbs*nh, s, s] causal softmax probabilities
+  T* P;            // [mbs*nh, s, s] causal softmax probabilities (materialised path only)
+  float* lse;      // [mbs*nh*s] log2-domain row logsumexp (flash path only)
   T* o;            // attention output [T, h]
   T* x1;           // x + o Wo + bo
   T* a2;           // LN2(x1)
@@ -50,8 +51,10 @@ struct BlockActs {
 
 template <typename T>
 struct Scratch {
-  float* S;        // [mbs*nh, s, s] fp32 scores / dP
-  T* dS;           // [mbs*nh, s, s]
+  float* S;        // [mbs*nh, s, s] fp32 scores / dP (materialised path only)
+  T* dS;           // [mbs*nh, s, s] (materialised path only)
+  float* dq;       // [T, h] fp32 dQ accumulator (flash path only)
+  float* dsum;     // [mbs*nh*s] rowsum(dO*O) (flash path only)
   T* big1;         // [T, 4h]
   T* t1;           // [T, h]
   T* t2;           // [T, h]
@@ -62,9 +65,19 @@ struct Scratch {
   float *mu, *rs;  // [T] (head LN)
 };
 
+// true when the fused tcgen05 attention is used (bf16, dh in {64,128}, s % 128 == 0)
+template <typename T>
+bool use_flash(const Shape& sh);
+// attention core: qkv -> o (fwd) and dO -> dqkv (bwd)
+template <typename T>
+int attention_fwd(const Shape& sh, const T* qkv, T* o, T* P, float* lse, Scratch<T>& sc, cudaStream_t st);
+template <typename T>
+int attention_bwd(const Shape& sh, const T* qkv, const T* o, const T* P, const float* lse, const T* dO, T* dqkv,
+                  Scratch<T>& sc, cudaStream_t st);
+
 // bytes of one BlockActs set / of the Scratch (for arena planning)
-int64_t block_acts_bytes(const Shape& sh, int elem);
-int64_t scratch_bytes(const Shape& sh, int elem, bool with_head);
+int64_t block_acts_bytes(const Shape& sh, int elem, bool flash);
+int64_t scratch_bytes(const Shape& sh, int elem, bool with_head, bool flash);
 template <typename T>
 void carve_block_acts(const Shape& sh, uint8_t* base, BlockActs<T>& a);
 template <typename T>

@@ -11,6 +11,7 @@
 
 #include "common.h"
 #include "elem.h"
+#include "flash.h"
 #include "ops.h"
 
 using namespace mobius;
@@ -25,7 +26,8 @@ int profile_impl(const mobius_model_cfg& c, mobius_layer_profile* out, int Lp) {
   EmbedLayout EL(h, c.vocab, c.seq_len);
   HeadLayout HL(h, c.vocab);
   int64_t wmax = std::max(BL.total, std::max(EL.total, HL.total));
-  int64_t ab = block_acts_bytes(sh, (int)e), sb = scratch_bytes(sh, (int)e, true);
+  const bool fl = use_flash<T>(sh);
+  int64_t ab = block_acts_bytes(sh, (int)e, fl), sb = scratch_bytes(sh, (int)e, true, fl);
   int64_t xb = (Tn * h * e + 255) & ~int64_t(255);
   int64_t tokb = ((int64_t)sh.mbs * (sh.s + 1) * 4 + 255) & ~int64_t(255);
   int64_t total = wmax * e + wmax * 4 + ab + sb + 4 * xb + tokb + 256 + 4096;

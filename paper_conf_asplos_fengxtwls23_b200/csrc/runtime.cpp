@@ -38,6 +38,7 @@
 #include "common.h"
 #include "elem.h"
 #include "host.h"
+#include "flash.h"
 #include "ops.h"
 
 namespace mobius {
@@ -795,7 +796,8 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
   const int M = plan->n_microbatches > 0 ? plan->n_microbatches : dist->world;
   ctx->max_M = M;
   ctx->slot_bytes = al256((int64_t)sh.T() * sh.h * esz);
-  ctx->acts_bytes = al256(block_acts_bytes(sh, esz));
+  const bool fl = esz == 2 && flash_supported(sh.dh(), sh.s);
+  ctx->acts_bytes = al256(block_acts_bytes(sh, esz, fl));
   int64_t off = al256(G);
   auto take = [&](int64_t bytes) {
     int64_t o = off;
@@ -810,7 +812,7 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
   ctx->off_bflag = take((int64_t)n * M * 4);
   int64_t o_acts = take(ctx->acts_bytes * std::max(1, ctx->max_blocks));
   int64_t o_xs = take(ctx->slot_bytes * (ctx->max_blocks + 3));
-  int64_t o_scr = take(scratch_bytes(sh, esz, true));
+  int64_t o_scr = take(scratch_bytes(sh, esz, true, fl));
   int64_t o_tok = take((int64_t)M * sh.mbs * (sh.s + 1) * 4);
   int64_t o_loss = take(8);
   ctx->arena_bytes = off;

@@ -313,3 +313,28 @@ def test_block_fwd_bwd(dtype, tol, wscale, h, nh, s, mbs):
         pos += n
     print(errs)
     assert max(errs.values()) < tol, errs
+
+
+@pytest.mark.parametrize("dtype", [BF16, F32])
+@pytest.mark.parametrize("mbs,s,nh,dh", [(2, 128, 2, 64), (1, 384, 3, 64), (2, 256, 2, 128), (1, 1024, 2, 64)])
+def test_attention_core(dtype, mbs, s, nh, dh):
+    """Causal attention fwd+bwd (fused tcgen05 flash kernels on the bf16 path)
+    vs the oracle's attention_fwd / attention_bwd in fp64."""
+    h = nh * dh
+    T = mbs * s
+    qkv = rnd(dtype, randn(T, 3 * h, scale=1.0))
+    dout = rnd(dtype, randn(T, h))
+    o_ref, cache = om.attention_fwd(qkv.astype(np.float64), mbs, s, nh)
+    dqkv_ref = om.attention_bwd(dout.astype(np.float64), cache, mbs, s, nh)
+    tq = to_dev(qkv, dtype)
+    to = torch.zeros((T, h), device=DEV, dtype=tq.dtype)
+    tdo = to_dev(dout, dtype)
+    tdq = torch.full((T, 3 * h), float("nan"), device=DEV, dtype=tq.dtype)
+    kt.attention(dtype, mbs, s, nh, dh, tq, to, tdo, tdq)
+    torch.cuda.synchronize()
+    tol = 2e-2 if dtype == BF16 else 1e-5
+    d = from_dev(tdq)
+    errs = {"o": rel(from_dev(to), o_ref)}
+    for part, name in ((0, "dq"), (1, "dk"), (2, "dv")):
+        errs[name] = rel(d[:, part * h:(part + 1) * h], dqkv_ref[:, part * h:(part + 1) * h])
+    assert max(errs.values()) < tol, errs
