@@ -377,7 +377,8 @@ struct BwdCfg {
   static constexpr int T_BYTES = 128 * DH * 2;       // one K / V / Q / dO tile
   static constexpr int QS = DH == 64 ? 2 : 1;        // Q/dO pipeline depth
   static constexpr int PT_BYTES = 128 * 128 * 2;     // P^T or dS^T tile
-  static constexpr int SMEM = 1024 + 2 * T_BYTES + QS * 2 * T_BYTES + 2 * PT_BYTES + 2 * 2 * 128 * 4 + 256;
+  static constexpr bool DQ_OWN = DH == 64;           // dQ has its own TMEM columns (else aliases S^T)
+  static constexpr int SMEM = 1024 + 2 * T_BYTES + QS * 2 * T_BYTES + 2 * PT_BYTES + QS * 1024 + 256;
 };
 
 struct BwdParams {
@@ -396,9 +397,21 @@ __device__ __forceinline__ void red_add_v4(float* addr, float a, float b, float 
                : "memory");
 }
 
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                   ptx::smem_u32(dst)),
+               "l"(reinterpret_cast<uint64_t>(src)), "r"(bytes), "r"(ptx::smem_u32(bar))
+               : "memory");
+}
+
+// One CTA per (batch, head, 128-key tile); loop over query tiles i >= kt.
+// MMA order per query tile: [S^T, dP^T](i) ... wait P^T/dS^T(i) ... dV, dK,
+// dQ(i), then [S^T, dP^T](i+1) right away (the softmax-gradient warps are
+// done with S^T(i)), so the next scores overlap the dQ read-out.
 template <int DH>
 __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_constant__ CUtensorMap tm,
-                                                          const __grid_constant__ CUtensorMap tdo, const BwdParams p) {
+                                                              const __grid_constant__ CUtensorMap tdo,
+                                                              const __grid_constant__ CUtensorMap tdq, const BwdParams p) {
   using C = BwdCfg<DH>;
   constexpr int QS = C::QS;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -409,27 +422,28 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
   uint8_t* sdO = sQ + QS * C::T_BYTES;       // [QS]
   uint8_t* sPT = sdO + QS * C::T_BYTES;
   uint8_t* sdST = sPT + C::PT_BYTES;
-  float* sLse = reinterpret_cast<float*>(sdST + C::PT_BYTES);  // [2][128]
-  float* sD = sLse + 2 * 128;                                  // [2][128]
-  uint64_t* bars = reinterpret_cast<uint64_t*>(sD + 2 * 128);
+  float* sLD = reinterpret_cast<float*>(sdST + C::PT_BYTES);  // [QS][lse 128 | D 128]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sLD + QS * 256);
   uint64_t* kv_full = bars;          // 1
-  uint64_t* q_full = bars + 1;       // [QS] (Q, dO, lse, D)
-  uint64_t* q_empty = bars + 3;      // [QS]
+  uint64_t* q_full = bars + 1;       // [2] (Q, dO, lse, D)
+  uint64_t* q_empty = bars + 3;      // [2]
   uint64_t* s_full = bars + 5;       // S^T and dP^T ready
-  uint64_t* p_full = bars + 6;       // P^T / dS^T in smem (count 4)
-  uint64_t* mm_done = bars + 7;      // dV/dK/dQ MMAs of this tile done (P^T/dS^T smem free, dQ ready)
-  uint64_t* dq_empty = bars + 8;     // dQ read out (count 4) -> TMEM S/dQ region free
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 9);
+  uint64_t* p_full = bars + 6;       // P^T / dS^T in smem (count 8)
+  uint64_t* mm_done = bars + 7;      // dV/dK/dQ of this tile done (P^T/dS^T smem free, dQ ready)
+  uint64_t* dq_empty = bars + 8;     // dQ read out (count 8)
+  uint64_t* st_empty = bars + 9;     // S^T / dP^T loaded into registers (count 8)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 10);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const int n_t = p.s / 128;
-  const int kt = (int)blockIdx.x;  // key tile (tile kt has n_t - kt query tiles; light-first is fine)
+  const int kt = (int)blockIdx.x;  // small kt = most query tiles: launched first
   const int hd = blockIdx.y, b = blockIdx.z;
   const int i0 = kt, nq = n_t - kt;
 
   if (threadIdx.x == 0) {
     ptx::tma_prefetch_desc(&tm);
     ptx::tma_prefetch_desc(&tdo);
+    ptx::tma_prefetch_desc(&tdq);
     ptx::mbar_init(kv_full, 1);
     for (int i = 0; i < 2; ++i) {
       ptx::mbar_init(&q_full[i], 1);
@@ -439,6 +453,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
     ptx::mbar_init(p_full, 8);
     ptx::mbar_init(mm_done, 1);
     ptx::mbar_init(dq_empty, 8);
+    ptx::mbar_init(st_empty, 8);
     ptx::fence_mbar_init();
   }
   if (warp == 1) ptx::tmem_alloc<512>(tmem_slot);
@@ -446,8 +461,10 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_slot;
-  const uint32_t T_S = tmem, T_DP = tmem + 128, T_DV = tmem + 256, T_DK = tmem + 256 + DH;
-  (void)T_DK;
+  // TMEM: S^T 0..127, dP^T 128..255, dV 256.., dK 256+DH.., dQ 384.. (dh 64) or aliasing S^T (dh 128)
+  const uint32_t T_S = tmem, T_DP = tmem + 128, T_DV = tmem + 256;
+  const uint32_t T_DQ = C::DQ_OWN ? tmem + 384 : tmem;
+  const int64_t ld_base = ((int64_t)b * p.nh + hd) * p.s;
 
   if (warp == 0) {
     if (lane == 0) {
@@ -462,31 +479,28 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
         const int ph = (it / QS) & 1;
         const int qi = i0 + it;
         ptx::mbar_wait(&q_empty[st], ph ^ 1);
-        ptx::mbar_arrive_expect_tx(&q_full[st], 2 * C::T_BYTES);
+        ptx::mbar_arrive_expect_tx(&q_full[st], 2 * C::T_BYTES + 1024);
 #pragma unroll
         for (int c = 0; c < DH / 64; ++c) {
           ptx::tma_load_4d(sQ + st * C::T_BYTES + c * 16384, &tm, &q_full[st], 64 * c, qi * 128, hd, b);
           ptx::tma_load_4d(sdO + st * C::T_BYTES + c * 16384, &tdo, &q_full[st], 64 * c, qi * 128, hd, b);
         }
+        bulk_g2s(sLD + st * 256, p.lse + ld_base + qi * 128, 512, &q_full[st]);
+        bulk_g2s(sLD + st * 256 + 128, p.Dsum + ld_base + qi * 128, 512, &q_full[st]);
       }
     }
   } else if (warp == 1) {
     if (lane == 0) {
-      // S^T (M=kv, N=q, K=d): A = K tile (K-major), B = Q tile (K-major)
-      constexpr uint32_t ID_ST = ptx::idesc_bf16(128, 128, 0, 0);
-      // dV (M=kv, N=d, K=q): A = P^T (K-major), B = dO (MN-major)
-      constexpr uint32_t ID_DV = ptx::idesc_bf16(128, DH, 0, 1);
-      // dQ (M=q, N=d, K=kv): A = dS (MN-major view of dS^T), B = K (MN-major)
-      constexpr uint32_t ID_DQ = ptx::idesc_bf16(128, DH, 1, 1);
+      constexpr uint32_t ID_ST = ptx::idesc_bf16(128, 128, 0, 0);  // S^T, dP^T
+      constexpr uint32_t ID_DV = ptx::idesc_bf16(128, DH, 0, 1);   // dV, dK
+      constexpr uint32_t ID_DQ = ptx::idesc_bf16(128, DH, 1, 1);   // dQ
       const uint32_t ak = ptx::smem_u32(sK), av = ptx::smem_u32(sV);
       const uint32_t apt = ptx::smem_u32(sPT), adst = ptx::smem_u32(sdST);
-      ptx::mbar_wait(kv_full, 0);
-      for (int it = 0; it < nq; ++it) {
-        const int st = it % QS;
-        const int ph = (it / QS) & 1;
+      auto issue_st = [&](int it) {
+        const int st = it % QS, ph = (it / QS) & 1;
         const uint32_t aq = ptx::smem_u32(sQ + st * C::T_BYTES), ado = ptx::smem_u32(sdO + st * C::T_BYTES);
         ptx::mbar_wait(&q_full[st], ph);
-        ptx::mbar_wait(dq_empty, (it & 1) ^ 1);  // S/dQ TMEM region free (dQ_{it-1} read)
+        if (!C::DQ_OWN && it >= 1) ptx::mbar_wait(dq_empty, (it - 1) & 1);  // S^T region holds dQ(it-1)
         ptx::tc_fence_after();
 #pragma unroll
         for (int t = 0; t < DH / 16; ++t) {
@@ -500,26 +514,34 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
                         t > 0);
         }
         ptx::mma_commit(s_full);
-        // wait for P^T / dS^T in smem
+      };
+      ptx::mbar_wait(kv_full, 0);
+      issue_st(0);
+      for (int it = 0; it < nq; ++it) {
+        const int st = it % QS;
+        const uint32_t aq = ptx::smem_u32(sQ + st * C::T_BYTES), ado = ptx::smem_u32(sdO + st * C::T_BYTES);
+        if (C::DQ_OWN && it + 1 < nq) {  // scores of the next query tile overlap this tile's softmax-gradient
+          ptx::mbar_wait(st_empty, it & 1);
+          issue_st(it + 1);
+        }
         ptx::mbar_wait(p_full, it & 1);
         ptx::tc_fence_after();
 #pragma unroll
         for (int t = 0; t < 128 / 16; ++t) {  // K = 128 queries
           const uint32_t offa = (t >> 2) * 16384 + (t & 3) * 32;
-          // dV += P^T dO
           ptx::mma_bf16(T_DV, ptx::sdesc_sw128(apt + offa, 16, 1024), ptx::sdesc_sw128(ado + t * 2048, 16384, 1024),
-                        ID_DV, (it > 0 || t > 0) ? 1u : 0u);
-          // dK += dS^T Q
+                        ID_DV, (it > 0 || t > 0) ? 1u : 0u);  // dV += P^T dO
           ptx::mma_bf16(T_DV + DH, ptx::sdesc_sw128(adst + offa, 16, 1024),
-                        ptx::sdesc_sw128(aq + t * 2048, 16384, 1024), ID_DV, (it > 0 || t > 0) ? 1u : 0u);
+                        ptx::sdesc_sw128(aq + t * 2048, 16384, 1024), ID_DV, (it > 0 || t > 0) ? 1u : 0u);  // dK += dS^T Q
         }
+        if (C::DQ_OWN && it >= 1) ptx::mbar_wait(dq_empty, (it - 1) & 1);  // dQ(it-1) read out
 #pragma unroll
-        for (int t = 0; t < 128 / 16; ++t) {  // K = 128 keys: dQ = dS K
-          ptx::mma_bf16(T_S, ptx::sdesc_sw128(adst + t * 2048, 16384, 1024),
+        for (int t = 0; t < 128 / 16; ++t)  // K = 128 keys: dQ = dS K
+          ptx::mma_bf16(T_DQ, ptx::sdesc_sw128(adst + t * 2048, 16384, 1024),
                         ptx::sdesc_sw128(ak + t * 2048, 16384, 1024), ID_DQ, t > 0);
-        }
         ptx::mma_commit(mm_done);
         ptx::mma_commit(&q_empty[st]);
+        if (!C::DQ_OWN && it + 1 < nq) issue_st(it + 1);
       }
     }
   } else {
@@ -528,48 +550,45 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
     // query columns [64 hf, 64 hf + 64)
     const int q4 = warp & 3;
     const int hf = (warp - 2) >> 2;
-    const int r = q4 * 32 + lane;     // key row of this thread (TMEM lane)
-    const int t8 = threadIdx.x - 64;  // 0..255
+    const int r = q4 * 32 + lane;  // key row of this thread (TMEM lane)
     const uint32_t lane_base = (uint32_t)(q4 * 32) << 16;
     const uint32_t spt = ptx::smem_u32(sPT), sdst = ptx::smem_u32(sdST);
     for (int it = 0; it < nq; ++it) {
-      const int st = it & 1;  // lse / D double buffer (independent of QS)
+      const int st = it % QS;
       const int qi = i0 + it;
       const bool diag = (qi == kt);
-      {  // stage lse / D of this query tile in smem
-        const int64_t base = ((int64_t)b * p.nh + hd) * p.s + qi * 128;
-        if (t8 < 128)
-          sts_f32(ptx::smem_u32(sLse + st * 128 + t8), p.lse[base + t8]);
-        else
-          sts_f32(ptx::smem_u32(sD + st * 128 + t8 - 128), p.Dsum[base + t8 - 128]);
-      }
-      named_bar(1, 256);
+      ptx::mbar_wait(&q_full[st], (it / QS) & 1);  // lse / D of this query tile in smem
       ptx::mbar_wait(s_full, it & 1);
       ptx::tc_fence_after();
-      // P^T / dS^T smem must be free: previous tile's MMAs done
-      if (it >= 1) ptx::mbar_wait(mm_done, (it - 1) & 1);
+      uint32_t vs[2][32], vd[2][32];
+      __syncwarp();
+      ptx::tmem_ld32(T_S + hf * 64 + lane_base, vs[0]);
+      ptx::tmem_ld32(T_S + hf * 64 + 32 + lane_base, vs[1]);
+      ptx::tmem_ld32(T_DP + hf * 64 + lane_base, vd[0]);
+      ptx::tmem_ld32(T_DP + hf * 64 + 32 + lane_base, vd[1]);
+      ptx::tmem_ld_wait();
+      ptx::tc_fence_before();
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(st_empty);  // S^T / dP^T TMEM may be overwritten
+      // P^T / dS^T smem (also the dQ staging tile) is free: the previous
+      // tile's dQ reduce finished reading it (named barrier below)
 #pragma unroll
       for (int cc = 0; cc < 2; ++cc) {
         const int c = hf * 2 + cc;
-        uint32_t vs[32], vd[32];
-        __syncwarp();
-        ptx::tmem_ld32(T_S + c * 32 + lane_base, vs);
-        ptx::tmem_ld32(T_DP + c * 32 + lane_base, vd);
-        ptx::tmem_ld_wait();
         uint32_t ppk[16], dpk[16];
-        const uint32_t aL = ptx::smem_u32(sLse + st * 128 + c * 32), aD = ptx::smem_u32(sD + st * 128 + c * 32);
+        const uint32_t aL = ptx::smem_u32(sLD + st * 256 + c * 32), aD = aL + 512;
 #pragma unroll
         for (int e = 0; e < 32; e += 2) {
           const int q = c * 32 + e;
           const float2 L = lds_f32x2(aL + e * 4), Dd = lds_f32x2(aD + e * 4);  // broadcast reads
-          float p0 = ex2(fmaf(__uint_as_float(vs[e]), p.scale_log2, -L.x));
-          float p1 = ex2(fmaf(__uint_as_float(vs[e + 1]), p.scale_log2, -L.y));
+          float p0 = ex2(fmaf(__uint_as_float(vs[cc][e]), p.scale_log2, -L.x));
+          float p1 = ex2(fmaf(__uint_as_float(vs[cc][e + 1]), p.scale_log2, -L.y));
           if (diag) {  // key r attends only from queries >= r
             if (q < r) p0 = 0.f;
             if (q + 1 < r) p1 = 0.f;
           }
-          const float d0 = p0 * (__uint_as_float(vd[e]) - Dd.x) * p.scale;
-          const float d1 = p1 * (__uint_as_float(vd[e + 1]) - Dd.y) * p.scale;
+          const float d0 = p0 * (__uint_as_float(vd[cc][e]) - Dd.x) * p.scale;
+          const float d1 = p1 * (__uint_as_float(vd[cc][e + 1]) - Dd.y) * p.scale;
           ppk[e >> 1] = pack_bf16(p0, p1);
           dpk[e >> 1] = pack_bf16(d0, d1);
         }
@@ -584,25 +603,41 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
       ptx::fence_proxy_async();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(p_full);
-      // dQ of this query tile: TMEM lane = query row; this warp's column half
+      // dQ of this query tile (TMEM lane = query row) -> fp32 staging tile in
+      // the P^T/dS^T smem (free once the MMAs completed) -> one TMA
+      // reduce-add into the fp32 dQ buffer
       ptx::mbar_wait(mm_done, it & 1);
       ptx::tc_fence_after();
-      float* dq = p.dQacc + ((int64_t)b * p.s + qi * 128 + r) * p.h + hd * DH;
+      const uint32_t stg = spt;  // [128 rows][DH] fp32, row-major
 #pragma unroll
       for (int cc = 0; cc < DH / 64; ++cc) {
         const int c = hf * (DH / 64) + cc;
         uint32_t v[32];
         __syncwarp();
-        ptx::tmem_ld32(T_S + c * 32 + lane_base, v);
+        ptx::tmem_ld32(T_DQ + c * 32 + lane_base, v);
         ptx::tmem_ld_wait();
 #pragma unroll
-        for (int e = 0; e < 32; e += 4)
-          red_add_v4(dq + c * 32 + e, __uint_as_float(v[e]), __uint_as_float(v[e + 1]), __uint_as_float(v[e + 2]),
-                     __uint_as_float(v[e + 3]));
+        for (int e = 0; e < 32; e += 4) {
+          // rotate the 16-byte chunk order by row to spread smem banks
+          const int ee = (e + 4 * (r & 7)) & 31;
+          st_shared_v4(stg + (uint32_t)(r * DH + c * 32 + ee) * 4, v[ee], v[ee + 1], v[ee + 2], v[ee + 3]);
+        }
       }
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(dq_empty);
+      ptx::fence_proxy_async();
+      named_bar(1, 256);
+      if (warp == 2 && lane == 0) {
+        asm volatile(
+            "cp.reduce.async.bulk.tensor.4d.global.shared::cta.add.tile.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
+                reinterpret_cast<uint64_t>(&tdq)),
+            "r"(stg), "r"(0), "r"(qi * 128), "r"(hd), "r"(b)
+            : "memory");
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+      }
+      named_bar(1, 256);
     }
     // dV (half 0) / dK (half 1) of this key tile (rows = keys)
     ptx::mbar_wait(mm_done, (nq - 1) & 1);
@@ -630,24 +665,31 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
   }
 }
 
-// D[b, h, q] = sum_d dO[q, d] * O[q, d]  (one warp per (row, head))
+// D[b, h, q] = sum_d dO[q, d] * O[q, d]; 8 lanes per (row, head) for dh=64
+// (16 for dh=128), 16-byte loads
 __global__ void flash_dsum_kernel(const __nv_bfloat16* dO, const __nv_bfloat16* O, float* D, int rows, int nh, int dh,
                                   int h, int s) {
-  const int64_t w = (int64_t)blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32;
-  const int lane = threadIdx.x % 32;
-  if (w >= (int64_t)rows * nh) return;
-  const int row = (int)(w / nh), hd = (int)(w % nh);
-  const __nv_bfloat16* a = dO + (int64_t)row * h + hd * dh;
-  const __nv_bfloat16* o = O + (int64_t)row * h + hd * dh;
+  const int lanes = dh / 8;
+  const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int64_t item = t / lanes;  // (row, head)
+  const int sub = (int)(t % lanes);
   float acc = 0.f;
-  for (int d = lane * 2; d < dh; d += 64) {
-    float2 x = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(a + d));
-    float2 y = __bfloat1622float2(*reinterpret_cast<const __nv_bfloat162*>(o + d));
-    acc += x.x * y.x + x.y * y.y;
-  }
+  if (item < (int64_t)rows * nh) {
+    const int row = (int)(item / nh), hd = (int)(item % nh);
+    const int64_t off = (int64_t)row * h + hd * dh + sub * 8;
+    const uint4 a = *reinterpret_cast<const uint4*>(dO + off);
+    const uint4 o = *reinterpret_cast<const uint4*>(O + off);
+    const __nv_bfloat162* a2 = reinterpret_cast<const __nv_bfloat162*>(&a);
+    const __nv_bfloat162* o2 = reinterpret_cast<const __nv_bfloat162*>(&o);
 #pragma unroll
-  for (int k = 16; k; k >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, k);
-  if (lane == 0) {
+    for (int k = 0; k < 4; ++k) {
+      const float2 x = __bfloat1622float2(a2[k]), y = __bfloat1622float2(o2[k]);
+      acc += x.x * y.x + x.y * y.y;
+    }
+  }
+  for (int k = lanes / 2; k; k >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, k);
+  if (sub == 0 && item < (int64_t)rows * nh) {
+    const int row = (int)(item / nh), hd = (int)(item % nh);
     const int b = row / s, q = row % s;
     D[((int64_t)b * nh + hd) * s + q] = acc;
   }
@@ -693,6 +735,21 @@ int head_map(CUtensorMap* m, const void* base, int64_t ld, int dh, int s, int n_
                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) MOBIUS_FAIL(MOBIUS_ECUDA, "flash tensor map (%d)", (int)r);
+  return MOBIUS_OK;
+}
+
+// fp32 {d, token, head, batch} map over the dQ accumulator [mbs*s, h]; box {dh, 128, 1, 1}
+int dq_map(CUtensorMap* m, const float* base, int h, int dh, int s, int nh, int mbs) {
+  EncodeTiledFn enc = encode_fn();
+  if (!enc) MOBIUS_FAIL(MOBIUS_ECUDA, "cuTensorMapEncodeTiled unavailable");
+  cuuint64_t dims[4] = {(cuuint64_t)dh, (cuuint64_t)s, (cuuint64_t)nh, (cuuint64_t)mbs};
+  cuuint64_t strides[3] = {(cuuint64_t)h * 4, (cuuint64_t)dh * 4, (cuuint64_t)s * h * 4};
+  cuuint32_t box[4] = {(cuuint32_t)dh, 128, 1, 1};
+  cuuint32_t es[4] = {1, 1, 1, 1};
+  CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, const_cast<float*>(base), dims, strides, box, es,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) MOBIUS_FAIL(MOBIUS_ECUDA, "flash dQ tensor map (%d)", (int)r);
   return MOBIUS_OK;
 }
 
@@ -750,14 +807,16 @@ int flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* o, const __nv_
   MOBIUS_CHECK_ARG(flash_supported(dh, s), "flash: dh %d / s %d unsupported", dh, s);
   const int h = nh * dh;
   const int64_t rows = (int64_t)mbs * s;
-  CUtensorMap tm, tdo;
+  CUtensorMap tm, tdo, tdq;
   int rc = head_map(&tm, qkv, 3 * h, dh, s, 3 * nh, mbs);
   if (rc) return rc;
   rc = head_map(&tdo, dout, h, dh, s, nh, mbs);
   if (rc) return rc;
+  rc = dq_map(&tdq, dq_ws, h, dh, s, nh, mbs);
+  if (rc) return rc;
   {
-    const int64_t warps = rows * nh;
-    flash_dsum_kernel<<<(unsigned)((warps + 7) / 8), 256, 0, st>>>(dout, o, dsum_ws, (int)rows, nh, dh, h, s);
+    const int64_t threads = rows * nh * (dh / 8);
+    flash_dsum_kernel<<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(dout, o, dsum_ws, (int)rows, nh, dh, h, s);
   }
   cudaError_t e = cudaMemsetAsync(dq_ws, 0, rows * h * sizeof(float), st);
   if (e != cudaSuccess) MOBIUS_FAIL(MOBIUS_ECUDA, "flash dq memset");
@@ -777,11 +836,11 @@ int flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* o, const __nv_
   if (dh == 64) {
     static bool once = false;
     if (!once) { rc = set_smem(flash_bwd_kernel<64>, BwdCfg<64>::SMEM); if (rc) return rc; once = true; }
-    flash_bwd_kernel<64><<<grid, NT_FWD, BwdCfg<64>::SMEM, st>>>(tm, tdo, p);
+    flash_bwd_kernel<64><<<grid, NT_FWD, BwdCfg<64>::SMEM, st>>>(tm, tdo, tdq, p);
   } else {
     static bool once = false;
     if (!once) { rc = set_smem(flash_bwd_kernel<128>, BwdCfg<128>::SMEM); if (rc) return rc; once = true; }
-    flash_bwd_kernel<128><<<grid, NT_FWD, BwdCfg<128>::SMEM, st>>>(tm, tdo, p);
+    flash_bwd_kernel<128><<<grid, NT_FWD, BwdCfg<128>::SMEM, st>>>(tm, tdo, tdq, p);
   }
   {
     const int64_t n = rows * h / 4;
