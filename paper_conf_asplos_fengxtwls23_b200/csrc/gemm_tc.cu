@@ -15,6 +15,7 @@
 #include <cuda.h>
 #include <cuda_runtime.h>
 
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 
@@ -58,14 +59,19 @@ struct Params {
   int64_t ldx, xbs1, xbs2;
 };
 
+__device__ __forceinline__ float tanh_fast(float x) {
+  float y;
+  asm("tanh.approx.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
 __device__ __forceinline__ float gelu_f(float u) {
   const float c = 0.7978845608028654f, a = 0.044715f;
-  float t = tanhf(c * (u + a * u * u * u));
+  float t = tanh_fast(c * (u + a * u * u * u));
   return 0.5f * u * (1.f + t);
 }
 __device__ __forceinline__ float gelu_grad_f(float u) {
   const float c = 0.7978845608028654f, a = 0.044715f;
-  float t = tanhf(c * (u + a * u * u * u));
+  float t = tanh_fast(c * (u + a * u * u * u));
   return 0.5f * (1.f + t) + 0.5f * u * (1.f - t * t) * c * (1.f + 3.f * a * u * u);
 }
 
@@ -100,6 +106,128 @@ __device__ __forceinline__ void kb_range(const Params& p, int mt, int& kb0, int&
     kb1 = (kend + BK - 1) / BK;
   } else if (p.causal == CAUSAL_K_GE_M0) {
     kb0 = (mt * BM) / BK;
+  }
+}
+
+// 8 bf16 (16 bytes) <-> floats
+__device__ __forceinline__ void ld_bf16x8(const __nv_bfloat16* g, float* f) {
+  const uint4 pk = *reinterpret_cast<const uint4*>(g);
+  const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&pk);
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    const float2 x = __bfloat1622float2(h2[j]);
+    f[2 * j] = x.x;
+    f[2 * j + 1] = x.y;
+  }
+}
+__device__ __forceinline__ void st_bf16x8(__nv_bfloat16* g, const float* f) {
+  uint4 pk;
+  __nv_bfloat162* h2 = reinterpret_cast<__nv_bfloat162*>(&pk);
+#pragma unroll
+  for (int j = 0; j < 4; ++j) h2[j] = __floats2bfloat162_rn(f[2 * j], f[2 * j + 1]);
+  *reinterpret_cast<uint4*>(g) = pk;
+}
+
+// Epilogue of one accumulator tile row-slice: this thread owns output row m
+// (TMEM lane), columns [nt*BN, nt*BN + BN); TMEM -> registers -> fused ops
+// -> global.  tmem_row = tmem base + lane quadrant + accumulator column base.
+// Full 32-column chunks use 16-byte vector accesses only (all indices are
+// compile-time, so nothing spills to local memory); a ragged last chunk
+// takes the predicated scalar path.
+template <int BN>
+__device__ __forceinline__ void epi_tile(const Params& p, uint32_t tmem_row, int m, int b1, int b2, int nt) {
+  const bool row_ok = m < p.M;
+  const int64_t crow = (int64_t)b1 * p.cbs1 + (int64_t)b2 * p.cbs2 + (int64_t)m * p.ldc;
+  const bool has_bias = p.epi == EPI_BIAS || p.epi == EPI_BIAS_GELU || p.epi == EPI_BIAS_RESID;
+  const bool has_r = p.epi == EPI_BIAS_RESID || p.epi == EPI_GELU_BWD;
+  const bool accum = p.epi == EPI_ACCUM && p.accumulate;
+#pragma unroll 1
+  for (int c = 0; c < BN; c += 32) {
+    uint32_t r[32];
+    __syncwarp();
+    ptx::tmem_ld32(tmem_row + c, r);
+    ptx::tmem_ld_wait();
+    const int n0 = nt * BN + c;
+    if (!row_ok || n0 >= p.N) continue;
+    float v[32];
+#pragma unroll
+    for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]) * p.alpha;
+    const __nv_bfloat16* rrow = has_r ? p.R + (int64_t)b1 * p.rbs1 + (int64_t)b2 * p.rbs2 + (int64_t)m * p.ldr + n0 : nullptr;
+    __nv_bfloat16* aux = p.epi == EPI_BIAS_GELU
+                             ? p.AUX + (int64_t)b1 * p.xbs1 + (int64_t)b2 * p.xbs2 + (int64_t)m * p.ldx + n0
+                             : nullptr;
+    if (n0 + 32 <= p.N) {
+      if (has_bias) {
+#pragma unroll
+        for (int i = 0; i < 32; i += 8) {
+          float bb[8];
+          ld_bf16x8(p.bias + n0 + i, bb);
+#pragma unroll
+          for (int j = 0; j < 8; ++j) v[i + j] += bb[j];
+        }
+      }
+      if (p.epi == EPI_BIAS_GELU) {
+#pragma unroll
+        for (int i = 0; i < 32; i += 8) st_bf16x8(aux + i, v + i);
+        // GeLU of the bf16-rounded pre-activation (what backward will see)
+#pragma unroll
+        for (int i = 0; i < 32; ++i) v[i] = gelu_f(__bfloat162float(__float2bfloat16_rn(v[i])));
+      }
+      if (has_r) {
+#pragma unroll
+        for (int i = 0; i < 32; i += 8) {
+          float rv[8];
+          ld_bf16x8(rrow + i, rv);
+          if (p.epi == EPI_BIAS_RESID) {
+#pragma unroll
+            for (int j = 0; j < 8; ++j) v[i + j] += rv[j];
+          } else {
+#pragma unroll
+            for (int j = 0; j < 8; ++j) v[i + j] *= gelu_grad_f(rv[j]);
+          }
+        }
+      }
+      if (p.c_f32) {
+        float* cp = reinterpret_cast<float*>(p.C) + crow + n0;
+#pragma unroll
+        for (int i = 0; i < 32; i += 4) {
+          float4 o = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
+          if (accum) {
+            const float4 old = *reinterpret_cast<const float4*>(cp + i);
+            o.x += old.x;
+            o.y += old.y;
+            o.z += old.z;
+            o.w += old.w;
+          }
+          *reinterpret_cast<float4*>(cp + i) = o;
+        }
+      } else {
+        __nv_bfloat16* cp = p.C + crow + n0;
+#pragma unroll
+        for (int i = 0; i < 32; i += 8) st_bf16x8(cp + i, v + i);
+      }
+    } else {
+      const int cnt = p.N - n0;
+#pragma unroll
+      for (int i = 0; i < 32; ++i) {
+        if (i < cnt) {
+          float x = v[i];
+          if (has_bias) x += __bfloat162float(p.bias[n0 + i]);
+          if (p.epi == EPI_BIAS_GELU) {
+            aux[i] = __float2bfloat16_rn(x);
+            x = gelu_f(__bfloat162float(__float2bfloat16_rn(x)));
+          }
+          if (p.epi == EPI_BIAS_RESID) x += __bfloat162float(rrow[i]);
+          if (p.epi == EPI_GELU_BWD) x *= gelu_grad_f(__bfloat162float(rrow[i]));
+          if (p.c_f32) {
+            float* cp = reinterpret_cast<float*>(p.C) + crow + n0;
+            cp[i] = x + (accum ? cp[i] : 0.f);
+          } else {
+            p.C[crow + n0 + i] = __float2bfloat16_rn(x);
+          }
+        }
+      }
+    }
   }
 }
 
@@ -232,104 +360,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       if (!tile_active<BN>(p, mt, nt)) continue;
       ptx::mbar_wait(&tfull[acc], aphase);
       ptx::tc_fence_after();
-      const int m = mt * BM + q * 32 + lane;
-      const bool row_ok = m < p.M;
-      const int64_t crow = (int64_t)b1 * p.cbs1 + (int64_t)b2 * p.cbs2 + (int64_t)m * p.ldc;
-#pragma unroll 1
-      for (int c = 0; c < BN; c += 32) {
-        uint32_t r[32];
-        __syncwarp();
-        ptx::tmem_ld32(tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + c, r);
-        ptx::tmem_ld_wait();
-        const int n0 = nt * BN + c;
-        if (row_ok && n0 < p.N) {
-        float v[32];
-#pragma unroll
-        for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]) * p.alpha;
-        const bool full_chunk = (n0 + 32 <= p.N);
-        const int cnt = full_chunk ? 32 : (p.N - n0);
-        if (p.epi == EPI_BIAS || p.epi == EPI_BIAS_GELU || p.epi == EPI_BIAS_RESID) {
-          for (int i = 0; i < cnt; ++i) v[i] += __bfloat162float(p.bias[n0 + i]);
-        }
-        if (p.epi == EPI_BIAS_GELU) {
-          __nv_bfloat16* aux = p.AUX + (int64_t)b1 * p.xbs1 + (int64_t)b2 * p.xbs2 + (int64_t)m * p.ldx + n0;
-          if (full_chunk) {
-#pragma unroll
-            for (int i = 0; i < 32; i += 8) {
-              uint4 pk;
-              __nv_bfloat162* h2 = reinterpret_cast<__nv_bfloat162*>(&pk);
-#pragma unroll
-              for (int j = 0; j < 4; ++j) h2[j] = __floats2bfloat162_rn(v[i + 2 * j], v[i + 2 * j + 1]);
-              *reinterpret_cast<uint4*>(aux + i) = pk;
-            }
-          } else {
-            for (int i = 0; i < cnt; ++i) aux[i] = __float2bfloat16_rn(v[i]);
-          }
-          // GeLU of the bf16-rounded pre-activation (what backward will see)
-#pragma unroll
-          for (int i = 0; i < 32; ++i) v[i] = gelu_f(__bfloat162float(__float2bfloat16_rn(v[i])));
-        }
-        if (p.epi == EPI_BIAS_RESID || p.epi == EPI_GELU_BWD) {
-          const __nv_bfloat16* rr = p.R + (int64_t)b1 * p.rbs1 + (int64_t)b2 * p.rbs2 + (int64_t)m * p.ldr + n0;
-          float rv[32];
-          if (full_chunk) {
-#pragma unroll
-            for (int i = 0; i < 32; i += 8) {
-              uint4 pk = *reinterpret_cast<const uint4*>(rr + i);
-              const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&pk);
-#pragma unroll
-              for (int j = 0; j < 4; ++j) {
-                float2 f = __bfloat1622float2(h2[j]);
-                rv[i + 2 * j] = f.x;
-                rv[i + 2 * j + 1] = f.y;
-              }
-            }
-          } else {
-            for (int i = 0; i < cnt; ++i) rv[i] = __bfloat162float(rr[i]);
-          }
-          if (p.epi == EPI_BIAS_RESID) {
-#pragma unroll
-            for (int i = 0; i < 32; ++i) v[i] += rv[i];
-          } else {
-#pragma unroll
-            for (int i = 0; i < 32; ++i) v[i] *= gelu_grad_f(rv[i]);
-          }
-        }
-        if (p.c_f32) {
-          float* cp = reinterpret_cast<float*>(p.C) + crow + n0;
-          if (full_chunk) {
-#pragma unroll
-            for (int i = 0; i < 32; i += 4) {
-              float4 o = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
-              if (p.epi == EPI_ACCUM && p.accumulate) {
-                float4 old = *reinterpret_cast<float4*>(cp + i);
-                o.x += old.x;
-                o.y += old.y;
-                o.z += old.z;
-                o.w += old.w;
-              }
-              *reinterpret_cast<float4*>(cp + i) = o;
-            }
-          } else {
-            for (int i = 0; i < cnt; ++i) cp[i] = v[i] + ((p.epi == EPI_ACCUM && p.accumulate) ? cp[i] : 0.f);
-          }
-        } else {
-          __nv_bfloat16* cp = p.C + crow + n0;
-          if (full_chunk) {
-#pragma unroll
-            for (int i = 0; i < 32; i += 8) {
-              uint4 pk;
-              __nv_bfloat162* h2 = reinterpret_cast<__nv_bfloat162*>(&pk);
-#pragma unroll
-              for (int j = 0; j < 4; ++j) h2[j] = __floats2bfloat162_rn(v[i + 2 * j], v[i + 2 * j + 1]);
-              *reinterpret_cast<uint4*>(cp + i) = pk;
-            }
-          } else {
-            for (int i = 0; i < cnt; ++i) cp[i] = __float2bfloat16_rn(v[i]);
-          }
-        }
-        }
-      }
+      epi_tile<BN>(p, tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN, mt * BM + q * 32 + lane, b1, b2, nt);
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(&tempty[acc]);
@@ -344,6 +375,167 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
   if (warp == 1) {
     ptx::tc_fence_after();
     ptx::tmem_dealloc<C::TMEM_COLS>(tmem_base);
+  }
+}
+
+
+// ======================================================================
+// 2-CTA variant (cta_group::2): a cluster of two CTAs on the two SMs of a
+// TPC computes a 256 x BN tile; each CTA loads its 128 rows of A and half of
+// B (BN/2 rows) into its own smem, the leader CTA issues
+// tcgen05.mma.cta_group::2 (M = 256) and multicasts the commits, each CTA's
+// epilogue drains its own 128 TMEM lanes.  Halves per-SM operand traffic.
+// Used for plain (non-batched, non-causal) GEMMs with N >= 256.
+template <int BN>
+struct Cfg2 {
+  static constexpr int A_BYTES = 128 * BK * 2;
+  static constexpr int B_BYTES = (BN / 2) * BK * 2;
+  static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+  static constexpr int STAGES = (200 * 1024) / STAGE_BYTES > 8 ? 8 : (200 * 1024) / STAGE_BYTES;
+  static constexpr int TMEM_COLS = 2 * BN;
+  static constexpr int SMEM = 1024 + STAGES * STAGE_BYTES + 256;
+};
+
+template <int BN, bool A_MN, bool B_MN>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
+    gemm_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, const Params p) {
+  using C = Cfg2<BN>;
+  constexpr int BM2 = 256;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* smA = smem;
+  uint8_t* smB = smem + C::STAGES * C::A_BYTES;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + C::STAGES * C::STAGE_BYTES);
+  uint64_t* empty = full + C::STAGES;
+  uint64_t* tfull = empty + C::STAGES;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+
+  const int warp = threadIdx.x / 32;
+  const int lane = threadIdx.x % 32;
+  const uint32_t rank = ptx::cluster_ctarank();
+  const bool leader = rank == 0;
+  const int cl = blockIdx.x / 2, ncl = gridDim.x / 2;
+
+  if (warp == 0 && lane == 0) {
+    ptx::tma_prefetch_desc(&tmA);
+    ptx::tma_prefetch_desc(&tmB);
+    for (int s = 0; s < C::STAGES; ++s) {
+      ptx::mbar_init(&full[s], 1);
+      ptx::mbar_init(&empty[s], 1);
+    }
+    for (int a = 0; a < 2; ++a) {
+      ptx::mbar_init(&tfull[a], 1);
+      ptx::mbar_init(&tempty[a], 8);  // 4 epilogue warps x 2 CTAs (leader's copy is the one used)
+    }
+    ptx::fence_mbar_init();
+  }
+  if (warp == 1) ptx::tmem_alloc_2sm<C::TMEM_COLS>(tmem_slot);
+  ptx::tc_fence_before();
+  ptx::cluster_sync();
+  ptx::tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+  const int total = p.nb1 * p.nb2 * p.tiles_m * p.tiles_n;
+
+  if (warp == 0) {
+    if (lane == 0) {  // TMA producer (both CTAs)
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int t = cl; t < total; t += ncl) {
+        int b1, b2, mt, nt;
+        decode_tile(p, t, b1, b2, mt, nt);
+        const int m0 = mt * BM2 + (int)rank * 128, n0 = nt * BN + (int)rank * (BN / 2);
+        for (int kb = 0; kb < p.num_kb; ++kb) {
+          ptx::mbar_wait_cluster(&empty[stage], phase ^ 1);
+          if (leader) ptx::mbar_arrive_expect_tx(&full[stage], 2 * C::STAGE_BYTES);
+          uint8_t* a = smA + stage * C::A_BYTES;
+          uint8_t* b = smB + stage * C::B_BYTES;
+          const int k0 = kb * BK;
+          if (A_MN) {
+#pragma unroll
+            for (int i = 0; i < 2; ++i) ptx::tma_load_4d_2sm(a + i * 8192, &tmA, &full[stage], m0 + 64 * i, k0, b2, b1);
+          } else {
+            ptx::tma_load_4d_2sm(a, &tmA, &full[stage], k0, m0, b2, b1);
+          }
+          if (B_MN) {
+#pragma unroll
+            for (int i = 0; i < BN / 128; ++i)
+              ptx::tma_load_4d_2sm(b + i * 8192, &tmB, &full[stage], n0 + 64 * i, k0, b2, b1);
+          } else {
+            ptx::tma_load_4d_2sm(b, &tmB, &full[stage], k0, n0, b2, b1);
+          }
+          if (++stage == C::STAGES) {
+            stage = 0;
+            phase ^= 1;
+          }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (leader && lane == 0) {  // MMA issuer (leader only)
+      constexpr uint32_t IDESC = ptx::idesc_bf16(BM2, BN, A_MN ? 1 : 0, B_MN ? 1 : 0);
+      int stage = 0;
+      uint32_t phase = 0;
+      int acc = 0;
+      uint32_t aphase = 0;
+      for (int t = cl; t < total; t += ncl) {
+        ptx::mbar_wait_cluster(&tempty[acc], aphase ^ 1);
+        ptx::tc_fence_after();
+        const uint32_t tmem_d = tmem_base + acc * BN;
+        for (int kb = 0; kb < p.num_kb; ++kb) {
+          ptx::mbar_wait_cluster(&full[stage], phase);
+          ptx::tc_fence_after();
+          const uint32_t a_base = ptx::smem_u32(smA + stage * C::A_BYTES);
+          const uint32_t b_base = ptx::smem_u32(smB + stage * C::B_BYTES);
+#pragma unroll
+          for (int k = 0; k < BK / 16; ++k) {
+            uint64_t ad = A_MN ? ptx::sdesc_sw128(a_base + k * 2048, 8192, 1024)
+                               : ptx::sdesc_sw128(a_base + k * 32, 16, 1024);
+            uint64_t bd = B_MN ? ptx::sdesc_sw128(b_base + k * 2048, 8192, 1024)
+                               : ptx::sdesc_sw128(b_base + k * 32, 16, 1024);
+            ptx::mma_bf16_2sm(tmem_d, ad, bd, IDESC, (kb > 0 || k > 0) ? 1u : 0u);
+          }
+          ptx::mma_commit_2sm(&empty[stage], 0x3);  // frees the slot in both CTAs
+          if (++stage == C::STAGES) {
+            stage = 0;
+            phase ^= 1;
+          }
+        }
+        ptx::mma_commit_2sm(&tfull[acc], 0x3);      // accumulator ready in both CTAs
+        if (++acc == 2) {
+          acc = 0;
+          aphase ^= 1;
+        }
+      }
+    }
+  } else {
+    // epilogue (warps 2..5) of both CTAs: rows mt*256 + rank*128 + lane quadrant
+    const int q = warp & 3;
+    const uint32_t tempty_leader = ptx::mapa_shared(ptx::smem_u32(&tempty[0]), 0);
+    int acc = 0;
+    uint32_t aphase = 0;
+    for (int t = cl; t < total; t += ncl) {
+      int b1, b2, mt, nt;
+      decode_tile(p, t, b1, b2, mt, nt);
+      ptx::mbar_wait_cluster(&tfull[acc], aphase);
+      ptx::tc_fence_after();
+      epi_tile<BN>(p, tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN, mt * BM2 + (int)rank * 128 + q * 32 + lane,
+                   b1, b2, nt);
+      ptx::tc_fence_before();
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive_cluster(tempty_leader + acc * 8);
+      if (++acc == 2) {
+        acc = 0;
+        aphase ^= 1;
+      }
+    }
+  }
+
+  __syncthreads();
+  ptx::cluster_sync();
+  if (warp == 1) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc_2sm<C::TMEM_COLS>(tmem_base);
   }
 }
 
@@ -411,6 +603,23 @@ int dispatch_major(bool amn, bool bmn, const CUtensorMap& ta, const CUtensorMap&
   return launch<BN, true, true>(ta, tb, p, total, s);
 }
 
+template <int BN, bool A_MN, bool B_MN>
+int launch2(const CUtensorMap& ta, const CUtensorMap& tb, const Params& p, int total, cudaStream_t s) {
+  auto k = gemm_tc2_kernel<BN, A_MN, B_MN>;
+  static bool attr_set = false;
+  if (!attr_set) {
+    if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg2<BN>::SMEM) != cudaSuccess)
+      MOBIUS_FAIL(MOBIUS_ECUDA, "cudaFuncSetAttribute(smem, 2cta) failed");
+    attr_set = true;
+  }
+  int clusters = total < num_sms() / 2 ? total : num_sms() / 2;
+  if (clusters < 1) clusters = 1;
+  k<<<2 * clusters, NUM_THREADS, Cfg2<BN>::SMEM, s>>>(ta, tb, p);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) MOBIUS_FAIL(MOBIUS_ECUDA, "gemm_tc2 launch: %s", cudaGetErrorString(e));
+  return MOBIUS_OK;
+}
+
 }  // namespace
 
 int num_sms() {
@@ -424,7 +633,49 @@ int num_sms() {
   return n;
 }
 
+static int gemm_bf16_2cta(const GemmDesc& d, cudaStream_t s) {
+  constexpr int BN = 256;
+  CUtensorMap ta, tb;
+  int rc;
+  if (d.a_mn)
+    rc = make_map(&ta, d.A, d.M, d.K, d.nb1, d.nb2, BK);
+  else
+    rc = make_map(&ta, d.A, d.K, d.M, d.nb1, d.nb2, 128);
+  if (rc) return rc;
+  if (d.b_mn)
+    rc = make_map(&tb, d.B, d.N, d.K, d.nb1, d.nb2, BK);
+  else
+    rc = make_map(&tb, d.B, d.K, d.N, d.nb1, d.nb2, BN / 2);
+  if (rc) return rc;
+  Params p;
+  std::memset(&p, 0, sizeof(p));
+  p.M = d.M; p.N = d.N; p.K = d.K; p.nb1 = 1; p.nb2 = 1;
+  p.tiles_m = (d.M + 255) / 256;
+  p.tiles_n = (d.N + BN - 1) / BN;
+  p.num_kb = (d.K + BK - 1) / BK;
+  p.causal = CAUSAL_NONE;
+  p.epi = d.epi; p.c_f32 = d.c_f32 ? 1 : 0; p.accumulate = d.accumulate ? 1 : 0; p.alpha = d.alpha;
+  p.C = (__nv_bfloat16*)d.C.ptr; p.ldc = d.C.ld;
+  p.bias = (const __nv_bfloat16*)d.bias;
+  p.R = (const __nv_bfloat16*)d.R.ptr; p.ldr = d.R.ld;
+  p.AUX = (__nv_bfloat16*)d.AUX.ptr; p.ldx = d.AUX.ld;
+  const int total = p.tiles_m * p.tiles_n;
+  if (!d.a_mn && !d.b_mn) return launch2<BN, false, false>(ta, tb, p, total, s);
+  if (!d.a_mn && d.b_mn) return launch2<BN, false, true>(ta, tb, p, total, s);
+  if (d.a_mn && !d.b_mn) return launch2<BN, true, false>(ta, tb, p, total, s);
+  return launch2<BN, true, true>(ta, tb, p, total, s);
+}
+
+static int g_gemm_mode = -1;  // -1 auto (env MOBIUS_GEMM_2CTA, default on), 0 off, 1 on
+
 int gemm_bf16(const GemmDesc& d, cudaStream_t s) {
+  if (g_gemm_mode < 0) {
+    const char* e = getenv("MOBIUS_GEMM_2CTA");
+    g_gemm_mode = (e && e[0] == '0') ? 0 : 1;
+  }
+  if (g_gemm_mode == 1 && d.causal == CAUSAL_NONE && d.nb1 == 1 && d.nb2 == 1 && d.N >= 256 && d.M >= 256 &&
+      d.K >= 64)
+    return gemm_bf16_2cta(d, s);
   MOBIUS_CHECK_ARG(d.M > 0 && d.N > 0 && d.K > 0, "gemm: empty shape %d x %d x %d", d.M, d.N, d.K);
   MOBIUS_CHECK_ARG(d.N % 8 == 0 || !true, "gemm: N must be a multiple of 8");
   int BN = d.N >= 256 ? 256 : (d.N > 64 ? 128 : 64);
