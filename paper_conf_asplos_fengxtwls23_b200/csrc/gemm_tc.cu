@@ -633,8 +633,8 @@ int num_sms() {
   return n;
 }
 
-static int gemm_bf16_2cta(const GemmDesc& d, cudaStream_t s) {
-  constexpr int BN = 256;
+template <int BN>
+static int gemm_bf16_2cta_bn(const GemmDesc& d, cudaStream_t s) {
   CUtensorMap ta, tb;
   int rc;
   if (d.a_mn)
@@ -665,6 +665,11 @@ static int gemm_bf16_2cta(const GemmDesc& d, cudaStream_t s) {
   if (d.a_mn && !d.b_mn) return launch2<BN, true, false>(ta, tb, p, total, s);
   return launch2<BN, true, true>(ta, tb, p, total, s);
 }
+
+// 256 x 256 tiles: at 64 B/clk/SM of operand traffic this is the only 2-CTA
+// shape that stays under the L2->SM feed rate (256 x 128 measured slower even
+// where it quantises better over the 74 SM pairs)
+static int gemm_bf16_2cta(const GemmDesc& d, cudaStream_t s) { return gemm_bf16_2cta_bn<256>(d, s); }
 
 static int g_gemm_mode = -1;  // -1 auto (env MOBIUS_GEMM_2CTA, default on), 0 off, 1 on
 
