@@ -139,6 +139,60 @@ __global__ void embed_bwd_wpe_k(const T* dx, float* dwpe, int mbs, int s, int h)
 }
 
 // ------------------------------------------------------------ LayerNorm
+// warp per row, the row held in registers (NV 16-byte vectors per lane)
+template <typename T, int NV>
+__global__ void __launch_bounds__(256) ln_fwd_warp_k(const T* __restrict__ x, const T* __restrict__ g,
+                                                     const T* __restrict__ b, T* __restrict__ y, float* mu_out,
+                                                     float* rstd_out, int rows, int h) {
+  constexpr int V = Vec<T>::N;
+  const int lane = threadIdx.x % 32;
+  const int r = blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32;
+  if (r >= rows) return;
+  const T* xr = x + (int64_t)r * h;
+  float v[NV][V];
+  float sum = 0.f;
+#pragma unroll
+  for (int k = 0; k < NV; ++k) {
+    const int c = (lane + 32 * k) * V;
+    if (c < h) {
+      Vec<T>::load(xr + c, v[k]);
+#pragma unroll
+      for (int e = 0; e < V; ++e) sum += v[k][e];
+    }
+  }
+  const float m = warp_sum(sum) / h;
+  float q = 0.f;
+#pragma unroll
+  for (int k = 0; k < NV; ++k) {
+    const int c = (lane + 32 * k) * V;
+    if (c < h) {
+#pragma unroll
+      for (int e = 0; e < V; ++e) {
+        const float d = v[k][e] - m;
+        q += d * d;
+      }
+    }
+  }
+  const float rs = rsqrtf(warp_sum(q) / h + 1e-5f);
+  if (lane == 0) {
+    mu_out[r] = m;
+    rstd_out[r] = rs;
+  }
+  T* yr = y + (int64_t)r * h;
+#pragma unroll
+  for (int k = 0; k < NV; ++k) {
+    const int c = (lane + 32 * k) * V;
+    if (c < h) {
+      float gg[V], bb[V], o[V];
+      Vec<T>::load(g + c, gg);
+      Vec<T>::load(b + c, bb);
+#pragma unroll
+      for (int e = 0; e < V; ++e) o[e] = (v[k][e] - m) * rs * gg[e] + bb[e];
+      Vec<T>::store(yr + c, o);
+    }
+  }
+}
+
 template <typename T, int LN_NT, int LN_MAXV>
 __global__ void __launch_bounds__(LN_NT) ln_fwd_k(const T* x, const T* g, const T* b, T* y, float* mu_out,
                                                    float* rstd_out, int h) {
@@ -187,74 +241,6 @@ __global__ void __launch_bounds__(LN_NT) ln_fwd_k(const T* x, const T* g, const 
 #pragma unroll
       for (int e = 0; e < V; ++e) o[e] = (v[k][e] - mu) * rs * gg[e] + bb[e];
       Vec<T>::store(yr + c, o);
-    }
-  }
-}
-
-constexpr int LNB_ROWS = 16;  // rows per CTA in backward (amortises dg/db atomics)
-
-template <typename T, int LN_NT, int LN_MAXV>
-__global__ void __launch_bounds__(LN_NT) ln_bwd_k(const T* dy, const T* x, const T* g, const float* mu,
-                                                   const float* rstd, const T* dres, T* dx, float* dg, float* db,
-                                                   int rows, int h) {
-  constexpr int V = Vec<T>::N;
-  __shared__ float red[33];
-  float gacc[LN_MAXV][V], bacc[LN_MAXV][V], gv[LN_MAXV][V];
-#pragma unroll
-  for (int k = 0; k < LN_MAXV; ++k) {
-    int c = (threadIdx.x + k * LN_NT) * V;
-#pragma unroll
-    for (int e = 0; e < V; ++e) gacc[k][e] = bacc[k][e] = 0.f;
-    if (c < h) Vec<T>::load(g + c, gv[k]);
-  }
-  const int r0 = blockIdx.x * LNB_ROWS;
-  for (int r = r0; r < min(rows, r0 + LNB_ROWS); ++r) {
-    const float m = mu[r], rs = rstd[r];
-    float xh[LN_MAXV][V], dyv[LN_MAXV][V];
-    float s1 = 0.f, s2 = 0.f;
-#pragma unroll
-    for (int k = 0; k < LN_MAXV; ++k) {
-      int c = (threadIdx.x + k * LN_NT) * V;
-      if (c < h) {
-        Vec<T>::load(x + (int64_t)r * h + c, xh[k]);
-        Vec<T>::load(dy + (int64_t)r * h + c, dyv[k]);
-#pragma unroll
-        for (int e = 0; e < V; ++e) {
-          xh[k][e] = (xh[k][e] - m) * rs;
-          float dh = dyv[k][e] * gv[k][e];
-          s1 += dh;
-          s2 += dh * xh[k][e];
-          gacc[k][e] += dyv[k][e] * xh[k][e];
-          bacc[k][e] += dyv[k][e];
-        }
-      }
-    }
-    const float c1 = block_sum<LN_NT>(s1, red) / h;
-    const float c2 = block_sum<LN_NT>(s2, red) / h;
-#pragma unroll
-    for (int k = 0; k < LN_MAXV; ++k) {
-      int c = (threadIdx.x + k * LN_NT) * V;
-      if (c < h) {
-        float o[V], rr[V];
-        if (dres) Vec<T>::load(dres + (int64_t)r * h + c, rr);
-#pragma unroll
-        for (int e = 0; e < V; ++e) {
-          o[e] = rs * (dyv[k][e] * gv[k][e] - c1 - xh[k][e] * c2);
-          if (dres) o[e] += rr[e];
-        }
-        Vec<T>::store(dx + (int64_t)r * h + c, o);
-      }
-    }
-  }
-#pragma unroll
-  for (int k = 0; k < LN_MAXV; ++k) {
-    int c = (threadIdx.x + k * LN_NT) * V;
-    if (c < h) {
-#pragma unroll
-      for (int e = 0; e < V; ++e) {
-        atomicAdd(dg + c + e, gacc[k][e]);
-        atomicAdd(db + c + e, bacc[k][e]);
-      }
     }
   }
 }
@@ -371,6 +357,116 @@ __global__ void loss_acc_k(const float* loss_rows, int rows, double* acc) {
 }
 
 // ----------------------------------------------------------- col sums
+// ---------------------------------------------- LayerNorm backward (v2)
+// dx only: one warp per row, two passes over the row (statistics, then dx),
+// 16-byte vectors, no atomics.  dg/db come from ln_param_grad_k.
+template <typename T>
+__global__ void __launch_bounds__(256) ln_bwd_dx_k(const T* __restrict__ dy, const T* __restrict__ x,
+                                                   const T* __restrict__ g, const float* __restrict__ mu,
+                                                   const float* __restrict__ rstd, const T* __restrict__ dres,
+                                                   T* __restrict__ dx, int rows, int h) {
+  constexpr int V = Vec<T>::N;
+  const int warps = blockDim.x / 32, lane = threadIdx.x % 32;
+  for (int r = blockIdx.x * warps + threadIdx.x / 32; r < rows; r += gridDim.x * warps) {
+    const float m = mu[r], rs = rstd[r];
+    const T* xr = x + (int64_t)r * h;
+    const T* dr = dy + (int64_t)r * h;
+    float s1 = 0.f, s2 = 0.f;
+#pragma unroll 4
+    for (int c = lane * V; c < h; c += 32 * V) {
+      float xv[V], dv[V], gv[V];
+      Vec<T>::load(xr + c, xv);
+      Vec<T>::load(dr + c, dv);
+      Vec<T>::load(g + c, gv);
+#pragma unroll
+      for (int e = 0; e < V; ++e) {
+        const float dh = dv[e] * gv[e];
+        s1 += dh;
+        s2 += dh * (xv[e] - m) * rs;
+      }
+    }
+    s1 = warp_sum(s1) / h;
+    s2 = warp_sum(s2) / h;
+    T* o = dx + (int64_t)r * h;
+    const T* rr = dres ? dres + (int64_t)r * h : nullptr;
+#pragma unroll 4
+    for (int c = lane * V; c < h; c += 32 * V) {
+      float xv[V], dv[V], gv[V], ov[V];
+      Vec<T>::load(xr + c, xv);
+      Vec<T>::load(dr + c, dv);
+      Vec<T>::load(g + c, gv);
+      if (rr) Vec<T>::load(rr + c, ov);
+#pragma unroll
+      for (int e = 0; e < V; ++e) {
+        const float val = rs * (dv[e] * gv[e] - s1 - (xv[e] - m) * rs * s2);
+        ov[e] = rr ? ov[e] + val : val;
+      }
+      Vec<T>::store(o + c, ov);
+    }
+  }
+}
+
+// Column reductions over `rows` rows, 16-byte vectors per thread, partial
+// sums in registers, CTA-level smem reduction, one atomic per column per
+// CTA.  mode 0: out0[c] += sum_r X[r,c].  mode 1 (LayerNorm parameters):
+// out0[c] += sum_r X[r,c] * (Y[r,c] - mu[r]) * rstd[r] (dgamma), out1[c] +=
+// sum_r X[r,c] (dbeta).
+constexpr int CS_THREADS = 256;
+constexpr int CS_COLV = 32;  // column vectors (of 8/4 elements) per CTA
+template <typename T, int MODE>
+__global__ void __launch_bounds__(CS_THREADS) colsum2_k(const T* __restrict__ X, int64_t ld, const T* __restrict__ Y,
+                                                        const float* __restrict__ mu, const float* __restrict__ rstd,
+                                                        int rows, int n, float* out0, float* out1, int rows_per_cta) {
+  constexpr int V = Vec<T>::N;
+  __shared__ float red0[CS_THREADS / CS_COLV][CS_COLV * V];
+  __shared__ float red1[MODE == 1 ? CS_THREADS / CS_COLV : 1][MODE == 1 ? CS_COLV * V : 1];
+  const int cv = threadIdx.x % CS_COLV;  // column vector within the CTA's slab
+  const int rg = threadIdx.x / CS_COLV;  // row group (CS_THREADS / CS_COLV groups)
+  const int c = (blockIdx.x * CS_COLV + cv) * V;
+  const int r0 = blockIdx.y * rows_per_cta, r1 = min(rows, r0 + rows_per_cta);
+  float a0[V], a1[V];
+#pragma unroll
+  for (int e = 0; e < V; ++e) a0[e] = a1[e] = 0.f;
+  if (c < n) {
+#pragma unroll 4
+    for (int r = r0 + rg; r < r1; r += CS_THREADS / CS_COLV) {
+      float xv[V];
+      Vec<T>::load(X + (int64_t)r * ld + c, xv);
+      if (MODE == 0) {
+#pragma unroll
+        for (int e = 0; e < V; ++e) a0[e] += xv[e];
+      } else {
+        float yv[V];
+        Vec<T>::load(Y + (int64_t)r * ld + c, yv);
+        const float m = mu[r], rs = rstd[r];
+#pragma unroll
+        for (int e = 0; e < V; ++e) {
+          a0[e] += xv[e] * (yv[e] - m) * rs;
+          a1[e] += xv[e];
+        }
+      }
+    }
+  }
+#pragma unroll
+  for (int e = 0; e < V; ++e) {
+    red0[rg][cv * V + e] = a0[e];
+    if (MODE == 1) red1[rg][cv * V + e] = a1[e];
+  }
+  __syncthreads();
+  for (int i = threadIdx.x; i < CS_COLV * V; i += CS_THREADS) {
+    const int col = blockIdx.x * CS_COLV * V + i;
+    if (col >= n) continue;
+    float t0 = 0.f, t1 = 0.f;
+#pragma unroll
+    for (int g2 = 0; g2 < CS_THREADS / CS_COLV; ++g2) {
+      t0 += red0[g2][i];
+      if (MODE == 1) t1 += red1[g2][i];
+    }
+    atomicAdd(out0 + col, t0);
+    if (MODE == 1) atomicAdd(out1 + col, t1);
+  }
+}
+
 template <typename T>
 __global__ void colsum_k(const T* X, int64_t ld, int rows, int n, float* out, int rows_per_block) {
   const int c = blockIdx.x * blockDim.x + threadIdx.x;
@@ -417,6 +513,13 @@ int check_launch(const char* what) {
   return MOBIUS_OK;
 }
 
+// rows per CTA so the column reduction launches >= ~4 waves of 148 SMs
+int colsum_rows_per_cta(int col_ctas, int rows) {
+  int rpc = 256;
+  while (rpc > 32 && (int64_t)col_ctas * ((rows + rpc - 1) / rpc) < 4 * 148) rpc /= 2;
+  return rpc;
+}
+
 template <typename T>
 bool aligned16(const T* p) {
   return (reinterpret_cast<uintptr_t>(p) & 15) == 0;
@@ -454,15 +557,34 @@ int embed_bwd(const int32_t* tok, const T* dx, float* dwte, float* dwpe, int mbs
 template <typename T>
 int layernorm_fwd(const T* x, const T* g, const T* b, T* y, float* mu, float* rstd, int rows, int h, cudaStream_t st) {
   MOBIUS_CHECK_ARG(h % Vec<T>::N == 0, "layernorm: unsupported h=%d", h);
-  LN_DISPATCH(ln_fwd_k, rows, x, g, b, y, mu, rstd, h);
+  const int nv = (h / Vec<T>::N + 31) / 32;  // vectors per lane
+  const unsigned blocks = (unsigned)((rows + 7) / 8);
+  if (nv <= 4)
+    ln_fwd_warp_k<T, 4><<<blocks, 256, 0, st>>>(x, g, b, y, mu, rstd, rows, h);
+  else if (nv <= 8)
+    ln_fwd_warp_k<T, 8><<<blocks, 256, 0, st>>>(x, g, b, y, mu, rstd, rows, h);
+  else
+    LN_DISPATCH(ln_fwd_k, rows, x, g, b, y, mu, rstd, h);
   return check_launch("layernorm_fwd");
 }
 template <typename T>
 int layernorm_bwd(const T* dy, const T* x, const T* g, const float* mu, const float* rstd, const T* dres, T* dx,
                   float* dg, float* db, int rows, int h, cudaStream_t st) {
   MOBIUS_CHECK_ARG(h % Vec<T>::N == 0, "layernorm: unsupported h=%d", h);
-  LN_DISPATCH(ln_bwd_k, (rows + LNB_ROWS - 1) / LNB_ROWS, dy, x, g, mu, rstd, dres, dx, dg, db, rows, h);
-  return check_launch("layernorm_bwd");
+  {
+    int blocks = (rows + 7) / 8;
+    if (blocks > 148 * 16) blocks = 148 * 16;
+    ln_bwd_dx_k<T><<<blocks, 256, 0, st>>>(dy, x, g, mu, rstd, dres, dx, rows, h);
+  }
+  int rc = check_launch("layernorm_bwd_dx");
+  if (rc) return rc;
+  {
+    const int gx = (h / Vec<T>::N + CS_COLV - 1) / CS_COLV;
+    const int rpc = colsum_rows_per_cta(gx, rows);
+    dim3 grid(gx, (rows + rpc - 1) / rpc);
+    colsum2_k<T, 1><<<grid, CS_THREADS, 0, st>>>(dy, h, x, mu, rstd, rows, h, dg, db, rpc);
+  }
+  return check_launch("layernorm_param_grad");
 }
 
 template <typename T>
@@ -493,6 +615,13 @@ int loss_accumulate(const float* loss_rows, int rows, double* acc, cudaStream_t 
 
 template <typename T>
 int colsum_accum(const T* X, int64_t ld, int rows, int n, float* out, cudaStream_t st) {
+  if (n % Vec<T>::N == 0 && ld % Vec<T>::N == 0 && aligned16(X)) {
+    const int gx = (n / Vec<T>::N + CS_COLV - 1) / CS_COLV;
+    const int rpc = colsum_rows_per_cta(gx, rows);
+    dim3 grid(gx, (rows + rpc - 1) / rpc);
+    colsum2_k<T, 0><<<grid, CS_THREADS, 0, st>>>(X, ld, (const T*)nullptr, nullptr, nullptr, rows, n, out, nullptr, rpc);
+    return check_launch("colsum");
+  }
   const int rpb = 128;
   dim3 grid((n + 255) / 256, (rows + rpb - 1) / rpb);
   colsum_k<T><<<grid, 256, 0, st>>>(X, ld, rows, n, out, rpb);

@@ -4,6 +4,7 @@
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
+#include <cstdlib>
 #include <vector>
 
 #include "../../include/mobius_kernels.h"
@@ -35,7 +36,12 @@ uint8_t* ws_get(int64_t bytes) {
 }
 int sync_rc(int rc) {
   if (rc) return rc;
-  cudaError_t e = cudaDeviceSynchronize();
+  static int nosync = -1;  // MOBIUS_KT_NOSYNC=1: timing loops (launch-only, errors via cudaGetLastError)
+  if (nosync < 0) {
+    const char* v = getenv("MOBIUS_KT_NOSYNC");
+    nosync = (v && v[0] == '1') ? 1 : 0;
+  }
+  cudaError_t e = nosync ? cudaGetLastError() : cudaDeviceSynchronize();
   if (e != cudaSuccess) MOBIUS_FAIL(MOBIUS_ECUDA, "kernel failed: %s", cudaGetErrorString(e));
   return MOBIUS_OK;
 }

@@ -1,4 +1,5 @@
 import sys, os
+os.environ.setdefault('MOBIUS_KT_NOSYNC', '1')
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
 from paper_conf_asplos_fengxtwls23_b200 import BF16, kt

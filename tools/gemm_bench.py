@@ -1,6 +1,7 @@
 """Time the tcgen05 GEMM / flash kernels at the 1.5B block shapes (kernel-level
 perf loop; not part of the bench contract)."""
 import sys, os
+os.environ.setdefault('MOBIUS_KT_NOSYNC', '1')
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
 from paper_conf_asplos_fengxtwls23_b200 import BF16, kt
