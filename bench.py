@@ -46,6 +46,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=3)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="1.5b")
+    ap.add_argument("--layers", type=int, default=0, help="override the block count (shape checks only)")
     ap.add_argument("--microbatches", type=int, default=0, help="M per GPU (default 16 for 1.5b)")
     ap.add_argument("--cap-gib", type=float, default=1.0, help="HBM stage-ring cap G per GPU")
     ap.add_argument("--impl", default="mobius", choices=["mobius", "reference"])
@@ -133,18 +134,25 @@ def cpu_oracle_sample(c: synth.GPTConfig, tokens_per_step: int, budget_s: float 
             for name, shape, init in c1.layer_specs(c1.n_layers + 1)}
     x = rng.standard_normal((s, h)).astype(np.float32)
     tok = rng.integers(0, V, size=(1, s + 1))
-    t0 = time.perf_counter()
-    y, cache = om.block_fwd(c1, blk, x, 1)
-    om.block_bwd(c1, blk, y, cache, 1)
-    t_block = time.perf_counter() - t0
-    t0 = time.perf_counter()
-    om.head_fwd_bwd(c1, head, x, tok[:, 1:], s)
-    t_head = time.perf_counter() - t0
+    tb, th = [], []
+    t_start = time.perf_counter()
+    while True:  # bounded sample: repeat until ~budget_s of CPU work, take medians
+        t0 = time.perf_counter()
+        y, cache = om.block_fwd(c1, blk, x, 1)
+        om.block_bwd(c1, blk, y, cache, 1)
+        tb.append(time.perf_counter() - t0)
+        t0 = time.perf_counter()
+        om.head_fwd_bwd(c1, head, x, tok[:, 1:], s)
+        th.append(time.perf_counter() - t0)
+        if time.perf_counter() - t_start > budget_s or len(tb) >= 50:
+            break
+    t_block, t_head = float(np.median(tb)), float(np.median(th))
     t_step = (c.n_layers * t_block + t_head) * tokens_per_step / s
     return {"value": tokens_per_step / t_step, "unit": "tokens/s", "cores": cores, "kind": "oracle",
-            "sample": f"numpy fp32 oracle: 1 block fwd+bwd ({t_block:.2f}s) + LM head fwd+bwd ({t_head:.2f}s) "
-                      f"at mbs=1 s={s} h={h} V={V}, extrapolated x{c.n_layers} blocks to the step's "
-                      f"{tokens_per_step} tokens (host AdamW and transfers not included)"}
+            "sample": f"numpy fp32 oracle: {len(tb)} x (1 block fwd+bwd, median {t_block:.2f}s + LM head fwd+bwd, "
+                      f"median {t_head:.2f}s) at mbs=1 s={s} h={h} V={V} (~{budget_s:.0f}s of CPU work), "
+                      f"extrapolated x{c.n_layers} blocks to the step's {tokens_per_step} tokens "
+                      f"(host AdamW and transfers not included)"}
 
 
 def run_reference(args, rank, world):
@@ -155,10 +163,10 @@ def run_reference(args, rank, world):
     tps = M * c.micro_batch * c.seq_len
     vals = []
     for _ in range(args.warmup):
-        cpu_oracle_sample(c, tps)
+        cpu_oracle_sample(c, tps, budget_s=3.0)
     t0 = time.perf_counter()
     for _ in range(args.steps):
-        vals.append(cpu_oracle_sample(c, tps))
+        vals.append(cpu_oracle_sample(c, tps, budget_s=10.0))
     wall = time.perf_counter() - t0
     v = float(np.median([x["value"] for x in vals]))
     cb = dict(vals[-1])
@@ -199,6 +207,9 @@ def run_mobius(args, rank, world, local):
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     c = synth.CONFIGS[args.config]
+    if args.layers:
+        import dataclasses
+        c = dataclasses.replace(c, n_layers=args.layers)
     M = (args.microbatches or 16) * world
     cfg = model_cfg(c.n_layers, c.hidden, c.n_heads, c.seq_len, c.vocab, c.micro_batch, dtype=BF16)
     G = int(args.cap_gib * GiB)
