@@ -203,9 +203,19 @@ def run_mobius(args, rank, world, local):
     from paper_conf_asplos_fengxtwls23_b200 import (BF16, FLAG_TIMING, MobiusContext, make_topology,
                                                     mobius_discover_topology, mobius_plan, mobius_profile,
                                                     model_cfg)
+    # MOBIUS_BENCH_SAME_GPU=1: every rank on device 0 (checks the N>1 code
+    # path on a 1-GPU box; ranks time-slice the GPU, numbers are not scaling
+    # numbers).  Plumbing then uses gloo (NCCL rejects duplicate GPUs).
+    same_gpu = os.environ.get("MOBIUS_BENCH_SAME_GPU") == "1"
+    if same_gpu:
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if same_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    pg_dev = "cpu" if same_gpu else "cuda"
     c = synth.CONFIGS[args.config]
     if args.layers:
         import dataclasses
@@ -214,16 +224,31 @@ def run_mobius(args, rank, world, local):
     cfg = model_cfg(c.n_layers, c.hidden, c.n_heads, c.seq_len, c.vocab, c.micro_batch, dtype=BF16)
     G = int(args.cap_gib * GiB)
     # profile (layer similarity) and plan (MIP + cross mapping)
+    t_prof0 = time.perf_counter()
     prof = mobius_profile(cfg, local)
+    prof_s = time.perf_counter() - t_prof0
     h2d_gbps = measure_h2d_GBps(torch)
     topo = mobius_discover_topology()
     groups = [topo.group[i] for i in range(topo.n_gpus)][:world]
     if len(groups) < world:
         groups = list(range(world))
+    # SPMD contract: every rank must plan from identical inputs -> rank 0's
+    # profile, link bandwidth and topology are broadcast (measured timings
+    # differ slightly per GPU, which would yield different partitions)
+    shared = [[(p.t_fwd_ns, p.t_bwd_ns, p.mem_fwd, p.mem_bwd, p.xfer_fwd, p.xfer_bwd, p.act_out) for p in prof],
+              h2d_gbps, groups]
+    if world > 1:
+        dist.broadcast_object_list(shared, src=0)
+        from paper_conf_asplos_fengxtwls23_b200._lib import LayerProfile
+        prof = [LayerProfile(*x) for x in shared[0]]
+        h2d_gbps, groups = shared[1], shared[2]
     t = make_topology(groups, host_bw_Bps=int(h2d_gbps * 1e9), p2p_bw_Bps=int(700e9))
     t0 = time.perf_counter()
     plan = mobius_plan(prof, world, G, M, t)
     plan_s = time.perf_counter() - t0
+    if world > 1:
+        from paper_conf_asplos_fengxtwls23_b200 import dist as mdist
+        assert mdist.check_same_plan(plan), "ranks derived different plans"
     ctx = MobiusContext(cfg, plan, rank=rank, world=world, device=local, seed=1234, flags=FLAG_TIMING)
     if world > 1:
         blobs = [None] * world
@@ -242,13 +267,18 @@ def run_mobius(args, rank, world, local):
     def max_over_ranks(x):
         if world == 1:
             return x
-        tt = torch.tensor([x], dtype=torch.float64, device="cuda")
+        tt = torch.tensor([x], dtype=torch.float64, device=pg_dev)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         return float(tt.item())
 
+    dbg = os.environ.get("MOBIUS_DEBUG") == "1"
+    if dbg:
+        print(f"[rank {rank}] ctx ready, K={plan.n_stages}", file=sys.stderr, flush=True)
     loss = float("nan")
-    for _ in range(args.warmup):
+    for w in range(args.warmup):
         loss = ctx.step_device(tok_dev, M)
+        if dbg:
+            print(f"[rank {rank}] warmup step {w} loss {loss}", file=sys.stderr, flush=True)
     sampler = ClockSampler(local)
     sampler.start()
     barrier()
@@ -304,6 +334,7 @@ def run_mobius(args, rank, world, local):
                        "n_stages": plan.n_stages, "stage_layers": [plan.stage_first_layer[j + 1] - plan.stage_first_layer[j]
                                                                    for j in range(plan.n_stages)],
                        "gpu_perm": [plan.gpu_perm[g] for g in range(world)], "plan_s": plan_s,
+                       "profile_s": prof_s, "plan_exhaustive": bool(plan.exhaustive),
                        "l2": "inputs larger than L2: every stage (3.1 GB bf16 total) streams from host DRAM each step"},
             "loss": loss,
             "e2e": e2e,

@@ -921,10 +921,36 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
 struct ExportBlob {
   uint32_t magic;
   int32_t rank;
+  uint64_t plan_digest;  // every rank must run the identical plan (SPMD contract)
   cudaIpcMemHandle_t handle;
   int64_t off_ckpt, off_gslot, off_fflag, off_bflag, slot_bytes;
   int32_t n_local, M;
 };
+
+static uint64_t plan_digest(const mobius_ctx* ctx) {
+  uint64_t h = 1469598103934665603ull;  // FNV-1a over the plan and model shape
+  auto mix = [&](int64_t v) {
+    for (int i = 0; i < 8; ++i) {
+      h ^= (uint64_t)((v >> (8 * i)) & 0xff);
+      h *= 1099511628211ull;
+    }
+  };
+  const mobius_plan_t& p = ctx->plan;
+  mix(p.n_stages);
+  mix(p.n_gpus);
+  mix(ctx->max_M);
+  for (int j = 0; j <= p.n_stages; ++j) mix(p.stage_first_layer[j]);
+  for (int j = 0; j < p.n_stages; ++j) mix(p.stage_gpu[j]);
+  const mobius_model_cfg& c = ctx->cfg;
+  mix(c.n_layers);
+  mix(c.hidden);
+  mix(c.n_heads);
+  mix(c.seq_len);
+  mix(c.vocab);
+  mix(c.micro_batch);
+  mix(c.dtype);
+  return h;
+}
 
 extern "C" int mobius_dist_export(mobius_ctx* ctx, void* buf, size_t cap, size_t* len) {
   int rc = check_ctx(ctx);
@@ -934,6 +960,7 @@ extern "C" int mobius_dist_export(mobius_ctx* ctx, void* buf, size_t cap, size_t
   std::memset(&b, 0, sizeof(b));
   b.magic = 0x4d4f4249;
   b.rank = ctx->dist.rank;
+  b.plan_digest = plan_digest(ctx);
   CU(cudaSetDevice(ctx->dist.device));
   CU(cudaIpcGetMemHandle(&b.handle, ctx->arena));
   b.off_ckpt = ctx->off_ckpt;
@@ -959,6 +986,8 @@ extern "C" int mobius_dist_connect(mobius_ctx* ctx, const void* all, size_t blob
     ExportBlob b;
     std::memcpy(&b, (const char*)all + r * blob_len, sizeof(b));
     MOBIUS_CHECK_ARG(b.magic == 0x4d4f4249 && b.rank == r, "blob %d is not a mobius export", r);
+    MOBIUS_CHECK_ARG(b.plan_digest == plan_digest(ctx), "rank %d runs a different plan / config than rank %d", r,
+                     ctx->dist.rank);
     PeerInfo& p = ctx->peers[r];
     p.rank = r;
     p.handle = b.handle;
