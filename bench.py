@@ -52,6 +52,7 @@ def parse():
     ap.add_argument("--impl", default="mobius", choices=["mobius", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-keep", action="store_true", help="always recompute (no kept activations)")
     return ap.parse_args()
 
 
@@ -200,7 +201,7 @@ def measure_h2d_GBps(torch, nbytes=512 << 20):
 def run_mobius(args, rank, world, local):
     import torch
     import torch.distributed as dist
-    from paper_conf_asplos_fengxtwls23_b200 import (BF16, FLAG_TIMING, MobiusContext, make_topology,
+    from paper_conf_asplos_fengxtwls23_b200 import (BF16, FLAG_KEEP_ACTS, FLAG_TIMING, MobiusContext, make_topology,
                                                     mobius_discover_topology, mobius_plan, mobius_profile,
                                                     model_cfg)
     # MOBIUS_BENCH_SAME_GPU=1: every rank on device 0 (checks the N>1 code
@@ -249,7 +250,8 @@ def run_mobius(args, rank, world, local):
     if world > 1:
         from paper_conf_asplos_fengxtwls23_b200 import dist as mdist
         assert mdist.check_same_plan(plan), "ranks derived different plans"
-    ctx = MobiusContext(cfg, plan, rank=rank, world=world, device=local, seed=1234, flags=FLAG_TIMING)
+    flags = FLAG_TIMING | (0 if args.no_keep else FLAG_KEEP_ACTS)
+    ctx = MobiusContext(cfg, plan, rank=rank, world=world, device=local, seed=1234, flags=flags)
     if world > 1:
         blobs = [None] * world
         dist.all_gather_object(blobs, ctx.dist_export())
@@ -352,6 +354,8 @@ def run_mobius(args, rank, world, local):
             "breakdown_ms": {"gemm": st.gemm_ns / 1e6, "attention": st.attn_ns / 1e6, "elementwise": st.elem_ns / 1e6,
                              "device_step": st.device_step_ns / 1e6, "host_update_total": st.host_update_ns / 1e6,
                              "update_tail": st.update_tail_ns / 1e6},
+            "memory": {"arena_GB": st.arena_bytes / 1e9, "ring_GB": st.ring_bytes / 1e9,
+                       "pinned_host_GB": st.pinned_bytes / 1e9, "recompute": bool(st.recompute)},
             "gpu_launches": int(sum(s.kernel_launches for s in stats)),
             "clocks": clocks,
         }

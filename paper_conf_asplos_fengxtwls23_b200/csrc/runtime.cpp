@@ -27,6 +27,7 @@
 #include <chrono>
 #include <cmath>
 #include <condition_variable>
+#include <cstdlib>
 #include <cstring>
 #include <deque>
 #include <memory>
@@ -164,6 +165,9 @@ struct mobius_ctx {
   int64_t slot_bytes = 0;
   int max_M = 0;
   uint8_t* acts_base = nullptr;   // per-block saved activations (recompute)
+  uint8_t* keep_pool = nullptr;   // kept activations (no recompute) for some stages
+  int64_t keep_bytes = 0;
+  std::vector<int64_t> keep_off;  // per local stage: offset into keep_pool, -1 if not kept
   int64_t acts_bytes = 0;
   int max_blocks = 0;
   uint8_t* xs_base = nullptr;     // [max_blocks+1] x buffers [T,h]
@@ -354,6 +358,20 @@ struct StepRunner {
     return tptr<T>(b + pi.off_gslot + ((int64_t)pv.ord * pi.M + m) * pi.slot_bytes);
   }
 
+  bool kept(int ls) const { return ctx->keep_off[ls] >= 0; }
+  uint8_t* keep_entry(int ls, int m, int bi) {
+    const StageDesc& st = ctx->all[ctx->mine[ls]];
+    const int64_t e = ctx->acts_bytes + ctx->slot_bytes;
+    return ctx->keep_pool + ctx->keep_off[ls] + ((int64_t)m * st.n_blocks + bi) * e;
+  }
+  // input x of block bi of a kept stage (block 0 of an embed stage too)
+  T* keep_x(int ls, int m, int bi) { return tptr<T>(keep_entry(ls, m, bi) + ctx->acts_bytes); }
+  BlockActs<T> keep_acts(int ls, int m, int bi) {
+    BlockActs<T> a;
+    carve_block_acts<T>(ctx->sh, keep_entry(ls, m, bi), a);
+    return a;
+  }
+
   const T* stage_w(int res, const StageDesc& st, int layer) {
     return tptr<T>(ctx->ring + ctx->loads[res].base) + st.layer_off[layer - st.first];
   }
@@ -439,7 +457,7 @@ struct StepRunner {
       if (st.n_blocks == 0 && !last_stage)
         out = fwd_dest(st.j, m, &flag);
       else
-        out = xbuf(0);
+        out = kept(ls) ? keep_x(ls, m, 0) : xbuf(0);
       RC(embed_layer_fwd<T>(sh, stage_w(res, st, 0), tok(m), out, s));
       if (flag) { RC(flag_set(flag, (int)seq, s)); ++ctx->launches_step; }
       x = out;
@@ -454,6 +472,16 @@ struct StepRunner {
       if (li == 0) continue;
       const bool last_block = (bi == st.n_blocks - 1);
       int* flag = nullptr;
+      if (kept(ls)) {  // keep every activation of this stage for its backward (no recompute)
+        T* y = last_block ? fwd_dest(st.j, m, &flag) : keep_x(ls, m, bi + 1);
+        BlockActs<T> ka = keep_acts(ls, m, bi);
+        ka.x = x;
+        RC(block_fwd<T>(sh, stage_w(res, st, li), ka, y, sc, s));
+        if (flag) { RC(flag_set(flag, (int)seq, s)); ++ctx->launches_step; }
+        x = y;
+        ++bi;
+        continue;
+      }
       T* y = last_block ? fwd_dest(st.j, m, &flag) : xbuf(1 + (bi % 2));
       acts[0].x = x;
       RC(block_fwd<T>(sh, stage_w(res, st, li), acts[0], y, sc, s));
@@ -470,22 +498,32 @@ struct StepRunner {
     const Shape& sh = ctx->sh;
     cudaStream_t s = ctx->s_comp;
     tr(1, st.j, m);
-    // recompute the stage forward from the checkpoint (a5/a7)
     const T* x;
-    if (st.has_embed) {
-      RC(embed_layer_fwd<T>(sh, stage_w(res, st, 0), tok(m), xbuf(0), s));
-      x = xbuf(0);
-    } else {
-      x = ckpt_slot(ls, m);
-    }
     int bi = 0;
-    for (int li = st.first; li < st.last; ++li) {
-      if (li == 0 || li == ctx->cfg.n_layers + 1) continue;
-      T* y = xbuf(bi + 1);
-      acts[bi].x = x;
-      RC(block_fwd<T>(sh, stage_w(res, st, li), acts[bi], y, sc, s));
-      x = y;
-      ++bi;
+    std::vector<BlockActs<T>> kacts;
+    if (kept(ls)) {  // activations kept from F_{j,m}: no recompute
+      for (int b = 0; b < st.n_blocks; ++b) {
+        kacts.push_back(keep_acts(ls, m, b));
+        kacts.back().x = (b == 0) ? (st.has_embed ? keep_x(ls, m, 0) : ckpt_slot(ls, m)) : keep_x(ls, m, b);
+      }
+      bi = st.n_blocks;
+      x = nullptr;  // the head is never in a kept stage
+    } else {
+      // recompute the stage forward from the checkpoint (a5/a7)
+      if (st.has_embed) {
+        RC(embed_layer_fwd<T>(sh, stage_w(res, st, 0), tok(m), xbuf(0), s));
+        x = xbuf(0);
+      } else {
+        x = ckpt_slot(ls, m);
+      }
+      for (int li = st.first; li < st.last; ++li) {
+        if (li == 0 || li == ctx->cfg.n_layers + 1) continue;
+        T* y = xbuf(bi + 1);
+        acts[bi].x = x;
+        RC(block_fwd<T>(sh, stage_w(res, st, li), acts[bi], y, sc, s));
+        x = y;
+        ++bi;
+      }
     }
     // gradient w.r.t. the stage output
     const T* dy;
@@ -517,7 +555,7 @@ struct StepRunner {
         pp ^= 1;
       }
       float* G = ctx->grad_acc + st.layer_off[li - st.first];
-      RC(block_bwd<T>(sh, stage_w(res, st, li), acts[bi], dy, dx, G, sc, s));
+      RC(block_bwd<T>(sh, stage_w(res, st, li), kept(ls) ? kacts[bi] : acts[bi], dy, dx, G, sc, s));
       if (flag) { RC(flag_set(flag, (int)seq, s)); ++ctx->launches_step; }
       dy = dx;
     }
@@ -678,7 +716,7 @@ int do_step(mobius_ctx* ctx, const int32_t* tok_dev, int M, float* loss_out) {
     }
   }
   S.kernel_launches = ctx->launches_step + g_kernel_launches;
-  S.arena_bytes = ctx->arena_bytes;
+  S.arena_bytes = ctx->arena_bytes + ctx->keep_bytes;
   S.ring_bytes = ctx->ring_bytes;
   int64_t pinned = 0;
   for (int ls = 0; ls < (int)ctx->mine.size(); ++ls) pinned += 2 * ctx->all[ctx->mine[ls]].n_params * ctx->esz;
@@ -686,7 +724,10 @@ int do_step(mobius_ctx* ctx, const int32_t* tok_dev, int M, float* loss_out) {
   S.host_update_ns = ctx->upd_ns;
   S.update_tail_ns = t1 - t_gpu_done;
   S.n_local_stages = (int)ctx->mine.size();
-  S.recompute = 1;
+  S.recompute = 0;
+  for (int ls = 0; ls < (int)ctx->mine.size(); ++ls)
+    if (ctx->keep_off[ls] < 0 && ctx->mine[ls] != ctx->plan.n_stages - 1 && ctx->all[ctx->mine[ls]].n_blocks > 0)
+      S.recompute = 1;  // block activations of this stage are recomputed in backward
   ctx->upd_ns = 0;
   ctx->step_count++;
   return MOBIUS_OK;
@@ -825,6 +866,29 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
     CU(cudaMalloc(&ctx->arena, ctx->arena_bytes));
     CU(cudaMemset(ctx->arena + o_gacc, 0, max_params * 4));
     ctx->ring = ctx->arena;
+    // kept activations (reading #17: keep instead of recompute when they fit):
+    // whole local stages, latest first, within the free HBM minus a margin
+    ctx->keep_off.assign(n, -1);
+    if (dist->flags & MOBIUS_FLAG_KEEP_ACTS) {
+      size_t fr = 0, tot = 0;
+      CU(cudaMemGetInfo(&fr, &tot));
+      int64_t budget = (int64_t)fr - (int64_t)6 * (1LL << 30);
+      if (const char* e = getenv("MOBIUS_KEEP_GIB")) budget = std::min<int64_t>(budget, (int64_t)(atof(e) * (1LL << 30)));
+      const int64_t entry = ctx->acts_bytes + ctx->slot_bytes;
+      int64_t off = 0;
+      for (int k = n - 1; k >= 0; --k) {
+        const StageDesc& st = ctx->all[ctx->mine[k]];
+        if (st.j == plan->n_stages - 1 || st.n_blocks == 0) continue;  // last stage: F is folded into B
+        const int64_t need = al256((int64_t)M * st.n_blocks * entry);
+        if (off + need > budget) continue;
+        ctx->keep_off[k] = off;
+        off += need;
+      }
+      if (off > 0) {
+        CU(cudaMalloc(&ctx->keep_pool, off));
+        ctx->keep_bytes = off;
+      }
+    }
     ctx->grad_acc = reinterpret_cast<float*>(ctx->arena + o_gacc);
     ctx->grad_stage = ctx->arena + o_gstage;
     ctx->ckpt = ctx->arena + ctx->off_ckpt;
@@ -1111,6 +1175,7 @@ extern "C" void mobius_destroy(mobius_ctx* ctx) {
   if (ctx->h_loss) cudaFreeHost(ctx->h_loss);
   if (ctx->h_tokens) cudaFreeHost(ctx->h_tokens);
   if (ctx->arena) cudaFree(ctx->arena);
+  if (ctx->keep_pool) cudaFree(ctx->keep_pool);
   if (ctx->s_comp) cudaStreamDestroy(ctx->s_comp);
   if (ctx->s_h2d) cudaStreamDestroy(ctx->s_h2d);
   if (ctx->s_d2h) cudaStreamDestroy(ctx->s_d2h);

@@ -134,3 +134,31 @@ def test_seeded_init_runs():
     loss = ctx.step(synth.gen_tokens(c, 2))
     ctx.close()
     assert abs(loss - np.log(c.vocab)) < 0.5
+
+
+@pytest.mark.parametrize("dtype,tol", [(BF16, 2e-2), (F32, 1e-4)])
+@pytest.mark.parametrize("sizes", [(3, 3), (1, 2, 1, 2), (2, 2, 2)])
+def test_tiny_step_keep_acts(dtype, tol, sizes):
+    """MOBIUS_FLAG_KEEP_ACTS (reading #17: keep activations instead of
+    recomputing when they fit): same loss / gradients, no recompute."""
+    from paper_conf_asplos_fengxtwls23_b200 import FLAG_KEEP_ACTS
+    c = synth.TINY
+    M = 2
+    w = synth.perturb_norm_params(c, synth.gen_params(c), scale=0.1)
+    if dtype == BF16:
+        w = synth.round_bf16(w)
+    tok = synth.gen_tokens(c, M)
+    cap = (4 * MiB) * (2 if dtype == F32 else 1)
+    ctx = MobiusContext(mk_cfg(c, dtype), plan_from_sizes(sizes, 1, M, hbm_cap_bytes=cap), init_params=w,
+                        flags=FLAG_KEEP_ACTS)
+    loss = ctx.step(tok)
+    g = ctx.read_grads(c.n_params)
+    st = ctx.stats()
+    loss2 = ctx.step(tok)
+    ctx.close()
+    assert st.recompute == 0
+    ref_loss, ref_g = om.reference_loss_and_grads(c, w, tok)
+    assert abs(loss - ref_loss) / abs(ref_loss) < tol
+    errs = tensor_errs(c, g, ref_g)
+    assert max(errs.values()) < tol, errs
+    assert np.isfinite(loss2)
