@@ -396,8 +396,13 @@ struct Cfg2 {
   static constexpr int SMEM = 1024 + STAGES * STAGE_BYTES + 256;
 };
 
-template <int BN, bool A_MN, bool B_MN>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
+// NP pairs per cluster (cluster = 2*NP CTAs along x).  Pairs of one cluster
+// compute horizontally adjacent 256 x BN tiles (same rows): with NP = 2 the
+// A tile is loaded once per cluster - each CTA loads half of its 128 A rows
+// and TMA-multicasts them to its counterpart in the other pair - cutting the
+// L2 -> SM operand traffic by a quarter.
+template <int BN, bool A_MN, bool B_MN, int NP>
+__global__ void __launch_bounds__(NUM_THREADS, 1)
     gemm_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, const Params p) {
   using C = Cfg2<BN>;
   constexpr int BM2 = 256;
@@ -414,19 +419,21 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
   const int warp = threadIdx.x / 32;
   const int lane = threadIdx.x % 32;
   const uint32_t rank = ptx::cluster_ctarank();
-  const bool leader = rank == 0;
-  const int cl = blockIdx.x / 2, ncl = gridDim.x / 2;
+  const uint32_t pair = rank >> 1, r2 = rank & 1;
+  const bool leader = r2 == 0;  // MMA-issuing CTA of this pair
+  const int cl = blockIdx.x / (2 * NP), ncl = gridDim.x / (2 * NP);
+  const int tiles_n2 = (p.tiles_n + NP - 1) / NP;  // column groups of NP tiles
 
   if (warp == 0 && lane == 0) {
     ptx::tma_prefetch_desc(&tmA);
     ptx::tma_prefetch_desc(&tmB);
     for (int s = 0; s < C::STAGES; ++s) {
       ptx::mbar_init(&full[s], 1);
-      ptx::mbar_init(&empty[s], 1);
+      ptx::mbar_init(&empty[s], NP);  // one commit per pair that reads this CTA's slot
     }
     for (int a = 0; a < 2; ++a) {
       ptx::mbar_init(&tfull[a], 1);
-      ptx::mbar_init(&tempty[a], 8);  // 4 epilogue warps x 2 CTAs (leader's copy is the one used)
+      ptx::mbar_init(&tempty[a], 8);  // 4 epilogue warps x 2 CTAs of the pair (leader's copy)
     }
     ptx::fence_mbar_init();
   }
@@ -435,34 +442,53 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
   ptx::cluster_sync();
   ptx::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
-  const int total = p.nb1 * p.nb2 * p.tiles_m * p.tiles_n;
+  const int total = p.tiles_m * tiles_n2;
+
+  auto tile_of = [&](int t, int& mt, int& nt) {  // grouped along M for L2 reuse
+    constexpr int GROUP = 8;
+    const int span = GROUP * tiles_n2;
+    const int g = t / span, first_m = g * GROUP;
+    const int gm = min(GROUP, p.tiles_m - first_m);
+    const int rr = t - g * span;
+    mt = first_m + rr % gm;
+    nt = (rr / gm) * NP + (int)pair;
+  };
 
   if (warp == 0) {
-    if (lane == 0) {  // TMA producer (both CTAs)
+    if (lane == 0) {  // TMA producer (every CTA)
       int stage = 0;
       uint32_t phase = 0;
+      const uint16_t amask = (uint16_t)((1u << r2) | (NP == 2 ? (1u << (r2 + 2)) : 0u));
       for (int t = cl; t < total; t += ncl) {
-        int b1, b2, mt, nt;
-        decode_tile(p, t, b1, b2, mt, nt);
-        const int m0 = mt * BM2 + (int)rank * 128, n0 = nt * BN + (int)rank * (BN / 2);
+        int mt, nt;
+        tile_of(t, mt, nt);
+        const int m0 = mt * BM2 + (int)r2 * 128, n0 = nt * BN + (int)r2 * (BN / 2);
         for (int kb = 0; kb < p.num_kb; ++kb) {
           ptx::mbar_wait_cluster(&empty[stage], phase ^ 1);
           if (leader) ptx::mbar_arrive_expect_tx(&full[stage], 2 * C::STAGE_BYTES);
           uint8_t* a = smA + stage * C::A_BYTES;
           uint8_t* b = smB + stage * C::B_BYTES;
           const int k0 = kb * BK;
-          if (A_MN) {
+          if (NP == 1) {
+            if (A_MN) {
 #pragma unroll
-            for (int i = 0; i < 2; ++i) ptx::tma_load_4d_2sm(a + i * 8192, &tmA, &full[stage], m0 + 64 * i, k0, b2, b1);
-          } else {
-            ptx::tma_load_4d_2sm(a, &tmA, &full[stage], k0, m0, b2, b1);
+              for (int i = 0; i < 2; ++i) ptx::tma_load_4d_2sm(a + i * 8192, &tmA, &full[stage], m0 + 64 * i, k0, 0, 0);
+            } else {
+              ptx::tma_load_4d_2sm(a, &tmA, &full[stage], k0, m0, 0, 0);
+            }
+          } else {  // this pair loads half h = pair of the 128 A rows and multicasts it
+            const int h = (int)pair;
+            if (A_MN)
+              ptx::tma_load_4d_2sm_mc(a + h * 8192, &tmA, &full[stage], amask, m0 + 64 * h, k0, 0, 0);
+            else
+              ptx::tma_load_4d_2sm_mc(a + h * 8192, &tmA, &full[stage], amask, k0, m0 + 64 * h, 0, 0);
           }
           if (B_MN) {
 #pragma unroll
             for (int i = 0; i < BN / 128; ++i)
-              ptx::tma_load_4d_2sm(b + i * 8192, &tmB, &full[stage], n0 + 64 * i, k0, b2, b1);
+              ptx::tma_load_4d_2sm(b + i * 8192, &tmB, &full[stage], n0 + 64 * i, k0, 0, 0);
           } else {
-            ptx::tma_load_4d_2sm(b, &tmB, &full[stage], k0, n0, b2, b1);
+            ptx::tma_load_4d_2sm(b, &tmB, &full[stage], k0, n0, 0, 0);
           }
           if (++stage == C::STAGES) {
             stage = 0;
@@ -472,8 +498,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
       }
     }
   } else if (warp == 1) {
-    if (leader && lane == 0) {  // MMA issuer (leader only)
+    if (leader && lane == 0) {  // MMA issuer (pair leader)
       constexpr uint32_t IDESC = ptx::idesc_bf16(BM2, BN, A_MN ? 1 : 0, B_MN ? 1 : 0);
+      const uint16_t all_mask = (uint16_t)((1u << (2 * NP)) - 1);
+      const uint16_t pair_mask = (uint16_t)(3u << (2 * pair));
       int stage = 0;
       uint32_t phase = 0;
       int acc = 0;
@@ -495,13 +523,15 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
                                : ptx::sdesc_sw128(b_base + k * 32, 16, 1024);
             ptx::mma_bf16_2sm(tmem_d, ad, bd, IDESC, (kb > 0 || k > 0) ? 1u : 0u);
           }
-          ptx::mma_commit_2sm(&empty[stage], 0x3);  // frees the slot in both CTAs
+          // the slot may be refilled by this pair's producers and (A halves)
+          // by the other pair's: free it in every CTA of the cluster
+          ptx::mma_commit_2sm(&empty[stage], all_mask);
           if (++stage == C::STAGES) {
             stage = 0;
             phase ^= 1;
           }
         }
-        ptx::mma_commit_2sm(&tfull[acc], 0x3);      // accumulator ready in both CTAs
+        ptx::mma_commit_2sm(&tfull[acc], pair_mask);  // accumulator ready in both CTAs of the pair
         if (++acc == 2) {
           acc = 0;
           aphase ^= 1;
@@ -509,18 +539,18 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(NUM_THREADS, 1)
       }
     }
   } else {
-    // epilogue (warps 2..5) of both CTAs: rows mt*256 + rank*128 + lane quadrant
+    // epilogue (warps 2..5): rows mt*256 + r2*128 + lane quadrant
     const int q = warp & 3;
-    const uint32_t tempty_leader = ptx::mapa_shared(ptx::smem_u32(&tempty[0]), 0);
+    const uint32_t tempty_leader = ptx::mapa_shared(ptx::smem_u32(&tempty[0]), pair * 2);
     int acc = 0;
     uint32_t aphase = 0;
     for (int t = cl; t < total; t += ncl) {
-      int b1, b2, mt, nt;
-      decode_tile(p, t, b1, b2, mt, nt);
+      int mt, nt;
+      tile_of(t, mt, nt);
       ptx::mbar_wait_cluster(&tfull[acc], aphase);
       ptx::tc_fence_after();
-      epi_tile<BN>(p, tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN, mt * BM2 + (int)rank * 128 + q * 32 + lane,
-                   b1, b2, nt);
+      epi_tile<BN>(p, tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN, mt * BM2 + (int)r2 * 128 + q * 32 + lane,
+                   0, 0, nt);
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive_cluster(tempty_leader + acc * 8);
@@ -603,19 +633,33 @@ int dispatch_major(bool amn, bool bmn, const CUtensorMap& ta, const CUtensorMap&
   return launch<BN, true, true>(ta, tb, p, total, s);
 }
 
-template <int BN, bool A_MN, bool B_MN>
-int launch2(const CUtensorMap& ta, const CUtensorMap& tb, const Params& p, int total, cudaStream_t s) {
-  auto k = gemm_tc2_kernel<BN, A_MN, B_MN>;
+template <int BN, bool A_MN, bool B_MN, int NP>
+int launch2(const CUtensorMap& ta, const CUtensorMap& tb, const Params& p, cudaStream_t s) {
+  auto k = gemm_tc2_kernel<BN, A_MN, B_MN, NP>;
   static bool attr_set = false;
   if (!attr_set) {
     if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg2<BN>::SMEM) != cudaSuccess)
       MOBIUS_FAIL(MOBIUS_ECUDA, "cudaFuncSetAttribute(smem, 2cta) failed");
     attr_set = true;
   }
-  int clusters = total < num_sms() / 2 ? total : num_sms() / 2;
+  const int total = p.tiles_m * ((p.tiles_n + NP - 1) / NP);
+  int clusters = num_sms() / (2 * NP);
+  if (total < clusters) clusters = total;
   if (clusters < 1) clusters = 1;
-  k<<<2 * clusters, NUM_THREADS, Cfg2<BN>::SMEM, s>>>(ta, tb, p);
-  cudaError_t e = cudaGetLastError();
+  cudaLaunchConfig_t cfg;
+  std::memset(&cfg, 0, sizeof(cfg));
+  cfg.gridDim = dim3(2 * NP * clusters);
+  cfg.blockDim = dim3(NUM_THREADS);
+  cfg.dynamicSmemBytes = Cfg2<BN>::SMEM;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = 2 * NP;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  cudaError_t e = cudaLaunchKernelEx(&cfg, k, ta, tb, p);
   if (e != cudaSuccess) MOBIUS_FAIL(MOBIUS_ECUDA, "gemm_tc2 launch: %s", cudaGetErrorString(e));
   return MOBIUS_OK;
 }
@@ -633,14 +677,24 @@ int num_sms() {
   return n;
 }
 
+// pairs per cluster for the 2-CTA kernel (MOBIUS_GEMM_NP=2 enables the A
+// multicast across two pairs; measured slower on the 1.5B shapes - the pairs
+// run in lock-step on every smem slot - so it is off by default)
+static int g_gemm_np = -1;
+
 template <int BN>
 static int gemm_bf16_2cta_bn(const GemmDesc& d, cudaStream_t s) {
+  if (g_gemm_np < 0) {
+    const char* e = getenv("MOBIUS_GEMM_NP");
+    g_gemm_np = (e && e[0] == '2') ? 2 : 1;
+  }
+  const bool mc = g_gemm_np == 2 && (d.N + BN - 1) / BN >= 2;
   CUtensorMap ta, tb;
   int rc;
   if (d.a_mn)
     rc = make_map(&ta, d.A, d.M, d.K, d.nb1, d.nb2, BK);
   else
-    rc = make_map(&ta, d.A, d.K, d.M, d.nb1, d.nb2, 128);
+    rc = make_map(&ta, d.A, d.K, d.M, d.nb1, d.nb2, mc ? 64 : 128);
   if (rc) return rc;
   if (d.b_mn)
     rc = make_map(&tb, d.B, d.N, d.K, d.nb1, d.nb2, BK);
@@ -659,11 +713,16 @@ static int gemm_bf16_2cta_bn(const GemmDesc& d, cudaStream_t s) {
   p.bias = (const __nv_bfloat16*)d.bias;
   p.R = (const __nv_bfloat16*)d.R.ptr; p.ldr = d.R.ld;
   p.AUX = (__nv_bfloat16*)d.AUX.ptr; p.ldx = d.AUX.ld;
-  const int total = p.tiles_m * p.tiles_n;
-  if (!d.a_mn && !d.b_mn) return launch2<BN, false, false>(ta, tb, p, total, s);
-  if (!d.a_mn && d.b_mn) return launch2<BN, false, true>(ta, tb, p, total, s);
-  if (d.a_mn && !d.b_mn) return launch2<BN, true, false>(ta, tb, p, total, s);
-  return launch2<BN, true, true>(ta, tb, p, total, s);
+  if (g_gemm_np == 2 && p.tiles_n >= 2) {  // A multicast across two pairs
+    if (!d.a_mn && !d.b_mn) return launch2<BN, false, false, 2>(ta, tb, p, s);
+    if (!d.a_mn && d.b_mn) return launch2<BN, false, true, 2>(ta, tb, p, s);
+    if (d.a_mn && !d.b_mn) return launch2<BN, true, false, 2>(ta, tb, p, s);
+    return launch2<BN, true, true, 2>(ta, tb, p, s);
+  }
+  if (!d.a_mn && !d.b_mn) return launch2<BN, false, false, 1>(ta, tb, p, s);
+  if (!d.a_mn && d.b_mn) return launch2<BN, false, true, 1>(ta, tb, p, s);
+  if (d.a_mn && !d.b_mn) return launch2<BN, true, false, 1>(ta, tb, p, s);
+  return launch2<BN, true, true, 1>(ta, tb, p, s);
 }
 
 // 256 x 256 tiles: at 64 B/clk/SM of operand traffic this is the only 2-CTA

@@ -167,6 +167,17 @@ __device__ __forceinline__ void tma_load_4d_2sm(void* smem, const CUtensorMap* m
       "l"(reinterpret_cast<uint64_t>(m)), "r"(mbar), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
       : "memory");
 }
+// as tma_load_4d_2sm, and the box is also written to every CTA of `mask`
+// (same smem offset); each destination's pair-leader barrier gets the bytes
+__device__ __forceinline__ void tma_load_4d_2sm_mc(void* smem, const CUtensorMap* m, uint64_t* bar_local, uint16_t mask,
+                                                   int c0, int c1, int c2, int c3) {
+  const uint32_t mbar = smem_u32(bar_local) & 0xFEFFFFFFu;
+  asm volatile(
+      "cp.async.bulk.tensor.4d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster "
+      "[%0], [%1, {%4, %5, %6, %7}], [%2], %3;" ::"r"(smem_u32(smem)),
+      "l"(reinterpret_cast<uint64_t>(m)), "r"(mbar), "h"(mask), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+      : "memory");
+}
 template <uint32_t NCOLS>
 __device__ __forceinline__ void tmem_alloc_2sm(uint32_t* dst_smem) {
   asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(dst_smem)),
