@@ -53,6 +53,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-keep", action="store_true", help="always recompute (no kept activations)")
+    ap.add_argument("--partition", default="mip", choices=["mip", "max", "min"],
+                    help="MIP (paper) or the Fig 9 max-stage / min-stage baselines")
     return ap.parse_args()
 
 
@@ -245,7 +247,13 @@ def run_mobius(args, rank, world, local):
         h2d_gbps, groups = shared[1], shared[2]
     t = make_topology(groups, host_bw_Bps=int(h2d_gbps * 1e9), p2p_bw_Bps=int(700e9))
     t0 = time.perf_counter()
-    plan = mobius_plan(prof, world, G, M, t)
+    if args.partition == "mip":
+        plan = mobius_plan(prof, world, G, M, t)
+    else:
+        from paper_conf_asplos_fengxtwls23_b200 import (PARTITION_MAX_STAGE, PARTITION_MIN_STAGE,
+                                                        mobius_plan_partition)
+        plan = mobius_plan_partition(prof, world, G, M,
+                                     PARTITION_MAX_STAGE if args.partition == "max" else PARTITION_MIN_STAGE, t)
     plan_s = time.perf_counter() - t0
     if world > 1:
         from paper_conf_asplos_fengxtwls23_b200 import dist as mdist
@@ -337,6 +345,7 @@ def run_mobius(args, rank, world, local):
                                                                    for j in range(plan.n_stages)],
                        "gpu_perm": [plan.gpu_perm[g] for g in range(world)], "plan_s": plan_s,
                        "profile_s": prof_s, "plan_exhaustive": bool(plan.exhaustive),
+                       "partition": args.partition, "plan_makespan_ms": plan.makespan_ns / 1e6,
                        "l2": "inputs larger than L2: every stage (3.1 GB bf16 total) streams from host DRAM each step"},
             "loss": loss,
             "e2e": e2e,

@@ -78,6 +78,7 @@ F = C.c_float
 # name -> (restype, argtypes); every symbol declared in include/*.h
 SIGNATURES = {
     "mobius_plan": (I, [C.POINTER(LayerProfile), I, I, I64, I, C.POINTER(Topology), C.POINTER(Plan)]),
+    "mobius_plan_partition": (I, [C.POINTER(LayerProfile), I, I, I64, I, C.POINTER(Topology), I, C.POINTER(Plan)]),
     "mobius_plan_cost": (I, [C.POINTER(LayerProfile), I, C.POINTER(C.c_int), I, I, I64, I, I64, I64,
                              C.POINTER(I64), C.POINTER(I64), C.POINTER(I64)]),
     "mobius_cross_map": (I, [I, I, C.POINTER(C.c_int), C.POINTER(C.c_int), C.POINTER(C.c_double),

@@ -11,7 +11,7 @@ import numpy as np
 from . import _lib as L
 from ._lib import BF16, F32, FLAG_KEEP_ACTS, FLAG_TIMING, MobiusError, check, lib  # noqa: F401
 
-__all__ = ["mobius_plan", "mobius_plan_cost", "mobius_cross_map", "mobius_mapping_contention",
+__all__ = ["mobius_plan", "mobius_plan_partition", "PARTITION_MIP", "PARTITION_MAX_STAGE", "PARTITION_MIN_STAGE", "mobius_plan_cost", "mobius_cross_map", "mobius_mapping_contention",
            "mobius_discover_topology", "mobius_layer_sizes", "mobius_profile", "MobiusContext", "model_cfg",
            "make_topology", "plan_from_sizes", "kt", "BF16", "F32", "FLAG_TIMING", "FLAG_KEEP_ACTS", "MobiusError",
            "build_info"]
@@ -59,6 +59,18 @@ def mobius_plan(layers, n_gpus: int, hbm_cap_bytes: int, n_microbatches: int,
     out = L.Plan()
     check(lib.mobius_plan(arr, len(layers), n_gpus, hbm_cap_bytes, n_microbatches,
                           C.byref(topo) if topo is not None else None, C.byref(out)))
+    return out
+
+
+PARTITION_MIP, PARTITION_MAX_STAGE, PARTITION_MIN_STAGE = 0, 1, 2
+
+
+def mobius_plan_partition(layers, n_gpus: int, hbm_cap_bytes: int, n_microbatches: int, algo: int,
+                          topo: Optional[L.Topology] = None) -> L.Plan:
+    arr = _profile_array(layers)
+    out = L.Plan()
+    check(lib.mobius_plan_partition(arr, len(layers), n_gpus, hbm_cap_bytes, n_microbatches,
+                                    C.byref(topo) if topo is not None else None, algo, C.byref(out)))
     return out
 
 

@@ -307,8 +307,8 @@ extern "C" int mobius_cross_map(int K, int N, const int* group, int* perm_out, d
   return MOBIUS_OK;
 }
 
-extern "C" int mobius_plan(const mobius_layer_profile* layers, int n_layers, int N, int64_t G, int M,
-                           const mobius_topology* topo_in, mobius_plan_t* out) {
+static int plan_impl(const mobius_layer_profile* layers, int n_layers, int N, int64_t G, int M,
+                     const mobius_topology* topo_in, int algo, mobius_plan_t* out) {
   int rc = validate_profile(layers, n_layers);
   if (rc) return rc;
   MOBIUS_CHECK_ARG(out && N >= 1 && N <= MOBIUS_MAX_GPUS && M >= 1 && G > 0, "bad arguments");
@@ -330,7 +330,29 @@ extern "C" int mobius_plan(const mobius_layer_profile* layers, int n_layers, int
   int64_t best_mk = -1;
   std::vector<int64_t> a, b;
   int exhaustive = 0;
-  if (n_layers <= 20) {
+  if (algo == MOBIUS_PARTITION_MAX_STAGE || algo == MOBIUS_PARTITION_MIN_STAGE) {
+    // Fig 9 baselines: as many layers per stage as memory
+    // allows (greedy, front to back), or one layer per stage
+    if (algo == MOBIUS_PARTITION_MIN_STAGE) {
+      best.assign(n_layers, 1);
+    } else {
+      int cur = 0;
+      int64_t sf = 0, sb = 0;
+      for (int i = 0; i < n_layers; ++i) {
+        if (cur && (sf + layers[i].mem_fwd > G || sb + layers[i].mem_bwd > G)) {
+          best.push_back(cur);
+          cur = 0;
+          sf = sb = 0;
+        }
+        ++cur;
+        sf += layers[i].mem_fwd;
+        sb += layers[i].mem_bwd;
+      }
+      best.push_back(cur);
+    }
+    best_mk = cost(layers, best.data(), (int)best.size(), N, G, M, Wh, Wp, nullptr, nullptr, a, b);
+    if (best_mk < 0) best.clear();
+  } else if (n_layers <= 20) {
     exhaustive = 1;
     std::vector<int> sizes;
     sizes.reserve(n_layers);
@@ -463,4 +485,17 @@ extern "C" int mobius_discover_topology(mobius_topology* out) {
     out->group[d] = it->second;
   }
   return MOBIUS_OK;
+}
+
+extern "C" int mobius_plan(const mobius_layer_profile* layers, int n_layers, int N, int64_t G, int M,
+                           const mobius_topology* topo_in, mobius_plan_t* out) {
+  return plan_impl(layers, n_layers, N, G, M, topo_in, MOBIUS_PARTITION_MIP, out);
+}
+
+extern "C" int mobius_plan_partition(const mobius_layer_profile* layers, int n_layers, int N, int64_t G, int M,
+                                     const mobius_topology* topo_in, int algo, mobius_plan_t* out) {
+  MOBIUS_CHECK_ARG(algo == MOBIUS_PARTITION_MIP || algo == MOBIUS_PARTITION_MAX_STAGE ||
+                       algo == MOBIUS_PARTITION_MIN_STAGE,
+                   "unknown partition algorithm %d", algo);
+  return plan_impl(layers, n_layers, N, G, M, topo_in, algo, out);
 }

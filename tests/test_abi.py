@@ -168,3 +168,26 @@ def test_tiny_config_cap_forces_swap(mb):
     assert plan.n_stages >= 2
     tot = sum(p.mem_fwd for p in prof)
     assert tot > 4 << 20
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_fig9_baseline_partitions(mb, seed):
+    """max-stage / min-stage (Fig 9) through the ABI equal the
+    oracle's construction, are scored by the same Eq 3-11 objective, and the
+    MIP optimum is never worse."""
+    rng = random.Random(500 + seed)
+    Lp = rng.randint(2, 12)
+    layers = _rand_layers(rng, Lp)
+    N, M = rng.randint(1, 4), rng.randint(1, 4)
+    G = max(l.mem_bwd for l in layers) + rng.randint(0, 120)
+    W = 10 ** 9
+    topo = mb.make_topology(list(range(N)), W, W)
+    mip = mb.mobius_plan(layers, N, G, M, topo)
+    for algo, ref in ((mb.PARTITION_MAX_STAGE, op.max_stage_sizes(layers, G)),
+                      (mb.PARTITION_MIN_STAGE, op.min_stage_sizes(layers))):
+        pl = mb.mobius_plan_partition(layers, N, G, M, algo, topo)
+        sizes = tuple(pl.stage_first_layer[j + 1] - pl.stage_first_layer[j] for j in range(pl.n_stages))
+        assert sizes == ref
+        r = op.stage_cost(layers, ref, N, M, G, W, W)
+        assert pl.makespan_ns == r[0]
+        assert mip.makespan_ns <= pl.makespan_ns

@@ -162,3 +162,24 @@ def test_tiny_step_keep_acts(dtype, tol, sizes):
     errs = tensor_errs(c, g, ref_g)
     assert max(errs.values()) < tol, errs
     assert np.isfinite(loss2)
+
+
+@pytest.mark.parametrize("dtype,tol", [(F32, 1e-5), (BF16, 2e-2)])
+def test_multistep_mobius_vs_gpipe_mode(dtype, tol):
+    """SURVEY f4 / P:L596-602, Fig 13 analog without a dataset: four
+    synthetic fine-tuning steps with stages swapped through DRAM (K=3 > N=1)
+    follow the same loss curve as the single-resident-stage run (K=N=1,
+    GPipe mode): the synchronous update makes the pipeline invisible."""
+    c = synth.TINY
+    M = 2
+    w = synth.perturb_norm_params(c, synth.gen_params(c), scale=0.1)
+    if dtype == BF16:
+        w = synth.round_bf16(w)
+    curves = []
+    for sizes, cap in (((6,), 64 * MiB), ((2, 2, 2), (4 * MiB) * (2 if dtype == F32 else 1))):
+        ctx = MobiusContext(mk_cfg(c, dtype), plan_from_sizes(sizes, 1, M, hbm_cap_bytes=cap), init_params=w)
+        curves.append([ctx.step(synth.gen_tokens(c, M, seed=100 + i)) for i in range(4)])
+        ctx.close()
+    a, b = np.array(curves[0]), np.array(curves[1])
+    assert np.all(np.abs(a - b) <= tol * np.abs(a)), (a, b)
+    assert a[-1] < a[0]
