@@ -378,7 +378,10 @@ struct BwdCfg {
   static constexpr int QS = DH == 64 ? 2 : 1;        // Q/dO pipeline depth
   static constexpr int PT_BYTES = 128 * 128 * 2;     // P^T or dS^T tile
   static constexpr bool DQ_OWN = DH == 64;           // dQ has its own TMEM columns (else aliases S^T)
-  static constexpr int SMEM = 1024 + 2 * T_BYTES + QS * 2 * T_BYTES + 2 * PT_BYTES + QS * 1024 + 256;
+  // dh 64: dQ(i-1) is drained from its own staging tile while the MMAs of
+  // tile i run; dh 128: staged in the P^T/dS^T tiles (smem budget)
+  static constexpr int STG_BYTES = DQ_OWN ? 128 * DH * 4 : 0;
+  static constexpr int SMEM = 1024 + 2 * T_BYTES + QS * 2 * T_BYTES + 2 * PT_BYTES + STG_BYTES + QS * 1024 + 256;
 };
 
 struct BwdParams {
@@ -422,7 +425,8 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
   uint8_t* sdO = sQ + QS * C::T_BYTES;       // [QS]
   uint8_t* sPT = sdO + QS * C::T_BYTES;
   uint8_t* sdST = sPT + C::PT_BYTES;
-  float* sLD = reinterpret_cast<float*>(sdST + C::PT_BYTES);  // [QS][lse 128 | D 128]
+  uint8_t* sSTG = sdST + C::PT_BYTES;  // dQ staging (dh 64)
+  float* sLD = reinterpret_cast<float*>(sSTG + C::STG_BYTES);  // [QS][lse 128 | D 128]
   uint64_t* bars = reinterpret_cast<uint64_t*>(sLD + QS * 256);
   uint64_t* kv_full = bars;          // 1
   uint64_t* q_full = bars + 1;       // [2] (Q, dO, lse, D)
@@ -553,6 +557,41 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
     const int r = q4 * 32 + lane;  // key row of this thread (TMEM lane)
     const uint32_t lane_base = (uint32_t)(q4 * 32) << 16;
     const uint32_t spt = ptx::smem_u32(sPT), sdst = ptx::smem_u32(sdST);
+    // dQ(it) (TMEM lane = query row) -> fp32 staging [DH/32 slabs][128 rows][128 B],
+    // 16-byte chunks XOR-swizzled by row (TMA SWIZZLE_128B, conflict-free
+    // stores) -> one TMA reduce-add per 32-column slab into the dQ buffer
+    auto dq_drain = [&](int itq, uint32_t stg) {
+      const int qiq = i0 + itq;
+#pragma unroll
+      for (int cc = 0; cc < DH / 64; ++cc) {
+        const int c = hf * (DH / 64) + cc;  // 32-column slab
+        uint32_t v[32];
+        __syncwarp();
+        ptx::tmem_ld32(T_DQ + c * 32 + lane_base, v);
+        ptx::tmem_ld_wait();
+#pragma unroll
+        for (int k = 0; k < 8; ++k)
+          st_shared_v4(stg + c * 16384 + r * 128 + ((k ^ (r & 7)) << 4), v[4 * k], v[4 * k + 1], v[4 * k + 2],
+                       v[4 * k + 3]);
+      }
+      ptx::tc_fence_before();
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(dq_empty);
+      ptx::fence_proxy_async();
+      named_bar(1, 256);
+      if (warp == 2 && lane == 0) {
+#pragma unroll
+        for (int c = 0; c < DH / 32; ++c)
+          asm volatile(
+              "cp.reduce.async.bulk.tensor.4d.global.shared::cta.add.tile.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
+                  reinterpret_cast<uint64_t>(&tdq)),
+              "r"(stg + c * 16384), "r"(c * 32), "r"(qiq * 128), "r"(hd), "r"(b)
+              : "memory");
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+      }
+      named_bar(1, 256);
+    };
     for (int it = 0; it < nq; ++it) {
       const int st = it % QS;
       const int qi = i0 + it;
@@ -570,8 +609,12 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(st_empty);  // S^T / dP^T TMEM may be overwritten
-      // P^T / dS^T smem (also the dQ staging tile) is free: the previous
-      // tile's dQ reduce finished reading it (named barrier below)
+      // P^T / dS^T smem must be free: dh 128 - the previous tile's dQ drain
+      // (staged there) completed; dh 64 - the previous tile's MMAs completed
+      if (C::DQ_OWN && it >= 1) {
+        ptx::mbar_wait(mm_done, (it - 1) & 1);
+        ptx::tc_fence_after();
+      }
 #pragma unroll
       for (int cc = 0; cc < 2; ++cc) {
         const int c = hf * 2 + cc;
@@ -603,41 +646,19 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
       ptx::fence_proxy_async();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(p_full);
-      // dQ of this query tile (TMEM lane = query row) -> fp32 staging tile in
-      // the P^T/dS^T smem (free once the MMAs completed) -> one TMA
-      // reduce-add into the fp32 dQ buffer
-      ptx::mbar_wait(mm_done, it & 1);
+      if (C::DQ_OWN) {
+        // drain dQ of the previous query tile while this tile's MMAs run
+        if (it >= 1) dq_drain(it - 1, ptx::smem_u32(sSTG));
+      } else {
+        ptx::mbar_wait(mm_done, it & 1);
+        ptx::tc_fence_after();
+        dq_drain(it, spt);  // staged in the (now free) P^T / dS^T tiles
+      }
+    }
+    if (C::DQ_OWN) {
+      ptx::mbar_wait(mm_done, (nq - 1) & 1);
       ptx::tc_fence_after();
-      const uint32_t stg = spt;  // [128 rows][DH] fp32, row-major
-#pragma unroll
-      for (int cc = 0; cc < DH / 64; ++cc) {
-        const int c = hf * (DH / 64) + cc;
-        uint32_t v[32];
-        __syncwarp();
-        ptx::tmem_ld32(T_DQ + c * 32 + lane_base, v);
-        ptx::tmem_ld_wait();
-#pragma unroll
-        for (int e = 0; e < 32; e += 4) {
-          // rotate the 16-byte chunk order by row to spread smem banks
-          const int ee = (e + 4 * (r & 7)) & 31;
-          st_shared_v4(stg + (uint32_t)(r * DH + c * 32 + ee) * 4, v[ee], v[ee + 1], v[ee + 2], v[ee + 3]);
-        }
-      }
-      ptx::tc_fence_before();
-      __syncwarp();
-      if (lane == 0) ptx::mbar_arrive(dq_empty);
-      ptx::fence_proxy_async();
-      named_bar(1, 256);
-      if (warp == 2 && lane == 0) {
-        asm volatile(
-            "cp.reduce.async.bulk.tensor.4d.global.shared::cta.add.tile.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
-                reinterpret_cast<uint64_t>(&tdq)),
-            "r"(stg), "r"(0), "r"(qi * 128), "r"(hd), "r"(b)
-            : "memory");
-        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-        asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
-      }
-      named_bar(1, 256);
+      dq_drain(nq - 1, ptx::smem_u32(sSTG));
     }
     // dV (half 0) / dK (half 1) of this key tile (rows = keys)
     ptx::mbar_wait(mm_done, (nq - 1) & 1);
@@ -738,16 +759,16 @@ int head_map(CUtensorMap* m, const void* base, int64_t ld, int dh, int s, int n_
   return MOBIUS_OK;
 }
 
-// fp32 {d, token, head, batch} map over the dQ accumulator [mbs*s, h]; box {dh, 128, 1, 1}
+// fp32 {d, token, head, batch} map over the dQ accumulator [mbs*s, h]; box {32, 128, 1, 1}, 128B swizzle
 int dq_map(CUtensorMap* m, const float* base, int h, int dh, int s, int nh, int mbs) {
   EncodeTiledFn enc = encode_fn();
   if (!enc) MOBIUS_FAIL(MOBIUS_ECUDA, "cuTensorMapEncodeTiled unavailable");
   cuuint64_t dims[4] = {(cuuint64_t)dh, (cuuint64_t)s, (cuuint64_t)nh, (cuuint64_t)mbs};
   cuuint64_t strides[3] = {(cuuint64_t)h * 4, (cuuint64_t)dh * 4, (cuuint64_t)s * h * 4};
-  cuuint32_t box[4] = {(cuuint32_t)dh, 128, 1, 1};
+  cuuint32_t box[4] = {32, 128, 1, 1};
   cuuint32_t es[4] = {1, 1, 1, 1};
   CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, const_cast<float*>(base), dims, strides, box, es,
-                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) MOBIUS_FAIL(MOBIUS_ECUDA, "flash dQ tensor map (%d)", (int)r);
   return MOBIUS_OK;
