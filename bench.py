@@ -326,6 +326,13 @@ def run_mobius(args, rank, world, local):
     gemm_flops = sum(s.gemm_flops for s in stats)
     achieved_tf = gemm_flops / (gemm_ns * 1e-9) / 1e12 if gemm_ns else 0.0
     peak_tf = peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops"))
+    traffic = traffic_alg = None
+    tr_path = os.path.join(ROOT, "profiles", "r1_gemm_traffic.json")
+    if os.path.exists(tr_path):  # ncu --set full capture of the block GEMM shapes (per launch)
+        with open(tr_path) as f:
+            tr = json.load(f)
+        traffic = float(np.mean([t["dram_bytes"] for t in tr]))
+        traffic_alg = float(np.mean([t["algorithmic_bytes"] for t in tr]))
     # step roofline (north_star): max(FLOP / P_tc, H2D bytes / host link), per GPU
     flop_step = model_flops_per_token(c) * tokens_per_step / world
     t_tc = flop_step / (peak_tf * 1e12)
@@ -351,7 +358,10 @@ def run_mobius(args, rank, world, local):
             "e2e": e2e,
             "roofline": {"bound": "tensor", "kernel": "gemm_tc (tcgen05 bf16, all block/head GEMMs)",
                          "achieved": achieved_tf, "peak": peak_tf, "unit": "TFLOP/s",
-                         "frac": achieved_tf / peak_tf if peak_tf else None, "traffic": None,
+                         "frac": achieved_tf / peak_tf if peak_tf else None, "traffic": traffic,
+                         "traffic_algorithmic_bytes": traffic_alg,
+                         "traffic_source": "profiles/r1_gemm_traffic.json: dram__bytes_read+write per launch, mean "
+                                           "over the fc1-fwd / fc2-fwd / fc1-dX / fc1-dW GEMMs (ncu --set full)",
                          "peak_source": f"MEASURED_PEAKS.json bf16_tflops_sustained ({peak_src})"},
             "step_roofline": {"t_tensor_ms": t_tc * 1e3, "t_link_ms": t_link * 1e3, "t_roofline_ms": t_roof * 1e3,
                               "frac": t_roof / (ms * 1e-3), "h2d_GBps_link": h2d_gbps,
