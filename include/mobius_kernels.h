@@ -34,6 +34,15 @@ int mobius_kt_gemm(int dtype, int M, int N, int K, int nb1, int nb2, const void*
                    int64_t ldc, int64_t cbs1, int64_t cbs2, int c_f32, int epi, float alpha, const void* bias,
                    const void* R, int64_t ldr, void* AUX, int64_t ldx, int causal, int accumulate);
 
+/* Process-wide bf16 GEMM kernel selection (perf A/B and tests; not part of
+ * the step contract): two_cta selects the cta_group::2 256x256 kernel for
+ * plain GEMMs, stream_k its Stream-K tail (the last partial wave's tiles are
+ * split along K over all SM pairs and reduced deterministically in segment
+ * order).  Each is -1 (environment default MOBIUS_GEMM_2CTA /
+ * MOBIUS_GEMM_SK, on unless set to 0), 0 or 1; anything else is
+ * MOBIUS_EINVAL.  Takes effect for GEMMs launched after the call. */
+int mobius_kt_gemm_config(int two_cta, int stream_k);
+
 int mobius_kt_layernorm_fwd(int dtype, const void* x, const void* g, const void* b, void* y, float* mu, float* rstd,
                             int rows, int h);
 int mobius_kt_layernorm_bwd(int dtype, const void* dy, const void* x, const void* g, const float* mu,

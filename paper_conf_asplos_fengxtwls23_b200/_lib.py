@@ -100,6 +100,7 @@ SIGNATURES = {
     "mobius_destroy": (None, [P]),
     "mobius_last_error": (C.c_char_p, []),
     "mobius_build_info": (C.c_char_p, []),
+    "mobius_kt_gemm_config": (I, [I, I]),
     "mobius_kt_gemm": (I, [I, I, I, I, I, I, P, I64, I64, I64, I, P, I64, I64, I64, I, P, I64, I64, I64, I, I, F,
                            P, P, I64, P, I64, I, I]),
     "mobius_kt_layernorm_fwd": (I, [I, P, P, P, P, P, P, I, I]),

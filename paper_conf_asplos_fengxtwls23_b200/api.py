@@ -238,6 +238,9 @@ class _KT:
                                  bbs[1], int(b_mn), pc, ldc, cbs[0], cbs[1], int(c_f32), epi, alpha, self._p(bias),
                                  self._p(R), ldr, self._p(AUX), ldx, causal, int(accumulate)))
 
+    def gemm_config(self, two_cta=-1, stream_k=-1):
+        check(lib.mobius_kt_gemm_config(int(two_cta), int(stream_k)))
+
     def layernorm_fwd(self, dtype, x, g, b, y, mu, rstd, rows, h):
         check(lib.mobius_kt_layernorm_fwd(dtype, *map(self._p, (x, g, b, y, mu, rstd)), rows, h))
 

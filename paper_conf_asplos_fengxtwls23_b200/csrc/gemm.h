@@ -60,4 +60,8 @@ int gemm_f32(const GemmDesc& d, cudaStream_t s);
 
 int num_sms();
 
+// Kernel selection knobs (tests / perf A-B): -1 = environment default
+// (MOBIUS_GEMM_2CTA, MOBIUS_GEMM_SK), 0 = off, 1 = on.
+void gemm_set_config(int two_cta, int stream_k);
+
 }  // namespace mobius

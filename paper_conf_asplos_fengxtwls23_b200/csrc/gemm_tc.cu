@@ -57,6 +57,14 @@ struct Params {
   int64_t ldr, rbs1, rbs2;
   __nv_bfloat16* AUX;
   int64_t ldx, xbs1, xbs2;
+  // Stream-K tail (2-CTA kernel only; sk_tiles == 0 disables): the first
+  // sk_tiles tiles' k-blocks are split evenly over all clusters; partial
+  // accumulators go to sk_ws, the last-arriving segment reduces them in
+  // segment order (deterministic) and runs the fused epilogue.
+  int sk_tiles, sk_maxseg;
+  int64_t sk_units;
+  float* sk_ws;
+  int* sk_cnt;
 };
 
 __device__ __forceinline__ float tanh_fast(float x) {
@@ -128,106 +136,110 @@ __device__ __forceinline__ void st_bf16x8(__nv_bfloat16* g, const float* f) {
   *reinterpret_cast<uint4*>(g) = pk;
 }
 
-// Epilogue of one accumulator tile row-slice: this thread owns output row m
-// (TMEM lane), columns [nt*BN, nt*BN + BN); TMEM -> registers -> fused ops
-// -> global.  tmem_row = tmem base + lane quadrant + accumulator column base.
-// Full 32-column chunks use 16-byte vector accesses only (all indices are
-// compile-time, so nothing spills to local memory); a ragged last chunk
-// takes the predicated scalar path.
-template <int BN>
-__device__ __forceinline__ void epi_tile(const Params& p, uint32_t tmem_row, int m, int b1, int b2, int nt) {
-  const bool row_ok = m < p.M;
+// Fused epilogue of one 32-column chunk of output row m: v[] holds
+// alpha * acc for columns [n0, n0 + 32); applies bias / GeLU / residual /
+// GeLU' / fp32 accumulate and stores.  Full chunks use 16-byte vector
+// accesses only (all indices compile-time, nothing spills); a ragged last
+// chunk takes the predicated scalar path.
+__device__ __forceinline__ void epi_vals(const Params& p, float (&v)[32], int m, int b1, int b2, int n0) {
+  if (m >= p.M || n0 >= p.N) return;
   const int64_t crow = (int64_t)b1 * p.cbs1 + (int64_t)b2 * p.cbs2 + (int64_t)m * p.ldc;
   const bool has_bias = p.epi == EPI_BIAS || p.epi == EPI_BIAS_GELU || p.epi == EPI_BIAS_RESID;
   const bool has_r = p.epi == EPI_BIAS_RESID || p.epi == EPI_GELU_BWD;
   const bool accum = p.epi == EPI_ACCUM && p.accumulate;
+  const __nv_bfloat16* rrow = has_r ? p.R + (int64_t)b1 * p.rbs1 + (int64_t)b2 * p.rbs2 + (int64_t)m * p.ldr + n0 : nullptr;
+  __nv_bfloat16* aux = p.epi == EPI_BIAS_GELU
+                           ? p.AUX + (int64_t)b1 * p.xbs1 + (int64_t)b2 * p.xbs2 + (int64_t)m * p.ldx + n0
+                           : nullptr;
+  if (n0 + 32 <= p.N) {
+    if (has_bias) {
+#pragma unroll
+      for (int i = 0; i < 32; i += 8) {
+        float bb[8];
+        ld_bf16x8(p.bias + n0 + i, bb);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) v[i + j] += bb[j];
+      }
+    }
+    if (p.epi == EPI_BIAS_GELU) {
+#pragma unroll
+      for (int i = 0; i < 32; i += 8) st_bf16x8(aux + i, v + i);
+      // GeLU of the bf16-rounded pre-activation (what backward will see)
+#pragma unroll
+      for (int i = 0; i < 32; ++i) v[i] = gelu_f(__bfloat162float(__float2bfloat16_rn(v[i])));
+    }
+    if (has_r) {
+#pragma unroll
+      for (int i = 0; i < 32; i += 8) {
+        float rv[8];
+        ld_bf16x8(rrow + i, rv);
+        if (p.epi == EPI_BIAS_RESID) {
+#pragma unroll
+          for (int j = 0; j < 8; ++j) v[i + j] += rv[j];
+        } else {
+#pragma unroll
+          for (int j = 0; j < 8; ++j) v[i + j] *= gelu_grad_f(rv[j]);
+        }
+      }
+    }
+    if (p.c_f32) {
+      float* cp = reinterpret_cast<float*>(p.C) + crow + n0;
+#pragma unroll
+      for (int i = 0; i < 32; i += 4) {
+        float4 o = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
+        if (accum) {
+          const float4 old = *reinterpret_cast<const float4*>(cp + i);
+          o.x += old.x;
+          o.y += old.y;
+          o.z += old.z;
+          o.w += old.w;
+        }
+        *reinterpret_cast<float4*>(cp + i) = o;
+      }
+    } else {
+      __nv_bfloat16* cp = p.C + crow + n0;
+#pragma unroll
+      for (int i = 0; i < 32; i += 8) st_bf16x8(cp + i, v + i);
+    }
+  } else {
+    const int cnt = p.N - n0;
+#pragma unroll
+    for (int i = 0; i < 32; ++i) {
+      if (i < cnt) {
+        float x = v[i];
+        if (has_bias) x += __bfloat162float(p.bias[n0 + i]);
+        if (p.epi == EPI_BIAS_GELU) {
+          aux[i] = __float2bfloat16_rn(x);
+          x = gelu_f(__bfloat162float(__float2bfloat16_rn(x)));
+        }
+        if (p.epi == EPI_BIAS_RESID) x += __bfloat162float(rrow[i]);
+        if (p.epi == EPI_GELU_BWD) x *= gelu_grad_f(__bfloat162float(rrow[i]));
+        if (p.c_f32) {
+          float* cp = reinterpret_cast<float*>(p.C) + crow + n0;
+          cp[i] = x + (accum ? cp[i] : 0.f);
+        } else {
+          p.C[crow + n0 + i] = __float2bfloat16_rn(x);
+        }
+      }
+    }
+  }
+}
+
+// Epilogue of one accumulator tile row-slice: this thread owns output row m
+// (TMEM lane), columns [nt*BN, nt*BN + BN); TMEM -> registers -> epi_vals.
+// tmem_row = tmem base + lane quadrant + accumulator column base.
+template <int BN>
+__device__ __forceinline__ void epi_tile(const Params& p, uint32_t tmem_row, int m, int b1, int b2, int nt) {
 #pragma unroll 1
   for (int c = 0; c < BN; c += 32) {
     uint32_t r[32];
     __syncwarp();
     ptx::tmem_ld32(tmem_row + c, r);
     ptx::tmem_ld_wait();
-    const int n0 = nt * BN + c;
-    if (!row_ok || n0 >= p.N) continue;
     float v[32];
 #pragma unroll
     for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]) * p.alpha;
-    const __nv_bfloat16* rrow = has_r ? p.R + (int64_t)b1 * p.rbs1 + (int64_t)b2 * p.rbs2 + (int64_t)m * p.ldr + n0 : nullptr;
-    __nv_bfloat16* aux = p.epi == EPI_BIAS_GELU
-                             ? p.AUX + (int64_t)b1 * p.xbs1 + (int64_t)b2 * p.xbs2 + (int64_t)m * p.ldx + n0
-                             : nullptr;
-    if (n0 + 32 <= p.N) {
-      if (has_bias) {
-#pragma unroll
-        for (int i = 0; i < 32; i += 8) {
-          float bb[8];
-          ld_bf16x8(p.bias + n0 + i, bb);
-#pragma unroll
-          for (int j = 0; j < 8; ++j) v[i + j] += bb[j];
-        }
-      }
-      if (p.epi == EPI_BIAS_GELU) {
-#pragma unroll
-        for (int i = 0; i < 32; i += 8) st_bf16x8(aux + i, v + i);
-        // GeLU of the bf16-rounded pre-activation (what backward will see)
-#pragma unroll
-        for (int i = 0; i < 32; ++i) v[i] = gelu_f(__bfloat162float(__float2bfloat16_rn(v[i])));
-      }
-      if (has_r) {
-#pragma unroll
-        for (int i = 0; i < 32; i += 8) {
-          float rv[8];
-          ld_bf16x8(rrow + i, rv);
-          if (p.epi == EPI_BIAS_RESID) {
-#pragma unroll
-            for (int j = 0; j < 8; ++j) v[i + j] += rv[j];
-          } else {
-#pragma unroll
-            for (int j = 0; j < 8; ++j) v[i + j] *= gelu_grad_f(rv[j]);
-          }
-        }
-      }
-      if (p.c_f32) {
-        float* cp = reinterpret_cast<float*>(p.C) + crow + n0;
-#pragma unroll
-        for (int i = 0; i < 32; i += 4) {
-          float4 o = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
-          if (accum) {
-            const float4 old = *reinterpret_cast<const float4*>(cp + i);
-            o.x += old.x;
-            o.y += old.y;
-            o.z += old.z;
-            o.w += old.w;
-          }
-          *reinterpret_cast<float4*>(cp + i) = o;
-        }
-      } else {
-        __nv_bfloat16* cp = p.C + crow + n0;
-#pragma unroll
-        for (int i = 0; i < 32; i += 8) st_bf16x8(cp + i, v + i);
-      }
-    } else {
-      const int cnt = p.N - n0;
-#pragma unroll
-      for (int i = 0; i < 32; ++i) {
-        if (i < cnt) {
-          float x = v[i];
-          if (has_bias) x += __bfloat162float(p.bias[n0 + i]);
-          if (p.epi == EPI_BIAS_GELU) {
-            aux[i] = __float2bfloat16_rn(x);
-            x = gelu_f(__bfloat162float(__float2bfloat16_rn(x)));
-          }
-          if (p.epi == EPI_BIAS_RESID) x += __bfloat162float(rrow[i]);
-          if (p.epi == EPI_GELU_BWD) x *= gelu_grad_f(__bfloat162float(rrow[i]));
-          if (p.c_f32) {
-            float* cp = reinterpret_cast<float*>(p.C) + crow + n0;
-            cp[i] = x + (accum ? cp[i] : 0.f);
-          } else {
-            p.C[crow + n0 + i] = __float2bfloat16_rn(x);
-          }
-        }
-      }
-    }
+    epi_vals(p, v, m, b1, b2, nt * BN + c);
   }
 }
 
@@ -396,6 +408,61 @@ struct Cfg2 {
   static constexpr int SMEM = 1024 + STAGES * STAGE_BYTES + 256;
 };
 
+// One unit of work of a cluster: k-blocks [k0, k1) of tile t, which is
+// segment seg of nseg (nseg == 1: a whole tile, no fixup).
+struct Work {
+  int t, k0, k1, seg, nseg;
+};
+
+__device__ __forceinline__ int64_t sk_start(const Params& p, int c, int ncl) {
+  return (int64_t)c * p.sk_units / ncl;
+}
+// cluster whose Stream-K range holds unit g
+__device__ __forceinline__ int sk_owner(const Params& p, int64_t g, int ncl) {
+  int c = (int)(g * ncl / p.sk_units);
+  while (c + 1 < ncl && sk_start(p, c + 1, ncl) <= g) ++c;
+  while (c > 0 && sk_start(p, c, ncl) > g) --c;
+  return c;
+}
+
+// Per-cluster schedule: its Stream-K range over the first sk_tiles tiles
+// (cut at tile boundaries), then whole tiles sk_tiles + cl, + ncl, ...
+// The producer, MMA issuer and epilogue walk identical sequences.
+struct Sched {
+  int64_t g, gend;
+  int t, cl, ncl;
+  __device__ __forceinline__ Sched(const Params& p, int cl_, int ncl_) : cl(cl_), ncl(ncl_) {
+    g = p.sk_tiles ? sk_start(p, cl, ncl) : 0;
+    gend = p.sk_tiles ? sk_start(p, cl + 1, ncl) : 0;
+    t = p.sk_tiles + cl;
+  }
+  __device__ __forceinline__ bool next(const Params& p, int total, Work& w) {
+    if (g < gend) {
+      const int nkb = p.num_kb;
+      const int tt = (int)(g / nkb);
+      w.t = tt;
+      w.k0 = (int)(g - (int64_t)tt * nkb);
+      w.k1 = (int)min((int64_t)nkb, (int64_t)w.k0 + (gend - g));
+      const int first = sk_owner(p, (int64_t)tt * nkb, ncl);
+      const int last = sk_owner(p, (int64_t)(tt + 1) * nkb - 1, ncl);
+      w.seg = cl - first;
+      w.nseg = last - first + 1;
+      g += w.k1 - w.k0;
+      return true;
+    }
+    if (t < total) {
+      w.t = t;
+      w.k0 = 0;
+      w.k1 = p.num_kb;
+      w.seg = 0;
+      w.nseg = 1;
+      t += ncl;
+      return true;
+    }
+    return false;
+  }
+};
+
 // NP pairs per cluster (cluster = 2*NP CTAs along x).  Pairs of one cluster
 // compute horizontally adjacent 256 x BN tiles (same rows): with NP = 2 the
 // A tile is loaded once per cluster - each CTA loads half of its 128 A rows
@@ -459,11 +526,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       int stage = 0;
       uint32_t phase = 0;
       const uint16_t amask = (uint16_t)((1u << r2) | (NP == 2 ? (1u << (r2 + 2)) : 0u));
-      for (int t = cl; t < total; t += ncl) {
+      Sched sc(p, cl, ncl);
+      Work w;
+      while (sc.next(p, total, w)) {
         int mt, nt;
-        tile_of(t, mt, nt);
+        tile_of(w.t, mt, nt);
         const int m0 = mt * BM2 + (int)r2 * 128, n0 = nt * BN + (int)r2 * (BN / 2);
-        for (int kb = 0; kb < p.num_kb; ++kb) {
+        for (int kb = w.k0; kb < w.k1; ++kb) {
           ptx::mbar_wait_cluster(&empty[stage], phase ^ 1);
           if (leader) ptx::mbar_arrive_expect_tx(&full[stage], 2 * C::STAGE_BYTES);
           uint8_t* a = smA + stage * C::A_BYTES;
@@ -506,11 +575,13 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
       uint32_t phase = 0;
       int acc = 0;
       uint32_t aphase = 0;
-      for (int t = cl; t < total; t += ncl) {
+      Sched sc(p, cl, ncl);
+      Work w;
+      while (sc.next(p, total, w)) {
         ptx::mbar_wait_cluster(&tempty[acc], aphase ^ 1);
         ptx::tc_fence_after();
         const uint32_t tmem_d = tmem_base + acc * BN;
-        for (int kb = 0; kb < p.num_kb; ++kb) {
+        for (int kb = w.k0; kb < w.k1; ++kb) {
           ptx::mbar_wait_cluster(&full[stage], phase);
           ptx::tc_fence_after();
           const uint32_t a_base = ptx::smem_u32(smA + stage * C::A_BYTES);
@@ -521,7 +592,7 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
                                : ptx::sdesc_sw128(a_base + k * 32, 16, 1024);
             uint64_t bd = B_MN ? ptx::sdesc_sw128(b_base + k * 2048, 8192, 1024)
                                : ptx::sdesc_sw128(b_base + k * 32, 16, 1024);
-            ptx::mma_bf16_2sm(tmem_d, ad, bd, IDESC, (kb > 0 || k > 0) ? 1u : 0u);
+            ptx::mma_bf16_2sm(tmem_d, ad, bd, IDESC, (kb > w.k0 || k > 0) ? 1u : 0u);
           }
           // the slot may be refilled by this pair's producers and (A halves)
           // by the other pair's: free it in every CTA of the cluster
@@ -544,16 +615,74 @@ __global__ void __launch_bounds__(NUM_THREADS, 1)
     const uint32_t tempty_leader = ptx::mapa_shared(ptx::smem_u32(&tempty[0]), pair * 2);
     int acc = 0;
     uint32_t aphase = 0;
-    for (int t = cl; t < total; t += ncl) {
+    Sched sc(p, cl, ncl);
+    Work w;
+    while (sc.next(p, total, w)) {
       int mt, nt;
-      tile_of(t, mt, nt);
+      tile_of(w.t, mt, nt);
+      const int m = mt * BM2 + (int)r2 * 128 + q * 32 + lane;
+      const uint32_t tmem_row = tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN;
       ptx::mbar_wait_cluster(&tfull[acc], aphase);
       ptx::tc_fence_after();
-      epi_tile<BN>(p, tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN, mt * BM2 + (int)r2 * 128 + q * 32 + lane,
-                   0, 0, nt);
-      ptx::tc_fence_before();
-      __syncwarp();
-      if (lane == 0) ptx::mbar_arrive_cluster(tempty_leader + acc * 8);
+      if (w.nseg == 1) {
+        epi_tile<BN>(p, tmem_row, m, 0, 0, nt);
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive_cluster(tempty_leader + acc * 8);
+      } else {
+        // Stream-K segment: raw partial (32 rows x BN fp32 per warp) to the
+        // workspace, lane-interleaved so every store is 512 contiguous bytes
+        const int wq = (int)r2 * 4 + q;
+        constexpr int SLOT = 32 * BN;  // floats per warp slot
+        float* base = p.sk_ws + ((int64_t)w.t * p.sk_maxseg * 8 + wq) * SLOT;
+        const int64_t seg_stride = 8 * (int64_t)SLOT;
+        float4* mine = reinterpret_cast<float4*>(base + w.seg * seg_stride) + lane;
+#pragma unroll 1
+        for (int c = 0; c < BN; c += 32) {
+          uint32_t r[32];
+          __syncwarp();
+          ptx::tmem_ld32(tmem_row + c, r);
+          ptx::tmem_ld_wait();
+#pragma unroll
+          for (int i = 0; i < 8; ++i)
+            __stcg(mine + ((c / 32) * 8 + i) * 32, make_float4(__uint_as_float(r[4 * i]), __uint_as_float(r[4 * i + 1]),
+                                                              __uint_as_float(r[4 * i + 2]), __uint_as_float(r[4 * i + 3])));
+        }
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive_cluster(tempty_leader + acc * 8);  // accumulator free: MMA runs on
+        __threadfence();
+        __syncwarp();
+        int old = 0;
+        int* cnt = p.sk_cnt + (int64_t)w.t * 8 + wq;
+        if (lane == 0) old = atomicAdd(cnt, 1);
+        old = __shfl_sync(0xffffffffu, old, 0);
+        if (old == w.nseg - 1) {  // last segment to arrive: reduce in segment order
+          __threadfence();
+#pragma unroll 1
+          for (int c = 0; c < BN; c += 32) {
+            float v[32];
+#pragma unroll
+            for (int i = 0; i < 32; ++i) v[i] = 0.f;
+#pragma unroll 1
+            for (int sgi = 0; sgi < w.nseg; ++sgi) {
+              const float4* src = reinterpret_cast<const float4*>(base + sgi * seg_stride) + lane;
+#pragma unroll
+              for (int i = 0; i < 8; ++i) {
+                const float4 x = __ldcg(src + ((c / 32) * 8 + i) * 32);
+                v[4 * i] += x.x;
+                v[4 * i + 1] += x.y;
+                v[4 * i + 2] += x.z;
+                v[4 * i + 3] += x.w;
+              }
+            }
+#pragma unroll
+            for (int i = 0; i < 32; ++i) v[i] *= p.alpha;
+            epi_vals(p, v, m, 0, 0, nt * BN + c);
+          }
+          if (lane == 0) *cnt = 0;  // self-cleaning for the next launch
+        }
+      }
       if (++acc == 2) {
         acc = 0;
         aphase ^= 1;
@@ -644,7 +773,7 @@ int launch2(const CUtensorMap& ta, const CUtensorMap& tb, const Params& p, cudaS
   }
   const int total = p.tiles_m * ((p.tiles_n + NP - 1) / NP);
   int clusters = num_sms() / (2 * NP);
-  if (total < clusters) clusters = total;
+  if (total < clusters && p.sk_tiles == 0) clusters = total;  // Stream-K needs every cluster
   if (clusters < 1) clusters = 1;
   cudaLaunchConfig_t cfg;
   std::memset(&cfg, 0, sizeof(cfg));
@@ -681,6 +810,100 @@ int num_sms() {
 // multicast across two pairs; measured slower on the 1.5B shapes - the pairs
 // run in lock-step on every smem slot - so it is off by default)
 static int g_gemm_np = -1;
+static int g_gemm_sk = -1;  // Stream-K tail: env MOBIUS_GEMM_SK=0 disables
+
+// Stream-K workspace, one per stream (GEMMs on different streams may run
+// concurrently).  Grows on demand; counters start at zero and are reset by
+// the reducing warp, so consecutive launches on one stream reuse them.
+struct SkWs {
+  cudaStream_t s;
+  float* ws;
+  size_t ws_bytes;
+  int* cnt;
+  size_t cnt_n;
+};
+static std::mutex g_sk_mu;
+static SkWs g_sk[16];
+static int g_sk_n = 0;
+
+static int sk_workspace(cudaStream_t s, size_t ws_bytes, size_t cnt_n, float** ws, int** cnt) {
+  std::lock_guard<std::mutex> lk(g_sk_mu);
+  SkWs* e = nullptr;
+  for (int i = 0; i < g_sk_n; ++i)
+    if (g_sk[i].s == s) e = &g_sk[i];
+  if (!e) {
+    if (g_sk_n == 16) MOBIUS_FAIL(MOBIUS_ENOMEM, "gemm: too many streams for Stream-K workspaces");
+    e = &g_sk[g_sk_n++];
+    std::memset(e, 0, sizeof(*e));
+    e->s = s;
+  }
+  if (e->ws_bytes < ws_bytes) {
+    if (e->ws) {
+      cudaStreamSynchronize(s);
+      cudaFree(e->ws);
+    }
+    e->ws = nullptr;
+    e->ws_bytes = 0;
+    if (cudaMalloc(&e->ws, ws_bytes) != cudaSuccess) MOBIUS_FAIL(MOBIUS_ENOMEM, "gemm: Stream-K workspace");
+    e->ws_bytes = ws_bytes;
+  }
+  if (e->cnt_n < cnt_n) {
+    if (e->cnt) {
+      cudaStreamSynchronize(s);
+      cudaFree(e->cnt);
+    }
+    e->cnt = nullptr;
+    e->cnt_n = 0;
+    if (cudaMalloc(&e->cnt, cnt_n * sizeof(int)) != cudaSuccess) MOBIUS_FAIL(MOBIUS_ENOMEM, "gemm: Stream-K counters");
+    if (cudaMemset(e->cnt, 0, cnt_n * sizeof(int)) != cudaSuccess) MOBIUS_FAIL(MOBIUS_ECUDA, "gemm: counter memset");
+    e->cnt_n = cnt_n;
+  }
+  *ws = e->ws;
+  *cnt = e->cnt;
+  return MOBIUS_OK;
+}
+
+// host copy of the device owner function (same integer arithmetic)
+static int sk_owner_h(int64_t units, int64_t g, int ncl) {
+  auto start = [&](int c) { return (int64_t)c * units / ncl; };
+  int c = (int)(g * ncl / units);
+  while (c + 1 < ncl && start(c + 1) <= g) ++c;
+  while (c > 0 && start(c) > g) --c;
+  return c;
+}
+
+// Wave quantisation: T tiles over P clusters take ceil(T/P) tile-times.
+// Stream-K keeps floor(T/P)-1 whole waves and spreads the remaining tiles'
+// k-blocks evenly (cost ~ T/P + fixup); used when that saves >= 5% of a
+// wave and every cluster gets a reasonable k-range.
+static void plan_stream_k(Params& p, int P) {
+  p.sk_tiles = 0;
+  p.sk_units = 0;
+  p.sk_maxseg = 0;
+  if (g_gemm_sk < 0) {
+    const char* e = getenv("MOBIUS_GEMM_SK");
+    g_gemm_sk = (e && e[0] == '0') ? 0 : 1;
+  }
+  if (!g_gemm_sk) return;
+  const int T = p.tiles_m * p.tiles_n, nkb = p.num_kb;
+  if (T % P == 0) return;
+  const int waves = (T + P - 1) / P;
+  const int dp_waves = T / P >= 1 ? T / P - 1 : 0;
+  const int sk_tiles = T - dp_waves * P;
+  const double cost = dp_waves + (double)sk_tiles / P + 0.25;
+  if (cost > waves - 0.05) return;
+  const int64_t units = (int64_t)sk_tiles * nkb;
+  const int64_t per = units / P;
+  if (per < 4 || per * 4 < nkb) return;
+  int maxseg = 1;
+  for (int t = 0; t < sk_tiles; ++t) {
+    const int n = sk_owner_h(units, (int64_t)(t + 1) * nkb - 1, P) - sk_owner_h(units, (int64_t)t * nkb, P) + 1;
+    if (n > maxseg) maxseg = n;
+  }
+  p.sk_tiles = sk_tiles;
+  p.sk_units = units;
+  p.sk_maxseg = maxseg;
+}
 
 template <int BN>
 static int gemm_bf16_2cta_bn(const GemmDesc& d, cudaStream_t s) {
@@ -713,6 +936,14 @@ static int gemm_bf16_2cta_bn(const GemmDesc& d, cudaStream_t s) {
   p.bias = (const __nv_bfloat16*)d.bias;
   p.R = (const __nv_bfloat16*)d.R.ptr; p.ldr = d.R.ld;
   p.AUX = (__nv_bfloat16*)d.AUX.ptr; p.ldx = d.AUX.ld;
+  if (g_gemm_np != 2) {
+    plan_stream_k(p, num_sms() / 2);
+    if (p.sk_tiles) {
+      const size_t ws = (size_t)p.sk_tiles * p.sk_maxseg * 8 * 32 * BN * sizeof(float);
+      int rc2 = sk_workspace(s, ws, (size_t)p.sk_tiles * 8, &p.sk_ws, &p.sk_cnt);
+      if (rc2) return rc2;
+    }
+  }
   if (g_gemm_np == 2 && p.tiles_n >= 2) {  // A multicast across two pairs
     if (!d.a_mn && !d.b_mn) return launch2<BN, false, false, 2>(ta, tb, p, s);
     if (!d.a_mn && d.b_mn) return launch2<BN, false, true, 2>(ta, tb, p, s);
@@ -731,6 +962,11 @@ static int gemm_bf16_2cta_bn(const GemmDesc& d, cudaStream_t s) {
 static int gemm_bf16_2cta(const GemmDesc& d, cudaStream_t s) { return gemm_bf16_2cta_bn<256>(d, s); }
 
 static int g_gemm_mode = -1;  // -1 auto (env MOBIUS_GEMM_2CTA, default on), 0 off, 1 on
+
+void gemm_set_config(int two_cta, int stream_k) {
+  g_gemm_mode = two_cta;
+  g_gemm_sk = stream_k;
+}
 
 int gemm_bf16(const GemmDesc& d, cudaStream_t s) {
   if (g_gemm_mode < 0) {

@@ -71,6 +71,13 @@ extern "C" int mobius_kt_gemm(int dtype, int M, int N, int K, int nb1, int nb2, 
   return sync_rc(dtype == MOBIUS_BF16 ? gemm_bf16(d, 0) : gemm_f32(d, 0));
 }
 
+extern "C" int mobius_kt_gemm_config(int two_cta, int stream_k) {
+  if (two_cta < -1 || two_cta > 1 || stream_k < -1 || stream_k > 1)
+    MOBIUS_FAIL(MOBIUS_EINVAL, "gemm_config: modes are -1, 0 or 1");
+  gemm_set_config(two_cta, stream_k);
+  return MOBIUS_OK;
+}
+
 extern "C" int mobius_kt_layernorm_fwd(int dtype, const void* x, const void* g, const void* b, void* y, float* mu,
                                        float* rstd, int rows, int h) {
   if (dtype == MOBIUS_BF16)

@@ -77,6 +77,62 @@ def test_gemm_layouts(dtype, a_mn, b_mn, shape):
         assert rel(from_dev(tC), ref) < tol, (shape, a_mn, b_mn, c_f32)
 
 
+# Stream-K tail of the 2-CTA kernel: shapes whose last wave is partial over
+# the 74 SM pairs (8192x1600 = 224 tiles -> 2 full waves + 76 split tiles;
+# 2000x1000 = 32 tiles, each split over up to 4 pairs, ragged M, N and K).
+SK_SHAPES = [(8192, 1600, 1600), (2000, 1000, 3000), (1600, 1600, 8192)]
+
+
+@pytest.mark.parametrize("shape", SK_SHAPES)
+@pytest.mark.parametrize("a_mn,b_mn", [(False, True), (True, True), (False, False)])
+def test_gemm_stream_k(shape, a_mn, b_mn):
+    M, N, K = shape
+    g = torch.Generator(device=DEV).manual_seed(7)
+    A = torch.randn(M, K, device=DEV, generator=g).to(torch.bfloat16)
+    B = torch.randn(N, K, device=DEV, generator=g).to(torch.bfloat16)
+    bias = torch.randn(N, device=DEV, generator=g).to(torch.bfloat16)
+    R = torch.randn(M, N, device=DEV, generator=g).to(torch.bfloat16)
+    ref = A.double() @ B.double().T
+    tA = A.T.contiguous() if a_mn else A
+    tB = B.T.contiguous() if b_mn else B
+
+    def run(sk, epi, **kw):
+        kt.gemm_config(-1, sk)
+        try:
+            tC = kw.pop("C")
+            kt.gemm(BF16, M, N, K, tA, M if a_mn else K, a_mn, tB, N if b_mn else K, b_mn, tC, N, epi=epi, **kw)
+            torch.cuda.synchronize()
+        finally:
+            kt.gemm_config(-1, -1)
+        return tC
+
+    def nrel(a, b):
+        return float((a.double() - b).norm() / b.norm())
+
+    # plain store, fp32 out: split-K partial sums reduce to the same product
+    c_sk = run(1, 0, C=torch.zeros(M, N, device=DEV), c_f32=True)
+    c_dp = run(0, 0, C=torch.zeros(M, N, device=DEV), c_f32=True)
+    assert nrel(c_sk, ref) < 1e-5 and nrel(c_dp, ref) < 1e-5
+    # deterministic: the reduction order is fixed by segment index
+    c_sk2 = run(1, 0, C=torch.zeros(M, N, device=DEV), c_f32=True)
+    assert torch.equal(c_sk, c_sk2)
+    # fused epilogues run once, on the reduced tile
+    out = run(1, 3, C=torch.zeros(M, N, device=DEV, dtype=torch.bfloat16), bias=bias, R=R, ldr=N)
+    assert nrel(out, ref + bias.double() + R.double()) < 1e-2
+    aux = torch.zeros(M, N, device=DEV, dtype=torch.bfloat16)
+    gl = run(1, 2, C=torch.zeros(M, N, device=DEV, dtype=torch.bfloat16), bias=bias, AUX=aux, ldx=N)
+    u = ref + bias.double()
+    assert nrel(aux, u) < 1e-2
+    assert nrel(gl, torch.nn.functional.gelu(u, approximate="tanh")) < 1e-2
+    # fp32 accumulate (dW): C = C0 + alpha * acc
+    C0 = torch.randn(M, N, device=DEV, generator=g)
+    acc = run(1, 5, C=C0.clone(), c_f32=True, accumulate=True, alpha=0.5)
+    assert nrel(acc, C0.double() + 0.5 * ref) < 1e-5
+    # counters self-reset: a second accumulate launch adds again
+    acc2 = run(1, 5, C=acc, c_f32=True, accumulate=True, alpha=0.5)
+    assert nrel(acc2, C0.double() + ref) < 1e-5
+
+
 @pytest.mark.parametrize("dtype", [BF16, F32])
 def test_gemm_epilogues(dtype):
     M, N, K = 300, 520, 200
