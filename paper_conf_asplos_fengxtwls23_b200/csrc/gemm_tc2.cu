@@ -1,0 +1,531 @@
+// 2-CTA (cta_group::2) persistent tcgen05 GEMM for plain (non-batched,
+// non-causal) products with M, N >= 256: 256 x 256 x 64 tiles over SM pairs,
+// 8 epilogue warps, and a deterministic Stream-K tail for the last partial
+// wave of long-K shapes.  Shared epilogue and parameters: gemm_common.cuh.
+#include "gemm_common.cuh"
+
+namespace mobius {
+namespace gemm_detail {
+
+// ======================================================================
+// 2-CTA variant (cta_group::2): a cluster of two CTAs on the two SMs of a
+// TPC computes a 256 x BN tile; each CTA loads its 128 rows of A and half of
+// B (BN/2 rows) into its own smem, the leader CTA issues
+// tcgen05.mma.cta_group::2 (M = 256) and multicasts the commits, each CTA's
+// epilogue drains its own 128 TMEM lanes.  Halves per-SM operand traffic.
+// Used for plain (non-batched, non-causal) GEMMs with N >= 256.
+template <int BN>
+struct Cfg2 {
+  static constexpr int A_BYTES = 128 * BK * 2;
+  static constexpr int B_BYTES = (BN / 2) * BK * 2;
+  static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+  static constexpr int STAGES = (200 * 1024) / STAGE_BYTES > 8 ? 8 : (200 * 1024) / STAGE_BYTES;
+  static constexpr int TMEM_COLS = 2 * BN;
+  static constexpr int SMEM = 1024 + STAGES * STAGE_BYTES + 256;
+};
+
+// One unit of work of a cluster: k-blocks [k0, k1) of tile t, which is
+// segment seg of nseg (nseg == 1: a whole tile, no fixup).
+struct Work {
+  int t, k0, k1, seg, nseg;
+};
+
+__device__ __forceinline__ int64_t sk_start(const Params& p, int c, int ncl) {
+  return (int64_t)c * p.sk_units / ncl;
+}
+// cluster whose Stream-K range holds unit g
+__device__ __forceinline__ int sk_owner(const Params& p, int64_t g, int ncl) {
+  int c = (int)(g * ncl / p.sk_units);
+  while (c + 1 < ncl && sk_start(p, c + 1, ncl) <= g) ++c;
+  while (c > 0 && sk_start(p, c, ncl) > g) --c;
+  return c;
+}
+
+// Per-cluster schedule: its Stream-K range over the first sk_tiles tiles
+// (cut at tile boundaries), then whole tiles sk_tiles + cl, + ncl, ...
+// The producer, MMA issuer and epilogue walk identical sequences.
+struct Sched {
+  int64_t g, gend;
+  int t, cl, ncl;
+  __device__ __forceinline__ Sched(const Params& p, int cl_, int ncl_) : cl(cl_), ncl(ncl_) {
+    g = p.sk_tiles ? sk_start(p, cl, ncl) : 0;
+    gend = p.sk_tiles ? sk_start(p, cl + 1, ncl) : 0;
+    t = p.sk_tiles + cl;
+  }
+  __device__ __forceinline__ bool next(const Params& p, int total, Work& w) {
+    if (g < gend) {
+      const int nkb = p.num_kb;
+      const int tt = (int)(g / nkb);
+      w.t = tt;
+      w.k0 = (int)(g - (int64_t)tt * nkb);
+      w.k1 = (int)min((int64_t)nkb, (int64_t)w.k0 + (gend - g));
+      const int first = sk_owner(p, (int64_t)tt * nkb, ncl);
+      const int last = sk_owner(p, (int64_t)(tt + 1) * nkb - 1, ncl);
+      w.seg = cl - first;
+      w.nseg = last - first + 1;
+      g += w.k1 - w.k0;
+      return true;
+    }
+    if (t < total) {
+      w.t = t;
+      w.k0 = 0;
+      w.k1 = p.num_kb;
+      w.seg = 0;
+      w.nseg = 1;
+      t += ncl;
+      return true;
+    }
+    return false;
+  }
+};
+
+// NP pairs per cluster (cluster = 2*NP CTAs along x).  Pairs of one cluster
+// compute horizontally adjacent 256 x BN tiles (same rows): with NP = 2 the
+// A tile is loaded once per cluster - each CTA loads half of its 128 A rows
+// and TMA-multicasts them to its counterpart in the other pair - cutting the
+// L2 -> SM operand traffic by a quarter.
+template <int BN, bool A_MN, bool B_MN, int NP>
+__global__ void __launch_bounds__(NUM_THREADS2, 1)
+    gemm_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, const Params p) {
+  using C = Cfg2<BN>;
+  constexpr int BM2 = 256;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* smA = smem;
+  uint8_t* smB = smem + C::STAGES * C::A_BYTES;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + C::STAGES * C::STAGE_BYTES);
+  uint64_t* empty = full + C::STAGES;
+  uint64_t* tfull = empty + C::STAGES;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+
+  const int warp = threadIdx.x / 32;
+  const int lane = threadIdx.x % 32;
+  const uint32_t rank = ptx::cluster_ctarank();
+  const uint32_t pair = rank >> 1, r2 = rank & 1;
+  const bool leader = r2 == 0;  // MMA-issuing CTA of this pair
+  const int cl = blockIdx.x / (2 * NP), ncl = gridDim.x / (2 * NP);
+  const int tiles_n2 = (p.tiles_n + NP - 1) / NP;  // column groups of NP tiles
+
+  if (warp == 0 && lane == 0) {
+    ptx::tma_prefetch_desc(&tmA);
+    ptx::tma_prefetch_desc(&tmB);
+    for (int s = 0; s < C::STAGES; ++s) {
+      ptx::mbar_init(&full[s], 1);
+      ptx::mbar_init(&empty[s], NP);  // one commit per pair that reads this CTA's slot
+    }
+    for (int a = 0; a < 2; ++a) {
+      ptx::mbar_init(&tfull[a], 1);
+      ptx::mbar_init(&tempty[a], 16);  // 8 epilogue warps x 2 CTAs of the pair (leader's copy)
+    }
+    ptx::fence_mbar_init();
+  }
+  if (warp == 1) ptx::tmem_alloc_2sm<C::TMEM_COLS>(tmem_slot);
+  ptx::tc_fence_before();
+  ptx::cluster_sync();
+  ptx::tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+  const int total = p.tiles_m * tiles_n2;
+
+  auto tile_of = [&](int t, int& mt, int& nt) {  // grouped along M for L2 reuse
+    constexpr int GROUP = 8;
+    const int span = GROUP * tiles_n2;
+    const int g = t / span, first_m = g * GROUP;
+    const int gm = min(GROUP, p.tiles_m - first_m);
+    const int rr = t - g * span;
+    mt = first_m + rr % gm;
+    nt = (rr / gm) * NP + (int)pair;
+  };
+
+  if (warp == 0) {
+    if (lane == 0) {  // TMA producer (every CTA)
+      int stage = 0;
+      uint32_t phase = 0;
+      const uint16_t amask = (uint16_t)((1u << r2) | (NP == 2 ? (1u << (r2 + 2)) : 0u));
+      Sched sc(p, cl, ncl);
+      Work w;
+      while (sc.next(p, total, w)) {
+        int mt, nt;
+        tile_of(w.t, mt, nt);
+        const int m0 = mt * BM2 + (int)r2 * 128, n0 = nt * BN + (int)r2 * (BN / 2);
+        for (int kb = w.k0; kb < w.k1; ++kb) {
+          ptx::mbar_wait_cluster(&empty[stage], phase ^ 1);
+          if (leader) ptx::mbar_arrive_expect_tx(&full[stage], 2 * C::STAGE_BYTES);
+          uint8_t* a = smA + stage * C::A_BYTES;
+          uint8_t* b = smB + stage * C::B_BYTES;
+          const int k0 = kb * BK;
+          if (NP == 1) {
+            if (A_MN) {
+#pragma unroll
+              for (int i = 0; i < 2; ++i) ptx::tma_load_4d_2sm(a + i * 8192, &tmA, &full[stage], m0 + 64 * i, k0, 0, 0);
+            } else {
+              ptx::tma_load_4d_2sm(a, &tmA, &full[stage], k0, m0, 0, 0);
+            }
+          } else {  // this pair loads half h = pair of the 128 A rows and multicasts it
+            const int h = (int)pair;
+            if (A_MN)
+              ptx::tma_load_4d_2sm_mc(a + h * 8192, &tmA, &full[stage], amask, m0 + 64 * h, k0, 0, 0);
+            else
+              ptx::tma_load_4d_2sm_mc(a + h * 8192, &tmA, &full[stage], amask, k0, m0 + 64 * h, 0, 0);
+          }
+          if (B_MN) {
+#pragma unroll
+            for (int i = 0; i < BN / 128; ++i)
+              ptx::tma_load_4d_2sm(b + i * 8192, &tmB, &full[stage], n0 + 64 * i, k0, 0, 0);
+          } else {
+            ptx::tma_load_4d_2sm(b, &tmB, &full[stage], k0, n0, 0, 0);
+          }
+          if (++stage == C::STAGES) {
+            stage = 0;
+            phase ^= 1;
+          }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (leader && lane == 0) {  // MMA issuer (pair leader)
+      constexpr uint32_t IDESC = ptx::idesc_bf16(BM2, BN, A_MN ? 1 : 0, B_MN ? 1 : 0);
+      const uint16_t all_mask = (uint16_t)((1u << (2 * NP)) - 1);
+      const uint16_t pair_mask = (uint16_t)(3u << (2 * pair));
+      int stage = 0;
+      uint32_t phase = 0;
+      int acc = 0;
+      uint32_t aphase = 0;
+      Sched sc(p, cl, ncl);
+      Work w;
+      while (sc.next(p, total, w)) {
+        ptx::mbar_wait_cluster(&tempty[acc], aphase ^ 1);
+        ptx::tc_fence_after();
+        const uint32_t tmem_d = tmem_base + acc * BN;
+        for (int kb = w.k0; kb < w.k1; ++kb) {
+          ptx::mbar_wait_cluster(&full[stage], phase);
+          ptx::tc_fence_after();
+          const uint32_t a_base = ptx::smem_u32(smA + stage * C::A_BYTES);
+          const uint32_t b_base = ptx::smem_u32(smB + stage * C::B_BYTES);
+#pragma unroll
+          for (int k = 0; k < BK / 16; ++k) {
+            uint64_t ad = A_MN ? ptx::sdesc_sw128(a_base + k * 2048, 8192, 1024)
+                               : ptx::sdesc_sw128(a_base + k * 32, 16, 1024);
+            uint64_t bd = B_MN ? ptx::sdesc_sw128(b_base + k * 2048, 8192, 1024)
+                               : ptx::sdesc_sw128(b_base + k * 32, 16, 1024);
+            ptx::mma_bf16_2sm(tmem_d, ad, bd, IDESC, (kb > w.k0 || k > 0) ? 1u : 0u);
+          }
+          // the slot may be refilled by this pair's producers and (A halves)
+          // by the other pair's: free it in every CTA of the cluster
+          ptx::mma_commit_2sm(&empty[stage], all_mask);
+          if (++stage == C::STAGES) {
+            stage = 0;
+            phase ^= 1;
+          }
+        }
+        ptx::mma_commit_2sm(&tfull[acc], pair_mask);  // accumulator ready in both CTAs of the pair
+        if (++acc == 2) {
+          acc = 0;
+          aphase ^= 1;
+        }
+      }
+    }
+  } else {
+    // epilogue (warps 2..9): warp w drains TMEM lane quadrant w % 4 (rows
+    // mt*256 + r2*128 + 32*(w%4) + lane), column half (w-2)/4 of the tile,
+    // 64 columns per step
+    const int q = warp & 3, hf = (warp - 2) >> 2;
+    constexpr int HALF = BN / 2;
+    const uint32_t tempty_leader = ptx::mapa_shared(ptx::smem_u32(&tempty[0]), pair * 2);
+    int acc = 0;
+    uint32_t aphase = 0;
+    Sched sc(p, cl, ncl);
+    Work w;
+    while (sc.next(p, total, w)) {
+      int mt, nt;
+      tile_of(w.t, mt, nt);
+      const int m = mt * BM2 + (int)r2 * 128 + q * 32 + lane;
+      const int ncol0 = nt * BN + hf * HALF;
+      const uint32_t tmem_row = tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + hf * HALF;
+      ptx::mbar_wait_cluster(&tfull[acc], aphase);
+      ptx::tc_fence_after();
+      if (w.nseg == 1) {
+#pragma unroll 1
+        for (int c = 0; c < HALF; c += 64) {
+          uint32_t r[64];
+          __syncwarp();
+          ptx::tmem_ld32(tmem_row + c, *reinterpret_cast<uint32_t(*)[32]>(&r[0]));
+          ptx::tmem_ld32(tmem_row + c + 32, *reinterpret_cast<uint32_t(*)[32]>(&r[32]));
+          ptx::tmem_ld_wait();
+          if (c + 64 >= HALF) {  // last TMEM read of this tile: hand the accumulator back early
+            ptx::tc_fence_before();
+            __syncwarp();
+            if (lane == 0) ptx::mbar_arrive_cluster(tempty_leader + acc * 8);
+          }
+          float v[64];
+#pragma unroll
+          for (int i = 0; i < 64; ++i) v[i] = __uint_as_float(r[i]) * p.alpha;
+          epi_vals<64>(p, v, m, 0, 0, ncol0 + c);
+        }
+      } else {
+        // Stream-K segment: raw partial (32 rows x BN/2 fp32 per warp) to the
+        // workspace, lane-interleaved so every store is 512 contiguous bytes
+        const int wq = (int)r2 * 8 + (warp - 2);
+        constexpr int SLOT = 32 * HALF;  // floats per warp slot
+        float* base = p.sk_ws + ((int64_t)w.t * p.sk_maxseg * 16 + wq) * SLOT;
+        const int64_t seg_stride = 16 * (int64_t)SLOT;
+        float4* mine = reinterpret_cast<float4*>(base + w.seg * seg_stride) + lane;
+#pragma unroll 1
+        for (int c = 0; c < HALF; c += 32) {
+          uint32_t r[32];
+          __syncwarp();
+          ptx::tmem_ld32(tmem_row + c, r);
+          ptx::tmem_ld_wait();
+#pragma unroll
+          for (int i = 0; i < 8; ++i)
+            __stcg(mine + ((c / 32) * 8 + i) * 32, make_float4(__uint_as_float(r[4 * i]), __uint_as_float(r[4 * i + 1]),
+                                                              __uint_as_float(r[4 * i + 2]), __uint_as_float(r[4 * i + 3])));
+        }
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive_cluster(tempty_leader + acc * 8);  // accumulator free: MMA runs on
+        __threadfence();
+        __syncwarp();
+        int old = 0;
+        int* cnt = p.sk_cnt + (int64_t)w.t * 16 + wq;
+        if (lane == 0) old = atomicAdd(cnt, 1);
+        old = __shfl_sync(0xffffffffu, old, 0);
+        if (old == w.nseg - 1) {  // last segment to arrive: reduce in segment order
+          __threadfence();
+#pragma unroll 1
+          for (int c = 0; c < HALF; c += 32) {
+            float v[32];
+#pragma unroll
+            for (int i = 0; i < 32; ++i) v[i] = 0.f;
+#pragma unroll 1
+            for (int sgi = 0; sgi < w.nseg; ++sgi) {
+              const float4* src = reinterpret_cast<const float4*>(base + sgi * seg_stride) + lane;
+              float4 x[8];
+#pragma unroll
+              for (int i = 0; i < 8; ++i) x[i] = __ldcg(src + ((c / 32) * 8 + i) * 32);
+#pragma unroll
+              for (int i = 0; i < 8; ++i) {
+                v[4 * i] += x[i].x;
+                v[4 * i + 1] += x[i].y;
+                v[4 * i + 2] += x[i].z;
+                v[4 * i + 3] += x[i].w;
+              }
+            }
+#pragma unroll
+            for (int i = 0; i < 32; ++i) v[i] *= p.alpha;
+            epi_vals<32>(p, v, m, 0, 0, ncol0 + c);
+          }
+          if (lane == 0) *cnt = 0;  // self-cleaning for the next launch
+        }
+      }
+      if (++acc == 2) {
+        acc = 0;
+        aphase ^= 1;
+      }
+    }
+  }
+
+  __syncthreads();
+  ptx::cluster_sync();
+  if (warp == 1) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc_2sm<C::TMEM_COLS>(tmem_base);
+  }
+}
+
+template <int BN, bool A_MN, bool B_MN, int NP>
+int launch2(const CUtensorMap& ta, const CUtensorMap& tb, const Params& p, cudaStream_t s) {
+  auto k = gemm_tc2_kernel<BN, A_MN, B_MN, NP>;
+  static bool attr_set = false;
+  if (!attr_set) {
+    if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg2<BN>::SMEM) != cudaSuccess)
+      MOBIUS_FAIL(MOBIUS_ECUDA, "cudaFuncSetAttribute(smem, 2cta) failed");
+    attr_set = true;
+  }
+  const int total = p.tiles_m * ((p.tiles_n + NP - 1) / NP);
+  int clusters = num_sms() / (2 * NP);
+  if (total < clusters && p.sk_tiles == 0) clusters = total;  // Stream-K needs every cluster
+  if (clusters < 1) clusters = 1;
+  cudaLaunchConfig_t cfg;
+  std::memset(&cfg, 0, sizeof(cfg));
+  cfg.gridDim = dim3(2 * NP * clusters);
+  cfg.blockDim = dim3(NUM_THREADS2);
+  cfg.dynamicSmemBytes = Cfg2<BN>::SMEM;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = 2 * NP;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  cudaError_t e = cudaLaunchKernelEx(&cfg, k, ta, tb, p);
+  if (e != cudaSuccess) MOBIUS_FAIL(MOBIUS_ECUDA, "gemm_tc2 launch: %s", cudaGetErrorString(e));
+  return MOBIUS_OK;
+}
+
+}  // namespace gemm_detail
+
+using namespace gemm_detail;
+
+// multicast across two pairs; measured slower on the 1.5B shapes - the pairs
+// run in lock-step on every smem slot - so it is off by default)
+static int g_gemm_np = -1;
+static int g_gemm_sk = -1;  // Stream-K tail: env MOBIUS_GEMM_SK=0 disables
+
+// Stream-K workspace, one per stream (GEMMs on different streams may run
+// concurrently).  Grows on demand; counters start at zero and are reset by
+// the reducing warp, so consecutive launches on one stream reuse them.
+struct SkWs {
+  cudaStream_t s;
+  float* ws;
+  size_t ws_bytes;
+  int* cnt;
+  size_t cnt_n;
+};
+static std::mutex g_sk_mu;
+static SkWs g_sk[16];
+static int g_sk_n = 0;
+
+static int sk_workspace(cudaStream_t s, size_t ws_bytes, size_t cnt_n, float** ws, int** cnt) {
+  std::lock_guard<std::mutex> lk(g_sk_mu);
+  SkWs* e = nullptr;
+  for (int i = 0; i < g_sk_n; ++i)
+    if (g_sk[i].s == s) e = &g_sk[i];
+  if (!e) {
+    if (g_sk_n == 16) MOBIUS_FAIL(MOBIUS_ENOMEM, "gemm: too many streams for Stream-K workspaces");
+    e = &g_sk[g_sk_n++];
+    std::memset(e, 0, sizeof(*e));
+    e->s = s;
+  }
+  if (e->ws_bytes < ws_bytes) {
+    if (e->ws) {
+      cudaStreamSynchronize(s);
+      cudaFree(e->ws);
+    }
+    e->ws = nullptr;
+    e->ws_bytes = 0;
+    if (cudaMalloc(&e->ws, ws_bytes) != cudaSuccess) MOBIUS_FAIL(MOBIUS_ENOMEM, "gemm: Stream-K workspace");
+    e->ws_bytes = ws_bytes;
+  }
+  if (e->cnt_n < cnt_n) {
+    if (e->cnt) {
+      cudaStreamSynchronize(s);
+      cudaFree(e->cnt);
+    }
+    e->cnt = nullptr;
+    e->cnt_n = 0;
+    if (cudaMalloc(&e->cnt, cnt_n * sizeof(int)) != cudaSuccess) MOBIUS_FAIL(MOBIUS_ENOMEM, "gemm: Stream-K counters");
+    if (cudaMemset(e->cnt, 0, cnt_n * sizeof(int)) != cudaSuccess) MOBIUS_FAIL(MOBIUS_ECUDA, "gemm: counter memset");
+    e->cnt_n = cnt_n;
+  }
+  *ws = e->ws;
+  *cnt = e->cnt;
+  return MOBIUS_OK;
+}
+
+// host copy of the device owner function (same integer arithmetic)
+static int sk_owner_h(int64_t units, int64_t g, int ncl) {
+  auto start = [&](int c) { return (int64_t)c * units / ncl; };
+  int c = (int)(g * ncl / units);
+  while (c + 1 < ncl && start(c + 1) <= g) ++c;
+  while (c > 0 && start(c) > g) --c;
+  return c;
+}
+
+// Wave quantisation: T tiles over P clusters take ceil(T/P) tile-times.
+// Stream-K keeps floor(T/P)-1 whole waves and spreads the remaining tiles'
+// k-blocks evenly (cost ~ T/P + fixup); used when that saves >= 5% of a
+// wave and every cluster gets a reasonable k-range.
+static void plan_stream_k(Params& p, int P) {
+  p.sk_tiles = 0;
+  p.sk_units = 0;
+  p.sk_maxseg = 0;
+  if (g_gemm_sk < 0) {
+    const char* e = getenv("MOBIUS_GEMM_SK");
+    g_gemm_sk = (e && e[0] == '0') ? 0 : 1;
+  }
+  if (!g_gemm_sk) return;
+  const int T = p.tiles_m * p.tiles_n, nkb = p.num_kb;
+  if (T % P == 0) return;
+  const int waves = (T + P - 1) / P;
+  const int dp_waves = T / P >= 1 ? T / P - 1 : 0;
+  const int sk_tiles = T - dp_waves * P;
+  const double cost = dp_waves + (double)sk_tiles / P + 0.25;
+  if (cost > waves - 0.3) return;
+  // Short K (< 64 k-blocks): the fp32 partial round trip costs more than the
+  // wave it saves (measured: 8192x1600x1600 46 -> 58 us); long K gains
+  // (8192x1600x6400 150 -> 137 us, 1600x6400x8192 165 -> 150 us, ncu).
+  if (nkb < 64) return;
+  const int64_t units = (int64_t)sk_tiles * nkb;
+  const int64_t per = units / P;
+  if (per < 4 || per * 4 < nkb) return;
+  int maxseg = 1;
+  for (int t = 0; t < sk_tiles; ++t) {
+    const int n = sk_owner_h(units, (int64_t)(t + 1) * nkb - 1, P) - sk_owner_h(units, (int64_t)t * nkb, P) + 1;
+    if (n > maxseg) maxseg = n;
+  }
+  p.sk_tiles = sk_tiles;
+  p.sk_units = units;
+  p.sk_maxseg = maxseg;
+}
+
+template <int BN>
+static int gemm_bf16_2cta_bn(const GemmDesc& d, cudaStream_t s) {
+  if (g_gemm_np < 0) {
+    const char* e = getenv("MOBIUS_GEMM_NP");
+    g_gemm_np = (e && e[0] == '2') ? 2 : 1;
+  }
+  const bool mc = g_gemm_np == 2 && (d.N + BN - 1) / BN >= 2;
+  CUtensorMap ta, tb;
+  int rc;
+  if (d.a_mn)
+    rc = make_map(&ta, d.A, d.M, d.K, d.nb1, d.nb2, BK);
+  else
+    rc = make_map(&ta, d.A, d.K, d.M, d.nb1, d.nb2, mc ? 64 : 128);
+  if (rc) return rc;
+  if (d.b_mn)
+    rc = make_map(&tb, d.B, d.N, d.K, d.nb1, d.nb2, BK);
+  else
+    rc = make_map(&tb, d.B, d.K, d.N, d.nb1, d.nb2, BN / 2);
+  if (rc) return rc;
+  Params p;
+  std::memset(&p, 0, sizeof(p));
+  p.M = d.M; p.N = d.N; p.K = d.K; p.nb1 = 1; p.nb2 = 1;
+  p.tiles_m = (d.M + 255) / 256;
+  p.tiles_n = (d.N + BN - 1) / BN;
+  p.num_kb = (d.K + BK - 1) / BK;
+  p.causal = CAUSAL_NONE;
+  p.epi = d.epi; p.c_f32 = d.c_f32 ? 1 : 0; p.accumulate = d.accumulate ? 1 : 0; p.alpha = d.alpha;
+  p.C = (__nv_bfloat16*)d.C.ptr; p.ldc = d.C.ld;
+  p.bias = (const __nv_bfloat16*)d.bias;
+  p.R = (const __nv_bfloat16*)d.R.ptr; p.ldr = d.R.ld;
+  p.AUX = (__nv_bfloat16*)d.AUX.ptr; p.ldx = d.AUX.ld;
+  if (g_gemm_np != 2) {
+    plan_stream_k(p, num_sms() / 2);
+    if (p.sk_tiles) {
+      const size_t ws = (size_t)p.sk_tiles * p.sk_maxseg * 16 * 32 * (BN / 2) * sizeof(float);
+      int rc2 = sk_workspace(s, ws, (size_t)p.sk_tiles * 16, &p.sk_ws, &p.sk_cnt);
+      if (rc2) return rc2;
+    }
+  }
+  if (g_gemm_np == 2 && p.tiles_n >= 2) {  // A multicast across two pairs
+    if (!d.a_mn && !d.b_mn) return launch2<BN, false, false, 2>(ta, tb, p, s);
+    if (!d.a_mn && d.b_mn) return launch2<BN, false, true, 2>(ta, tb, p, s);
+    if (d.a_mn && !d.b_mn) return launch2<BN, true, false, 2>(ta, tb, p, s);
+    return launch2<BN, true, true, 2>(ta, tb, p, s);
+  }
+  if (!d.a_mn && !d.b_mn) return launch2<BN, false, false, 1>(ta, tb, p, s);
+  if (!d.a_mn && d.b_mn) return launch2<BN, false, true, 1>(ta, tb, p, s);
+  if (d.a_mn && !d.b_mn) return launch2<BN, true, false, 1>(ta, tb, p, s);
+  return launch2<BN, true, true, 1>(ta, tb, p, s);
+}
+
+// 256 x 256 tiles: at 64 B/clk/SM of operand traffic this is the only 2-CTA
+// shape that stays under the L2->SM feed rate (256 x 128 measured slower even
+// where it quantises better over the 74 SM pairs)
+int gemm_bf16_2cta(const GemmDesc& d, cudaStream_t s) { return gemm_bf16_2cta_bn<256>(d, s); }
+
+void gemm_2cta_set_stream_k(int stream_k) { g_gemm_sk = stream_k; }
+
+}  // namespace mobius

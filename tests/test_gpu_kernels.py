@@ -77,10 +77,11 @@ def test_gemm_layouts(dtype, a_mn, b_mn, shape):
         assert rel(from_dev(tC), ref) < tol, (shape, a_mn, b_mn, c_f32)
 
 
-# Stream-K tail of the 2-CTA kernel: shapes whose last wave is partial over
-# the 74 SM pairs (8192x1600 = 224 tiles -> 2 full waves + 76 split tiles;
-# 2000x1000 = 32 tiles, each split over up to 4 pairs, ragged M, N and K).
-SK_SHAPES = [(8192, 1600, 1600), (2000, 1000, 3000), (1600, 1600, 8192)]
+# Stream-K tail of the 2-CTA kernel (long K only): shapes whose last wave is
+# partial over the 74 SM pairs (8192x1600 = 224 tiles -> 2 full waves + 76
+# split tiles; 2000x1000 = 32 tiles, each split over up to 4 pairs, ragged
+# M, N and K; 1600x6400 = 175 tiles, the fc1 dW shape).
+SK_SHAPES = [(8192, 1600, 6400), (2000, 1000, 4104), (1600, 6400, 8192)]
 
 
 @pytest.mark.parametrize("shape", SK_SHAPES)
