@@ -374,7 +374,8 @@ def run_mobius(args, rank, world, local):
                              "device_step": st.device_step_ns / 1e6, "host_update_total": st.host_update_ns / 1e6,
                              "update_tail": st.update_tail_ns / 1e6},
             "memory": {"arena_GB": st.arena_bytes / 1e9, "ring_GB": st.ring_bytes / 1e9,
-                       "pinned_host_GB": st.pinned_bytes / 1e9, "recompute": bool(st.recompute)},
+                       "pinned_host_GB": st.pinned_bytes / 1e9, "recompute_blocks": int(st.recompute),
+                       "kept_layout": "compact (x, qkv, o, x1, u, lse, LN stats)"},
             "gpu_launches": int(sum(s.kernel_launches for s in stats)),
             "clocks": clocks,
         }

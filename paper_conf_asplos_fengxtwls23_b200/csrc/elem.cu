@@ -638,6 +638,38 @@ int cast_from_f32(const float* src, T* dst, int64_t n, cudaStream_t st) {
   return check_launch("cast");
 }
 
+namespace {
+__device__ __forceinline__ float gelu_tanh_approx(float u) {  // == gemm_common.cuh gelu_f
+  const float c = 0.7978845608028654f, a = 0.044715f;
+  float t;
+  asm("tanh.approx.f32 %0, %1;" : "=f"(t) : "f"(c * (u + a * u * u * u)));
+  return 0.5f * u * (1.f + t);
+}
+__global__ void gelu_fwd_k(const uint4* __restrict__ u, uint4* __restrict__ g, int64_t n8) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n8; i += (int64_t)gridDim.x * blockDim.x) {
+    uint4 x = u[i];
+    __nv_bfloat162* h = reinterpret_cast<__nv_bfloat162*>(&x);
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const float2 f = __bfloat1622float2(h[j]);
+      h[j] = __floats2bfloat162_rn(gelu_tanh_approx(f.x), gelu_tanh_approx(f.y));
+    }
+    g[i] = x;
+  }
+}
+}  // namespace
+
+int gelu_fwd_bf16(const __nv_bfloat16* u, __nv_bfloat16* g, int64_t n, cudaStream_t st) {
+  if (n <= 0) return MOBIUS_OK;
+  if (n % 8 || (reinterpret_cast<uintptr_t>(u) | reinterpret_cast<uintptr_t>(g)) & 15)
+    MOBIUS_FAIL(MOBIUS_EINVAL, "gelu_fwd: n %% 8 and 16-byte alignment required");
+  const int64_t n8 = n / 8;
+  int64_t blocks = (n8 + 255) / 256;
+  if (blocks > 148 * 8) blocks = 148 * 8;
+  gelu_fwd_k<<<(unsigned)blocks, 256, 0, st>>>(reinterpret_cast<const uint4*>(u), reinterpret_cast<uint4*>(g), n8);
+  return check_launch("gelu_fwd");
+}
+
 int flag_wait(const volatile int* flag, int value, cudaStream_t st) {
   flag_wait_k<<<1, 1, 0, st>>>(flag, value);
   return check_launch("flag_wait");

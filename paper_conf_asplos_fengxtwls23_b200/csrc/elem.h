@@ -46,6 +46,11 @@ int loss_accumulate(const float* loss_rows, int rows, double* acc, cudaStream_t 
 template <typename T>
 int colsum_accum(const T* X, int64_t ld, int rows, int n, float* out, cudaStream_t st);
 
+// g = gelu_tanh(u) elementwise, the same arithmetic (tanh.approx, bf16
+// rounding of the result) as the GEMM's EPI_BIAS_GELU epilogue, so a
+// recomputed g is bit-identical to the one the forward wrote (bf16 only).
+int gelu_fwd_bf16(const __nv_bfloat16* u, __nv_bfloat16* g, int64_t n, cudaStream_t st);
+
 // dst = (T) src
 template <typename T>
 int cast_from_f32(const float* src, T* dst, int64_t n, cudaStream_t st);

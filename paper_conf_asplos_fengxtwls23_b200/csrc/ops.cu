@@ -119,10 +119,11 @@ bool use_flash<__nv_bfloat16>(const Shape& sh) {
   return flash_supported(sh.dh(), sh.s) != 0;
 }
 
-int64_t block_acts_bytes(const Shape& sh, int e, bool flash) {
+int64_t block_acts_bytes(const Shape& sh, int e, bool flash, bool compact) {
   Carver c{nullptr};
   const int64_t T = sh.T(), h = sh.h, B = (int64_t)sh.mbs * sh.nh, s = sh.s;
-  c.take<char>(T * h * e);      // a
+  const int64_t full = compact ? 0 : 1;
+  c.take<char>(full * T * h * e);      // a
   c.take<char>(T * 4);          // mu1
   c.take<char>(T * 4);          // rs1
   c.take<char>(T * 3 * h * e);  // qkv
@@ -130,19 +131,20 @@ int64_t block_acts_bytes(const Shape& sh, int e, bool flash) {
   c.take<char>(flash ? B * s * 4 : 0);      // lse
   c.take<char>(T * h * e);      // o
   c.take<char>(T * h * e);      // x1
-  c.take<char>(T * h * e);      // a2
+  c.take<char>(full * T * h * e);      // a2
   c.take<char>(T * 4);
   c.take<char>(T * 4);
   c.take<char>(T * 4 * h * e);  // u
-  c.take<char>(T * 4 * h * e);  // g
+  c.take<char>(full * T * 4 * h * e);  // g
   return c.off;
 }
 
 template <typename T>
-void carve_block_acts(const Shape& sh, uint8_t* base, BlockActs<T>& a) {
+void carve_block_acts(const Shape& sh, uint8_t* base, BlockActs<T>& a, bool compact) {
   Carver c{base};
   const int64_t Tn = sh.T(), h = sh.h, B = (int64_t)sh.mbs * sh.nh, s = sh.s, e = sizeof(T);
-  a.a = c.take<T>(Tn * h * e);
+  const int64_t full = compact ? 0 : 1;
+  a.a = compact ? nullptr : c.take<T>(Tn * h * e);
   a.mu1 = c.take<float>(Tn * 4);
   a.rs1 = c.take<float>(Tn * 4);
   const bool fl = use_flash<T>(sh);
@@ -151,11 +153,12 @@ void carve_block_acts(const Shape& sh, uint8_t* base, BlockActs<T>& a) {
   a.lse = c.take<float>(fl ? B * s * 4 : 0);
   a.o = c.take<T>(Tn * h * e);
   a.x1 = c.take<T>(Tn * h * e);
-  a.a2 = c.take<T>(Tn * h * e);
+  a.a2 = compact ? nullptr : c.take<T>(Tn * h * e);
   a.mu2 = c.take<float>(Tn * 4);
   a.rs2 = c.take<float>(Tn * 4);
   a.u = c.take<T>(Tn * 4 * h * e);
-  a.g = c.take<T>(Tn * 4 * h * e);
+  a.g = compact ? nullptr : c.take<T>(Tn * 4 * h * e);
+  (void)full;
 }
 
 int64_t scratch_bytes(const Shape& sh, int e, bool with_head, bool flash) {
@@ -174,6 +177,9 @@ int64_t scratch_bytes(const Shape& sh, int e, bool with_head, bool flash) {
   c.take<char>(T * 4);
   c.take<char>(T * 4);
   c.take<char>(T * 4);
+  c.take<char>(T * h * e);      // ra
+  c.take<char>(T * h * e);      // ra2
+  c.take<char>(T * 4 * h * e);  // rg
   return c.off;
 }
 
@@ -195,6 +201,9 @@ void carve_scratch(const Shape& sh, uint8_t* base, bool with_head, Scratch<T>& s
   sc.loss_rows = c.take<float>(Tn * 4);
   sc.mu = c.take<float>(Tn * 4);
   sc.rs = c.take<float>(Tn * 4);
+  sc.ra = c.take<T>(Tn * h * e);
+  sc.ra2 = c.take<T>(Tn * h * e);
+  sc.rg = c.take<T>(Tn * 4 * h * e);
 }
 
 // ------------------------------------------------------------ attention
@@ -297,8 +306,14 @@ int attention_bwd(const Shape& sh, const T* qkv, const T* o, const T* P, const f
 
 // ------------------------------------------------------------------ block
 template <typename T>
-int block_fwd(const Shape& sh, const T* w, BlockActs<T>& A, T* y, Scratch<T>& sc, cudaStream_t st) {
+int block_fwd(const Shape& sh, const T* w, BlockActs<T>& A_in, T* y, Scratch<T>& sc, cudaStream_t st) {
   const BlockLayout L(sh.h);
+  BlockActs<T> A = A_in;
+  if (!A.a) {  // compact kept activations: a, a2, g go to scratch (recomputed in backward)
+    A.a = sc.ra;
+    A.a2 = sc.ra2;
+    A.g = sc.rg;
+  }
   const int Tn = sh.T(), h = sh.h, nh = sh.nh, s = sh.s, dh = sh.dh(), mbs = sh.mbs;
   const int64_t Sbs2 = (int64_t)s * s, Sbs1 = nh * Sbs2;
   {
@@ -350,12 +365,26 @@ int block_fwd(const Shape& sh, const T* w, BlockActs<T>& A, T* y, Scratch<T>& sc
 }
 
 template <typename T>
-int block_bwd(const Shape& sh, const T* w, const BlockActs<T>& A, const T* dy, T* dx, float* G, Scratch<T>& sc,
+int block_bwd(const Shape& sh, const T* w, const BlockActs<T>& A_in, const T* dy, T* dx, float* G, Scratch<T>& sc,
               cudaStream_t st) {
   const BlockLayout L(sh.h);
   const int Tn = sh.T(), h = sh.h, nh = sh.nh, s = sh.s, dh = sh.dh(), mbs = sh.mbs;
   const int64_t Sbs2 = (int64_t)s * s, Sbs1 = nh * Sbs2;
   const float scale = 1.0f / sqrtf((float)dh);
+  BlockActs<T> A = A_in;
+  if (!A.a) {  // compact kept activations: recompute a, a2 (LN forwards) and g = gelu(u)
+    if constexpr (sizeof(T) != 2) {
+      MOBIUS_FAIL(MOBIUS_EINVAL, "block_bwd: compact activations are bf16-only");
+    } else {
+      ElemScope es(st, 1);
+      A.a = sc.ra;
+      A.a2 = sc.ra2;
+      A.g = sc.rg;
+      RC(layernorm_fwd<T>(A.x, w + L.ln1_g, w + L.ln1_b, A.a, A.mu1, A.rs1, Tn, h, st));
+      RC(layernorm_fwd<T>(A.x1, w + L.ln2_g, w + L.ln2_b, A.a2, A.mu2, A.rs2, Tn, h, st));
+      RC(gelu_fwd_bf16(A.u, A.g, (int64_t)Tn * 4 * h, st));
+    }
+  }
   T* du = sc.big1;
   {  // du = (dy W2^T) * gelu'(u)
     GemmDesc d;
@@ -516,7 +545,7 @@ int head_layer_fwd_bwd(const Shape& sh, const T* w, const T* x, const int32_t* t
 }
 
 #define INST(T)                                                                                                   \
-  template void carve_block_acts<T>(const Shape&, uint8_t*, BlockActs<T>&);                                      \
+  template void carve_block_acts<T>(const Shape&, uint8_t*, BlockActs<T>&, bool);                                      \
   template void carve_scratch<T>(const Shape&, uint8_t*, bool, Scratch<T>&);                                     \
   template int block_fwd<T>(const Shape&, const T*, BlockActs<T>&, T*, Scratch<T>&, cudaStream_t);               \
   template int block_bwd<T>(const Shape&, const T*, const BlockActs<T>&, const T*, T*, float*, Scratch<T>&,      \

@@ -63,6 +63,7 @@ struct Scratch {
   T* logits;       // [T, V]
   float* loss_rows;  // [T]
   float *mu, *rs;  // [T] (head LN)
+  T *ra, *ra2, *rg;  // recompute targets of a compact BlockActs: [T, h], [T, h], [T, 4h]
 };
 
 // true when the fused tcgen05 attention is used (bf16, dh in {64,128}, s % 128 == 0)
@@ -76,10 +77,14 @@ int attention_bwd(const Shape& sh, const T* qkv, const T* o, const T* P, const f
                   Scratch<T>& sc, cudaStream_t st);
 
 // bytes of one BlockActs set / of the Scratch (for arena planning)
-int64_t block_acts_bytes(const Shape& sh, int elem, bool flash);
+// compact: the kept-activation layout (bf16 flash path) without the LN
+// outputs a, a2 and g = gelu(u); block_bwd recomputes those three (two LN
+// forwards and an elementwise GeLU, bit-identical to the forward's values)
+// into scratch.  The stored set is x, qkv, o, x1, u, lse and the LN stats.
+int64_t block_acts_bytes(const Shape& sh, int elem, bool flash, bool compact = false);
 int64_t scratch_bytes(const Shape& sh, int elem, bool with_head, bool flash);
 template <typename T>
-void carve_block_acts(const Shape& sh, uint8_t* base, BlockActs<T>& a);
+void carve_block_acts(const Shape& sh, uint8_t* base, BlockActs<T>& a, bool compact = false);
 template <typename T>
 void carve_scratch(const Shape& sh, uint8_t* base, bool with_head, Scratch<T>& s);
 

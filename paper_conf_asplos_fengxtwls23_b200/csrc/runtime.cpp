@@ -169,6 +169,8 @@ struct mobius_ctx {
   int64_t keep_bytes = 0;
   std::vector<int64_t> keep_off;  // per local stage: offset into keep_pool, -1 if not kept
   int64_t acts_bytes = 0;
+  int64_t keep_acts_bytes = 0;  // per kept block-microbatch (compact layout on the bf16 flash path)
+  bool keep_compact = false;
   int max_blocks = 0;
   uint8_t* xs_base = nullptr;     // [max_blocks+1] x buffers [T,h]
   uint8_t* scratch_base = nullptr;
@@ -361,14 +363,14 @@ struct StepRunner {
   bool kept(int ls) const { return ctx->keep_off[ls] >= 0; }
   uint8_t* keep_entry(int ls, int m, int bi) {
     const StageDesc& st = ctx->all[ctx->mine[ls]];
-    const int64_t e = ctx->acts_bytes + ctx->slot_bytes;
+    const int64_t e = ctx->keep_acts_bytes + ctx->slot_bytes;
     return ctx->keep_pool + ctx->keep_off[ls] + ((int64_t)m * st.n_blocks + bi) * e;
   }
   // input x of block bi of a kept stage (block 0 of an embed stage too)
-  T* keep_x(int ls, int m, int bi) { return tptr<T>(keep_entry(ls, m, bi) + ctx->acts_bytes); }
+  T* keep_x(int ls, int m, int bi) { return tptr<T>(keep_entry(ls, m, bi) + ctx->keep_acts_bytes); }
   BlockActs<T> keep_acts(int ls, int m, int bi) {
     BlockActs<T> a;
-    carve_block_acts<T>(ctx->sh, keep_entry(ls, m, bi), a);
+    carve_block_acts<T>(ctx->sh, keep_entry(ls, m, bi), a, ctx->keep_compact);
     return a;
   }
 
@@ -727,7 +729,7 @@ int do_step(mobius_ctx* ctx, const int32_t* tok_dev, int M, float* loss_out) {
   S.recompute = 0;
   for (int ls = 0; ls < (int)ctx->mine.size(); ++ls)
     if (ctx->keep_off[ls] < 0 && ctx->mine[ls] != ctx->plan.n_stages - 1 && ctx->all[ctx->mine[ls]].n_blocks > 0)
-      S.recompute = 1;  // block activations of this stage are recomputed in backward
+      S.recompute += ctx->all[ctx->mine[ls]].n_blocks;  // this stage's blocks are recomputed in backward
   ctx->upd_ns = 0;
   ctx->step_count++;
   return MOBIUS_OK;
@@ -839,6 +841,8 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
   ctx->slot_bytes = al256((int64_t)sh.T() * sh.h * esz);
   const bool fl = esz == 2 && flash_supported(sh.dh(), sh.s);
   ctx->acts_bytes = al256(block_acts_bytes(sh, esz, fl));
+  ctx->keep_compact = fl && !getenv("MOBIUS_KEEP_FULL");
+  ctx->keep_acts_bytes = al256(block_acts_bytes(sh, esz, fl, ctx->keep_compact));
   int64_t off = al256(G);
   auto take = [&](int64_t bytes) {
     int64_t o = off;
@@ -874,7 +878,7 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
       CU(cudaMemGetInfo(&fr, &tot));
       int64_t budget = (int64_t)fr - (int64_t)6 * (1LL << 30);
       if (const char* e = getenv("MOBIUS_KEEP_GIB")) budget = std::min<int64_t>(budget, (int64_t)(atof(e) * (1LL << 30)));
-      const int64_t entry = ctx->acts_bytes + ctx->slot_bytes;
+      const int64_t entry = ctx->keep_acts_bytes + ctx->slot_bytes;
       int64_t off = 0;
       for (int k = n - 1; k >= 0; --k) {
         const StageDesc& st = ctx->all[ctx->mine[k]];

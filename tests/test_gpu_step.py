@@ -138,10 +138,17 @@ def test_seeded_init_runs():
 
 @pytest.mark.parametrize("dtype,tol", [(BF16, 2e-2), (F32, 1e-4)])
 @pytest.mark.parametrize("sizes", [(3, 3), (1, 2, 1, 2), (2, 2, 2)])
-def test_tiny_step_keep_acts(dtype, tol, sizes):
+@pytest.mark.parametrize("layout", ["compact", "full"])
+def test_tiny_step_keep_acts(dtype, tol, sizes, layout, monkeypatch):
     """MOBIUS_FLAG_KEEP_ACTS (reading #17: keep activations instead of
-    recomputing when they fit): same loss / gradients, no recompute."""
+    recomputing when they fit): same loss / gradients, no recompute.  The
+    bf16 path keeps the compact set (LN outputs and GeLU recomputed in
+    backward) unless MOBIUS_KEEP_FULL is set."""
     from paper_conf_asplos_fengxtwls23_b200 import FLAG_KEEP_ACTS
+    if layout == "full":
+        monkeypatch.setenv("MOBIUS_KEEP_FULL", "1")
+    else:
+        monkeypatch.delenv("MOBIUS_KEEP_FULL", raising=False)
     c = synth.TINY
     M = 2
     w = synth.perturb_norm_params(c, synth.gen_params(c), scale=0.1)
