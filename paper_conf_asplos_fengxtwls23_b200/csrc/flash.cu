@@ -560,23 +560,35 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
     // dQ(it) (TMEM lane = query row) -> fp32 staging [DH/32 slabs][128 rows][128 B],
     // 16-byte chunks XOR-swizzled by row (TMA SWIZZLE_128B, conflict-free
     // stores) -> one TMA reduce-add per 32-column slab into the dQ buffer
+    // The reduce is not waited for here: the staging memory is next written
+    // one query tile later (stage_free() before that write), by which time
+    // the bulk copy has long finished reading it - so no warp stalls on it.
+    auto stage_free = [&]() {
+      if (warp == 2 && lane == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+      named_bar(1, 256);
+    };
     auto dq_drain = [&](int itq, uint32_t stg) {
       const int qiq = i0 + itq;
+      uint32_t v[DH / 64][32];
 #pragma unroll
       for (int cc = 0; cc < DH / 64; ++cc) {
         const int c = hf * (DH / 64) + cc;  // 32-column slab
-        uint32_t v[32];
         __syncwarp();
-        ptx::tmem_ld32(T_DQ + c * 32 + lane_base, v);
-        ptx::tmem_ld_wait();
-#pragma unroll
-        for (int k = 0; k < 8; ++k)
-          st_shared_v4(stg + c * 16384 + r * 128 + ((k ^ (r & 7)) << 4), v[4 * k], v[4 * k + 1], v[4 * k + 2],
-                       v[4 * k + 3]);
+        ptx::tmem_ld32(T_DQ + c * 32 + lane_base, v[cc]);
       }
+      ptx::tmem_ld_wait();
       ptx::tc_fence_before();
       __syncwarp();
-      if (lane == 0) ptx::mbar_arrive(dq_empty);
+      if (lane == 0) ptx::mbar_arrive(dq_empty);  // dQ TMEM may be overwritten
+      if (C::DQ_OWN) stage_free();                 // dh 128: done before the P^T / dS^T writes
+#pragma unroll
+      for (int cc = 0; cc < DH / 64; ++cc) {
+        const int c = hf * (DH / 64) + cc;
+#pragma unroll
+        for (int k = 0; k < 8; ++k)
+          st_shared_v4(stg + c * 16384 + r * 128 + ((k ^ (r & 7)) << 4), v[cc][4 * k], v[cc][4 * k + 1],
+                       v[cc][4 * k + 2], v[cc][4 * k + 3]);
+      }
       ptx::fence_proxy_async();
       named_bar(1, 256);
       if (warp == 2 && lane == 0) {
@@ -588,9 +600,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
               "r"(stg + c * 16384), "r"(c * 32), "r"(qiq * 128), "r"(hd), "r"(b)
               : "memory");
         asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-        asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
       }
-      named_bar(1, 256);
     };
     for (int it = 0; it < nq; ++it) {
       const int st = it % QS;
@@ -615,6 +625,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
         ptx::mbar_wait(mm_done, (it - 1) & 1);
         ptx::tc_fence_after();
       }
+      if (!C::DQ_OWN && it >= 1) stage_free();  // dQ(it-1) staged in P^T / dS^T: reduce must have read it
 #pragma unroll
       for (int cc = 0; cc < 2; ++cc) {
         const int c = hf * 2 + cc;
@@ -660,6 +671,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
       ptx::tc_fence_after();
       dq_drain(nq - 1, ptx::smem_u32(sSTG));
     }
+    if (warp == 2 && lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");  // last dQ reduce
     // dV (half 0) / dK (half 1) of this key tile (rows = keys)
     ptx::mbar_wait(mm_done, (nq - 1) & 1);
     ptx::tc_fence_after();
