@@ -288,6 +288,10 @@ __device__ __forceinline__ void epi_tile(const Params& p, uint32_t tmem_row, int
 
 // TMA map over a bf16 MatView (gemm_tc.cu)
 int make_map(CUtensorMap* map, const MatView& v, int64_t inner, int64_t outer, int nb1, int nb2, int box_outer);
+// plain 2-D (as 4-D) row-major map [outer][inner] with row stride ld
+// elements, bf16 or fp32, box {box_inner, box_outer}, SWIZZLE_128B
+int make_map_2d(CUtensorMap* map, const void* ptr, bool f32, int64_t ld, int64_t inner, int64_t outer, int box_inner,
+                int box_outer);
 
 }  // namespace gemm_detail
 }  // namespace mobius

@@ -203,6 +203,24 @@ int make_map(CUtensorMap* map, const MatView& v, int64_t inner, int64_t outer, i
   return MOBIUS_OK;
 }
 
+int make_map_2d(CUtensorMap* map, const void* ptr, bool f32, int64_t ld, int64_t inner, int64_t outer, int box_inner,
+                int box_outer) {
+  EncodeTiledFn enc = get_encode();
+  if (!enc) MOBIUS_FAIL(MOBIUS_ECUDA, "cuTensorMapEncodeTiled unavailable");
+  const int64_t es = f32 ? 4 : 2;
+  if ((reinterpret_cast<uintptr_t>(ptr) & 15) != 0 || (ld * es) % 16 != 0)
+    MOBIUS_FAIL(MOBIUS_EINVAL, "TMA epilogue map: base and row stride must be 16-byte aligned");
+  cuuint64_t dims[4] = {(cuuint64_t)inner, (cuuint64_t)outer, 1, 1};
+  cuuint64_t strides[3] = {(cuuint64_t)(ld * es), (cuuint64_t)(ld * es * outer), (cuuint64_t)(ld * es * outer)};
+  cuuint32_t box[4] = {(cuuint32_t)box_inner, (cuuint32_t)box_outer, 1, 1};
+  cuuint32_t estr[4] = {1, 1, 1, 1};
+  CUresult r = enc(map, f32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void*>(ptr),
+                   dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) MOBIUS_FAIL(MOBIUS_ECUDA, "cuTensorMapEncodeTiled (epilogue) failed (%d)", (int)r);
+  return MOBIUS_OK;
+}
+
 template <int BN, bool A_MN, bool B_MN>
 int launch(const CUtensorMap& ta, const CUtensorMap& tb, const Params& p, int total, cudaStream_t s) {
   auto k = gemm_tc_kernel<BN, A_MN, B_MN>;

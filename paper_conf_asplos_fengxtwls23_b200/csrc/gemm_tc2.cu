@@ -19,10 +19,205 @@ struct Cfg2 {
   static constexpr int A_BYTES = 128 * BK * 2;
   static constexpr int B_BYTES = (BN / 2) * BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int STAGES = (200 * 1024) / STAGE_BYTES > 8 ? 8 : (200 * 1024) / STAGE_BYTES;
+  static constexpr int STAGES = (160 * 1024) / STAGE_BYTES > 8 ? 8 : (160 * 1024) / STAGE_BYTES;
   static constexpr int TMEM_COLS = 2 * BN;
-  static constexpr int SMEM = 1024 + STAGES * STAGE_BYTES + 256;
+  // epilogue staging: per epilogue warp two 4 KiB boxes (32 rows x 128 B,
+  // SWIZZLE_128B) for TMA stores / reduce-adds of C and TMA loads of R
+  static constexpr int EPI_BOX = 4096;
+  static constexpr int EPI_BYTES = 8 * 2 * EPI_BOX;
+  static constexpr int SMEM = 1024 + STAGES * STAGE_BYTES + EPI_BYTES + 512;
 };
+
+// ---------------------------------------------------- TMA-store epilogue
+__device__ __forceinline__ void tma_store_2d(const CUtensorMap* m, uint32_t src, int c0, int c1) {
+  asm volatile("cp.async.bulk.tensor.4d.global.shared::cta.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
+                   reinterpret_cast<uint64_t>(m)),
+               "r"(src), "r"(c0), "r"(c1), "r"(0), "r"(0)
+               : "memory");
+}
+__device__ __forceinline__ void tma_reduce_add_2d(const CUtensorMap* m, uint32_t src, int c0, int c1) {
+  asm volatile(
+      "cp.reduce.async.bulk.tensor.4d.global.shared::cta.add.tile.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
+          reinterpret_cast<uint64_t>(m)),
+      "r"(src), "r"(c0), "r"(c1), "r"(0), "r"(0)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() {
+  asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+// byte offset of 16-byte chunk c of row r in a 32 x 128 B SWIZZLE_128B box
+__device__ __forceinline__ uint32_t box_off(int r, int c) { return (uint32_t)(r * 128 + ((c ^ (r & 7)) << 4)); }
+
+struct EpiMaps {
+  const CUtensorMap* C;  // bf16 box {64, 32} or fp32 box {32, 32}
+  const CUtensorMap* R;  // bf16 box {64, 32} (residual / GeLU input)
+  const CUtensorMap* X;  // bf16 box {64, 32} (pre-activation output)
+};
+
+// One warp's share of an accumulator tile: 32 rows (its TMEM lane quadrant)
+// x 128 columns (half the tile), starting at (m0w, n0w).  Values leave TMEM
+// 64 (bf16) or 32 (fp32) columns at a time, get the fused ops in registers,
+// are written swizzled into this warp's staging boxes and leave with one
+// TMA store (or, for the fp32 dW accumulate, a TMA reduce-add: L2 does the
+// read-modify-write) per box; R boxes arrive by TMA before the accumulator
+// is ready.  Partial boxes at the matrix edge are clipped by the TMA unit.
+// `release` is called after the last TMEM read (accumulator handed back).
+template <int EPI, bool CF32, bool ACC, typename Rel>
+__device__ __forceinline__ void epi_tma(const Params& p, const EpiMaps& mp, uint32_t tmem_row, uint32_t stg,
+                                        uint64_t* rbar, uint32_t rph, int m0w, int n0w, int lane, Rel release) {
+  constexpr bool has_bias = EPI == EPI_BIAS || EPI == EPI_BIAS_GELU || EPI == EPI_BIAS_RESID;
+  constexpr bool has_r = EPI == EPI_BIAS_RESID || EPI == EPI_GELU_BWD;
+  if constexpr (CF32) {
+    // fp32 C: four 32-column boxes, alternating between the two staging boxes
+#pragma unroll 1
+    for (int j = 0; j < 4; ++j) {
+      uint32_t r[32];
+      __syncwarp();
+      ptx::tmem_ld32(tmem_row + j * 32, r);
+      ptx::tmem_ld_wait();
+      if (j == 3) release();
+      const int n0 = n0w + 32 * j;
+      if (n0 >= p.N) continue;
+      const uint32_t box = stg + (j & 1) * 4096;
+      if (j >= 2) {
+        if (lane == 0) bulk_wait_read<1>();  // the store from this box two chunks ago has read it
+        __syncwarp();
+      }
+#pragma unroll
+      for (int c = 0; c < 8; ++c) {
+        float4 o = make_float4(__uint_as_float(r[4 * c]) * p.alpha, __uint_as_float(r[4 * c + 1]) * p.alpha,
+                               __uint_as_float(r[4 * c + 2]) * p.alpha, __uint_as_float(r[4 * c + 3]) * p.alpha);
+        asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(box + box_off(lane, c)), "f"(o.x), "f"(o.y),
+                     "f"(o.z), "f"(o.w)
+                     : "memory");
+      }
+      ptx::fence_proxy_async();
+      __syncwarp();
+      if (lane == 0) {
+        if (ACC)
+          tma_reduce_add_2d(mp.C, box, n0, m0w);
+        else
+          tma_store_2d(mp.C, box, n0, m0w);
+        bulk_commit();
+      }
+    }
+  } else {
+    // bf16 C: two 64-column chunks; GeLU uses both boxes per chunk (u, g)
+    constexpr int NCH = 2;
+#pragma unroll 1
+    for (int j = 0; j < NCH; ++j) {
+      const int n0 = n0w + 64 * j;
+      uint32_t ra[32], rb[32];
+      __syncwarp();
+      ptx::tmem_ld32(tmem_row + j * 64, ra);
+      ptx::tmem_ld32(tmem_row + j * 64 + 32, rb);
+      ptx::tmem_ld_wait();
+      if (j == NCH - 1) release();
+      if (n0 >= p.N) continue;
+      float v[64];
+#pragma unroll
+      for (int i = 0; i < 32; ++i) {
+        v[i] = __uint_as_float(ra[i]) * p.alpha;
+        v[32 + i] = __uint_as_float(rb[i]) * p.alpha;
+      }
+      if constexpr (has_bias) {
+        if (n0 + 64 <= p.N) {
+#pragma unroll
+          for (int i = 0; i < 8; ++i) {
+            const uint4 pk = __ldg(reinterpret_cast<const uint4*>(p.bias + n0) + i);
+            const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&pk);
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+              const float2 x = __bfloat1622float2(h2[k]);
+              v[8 * i + 2 * k] += x.x;
+              v[8 * i + 2 * k + 1] += x.y;
+            }
+          }
+        } else {
+#pragma unroll
+          for (int i = 0; i < 64; ++i)
+            if (n0 + i < p.N) v[i] += __bfloat162float(p.bias[n0 + i]);
+        }
+      }
+      const uint32_t box = stg + (has_r ? j * 4096 : 0);
+      if constexpr (has_r) {
+        ptx::mbar_wait(&rbar[j], (rph >> j) & 1u);  // R box j landed
+#pragma unroll
+        for (int c = 0; c < 8; ++c) {
+          uint4 pk;
+          asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];"
+                       : "=r"(pk.x), "=r"(pk.y), "=r"(pk.z), "=r"(pk.w)
+                       : "r"(box + box_off(lane, c)));
+          const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&pk);
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            const float2 x = __bfloat1622float2(h2[k]);
+            if constexpr (EPI == EPI_BIAS_RESID) {
+              v[8 * c + 2 * k] += x.x;
+              v[8 * c + 2 * k + 1] += x.y;
+            } else {
+              v[8 * c + 2 * k] *= gelu_grad_f(x.x);
+              v[8 * c + 2 * k + 1] *= gelu_grad_f(x.y);
+            }
+          }
+        }
+      } else if (j > 0) {
+        if (lane == 0) bulk_wait_read<0>();  // previous chunk's stores have read the boxes
+        __syncwarp();
+      }
+      if constexpr (EPI == EPI_BIAS_GELU) {
+        // u (bf16) -> box 0 (AUX), g = gelu(bf16(u)) -> box 1 (C)
+#pragma unroll
+        for (int c = 0; c < 8; ++c) {
+          uint32_t pu[4], pg[4];
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            const __nv_bfloat162 u2 = __floats2bfloat162_rn(v[8 * c + 2 * k], v[8 * c + 2 * k + 1]);
+            const float2 uf = __bfloat1622float2(u2);
+            const __nv_bfloat162 g2 = __floats2bfloat162_rn(gelu_f(uf.x), gelu_f(uf.y));
+            pu[k] = *reinterpret_cast<const uint32_t*>(&u2);
+            pg[k] = *reinterpret_cast<const uint32_t*>(&g2);
+          }
+          asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(stg + box_off(lane, c)), "r"(pu[0]), "r"(pu[1]),
+                       "r"(pu[2]), "r"(pu[3])
+                       : "memory");
+          asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(stg + 4096 + box_off(lane, c)), "r"(pg[0]),
+                       "r"(pg[1]), "r"(pg[2]), "r"(pg[3])
+                       : "memory");
+        }
+        ptx::fence_proxy_async();
+        __syncwarp();
+        if (lane == 0) {
+          tma_store_2d(mp.X, stg, n0, m0w);
+          tma_store_2d(mp.C, stg + 4096, n0, m0w);
+          bulk_commit();
+        }
+      } else {
+#pragma unroll
+        for (int c = 0; c < 8; ++c) {
+          uint32_t pk[4];
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            const __nv_bfloat162 o2 = __floats2bfloat162_rn(v[8 * c + 2 * k], v[8 * c + 2 * k + 1]);
+            pk[k] = *reinterpret_cast<const uint32_t*>(&o2);
+          }
+          asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(box + box_off(lane, c)), "r"(pk[0]), "r"(pk[1]),
+                       "r"(pk[2]), "r"(pk[3])
+                       : "memory");
+        }
+        ptx::fence_proxy_async();
+        __syncwarp();
+        if (lane == 0) {
+          tma_store_2d(mp.C, box, n0, m0w);
+          bulk_commit();
+        }
+      }
+    }
+  }
+}
 
 // One unit of work of a cluster: k-blocks [k0, k1) of tile t, which is
 // segment seg of nseg (nseg == 1: a whole tile, no fixup).
@@ -86,18 +281,22 @@ struct Sched {
 // L2 -> SM operand traffic by a quarter.
 template <int BN, bool A_MN, bool B_MN, int NP>
 __global__ void __launch_bounds__(NUM_THREADS2, 1)
-    gemm_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, const Params p) {
+    gemm_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                    const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmR,
+                    const __grid_constant__ CUtensorMap tmX, const Params p) {
   using C = Cfg2<BN>;
   constexpr int BM2 = 256;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* smA = smem;
   uint8_t* smB = smem + C::STAGES * C::A_BYTES;
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + C::STAGES * C::STAGE_BYTES);
+  uint8_t* smE = smem + C::STAGES * C::STAGE_BYTES;  // [8 warps][2 boxes][4 KiB]
+  uint64_t* full = reinterpret_cast<uint64_t*>(smE + C::EPI_BYTES);
   uint64_t* empty = full + C::STAGES;
   uint64_t* tfull = empty + C::STAGES;
   uint64_t* tempty = tfull + 2;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+  uint64_t* rbar = tempty + 2;  // [8 warps][2] R-box arrivals
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(rbar + 16);
 
   const int warp = threadIdx.x / 32;
   const int lane = threadIdx.x % 32;
@@ -118,6 +317,7 @@ __global__ void __launch_bounds__(NUM_THREADS2, 1)
       ptx::mbar_init(&tfull[a], 1);
       ptx::mbar_init(&tempty[a], 16);  // 8 epilogue warps x 2 CTAs of the pair (leader's copy)
     }
+    for (int i = 0; i < 16; ++i) ptx::mbar_init(&rbar[i], 1);
     ptx::fence_mbar_init();
   }
   if (warp == 1) ptx::tmem_alloc_2sm<C::TMEM_COLS>(tmem_slot);
@@ -234,6 +434,11 @@ __global__ void __launch_bounds__(NUM_THREADS2, 1)
     const uint32_t tempty_leader = ptx::mapa_shared(ptx::smem_u32(&tempty[0]), pair * 2);
     int acc = 0;
     uint32_t aphase = 0;
+    const uint32_t stg = ptx::smem_u32(smE) + (uint32_t)(warp - 2) * (2 * C::EPI_BOX);
+    uint64_t* wrbar = rbar + (warp - 2) * 2;
+    uint32_t rph = 0;  // phase bit per R box barrier
+    const EpiMaps mp{&tmC, &tmR, &tmX};
+    const bool has_r = p.epi == EPI_BIAS_RESID || p.epi == EPI_GELU_BWD;
     Sched sc(p, cl, ncl);
     Work w;
     while (sc.next(p, total, w)) {
@@ -242,25 +447,53 @@ __global__ void __launch_bounds__(NUM_THREADS2, 1)
       const int m = mt * BM2 + (int)r2 * 128 + q * 32 + lane;
       const int ncol0 = nt * BN + hf * HALF;
       const uint32_t tmem_row = tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + hf * HALF;
+      if (has_r && w.nseg == 1 && lane == 0) {
+        // R boxes of this tile into the staging boxes while the mainloop runs
+        bulk_wait_read<0>();  // the previous tile's stores have read them
+        const int m0w = mt * BM2 + (int)r2 * 128 + q * 32;
+#pragma unroll
+        for (int j = 0; j < 2; ++j)
+          if (ncol0 + 64 * j < p.N) {
+            ptx::mbar_arrive_expect_tx(&wrbar[j], C::EPI_BOX);
+            ptx::tma_load_4d(smE + (warp - 2) * (2 * C::EPI_BOX) + j * C::EPI_BOX, &tmR, &wrbar[j], ncol0 + 64 * j,
+                             m0w, 0, 0);
+          }
+      }
       ptx::mbar_wait_cluster(&tfull[acc], aphase);
       ptx::tc_fence_after();
       if (w.nseg == 1) {
-#pragma unroll 1
-        for (int c = 0; c < HALF; c += 64) {
-          uint32_t r[64];
+        auto release = [&]() {  // last TMEM read of this tile: hand the accumulator back early
+          ptx::tc_fence_before();
           __syncwarp();
-          ptx::tmem_ld32(tmem_row + c, *reinterpret_cast<uint32_t(*)[32]>(&r[0]));
-          ptx::tmem_ld32(tmem_row + c + 32, *reinterpret_cast<uint32_t(*)[32]>(&r[32]));
-          ptx::tmem_ld_wait();
-          if (c + 64 >= HALF) {  // last TMEM read of this tile: hand the accumulator back early
-            ptx::tc_fence_before();
-            __syncwarp();
-            if (lane == 0) ptx::mbar_arrive_cluster(tempty_leader + acc * 8);
-          }
-          float v[64];
+          if (lane == 0) ptx::mbar_arrive_cluster(tempty_leader + acc * 8);
+        };
+        const int m0w = mt * BM2 + (int)r2 * 128 + q * 32;
+        switch (p.epi) {
+          case EPI_BIAS: epi_tma<EPI_BIAS, false, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release); break;
+          case EPI_BIAS_GELU:
+            epi_tma<EPI_BIAS_GELU, false, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
+            break;
+          case EPI_BIAS_RESID:
+          case EPI_GELU_BWD:
+            if (p.epi == EPI_BIAS_RESID)
+              epi_tma<EPI_BIAS_RESID, false, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
+            else
+              epi_tma<EPI_GELU_BWD, false, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
 #pragma unroll
-          for (int i = 0; i < 64; ++i) v[i] = __uint_as_float(r[i]) * p.alpha;
-          epi_vals<64>(p, v, m, 0, 0, ncol0 + c);
+            for (int j = 0; j < 2; ++j)
+              if (ncol0 + 64 * j < p.N) rph ^= 1u << j;
+            break;
+          case EPI_ACCUM:
+            if (p.accumulate)
+              epi_tma<EPI_ACCUM, true, true>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
+            else
+              epi_tma<EPI_STORE, true, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
+            break;
+          default:
+            if (p.c_f32)
+              epi_tma<EPI_STORE, true, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
+            else
+              epi_tma<EPI_STORE, false, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
         }
       } else {
         // Stream-K segment: raw partial (32 rows x BN/2 fp32 per warp) to the
@@ -323,6 +556,7 @@ __global__ void __launch_bounds__(NUM_THREADS2, 1)
         aphase ^= 1;
       }
     }
+    if (lane == 0) bulk_wait_all();  // staged stores complete before the CTA exits
   }
 
   __syncthreads();
@@ -334,7 +568,8 @@ __global__ void __launch_bounds__(NUM_THREADS2, 1)
 }
 
 template <int BN, bool A_MN, bool B_MN, int NP>
-int launch2(const CUtensorMap& ta, const CUtensorMap& tb, const Params& p, cudaStream_t s) {
+int launch2(const CUtensorMap& ta, const CUtensorMap& tb, const CUtensorMap& tc, const CUtensorMap& tr,
+            const CUtensorMap& tx, const Params& p, cudaStream_t s) {
   auto k = gemm_tc2_kernel<BN, A_MN, B_MN, NP>;
   static bool attr_set = false;
   if (!attr_set) {
@@ -359,7 +594,7 @@ int launch2(const CUtensorMap& ta, const CUtensorMap& tb, const Params& p, cudaS
   attr[0].val.clusterDim.z = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  cudaError_t e = cudaLaunchKernelEx(&cfg, k, ta, tb, p);
+  cudaError_t e = cudaLaunchKernelEx(&cfg, k, ta, tb, tc, tr, tx, p);
   if (e != cudaSuccess) MOBIUS_FAIL(MOBIUS_ECUDA, "gemm_tc2 launch: %s", cudaGetErrorString(e));
   return MOBIUS_OK;
 }
@@ -368,9 +603,6 @@ int launch2(const CUtensorMap& ta, const CUtensorMap& tb, const Params& p, cudaS
 
 using namespace gemm_detail;
 
-// multicast across two pairs; measured slower on the 1.5B shapes - the pairs
-// run in lock-step on every smem slot - so it is off by default)
-static int g_gemm_np = -1;
 static int g_gemm_sk = -1;  // Stream-K tail: env MOBIUS_GEMM_SK=0 disables
 
 // Stream-K workspace, one per stream (GEMMs on different streams may run
@@ -472,23 +704,32 @@ static void plan_stream_k(Params& p, int P) {
 
 template <int BN>
 static int gemm_bf16_2cta_bn(const GemmDesc& d, cudaStream_t s) {
-  if (g_gemm_np < 0) {
-    const char* e = getenv("MOBIUS_GEMM_NP");
-    g_gemm_np = (e && e[0] == '2') ? 2 : 1;
-  }
-  const bool mc = g_gemm_np == 2 && (d.N + BN - 1) / BN >= 2;
-  CUtensorMap ta, tb;
+  CUtensorMap ta, tb, tc, tr, tx;
   int rc;
   if (d.a_mn)
     rc = make_map(&ta, d.A, d.M, d.K, d.nb1, d.nb2, BK);
   else
-    rc = make_map(&ta, d.A, d.K, d.M, d.nb1, d.nb2, mc ? 64 : 128);
+    rc = make_map(&ta, d.A, d.K, d.M, d.nb1, d.nb2, 128);
   if (rc) return rc;
   if (d.b_mn)
     rc = make_map(&tb, d.B, d.N, d.K, d.nb1, d.nb2, BK);
   else
     rc = make_map(&tb, d.B, d.K, d.N, d.nb1, d.nb2, BN / 2);
   if (rc) return rc;
+  // epilogue maps: 32-row boxes of 128 B (64 bf16 or 32 fp32 columns)
+  const bool cf = d.c_f32;
+  if ((rc = make_map_2d(&tc, d.C.ptr, cf, d.C.ld, d.N, d.M, cf ? 32 : 64, 32))) return rc;
+  const bool has_r = d.epi == EPI_BIAS_RESID || d.epi == EPI_GELU_BWD;
+  if (has_r) {
+    if ((rc = make_map_2d(&tr, d.R.ptr, false, d.R.ld, d.N, d.M, 64, 32))) return rc;
+  } else {
+    tr = tc;
+  }
+  if (d.epi == EPI_BIAS_GELU) {
+    if ((rc = make_map_2d(&tx, d.AUX.ptr, false, d.AUX.ld, d.N, d.M, 64, 32))) return rc;
+  } else {
+    tx = tc;
+  }
   Params p;
   std::memset(&p, 0, sizeof(p));
   p.M = d.M; p.N = d.N; p.K = d.K; p.nb1 = 1; p.nb2 = 1;
@@ -501,24 +742,16 @@ static int gemm_bf16_2cta_bn(const GemmDesc& d, cudaStream_t s) {
   p.bias = (const __nv_bfloat16*)d.bias;
   p.R = (const __nv_bfloat16*)d.R.ptr; p.ldr = d.R.ld;
   p.AUX = (__nv_bfloat16*)d.AUX.ptr; p.ldx = d.AUX.ld;
-  if (g_gemm_np != 2) {
-    plan_stream_k(p, num_sms() / 2);
-    if (p.sk_tiles) {
-      const size_t ws = (size_t)p.sk_tiles * p.sk_maxseg * 16 * 32 * (BN / 2) * sizeof(float);
-      int rc2 = sk_workspace(s, ws, (size_t)p.sk_tiles * 16, &p.sk_ws, &p.sk_cnt);
-      if (rc2) return rc2;
-    }
+  plan_stream_k(p, num_sms() / 2);
+  if (p.sk_tiles) {
+    const size_t ws = (size_t)p.sk_tiles * p.sk_maxseg * 16 * 32 * (BN / 2) * sizeof(float);
+    int rc2 = sk_workspace(s, ws, (size_t)p.sk_tiles * 16, &p.sk_ws, &p.sk_cnt);
+    if (rc2) return rc2;
   }
-  if (g_gemm_np == 2 && p.tiles_n >= 2) {  // A multicast across two pairs
-    if (!d.a_mn && !d.b_mn) return launch2<BN, false, false, 2>(ta, tb, p, s);
-    if (!d.a_mn && d.b_mn) return launch2<BN, false, true, 2>(ta, tb, p, s);
-    if (d.a_mn && !d.b_mn) return launch2<BN, true, false, 2>(ta, tb, p, s);
-    return launch2<BN, true, true, 2>(ta, tb, p, s);
-  }
-  if (!d.a_mn && !d.b_mn) return launch2<BN, false, false, 1>(ta, tb, p, s);
-  if (!d.a_mn && d.b_mn) return launch2<BN, false, true, 1>(ta, tb, p, s);
-  if (d.a_mn && !d.b_mn) return launch2<BN, true, false, 1>(ta, tb, p, s);
-  return launch2<BN, true, true, 1>(ta, tb, p, s);
+  if (!d.a_mn && !d.b_mn) return launch2<BN, false, false, 1>(ta, tb, tc, tr, tx, p, s);
+  if (!d.a_mn && d.b_mn) return launch2<BN, false, true, 1>(ta, tb, tc, tr, tx, p, s);
+  if (d.a_mn && !d.b_mn) return launch2<BN, true, false, 1>(ta, tb, tc, tr, tx, p, s);
+  return launch2<BN, true, true, 1>(ta, tb, tc, tr, tx, p, s);
 }
 
 // 256 x 256 tiles: at 64 B/clk/SM of operand traffic this is the only 2-CTA
