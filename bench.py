@@ -258,7 +258,8 @@ def run_mobius(args, rank, world, local):
     if world > 1:
         from paper_conf_asplos_fengxtwls23_b200 import dist as mdist
         assert mdist.check_same_plan(plan), "ranks derived different plans"
-    flags = FLAG_TIMING | (0 if args.no_keep else FLAG_KEEP_ACTS)
+    timing = os.environ.get("MOBIUS_BENCH_TIMING", "1") != "0"  # per-kernel CUDA events (roofline)
+    flags = (FLAG_TIMING if timing else 0) | (0 if args.no_keep else FLAG_KEEP_ACTS)
     ctx = MobiusContext(cfg, plan, rank=rank, world=world, device=local, seed=1234, flags=flags)
     if world > 1:
         blobs = [None] * world
@@ -321,6 +322,9 @@ def run_mobius(args, rank, world, local):
                "d2h_bytes_per_step": 8, "ms_per_step": ems}
 
     st = stats[-1]
+
+    def avg(field):
+        return sum(getattr(x, field) for x in stats) / len(stats)
     peaks, peak_src = load_peaks()
     gemm_ns = sum(s.gemm_ns for s in stats)
     gemm_flops = sum(s.gemm_flops for s in stats)
@@ -370,7 +374,10 @@ def run_mobius(args, rank, world, local):
             "swap_in": {"h2d_bytes_per_step": st.h2d_bytes, "d2h_bytes_per_step": st.d2h_bytes,
                         "copies": st.n_h2d_copies, "GBps_median": st.h2d_GBps_median, "GBps_max": st.h2d_GBps_max,
                         "link_peak_GBps": h2d_gbps, "exposed_load_ms": st.exposed_load_ns / 1e6},
-            "breakdown_ms": {"gemm": st.gemm_ns / 1e6, "attention": st.attn_ns / 1e6, "elementwise": st.elem_ns / 1e6,
+            "breakdown_ms": {"gemm": avg("gemm_ns") / 1e6, "attention": avg("attn_ns") / 1e6,
+                             "elementwise": avg("elem_ns") / 1e6,
+                             "timing": f"CUDA events around every {st.timing_stride}th launch of each kernel class "
+                                       "inside the timed steps, scaled by the stride (sampled estimate)",
                              "device_step": st.device_step_ns / 1e6, "host_update_total": st.host_update_ns / 1e6,
                              "update_tail": st.update_tail_ns / 1e6},
             "memory": {"arena_GB": st.arena_bytes / 1e9, "ring_GB": st.ring_bytes / 1e9,

@@ -64,7 +64,7 @@ class StepStats(C.Structure):
                 ("elem_ns", C.c_int64), ("kernel_launches", C.c_int64), ("exposed_load_ns", C.c_int64),
                 ("update_tail_ns", C.c_int64), ("arena_bytes", C.c_int64), ("ring_bytes", C.c_int64),
                 ("pinned_bytes", C.c_int64), ("host_update_ns", C.c_int64), ("n_local_stages", C.c_int),
-                ("recompute", C.c_int)]
+                ("recompute", C.c_int), ("timing_stride", C.c_int)]
 
 
 FLAG_TIMING = 1
