@@ -4,6 +4,8 @@
 // path.  Auto-vectorised (AVX-512 / AVX2 clones).
 #include "host.h"
 
+#include <immintrin.h>
+
 #include <cmath>
 #include <cstring>
 
@@ -112,6 +114,60 @@ __attribute__((target_clones("avx512f", "avx2", "default"))) void adamw_chunk(
   }
 }
 
+// bf16 grad -> bf16 weights (the bf16 path), explicit AVX-512: 16 params
+// per iteration, the two bias-correction divisions folded into multiplies,
+// and non-temporal stores for master/m/v/weights (no read-for-ownership:
+// 28 B/param of DRAM traffic instead of ~42).  Same AdamW as adamw_chunk to
+// fp32 rounding (FMA contraction and the folded reciprocals differ in the
+// last bits; the oracle parity test allows 1e-6).
+__attribute__((target("avx512f,avx512bw,avx512vl"))) void adamw_chunk_bf16_avx512(
+    float* __restrict__ w, float* __restrict__ m, float* __restrict__ v, const uint16_t* __restrict__ g,
+    uint16_t* __restrict__ wo, int64_t n, float lr, float b1, float b2, float eps, float wd, float bc1, float bc2) {
+  const __m512 vb1 = _mm512_set1_ps(b1), vb2 = _mm512_set1_ps(b2);
+  const __m512 vomb1 = _mm512_set1_ps(1.f - b1), vomb2 = _mm512_set1_ps(1.f - b2);
+  const __m512 vlr = _mm512_set1_ps(lr), vlrwd = _mm512_set1_ps(lr * wd), veps = _mm512_set1_ps(eps);
+  const __m512 vr1 = _mm512_set1_ps(1.f / bc1), vr2 = _mm512_set1_ps(1.f / bc2);
+  const __m512i rnd = _mm512_set1_epi32(0x7FFF), one = _mm512_set1_epi32(1);
+  const bool nt = ((reinterpret_cast<uintptr_t>(w) | reinterpret_cast<uintptr_t>(m) | reinterpret_cast<uintptr_t>(v)) &
+                   63) == 0 &&
+                  (reinterpret_cast<uintptr_t>(wo) & 31) == 0;
+  int64_t i = 0;
+  for (; i + 16 <= n; i += 16) {
+    const __m256i gb = _mm256_loadu_si256(reinterpret_cast<const __m256i*>(g + i));
+    const __m512 gv = _mm512_castsi512_ps(_mm512_slli_epi32(_mm512_cvtepu16_epi32(gb), 16));
+    __m512 x = _mm512_loadu_ps(w + i);
+    x = _mm512_fnmadd_ps(vlrwd, x, x);
+    const __m512 mi = _mm512_fmadd_ps(vb1, _mm512_loadu_ps(m + i), _mm512_mul_ps(vomb1, gv));
+    const __m512 vi = _mm512_fmadd_ps(vb2, _mm512_loadu_ps(v + i), _mm512_mul_ps(_mm512_mul_ps(vomb2, gv), gv));
+    const __m512 den = _mm512_add_ps(_mm512_sqrt_ps(_mm512_mul_ps(vi, vr2)), veps);
+    x = _mm512_sub_ps(x, _mm512_div_ps(_mm512_mul_ps(vlr, _mm512_mul_ps(mi, vr1)), den));
+    // round-to-nearest-even to bf16
+    const __m512i u = _mm512_castps_si512(x);
+    const __m512i r = _mm512_add_epi32(u, _mm512_add_epi32(rnd, _mm512_and_si512(_mm512_srli_epi32(u, 16), one)));
+    const __m256i wb = _mm512_cvtepi32_epi16(_mm512_srli_epi32(r, 16));
+    if (nt) {
+      _mm512_stream_ps(m + i, mi);
+      _mm512_stream_ps(v + i, vi);
+      _mm512_stream_ps(w + i, x);
+      _mm256_stream_si256(reinterpret_cast<__m256i*>(wo + i), wb);
+    } else {
+      _mm512_storeu_ps(m + i, mi);
+      _mm512_storeu_ps(v + i, vi);
+      _mm512_storeu_ps(w + i, x);
+      _mm256_storeu_si256(reinterpret_cast<__m256i*>(wo + i), wb);
+    }
+  }
+  _mm_sfence();  // non-temporal stores visible before the chunk is reported done
+  if (i < n)
+    adamw_chunk<0, 0>(w + i, m + i, v + i, g + i, wo + i, n - i, lr, b1, b2, eps, wd, bc1, bc2);
+}
+
+bool have_avx512() {
+  static const int ok = __builtin_cpu_supports("avx512f") && __builtin_cpu_supports("avx512bw") &&
+                        __builtin_cpu_supports("avx512vl");
+  return ok != 0;
+}
+
 }  // namespace
 
 void adamw_update(float* master, float* m, float* v, const void* grad, int grad_kind, void* weights_out,
@@ -125,7 +181,10 @@ void adamw_update(float* master, float* m, float* v, const void* grad, int grad_
     int64_t b = (int64_t)t * chunk, e = std::min<int64_t>(n, b + chunk);
     const void* g = (const char*)grad + b * gs;
     void* wo = (char*)weights_out + b * ws;
-    if (grad_kind == 0 && weights_kind == 0)
+    if (grad_kind == 0 && weights_kind == 0 && have_avx512())
+      adamw_chunk_bf16_avx512(master + b, m + b, v + b, (const uint16_t*)g, (uint16_t*)wo, e - b, a.lr, a.beta1,
+                              a.beta2, a.eps, a.wd, bc1, bc2);
+    else if (grad_kind == 0 && weights_kind == 0)
       adamw_chunk<0, 0>(master + b, m + b, v + b, g, wo, e - b, a.lr, a.beta1, a.beta2, a.eps, a.wd, bc1, bc2);
     else if (grad_kind == 1 && weights_kind == 1)
       adamw_chunk<1, 1>(master + b, m + b, v + b, g, wo, e - b, a.lr, a.beta1, a.beta2, a.eps, a.wd, bc1, bc2);

@@ -964,9 +964,11 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
       const int64_t np = st.n_params;
       CU(cudaHostAlloc(&ctx->h_weights[k], al256(np * esz), cudaHostAllocDefault));
       CU(cudaHostAlloc(&ctx->h_grads[k], al256(np * esz), cudaHostAllocDefault));
-      float* mst = (float*)std::malloc(np * 4);
-      float* mm = (float*)std::malloc(np * 4);
-      float* vv = (float*)std::malloc(np * 4);
+      // 64-byte aligned so the AVX-512 update can use non-temporal stores
+      const size_t nb = (size_t)((np * 4 + 63) / 64 * 64);
+      float* mst = (float*)std::aligned_alloc(64, nb);
+      float* mm = (float*)std::aligned_alloc(64, nb);
+      float* vv = (float*)std::aligned_alloc(64, nb);
       if (!mst || !mm || !vv) MOBIUS_FAIL(MOBIUS_ENOMEM, "host optimizer state (%lld params)", (long long)np);
       ctx->h_master[k] = mst;
       ctx->h_m[k] = mm;
