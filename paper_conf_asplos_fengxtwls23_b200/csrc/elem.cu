@@ -123,8 +123,12 @@ __global__ void embed_bwd_wte_k(const int32_t* tok, const T* dx, float* dwte, in
   for (int c = threadIdx.x * V; c < h; c += blockDim.x * V) {
     float a[V];
     Vec<T>::load(g + c, a);
+    // vector reductions (sm_90+): a quarter of the atomic operations
 #pragma unroll
-    for (int k = 0; k < V; ++k) atomicAdd(o + c + k, a[k]);
+    for (int k = 0; k < V; k += 4)
+      asm volatile("red.relaxed.gpu.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(o + c + k), "f"(a[k]),
+                   "f"(a[k + 1]), "f"(a[k + 2]), "f"(a[k + 3])
+                   : "memory");
   }
 }
 
@@ -535,6 +539,8 @@ int embed_fwd(const int32_t* tok, const T* wte, const T* wpe, T* x, int mbs, int
 }
 template <typename T>
 int embed_bwd(const int32_t* tok, const T* dx, float* dwte, float* dwpe, int mbs, int s, int h, cudaStream_t st) {
+  MOBIUS_CHECK_ARG(h % 8 == 0 && (reinterpret_cast<uintptr_t>(dwte) & 15) == 0,
+                   "embed_bwd: h %% 8 and a 16-byte aligned dWte are required (vector reductions)");
   embed_bwd_wte_k<T><<<mbs * s, 128, 0, st>>>(tok, dx, dwte, s, h);
   int rc = check_launch("embed_bwd_wte");
   if (rc) return rc;

@@ -440,8 +440,12 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const int n_t = p.s / 128;
-  const int kt = (int)blockIdx.x;  // small kt = most query tiles: launched first
-  const int hd = blockIdx.y, b = blockIdx.z;
+  // linear grid, heaviest first: every (b, head) with key tile 0 (n_t query
+  // tiles to visit) launches before any with key tile 1, ..., so the last
+  // wave holds the one-tile CTAs (longest-processing-time-first order)
+  const int nbh = (int)gridDim.x / (p.s / 128);  // nh * mbs
+  const int kt = (int)blockIdx.x / nbh;
+  const int hd = ((int)blockIdx.x % nbh) % p.nh, b = ((int)blockIdx.x % nbh) / p.nh;
   const int i0 = kt, nq = n_t - kt;
 
   if (threadIdx.x == 0) {
@@ -865,7 +869,7 @@ int flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* o, const __nv_
   p.h = h;
   p.scale_log2 = 1.4426950408889634f / sqrtf((float)dh);
   p.scale = 1.0f / sqrtf((float)dh);
-  dim3 grid(s / 128, nh, mbs);
+  dim3 grid((s / 128) * nh * mbs);
   if (dh == 64) {
     static bool once = false;
     if (!once) { rc = set_smem(flash_bwd_kernel<64>, BwdCfg<64>::SMEM); if (rc) return rc; once = true; }

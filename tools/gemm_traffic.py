@@ -28,7 +28,7 @@ def col(r, name):
     return float(v) * SCALE.get(units[h.index(name)], 1)
 
 
-tcol = next((c for c in h if "sm__pipe_tensor_cycles_active_realtime.avg.pct_of_peak_sustained_elapsed" in c), None)
+tcol = "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed" if "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed" in h else None
 out = []
 for (name, M, N, K, amn, bmn, epi, cf), r in zip(SHAPES, data):
     dur_ns = col(r, "gpu__time_duration.sum")
