@@ -331,7 +331,7 @@ def run_mobius(args, rank, world, local):
     achieved_tf = gemm_flops / (gemm_ns * 1e-9) / 1e12 if gemm_ns else 0.0
     peak_tf = peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops"))
     traffic = traffic_alg = None
-    tr_path = os.path.join(ROOT, "profiles", "r1_gemm_traffic.json")
+    tr_path = os.path.join(ROOT, "profiles", "r1_gemm_traffic_v3.json")
     if os.path.exists(tr_path):  # ncu --set full capture of the block GEMM shapes (per launch)
         with open(tr_path) as f:
             tr = json.load(f)
@@ -364,8 +364,9 @@ def run_mobius(args, rank, world, local):
                          "achieved": achieved_tf, "peak": peak_tf, "unit": "TFLOP/s",
                          "frac": achieved_tf / peak_tf if peak_tf else None, "traffic": traffic,
                          "traffic_algorithmic_bytes": traffic_alg,
-                         "traffic_source": "profiles/r1_gemm_traffic.json: dram__bytes_read+write per launch, mean "
-                                           "over the fc1-fwd / fc2-fwd / fc1-dX / fc1-dW GEMMs (ncu --set full)",
+                         "traffic_source": "profiles/r1_gemm_traffic_v3.json: dram__bytes_read+write per launch, mean "
+                                           "over the 8 captured 1.5B block GEMM shapes (ncu --set full, cold L2; "
+                                           "tools/gemm_traffic.py)",
                          "peak_source": f"MEASURED_PEAKS.json bf16_tflops_sustained ({peak_src})"},
             "step_roofline": {"t_tensor_ms": t_tc * 1e3, "t_link_ms": t_link * 1e3, "t_roofline_ms": t_roof * 1e3,
                               "frac": t_roof / (ms * 1e-3), "h2d_GBps_link": h2d_gbps,
