@@ -65,20 +65,21 @@ struct EpiMaps {
 // read-modify-write) per box; R boxes arrive by TMA before the accumulator
 // is ready.  Partial boxes at the matrix edge are clipped by the TMA unit.
 // `release` is called after the last TMEM read (accumulator handed back).
-template <int EPI, bool CF32, bool ACC, typename Rel>
+template <int HALF, int EPI, bool CF32, bool ACC, typename Rel>
 __device__ __forceinline__ void epi_tma(const Params& p, const EpiMaps& mp, uint32_t tmem_row, uint32_t stg,
                                         uint64_t* rbar, uint32_t rph, int m0w, int n0w, int lane, Rel release) {
   constexpr bool has_bias = EPI == EPI_BIAS || EPI == EPI_BIAS_GELU || EPI == EPI_BIAS_RESID;
   constexpr bool has_r = EPI == EPI_BIAS_RESID || EPI == EPI_GELU_BWD;
   if constexpr (CF32) {
-    // fp32 C: four 32-column boxes, alternating between the two staging boxes
+    // fp32 C: HALF/32 32-column boxes, alternating between the two staging boxes
+    constexpr int NF = HALF / 32;
 #pragma unroll 1
-    for (int j = 0; j < 4; ++j) {
+    for (int j = 0; j < NF; ++j) {
       uint32_t r[32];
       __syncwarp();
       ptx::tmem_ld32(tmem_row + j * 32, r);
       ptx::tmem_ld_wait();
-      if (j == 3) release();
+      if (j == NF - 1) release();
       const int n0 = n0w + 32 * j;
       if (n0 >= p.N) continue;
       const uint32_t box = stg + (j & 1) * 4096;
@@ -105,8 +106,8 @@ __device__ __forceinline__ void epi_tma(const Params& p, const EpiMaps& mp, uint
       }
     }
   } else {
-    // bf16 C: two 64-column chunks; GeLU uses both boxes per chunk (u, g)
-    constexpr int NCH = 2;
+    // bf16 C: HALF/64 64-column chunks; GeLU uses both boxes per chunk (u, g)
+    constexpr int NCH = HALF / 64;
 #pragma unroll 1
     for (int j = 0; j < NCH; ++j) {
       const int n0 = n0w + 64 * j;
@@ -452,7 +453,7 @@ __global__ void __launch_bounds__(NUM_THREADS2, 1)
         bulk_wait_read<0>();  // the previous tile's stores have read them
         const int m0w = mt * BM2 + (int)r2 * 128 + q * 32;
 #pragma unroll
-        for (int j = 0; j < 2; ++j)
+        for (int j = 0; j < HALF / 64; ++j)
           if (ncol0 + 64 * j < p.N) {
             ptx::mbar_arrive_expect_tx(&wrbar[j], C::EPI_BOX);
             ptx::tma_load_4d(smE + (warp - 2) * (2 * C::EPI_BOX) + j * C::EPI_BOX, &tmR, &wrbar[j], ncol0 + 64 * j,
@@ -469,31 +470,31 @@ __global__ void __launch_bounds__(NUM_THREADS2, 1)
         };
         const int m0w = mt * BM2 + (int)r2 * 128 + q * 32;
         switch (p.epi) {
-          case EPI_BIAS: epi_tma<EPI_BIAS, false, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release); break;
+          case EPI_BIAS: epi_tma<HALF, EPI_BIAS, false, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release); break;
           case EPI_BIAS_GELU:
-            epi_tma<EPI_BIAS_GELU, false, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
+            epi_tma<HALF, EPI_BIAS_GELU, false, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
             break;
           case EPI_BIAS_RESID:
           case EPI_GELU_BWD:
             if (p.epi == EPI_BIAS_RESID)
-              epi_tma<EPI_BIAS_RESID, false, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
+              epi_tma<HALF, EPI_BIAS_RESID, false, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
             else
-              epi_tma<EPI_GELU_BWD, false, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
+              epi_tma<HALF, EPI_GELU_BWD, false, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
 #pragma unroll
-            for (int j = 0; j < 2; ++j)
+            for (int j = 0; j < HALF / 64; ++j)
               if (ncol0 + 64 * j < p.N) rph ^= 1u << j;
             break;
           case EPI_ACCUM:
             if (p.accumulate)
-              epi_tma<EPI_ACCUM, true, true>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
+              epi_tma<HALF, EPI_ACCUM, true, true>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
             else
-              epi_tma<EPI_STORE, true, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
+              epi_tma<HALF, EPI_STORE, true, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
             break;
           default:
             if (p.c_f32)
-              epi_tma<EPI_STORE, true, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
+              epi_tma<HALF, EPI_STORE, true, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
             else
-              epi_tma<EPI_STORE, false, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
+              epi_tma<HALF, EPI_STORE, false, false>(p, mp, tmem_row, stg, wrbar, rph, m0w, ncol0, lane, release);
         }
       } else {
         // Stream-K segment: raw partial (32 rows x BN/2 fp32 per warp) to the
