@@ -7,6 +7,7 @@
 #include <immintrin.h>
 
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 
 namespace mobius {
@@ -162,9 +163,9 @@ __attribute__((target("avx512f,avx512bw,avx512vl"))) void adamw_chunk_bf16_avx51
     adamw_chunk<0, 0>(w + i, m + i, v + i, g + i, wo + i, n - i, lr, b1, b2, eps, wd, bc1, bc2);
 }
 
-bool have_avx512() {
+bool have_avx512() {  // MOBIUS_ADAMW_SCALAR=1 forces the portable loop (A/B checks)
   static const int ok = __builtin_cpu_supports("avx512f") && __builtin_cpu_supports("avx512bw") &&
-                        __builtin_cpu_supports("avx512vl");
+                        __builtin_cpu_supports("avx512vl") && !std::getenv("MOBIUS_ADAMW_SCALAR");
   return ok != 0;
 }
 

@@ -116,12 +116,16 @@ def test_full_1p5b_step_properties():
     st = ctx.stats()
     l2 = ctx.step(tok)
     l3 = ctx.step(tok)
+    l4 = ctx.step(tok)
     ctx.close()
     # at init LN_f(x) has unit-variance entries, so the logits are
     # ~N(0, h * 0.02^2) and E[CE] = log V + sigma^2 / 2 (lognormal mean)
     expect = math.log(c.vocab) + c.hidden * 0.02 ** 2 / 2
     assert abs(l1 - expect) < 0.05, (l1, expect)
-    assert l2 < l1 and l3 < l1  # training signal (Adam's sign-like first steps may oscillate)
+    # training signal: Adam's sign-like first updates (every weight moves by
+    # ~lr) overshoot on step 3 for this init and lr (measured 11.147, 11.007,
+    # 11.18, 10.84 with every GEMM / optimizer variant), so check the trend
+    assert l2 < l1 and l4 < l2 and np.isfinite(l3), (l1, l2, l3, l4)
     sizes = [plan.stage_first_layer[j + 1] - plan.stage_first_layer[j] for j in range(K)]
     sg = [0] * K
     assert trace == osch.per_gpu_ops(sg, M)[0]
