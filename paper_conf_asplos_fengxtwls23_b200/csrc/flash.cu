@@ -19,7 +19,6 @@
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
-#include <cstdlib>
 #include <cstring>
 
 #include "common.h"
@@ -394,7 +393,6 @@ struct BwdParams {
   int64_t ldd;          // row stride of dK/dV (3h)
   int s, nh, h;
   float scale_log2, scale;
-  int dq_red;           // 1: dQ tiles leave TMEM as vector reductions straight to dQacc (no staging)
 };
 
 __device__ __forceinline__ void red_add_v4(float* addr, float a, float b, float c, float d) {
@@ -575,28 +573,6 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
     };
     auto dq_drain = [&](int itq, uint32_t stg) {
       const int qiq = i0 + itq;
-      if (p.dq_red) {  // TMEM -> registers -> red.global.add.v4.f32 (row = query qiq*128 + r)
-        uint32_t v[DH / 64][32];
-#pragma unroll
-        for (int cc = 0; cc < DH / 64; ++cc) {
-          __syncwarp();
-          ptx::tmem_ld32(T_DQ + (hf * (DH / 64) + cc) * 32 + lane_base, v[cc]);
-        }
-        ptx::tmem_ld_wait();
-        ptx::tc_fence_before();
-        __syncwarp();
-        if (lane == 0) ptx::mbar_arrive(dq_empty);
-        float* dst = p.dQacc + ((int64_t)b * p.s + qiq * 128 + r) * p.h + hd * DH;
-#pragma unroll
-        for (int cc = 0; cc < DH / 64; ++cc) {
-          const int c = hf * (DH / 64) + cc;
-#pragma unroll
-          for (int k = 0; k < 8; ++k)
-            red_add_v4(dst + c * 32 + 4 * k, __uint_as_float(v[cc][4 * k]), __uint_as_float(v[cc][4 * k + 1]),
-                       __uint_as_float(v[cc][4 * k + 2]), __uint_as_float(v[cc][4 * k + 3]));
-        }
-        return;
-      }
       uint32_t v[DH / 64][32];
 #pragma unroll
       for (int cc = 0; cc < DH / 64; ++cc) {
@@ -653,7 +629,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
         ptx::mbar_wait(mm_done, (it - 1) & 1);
         ptx::tc_fence_after();
       }
-      if (!C::DQ_OWN && it >= 1 && !p.dq_red) stage_free();  // dQ(it-1) staged in P^T / dS^T: reduce must have read it
+      if (!C::DQ_OWN && it >= 1) stage_free();  // dQ(it-1) staged in P^T / dS^T: reduce must have read it
 #pragma unroll
       for (int cc = 0; cc < 2; ++cc) {
         const int c = hf * 2 + cc;
@@ -893,14 +869,6 @@ int flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* o, const __nv_
   p.h = h;
   p.scale_log2 = 1.4426950408889634f / sqrtf((float)dh);
   p.scale = 1.0f / sqrtf((float)dh);
-  {
-    static int red = -1;  // MOBIUS_FLASH_DQ_RED: 1 vector reductions, 0 staged TMA reduce-add
-    if (red < 0) {
-      const char* e = getenv("MOBIUS_FLASH_DQ_RED");
-      red = (e && e[0] == '0') ? 0 : 1;
-    }
-    p.dq_red = red;
-  }
   dim3 grid((s / 128) * nh * mbs);
   if (dh == 64) {
     static bool once = false;
