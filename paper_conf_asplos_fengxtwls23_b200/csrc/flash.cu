@@ -378,6 +378,9 @@ struct BwdCfg {
   static constexpr int QS = DH == 64 ? 2 : 1;        // Q/dO pipeline depth
   static constexpr int PT_BYTES = 128 * 128 * 2;     // P^T or dS^T tile
   static constexpr bool DQ_OWN = DH == 64;           // dQ has its own TMEM columns (else aliases S^T)
+  // dh 64: P^T lives in TMEM columns 448..511 and feeds dV += P^T dO as the
+  // A operand of a TS-MMA; the smem it used becomes the second dS^T buffer
+  static constexpr bool PT_TMEM = DH == 64;
   // dh 64: dQ(i-1) is drained from its own staging tile while the MMAs of
   // tile i run; dh 128: staged in the P^T/dS^T tiles (smem budget)
   static constexpr int STG_BYTES = DQ_OWN ? 128 * DH * 4 : 0;
@@ -436,7 +439,10 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
   uint64_t* mm_done = bars + 7;      // dV/dK/dQ of this tile done (P^T/dS^T smem free, dQ ready)
   uint64_t* dq_empty = bars + 8;     // dQ read out (count 8)
   uint64_t* st_empty = bars + 9;     // S^T / dP^T loaded into registers (count 8)
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 10);
+  uint64_t* pt_free = bars + 10;     // dV MMAs of this tile done: P^T (TMEM) may be overwritten
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 11);
+  // dS^T buffers: [it & 1] with P^T in TMEM, else a single tile
+  uint8_t* const sdS_buf[2] = {C::PT_TMEM ? sPT : sdST, sdST};
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const int n_t = p.s / 128;
@@ -462,6 +468,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
     ptx::mbar_init(mm_done, 1);
     ptx::mbar_init(dq_empty, 8);
     ptx::mbar_init(st_empty, 8);
+    ptx::mbar_init(pt_free, 1);
     ptx::fence_mbar_init();
   }
   if (warp == 1) ptx::tmem_alloc<512>(tmem_slot);
@@ -472,6 +479,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
   // TMEM: S^T 0..127, dP^T 128..255, dV 256.., dK 256+DH.., dQ 384.. (dh 64) or aliasing S^T (dh 128)
   const uint32_t T_S = tmem, T_DP = tmem + 128, T_DV = tmem + 256;
   const uint32_t T_DQ = C::DQ_OWN ? tmem + 384 : tmem;
+  const uint32_t T_PT = tmem + 448;  // PT_TMEM only
   const int64_t ld_base = ((int64_t)b * p.nh + hd) * p.s;
 
   if (warp == 0) {
@@ -534,19 +542,39 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
         }
         ptx::mbar_wait(p_full, it & 1);
         ptx::tc_fence_after();
+        if (C::PT_TMEM) {
+          const uint32_t ads = ptx::smem_u32(sdS_buf[it & 1]);
 #pragma unroll
-        for (int t = 0; t < 128 / 16; ++t) {  // K = 128 queries
-          const uint32_t offa = (t >> 2) * 16384 + (t & 3) * 32;
-          ptx::mma_bf16(T_DV, ptx::sdesc_sw128(apt + offa, 16, 1024), ptx::sdesc_sw128(ado + t * 2048, 16384, 1024),
-                        ID_DV, (it > 0 || t > 0) ? 1u : 0u);  // dV += P^T dO
-          ptx::mma_bf16(T_DV + DH, ptx::sdesc_sw128(adst + offa, 16, 1024),
-                        ptx::sdesc_sw128(aq + t * 2048, 16384, 1024), ID_DV, (it > 0 || t > 0) ? 1u : 0u);  // dK += dS^T Q
+          for (int t = 0; t < 128 / 16; ++t)  // dV += P^T dO, P^T from TMEM (8 columns per 16 queries)
+            ptx::mma_bf16_ts(T_DV, T_PT + 8 * t, ptx::sdesc_sw128(ado + t * 2048, 16384, 1024), ID_DV,
+                             (it > 0 || t > 0) ? 1u : 0u);
+          ptx::mma_commit(pt_free);
+#pragma unroll
+          for (int t = 0; t < 128 / 16; ++t) {  // dK += dS^T Q
+            const uint32_t offa = (t >> 2) * 16384 + (t & 3) * 32;
+            ptx::mma_bf16(T_DV + DH, ptx::sdesc_sw128(ads + offa, 16, 1024), ptx::sdesc_sw128(aq + t * 2048, 16384, 1024),
+                          ID_DV, (it > 0 || t > 0) ? 1u : 0u);
+          }
+          if (it >= 1) ptx::mbar_wait(dq_empty, (it - 1) & 1);  // dQ(it-1) read out
+#pragma unroll
+          for (int t = 0; t < 128 / 16; ++t)  // K = 128 keys: dQ = dS K
+            ptx::mma_bf16(T_DQ, ptx::sdesc_sw128(ads + t * 2048, 16384, 1024),
+                          ptx::sdesc_sw128(ak + t * 2048, 16384, 1024), ID_DQ, t > 0);
+        } else {
+#pragma unroll
+          for (int t = 0; t < 128 / 16; ++t) {  // K = 128 queries
+            const uint32_t offa = (t >> 2) * 16384 + (t & 3) * 32;
+            ptx::mma_bf16(T_DV, ptx::sdesc_sw128(apt + offa, 16, 1024), ptx::sdesc_sw128(ado + t * 2048, 16384, 1024),
+                          ID_DV, (it > 0 || t > 0) ? 1u : 0u);  // dV += P^T dO
+            ptx::mma_bf16(T_DV + DH, ptx::sdesc_sw128(adst + offa, 16, 1024),
+                          ptx::sdesc_sw128(aq + t * 2048, 16384, 1024), ID_DV, (it > 0 || t > 0) ? 1u : 0u);  // dK += dS^T Q
+          }
+          if (C::DQ_OWN && it >= 1) ptx::mbar_wait(dq_empty, (it - 1) & 1);  // dQ(it-1) read out
+#pragma unroll
+          for (int t = 0; t < 128 / 16; ++t)  // K = 128 keys: dQ = dS K
+            ptx::mma_bf16(T_DQ, ptx::sdesc_sw128(adst + t * 2048, 16384, 1024),
+                          ptx::sdesc_sw128(ak + t * 2048, 16384, 1024), ID_DQ, t > 0);
         }
-        if (C::DQ_OWN && it >= 1) ptx::mbar_wait(dq_empty, (it - 1) & 1);  // dQ(it-1) read out
-#pragma unroll
-        for (int t = 0; t < 128 / 16; ++t)  // K = 128 keys: dQ = dS K
-          ptx::mma_bf16(T_DQ, ptx::sdesc_sw128(adst + t * 2048, 16384, 1024),
-                        ptx::sdesc_sw128(ak + t * 2048, 16384, 1024), ID_DQ, t > 0);
         ptx::mma_commit(mm_done);
         ptx::mma_commit(&q_empty[st]);
         if (!C::DQ_OWN && it + 1 < nq) issue_st(it + 1);
@@ -560,7 +588,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
     const int hf = (warp - 2) >> 2;
     const int r = q4 * 32 + lane;  // key row of this thread (TMEM lane)
     const uint32_t lane_base = (uint32_t)(q4 * 32) << 16;
-    const uint32_t spt = ptx::smem_u32(sPT), sdst = ptx::smem_u32(sdST);
+    const uint32_t spt = ptx::smem_u32(sPT);
     // dQ(it) (TMEM lane = query row) -> fp32 staging [DH/32 slabs][128 rows][128 B],
     // 16-byte chunks XOR-swizzled by row (TMA SWIZZLE_128B, conflict-free
     // stores) -> one TMA reduce-add per 32-column slab into the dQ buffer
@@ -625,11 +653,20 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
       if (lane == 0) ptx::mbar_arrive(st_empty);  // S^T / dP^T TMEM may be overwritten
       // P^T / dS^T smem must be free: dh 128 - the previous tile's dQ drain
       // (staged there) completed; dh 64 - the previous tile's MMAs completed
-      if (C::DQ_OWN && it >= 1) {
+      if (C::PT_TMEM) {
+        // P^T (TMEM) free once the dV MMAs of the previous tile completed;
+        // dS^T buffer it&1 was last read by the MMAs of tile it-2, whose
+        // completion the dQ drain of tile it-2 already waited for
+        if (it >= 1) {
+          ptx::mbar_wait(pt_free, (it - 1) & 1);
+          ptx::tc_fence_after();
+        }
+      } else if (C::DQ_OWN && it >= 1) {
         ptx::mbar_wait(mm_done, (it - 1) & 1);
         ptx::tc_fence_after();
       }
       if (!C::DQ_OWN && it >= 1) stage_free();  // dQ(it-1) staged in P^T / dS^T: reduce must have read it
+      const uint32_t sds = ptx::smem_u32(sdS_buf[C::PT_TMEM ? (it & 1) : 0]);
 #pragma unroll
       for (int cc = 0; cc < 2; ++cc) {
         const int c = hf * 2 + cc;
@@ -650,19 +687,31 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
           ppk[e >> 1] = pack_bf16(p0, p1);
           dpk[e >> 1] = pack_bf16(d0, d1);
         }
+        if (C::PT_TMEM) {  // P^T row r, queries c*32.. -> TMEM columns (2 bf16 per column)
+          ptx::tmem_st16(T_PT + c * 16 + lane_base, ppk);
 #pragma unroll
-        for (int k = 0; k < 4; ++k) {
-          const uint32_t o = sw128_off(r, c * 4 + k);
-          st_shared_v4(spt + o, ppk[4 * k], ppk[4 * k + 1], ppk[4 * k + 2], ppk[4 * k + 3]);
-          st_shared_v4(sdst + o, dpk[4 * k], dpk[4 * k + 1], dpk[4 * k + 2], dpk[4 * k + 3]);
+          for (int k = 0; k < 4; ++k)
+            st_shared_v4(sds + sw128_off(r, c * 4 + k), dpk[4 * k], dpk[4 * k + 1], dpk[4 * k + 2], dpk[4 * k + 3]);
+        } else {
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            const uint32_t o = sw128_off(r, c * 4 + k);
+            st_shared_v4(spt + o, ppk[4 * k], ppk[4 * k + 1], ppk[4 * k + 2], ppk[4 * k + 3]);
+            st_shared_v4(sds + o, dpk[4 * k], dpk[4 * k + 1], dpk[4 * k + 2], dpk[4 * k + 3]);
+          }
         }
       }
+      if (C::PT_TMEM) ptx::tmem_st_wait();
       ptx::tc_fence_before();
       ptx::fence_proxy_async();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(p_full);
       if (C::DQ_OWN) {
         // drain dQ of the previous query tile while this tile's MMAs run
+        if (C::PT_TMEM && it >= 1) {
+          ptx::mbar_wait(mm_done, (it - 1) & 1);
+          ptx::tc_fence_after();
+        }
         if (it >= 1) dq_drain(it - 1, ptx::smem_u32(sSTG));
       } else {
         ptx::mbar_wait(mm_done, it & 1);
