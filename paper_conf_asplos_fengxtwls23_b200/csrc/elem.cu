@@ -197,6 +197,83 @@ __global__ void __launch_bounds__(256) ln_fwd_warp_k(const T* __restrict__ x, co
   }
 }
 
+// bf16 LayerNorm, warp per row, the row held PACKED (8 bf16 per uint4
+// register quad) so a warp needs 4*NV registers for it: ~2x the resident
+// warps of the float-cached version, all row loads issued up front.  Same
+// arithmetic and summation order as ln_fwd_warp_k / ln_bwd_dx_k, so the
+// results are bit-identical to them.
+__device__ __forceinline__ void unpack8(const uint4& u, float* f) {
+  const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&u);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const float2 t = __bfloat1622float2(h2[i]);
+    f[2 * i] = t.x;
+    f[2 * i + 1] = t.y;
+  }
+}
+__device__ __forceinline__ uint4 pack8(const float* f) {
+  uint4 v;
+  __nv_bfloat162* h2 = reinterpret_cast<__nv_bfloat162*>(&v);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) h2[i] = __floats2bfloat162_rn(f[2 * i], f[2 * i + 1]);
+  return v;
+}
+
+template <int NV>
+__global__ void __launch_bounds__(256, 3) ln_fwd_bf16_k(const __nv_bfloat16* __restrict__ x,
+                                                     const __nv_bfloat16* __restrict__ g,
+                                                     const __nv_bfloat16* __restrict__ b, __nv_bfloat16* __restrict__ y,
+                                                     float* mu_out, float* rstd_out, int rows, int h) {
+  const int lane = threadIdx.x % 32;
+  const int r = blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32;
+  if (r >= rows) return;
+  const int nvec = h / 8;
+  const uint4* xr = reinterpret_cast<const uint4*>(x + (int64_t)r * h);
+  uint4 xv[NV];
+#pragma unroll
+  for (int k = 0; k < NV; ++k)
+    if (lane + 32 * k < nvec) xv[k] = xr[lane + 32 * k];
+  float sum = 0.f;
+#pragma unroll
+  for (int k = 0; k < NV; ++k)
+    if (lane + 32 * k < nvec) {
+      float f[8];
+      unpack8(xv[k], f);
+#pragma unroll
+      for (int e = 0; e < 8; ++e) sum += f[e];
+    }
+  const float m = warp_sum(sum) / h;
+  float q = 0.f;
+#pragma unroll
+  for (int k = 0; k < NV; ++k)
+    if (lane + 32 * k < nvec) {
+      float f[8];
+      unpack8(xv[k], f);
+#pragma unroll
+      for (int e = 0; e < 8; ++e) {
+        const float d = f[e] - m;
+        q += d * d;
+      }
+    }
+  const float rs = rsqrtf(warp_sum(q) / h + 1e-5f);
+  if (lane == 0) {
+    mu_out[r] = m;
+    rstd_out[r] = rs;
+  }
+  uint4* yr = reinterpret_cast<uint4*>(y + (int64_t)r * h);
+#pragma unroll
+  for (int k = 0; k < NV; ++k)
+    if (lane + 32 * k < nvec) {
+      float f[8], gg[8], bb[8], o[8];
+      unpack8(xv[k], f);
+      unpack8(__ldg(reinterpret_cast<const uint4*>(g) + lane + 32 * k), gg);
+      unpack8(__ldg(reinterpret_cast<const uint4*>(b) + lane + 32 * k), bb);
+#pragma unroll
+      for (int e = 0; e < 8; ++e) o[e] = (f[e] - m) * rs * gg[e] + bb[e];
+      yr[lane + 32 * k] = pack8(o);
+    }
+}
+
 template <typename T, int LN_NT, int LN_MAXV>
 __global__ void __launch_bounds__(LN_NT) ln_fwd_k(const T* x, const T* g, const T* b, T* y, float* mu_out,
                                                    float* rstd_out, int h) {
@@ -560,11 +637,33 @@ int embed_bwd(const int32_t* tok, const T* dx, float* dwte, float* dwpe, int mbs
     else MOBIUS_FAIL(MOBIUS_EINVAL, "layernorm: h=%d too large", h);          \
   } while (0)
 
+// MOBIUS_LN_FLOATROW=1 selects the float-cached row LN forward (A/B timing)
+static bool ln_packed() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("MOBIUS_LN_FLOATROW");
+    v = (e && e[0] == '1') ? 0 : 1;
+  }
+  return v == 1;
+}
+
 template <typename T>
 int layernorm_fwd(const T* x, const T* g, const T* b, T* y, float* mu, float* rstd, int rows, int h, cudaStream_t st) {
   MOBIUS_CHECK_ARG(h % Vec<T>::N == 0, "layernorm: unsupported h=%d", h);
   const int nv = (h / Vec<T>::N + 31) / 32;  // vectors per lane
   const unsigned blocks = (unsigned)((rows + 7) / 8);
+  if constexpr (sizeof(T) == 2) {
+    if (ln_packed() && nv <= 8 && aligned16(x) && aligned16(y) && aligned16(g) && aligned16(b)) {
+#define LNF(NV) ln_fwd_bf16_k<NV><<<blocks, 256, 0, st>>>(x, g, b, y, mu, rstd, rows, h)
+      if (nv <= 4) LNF(4);
+      else if (nv == 5) LNF(5);
+      else if (nv == 6) LNF(6);
+      else if (nv == 7) LNF(7);
+      else LNF(8);
+#undef LNF
+      return check_launch("layernorm_fwd");
+    }
+  }
   if (nv <= 4)
     ln_fwd_warp_k<T, 4><<<blocks, 256, 0, st>>>(x, g, b, y, mu, rstd, rows, h);
   else if (nv <= 8)

@@ -146,7 +146,10 @@ __device__ __forceinline__ void epi_vals_t(const Params& p, float (&v)[W], int m
   constexpr bool has_r = EPI == EPI_BIAS_RESID || EPI == EPI_GELU_BWD;
   constexpr bool accum = EPI == EPI_ACCUM && ACC;
   const __nv_bfloat16* rrow = has_r ? p.R + (int64_t)b1 * p.rbs1 + (int64_t)b2 * p.rbs2 + (int64_t)m * p.ldr + n0 : nullptr;
-  __nv_bfloat16* aux = EPI == EPI_BIAS_GELU
+  // AUX: the pre-activation u (EPI_BIAS_GELU), or, when set for
+  // EPI_GELU_BWD, g = gelu(R) - the forward's activation recomputed from the
+  // R (= u) values this epilogue reads anyway
+  __nv_bfloat16* aux = (EPI == EPI_BIAS_GELU || (EPI == EPI_GELU_BWD && p.AUX))
                            ? p.AUX + (int64_t)b1 * p.xbs1 + (int64_t)b2 * p.xbs2 + (int64_t)m * p.ldx + n0
                            : nullptr;
   if (n0 + W <= p.N) {
@@ -183,6 +186,22 @@ __device__ __forceinline__ void epi_vals_t(const Params& p, float (&v)[W], int m
       // GeLU of the bf16-rounded pre-activation (what backward will see)
 #pragma unroll
       for (int i = 0; i < W; ++i) v[i] = gelu_f(__bfloat162float(__float2bfloat16_rn(v[i])));
+    }
+    if constexpr (EPI == EPI_GELU_BWD) {
+      if (aux) {
+#pragma unroll
+        for (int i = 0; i < W / 8; ++i) {
+          float gf[8];
+          const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&lr[i]);
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            const float2 x = __bfloat1622float2(h2[j]);
+            gf[2 * j] = gelu_f(x.x);
+            gf[2 * j + 1] = gelu_f(x.y);
+          }
+          st_bf16x8(aux + 8 * i, gf);
+        }
+      }
     }
     if constexpr (has_r) {
 #pragma unroll
@@ -230,7 +249,11 @@ __device__ __forceinline__ void epi_vals_t(const Params& p, float (&v)[W], int m
           x = gelu_f(__bfloat162float(__float2bfloat16_rn(x)));
         }
         if (EPI == EPI_BIAS_RESID) x += __bfloat162float(rrow[i]);
-        if (EPI == EPI_GELU_BWD) x *= gelu_grad_f(__bfloat162float(rrow[i]));
+        if (EPI == EPI_GELU_BWD) {
+          const float u = __bfloat162float(rrow[i]);
+          if (aux) aux[i] = __float2bfloat16_rn(gelu_f(u));
+          x *= gelu_grad_f(u);
+        }
         if constexpr (CF32) {
           float* cp = reinterpret_cast<float*>(p.C) + crow + n0;
           cp[i] = x + (accum ? cp[i] : 0.f);

@@ -144,6 +144,7 @@ __device__ __forceinline__ void epi_tma(const Params& p, const EpiMaps& mp, uint
         }
       }
       const uint32_t box = stg + (has_r ? j * 4096 : 0);
+      uint32_t gk[EPI == EPI_GELU_BWD ? 8 : 1][4];  // EPI_GELU_BWD with AUX: packed g of this chunk
       if constexpr (has_r) {
         ptx::mbar_wait(&rbar[j], (rph >> j) & 1u);  // R box j landed
 #pragma unroll
@@ -160,6 +161,10 @@ __device__ __forceinline__ void epi_tma(const Params& p, const EpiMaps& mp, uint
               v[8 * c + 2 * k] += x.x;
               v[8 * c + 2 * k + 1] += x.y;
             } else {
+              if (p.AUX) {  // g = gelu(u), bf16, as the forward epilogue computed it
+                const __nv_bfloat162 g2 = __floats2bfloat162_rn(gelu_f(x.x), gelu_f(x.y));
+                gk[c][k] = *reinterpret_cast<const uint32_t*>(&g2);
+              }
               v[8 * c + 2 * k] *= gelu_grad_f(x.x);
               v[8 * c + 2 * k + 1] *= gelu_grad_f(x.y);
             }
@@ -214,6 +219,23 @@ __device__ __forceinline__ void epi_tma(const Params& p, const EpiMaps& mp, uint
         if (lane == 0) {
           tma_store_2d(mp.C, box, n0, m0w);
           bulk_commit();
+        }
+        if constexpr (EPI == EPI_GELU_BWD) {
+          if (p.AUX) {  // g leaves through the same box once the dU store has read it
+            if (lane == 0) bulk_wait_read<0>();
+            __syncwarp();
+#pragma unroll
+            for (int c = 0; c < 8; ++c)
+              asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(box + box_off(lane, c)), "r"(gk[c][0]),
+                           "r"(gk[c][1]), "r"(gk[c][2]), "r"(gk[c][3])
+                           : "memory");
+            ptx::fence_proxy_async();
+            __syncwarp();
+            if (lane == 0) {
+              tma_store_2d(mp.X, box, n0, m0w);
+              bulk_commit();
+            }
+          }
         }
       }
     }
@@ -726,7 +748,7 @@ static int gemm_bf16_2cta_bn(const GemmDesc& d, cudaStream_t s) {
   } else {
     tr = tc;
   }
-  if (d.epi == EPI_BIAS_GELU) {
+  if (d.epi == EPI_BIAS_GELU || (d.epi == EPI_GELU_BWD && d.AUX.ptr)) {
     if ((rc = make_map_2d(&tx, d.AUX.ptr, false, d.AUX.ld, d.N, d.M, 64, 32))) return rc;
   } else {
     tx = tc;

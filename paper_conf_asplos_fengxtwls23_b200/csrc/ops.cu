@@ -372,27 +372,28 @@ int block_bwd(const Shape& sh, const T* w, const BlockActs<T>& A_in, const T* dy
   const int64_t Sbs2 = (int64_t)s * s, Sbs1 = nh * Sbs2;
   const float scale = 1.0f / sqrtf((float)dh);
   BlockActs<T> A = A_in;
-  if (!A.a) {  // compact kept activations: recompute a, a2 (LN forwards) and g = gelu(u)
+  const bool compact = !A.a;
+  if (compact) {  // compact kept activations: recompute a, a2 (LN forwards); g = gelu(u) comes from the du GEMM
     if constexpr (sizeof(T) != 2) {
       MOBIUS_FAIL(MOBIUS_EINVAL, "block_bwd: compact activations are bf16-only");
     } else {
-      ElemScope es(st, 1);
+      ElemScope es(st, 2);
       A.a = sc.ra;
       A.a2 = sc.ra2;
       A.g = sc.rg;
       RC(layernorm_fwd<T>(A.x, w + L.ln1_g, w + L.ln1_b, A.a, A.mu1, A.rs1, Tn, h, st));
       RC(layernorm_fwd<T>(A.x1, w + L.ln2_g, w + L.ln2_b, A.a2, A.mu2, A.rs2, Tn, h, st));
-      RC(gelu_fwd_bf16(A.u, A.g, (int64_t)Tn * 4 * h, st));
     }
   }
   T* du = sc.big1;
-  {  // du = (dy W2^T) * gelu'(u)
+  {  // du = (dy W2^T) * gelu'(u); compact: also g = gelu(u) (AUX), bit-identical to the forward's
     GemmDesc d;
     d.M = Tn; d.N = 4 * h; d.K = h;
     d.A = mv(dy, h);
     d.B = mv(w + L.w_2, h);
     d.C = mv(du, 4 * h);
     d.epi = EPI_GELU_BWD; d.R = mv(A.u, 4 * h);
+    if (compact) d.AUX = mv(A.g, 4 * h);
     RC(run_gemm<T>(d, st, KCLS_GEMM));
   }
   {  // dW2 += g^T dy
