@@ -11,9 +11,10 @@
 //                            merged from TMEM; writes O (bf16) and lse (log2).
 // Backward, one CTA per (batch, head, 128-key tile), loop over query tiles
 // i >= j:  S^T = K Q_i^T, dP^T = V dO_i^T (TMEM); thread = key row computes
-// P^T = 2^(S^T*c - lse_q), dS^T = P^T (dP^T - D_q) * scale into smem; then
+// P^T = 2^(S^T*c - lse_q), dS^T = P^T (dP^T - D_q) into smem; then
 // dV += P^T dO_i, dK += dS^T Q_i (TMEM accumulators), dQ_i = dS K_j (TMEM,
-// red.global.add.f32 into an fp32 dQ buffer).  The same smem tiles serve as
+// TMA reduce-add into an fp32 dQ buffer); the 1/sqrt(dh) of dS is applied to
+// dK at its store and to dQ in the final cast.  The same smem tiles serve as
 // K-major and MN-major UMMA operands, so no transposes are materialised.
 #include <cuda.h>
 #include <cuda_bf16.h>
@@ -31,7 +32,6 @@ namespace {
 
 constexpr int BQ = 128;
 constexpr int BKV = 128;
-constexpr int NT = 192;
 
 __device__ __forceinline__ void named_bar(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
 
@@ -58,9 +58,11 @@ __device__ __forceinline__ float lds_f32(uint32_t addr) {
   asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(addr) : "memory");
   return v;
 }
-__device__ __forceinline__ float2 lds_f32x2(uint32_t addr) {
-  float2 v;
-  asm volatile("ld.shared.v2.f32 {%0, %1}, [%2];" : "=f"(v.x), "=f"(v.y) : "r"(addr) : "memory");
+
+__device__ __forceinline__ float4 lds_f32x4(uint32_t addr) {
+  float4 v;
+  asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(addr)
+               : "memory");
   return v;
 }
 
@@ -68,6 +70,43 @@ __device__ __forceinline__ float ex2(float x) {
   float y;
   asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
   return y;
+}
+
+__device__ __forceinline__ uint32_t pack_bf16x2(float2 v) { return pack_bf16(v.x, v.y); }
+
+// Softmax-gradient math of one 32-query slab of a key row (flash bwd):
+//   P^T[r, q]  = 2^(S^T[r, q] * c - lse_q)          (masked to q >= r on the diagonal tile)
+//   dS^T[r, q] = P^T[r, q] * (dP^T[r, q] - D_q)      (the 1/sqrt(dh) factor is applied to
+//                                                     dK / dQ after accumulation)
+// sLDq: smem address of lse[q0..q0+31] (fp32), followed 512 bytes later by -D.
+// Packed f32x2 arithmetic (FADD2/FMUL2); the non-diagonal instantiation
+// carries no masking code at all.
+template <bool DIAG>
+__device__ __forceinline__ void bwd_slab_math(const uint32_t (&vs)[32], const uint32_t (&vd)[32], uint32_t sLDq,
+                                              int q0, int r, float sl2, uint32_t (&ppk)[16], uint32_t (&dpk)[16]) {
+#pragma unroll
+  for (int e = 0; e < 32; e += 4) {
+    const float4 L = lds_f32x4(sLDq + e * 4), nD = lds_f32x4(sLDq + 512 + e * 4);  // broadcast reads
+    float p0 = ex2(fmaf(__uint_as_float(vs[e]), sl2, -L.x));
+    float p1 = ex2(fmaf(__uint_as_float(vs[e + 1]), sl2, -L.y));
+    float p2 = ex2(fmaf(__uint_as_float(vs[e + 2]), sl2, -L.z));
+    float p3 = ex2(fmaf(__uint_as_float(vs[e + 3]), sl2, -L.w));
+    if (DIAG) {  // key r attends only from queries >= r
+      const int q = q0 + e;
+      if (q < r) p0 = 0.f;
+      if (q + 1 < r) p1 = 0.f;
+      if (q + 2 < r) p2 = 0.f;
+      if (q + 3 < r) p3 = 0.f;
+    }
+    const float2 P01 = make_float2(p0, p1), P23 = make_float2(p2, p3);
+    const float2 t01 = __fadd2_rn(make_float2(__uint_as_float(vd[e]), __uint_as_float(vd[e + 1])), make_float2(nD.x, nD.y));
+    const float2 t23 =
+        __fadd2_rn(make_float2(__uint_as_float(vd[e + 2]), __uint_as_float(vd[e + 3])), make_float2(nD.z, nD.w));
+    ppk[e >> 1] = pack_bf16x2(P01);
+    ppk[(e >> 1) + 1] = pack_bf16x2(P23);
+    dpk[e >> 1] = pack_bf16x2(__fmul2_rn(P01, t01));
+    dpk[(e >> 1) + 1] = pack_bf16x2(__fmul2_rn(P23, t23));
+  }
 }
 
 constexpr int NT_FWD = 320;  // 10 warps: TMA, MMA, 8 softmax warps (4 lane quadrants x 2 column halves)
@@ -389,19 +428,14 @@ struct BwdCfg {
 
 struct BwdParams {
   const float* lse;     // [mbs, nh, s] log2 domain
-  const float* Dsum;    // [mbs, nh, s] rowsum(dO * O)
+  const float* Dsum;    // [mbs, nh, s] -rowsum(dO * O) (negated)
   float* dQacc;         // [mbs*s, h] fp32 (head view), accumulated with red.add
   __nv_bfloat16* dK;    // head view into dqkv (k part)
   __nv_bfloat16* dV;    // head view into dqkv (v part)
   int64_t ldd;          // row stride of dK/dV (3h)
-  int s, nh, h;
+  int s, nh, h, mbs;
   float scale_log2, scale;
 };
-
-__device__ __forceinline__ void red_add_v4(float* addr, float a, float b, float c, float d) {
-  asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(addr), "f"(a), "f"(b), "f"(c), "f"(d)
-               : "memory");
-}
 
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
@@ -410,10 +444,19 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
                : "memory");
 }
 
-// One CTA per (batch, head, 128-key tile); loop over query tiles i >= kt.
+// Item = (batch, head, 128-key tile kt); it visits query tiles i >= kt.
+// Persistent: one CTA per SM walks its items (snake order over the list
+// sorted heaviest first, so per-CTA work balances to ~5%); all barrier
+// phases run on a per-CTA global tile counter g, so the TMA warp prefetches
+// the next item's Q/dO tiles and K/V while the current item finishes, and
+// the next item's scores start while its predecessor's dV/dK leave TMEM.
 // MMA order per query tile: [S^T, dP^T](i) ... wait P^T/dS^T(i) ... dV, dK,
 // dQ(i), then [S^T, dP^T](i+1) right away (the softmax-gradient warps are
 // done with S^T(i)), so the next scores overlap the dQ read-out.
+__device__ __forceinline__ int bwd_item_of(int pass, int ncta, int cta) {
+  return pass * ncta + ((pass & 1) ? ncta - 1 - cta : cta);
+}
+
 template <int DH>
 __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_constant__ CUtensorMap tm,
                                                               const __grid_constant__ CUtensorMap tdo,
@@ -429,9 +472,9 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
   uint8_t* sPT = sdO + QS * C::T_BYTES;
   uint8_t* sdST = sPT + C::PT_BYTES;
   uint8_t* sSTG = sdST + C::PT_BYTES;  // dQ staging (dh 64)
-  float* sLD = reinterpret_cast<float*>(sSTG + C::STG_BYTES);  // [QS][lse 128 | D 128]
+  float* sLD = reinterpret_cast<float*>(sSTG + C::STG_BYTES);  // [QS][lse 128 | -D 128]
   uint64_t* bars = reinterpret_cast<uint64_t*>(sLD + QS * 256);
-  uint64_t* kv_full = bars;          // 1
+  uint64_t* kv_full = bars;          // K/V of the current item landed
   uint64_t* q_full = bars + 1;       // [2] (Q, dO, lse, D)
   uint64_t* q_empty = bars + 3;      // [2]
   uint64_t* s_full = bars + 5;       // S^T and dP^T ready
@@ -440,19 +483,25 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
   uint64_t* dq_empty = bars + 8;     // dQ read out (count 8)
   uint64_t* st_empty = bars + 9;     // S^T / dP^T loaded into registers (count 8)
   uint64_t* pt_free = bars + 10;     // dV MMAs of this tile done: P^T (TMEM) may be overwritten
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 11);
-  // dS^T buffers: [it & 1] with P^T in TMEM, else a single tile
+  uint64_t* kv_empty = bars + 11;    // every MMA of an item done: K/V smem may be reloaded
+  uint64_t* acc_empty = bars + 12;   // dV/dK of an item read out of TMEM (count 8)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 13);
+  // dS^T buffers: [g & 1] with P^T in TMEM, else a single tile
   uint8_t* const sdS_buf[2] = {C::PT_TMEM ? sPT : sdST, sdST};
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const int n_t = p.s / 128;
-  // linear grid, heaviest first: every (b, head) with key tile 0 (n_t query
-  // tiles to visit) launches before any with key tile 1, ..., so the last
-  // wave holds the one-tile CTAs (longest-processing-time-first order)
-  const int nbh = (int)gridDim.x / (p.s / 128);  // nh * mbs
-  const int kt = (int)blockIdx.x / nbh;
-  const int hd = ((int)blockIdx.x % nbh) % p.nh, b = ((int)blockIdx.x % nbh) / p.nh;
-  const int i0 = kt, nq = n_t - kt;
+  const int nbh = p.nh * p.mbs;
+  const int n_items = n_t * nbh;
+  const int ncta = (int)gridDim.x, cta = (int)blockIdx.x;
+  // item index -> (key tile, head, batch); the list is sorted heaviest
+  // first: every (b, head) with key tile 0 (n_t query tiles) before key tile 1 ...
+  auto decode = [&](int item, int& kt, int& hd, int& b) {
+    kt = item / nbh;
+    const int r = item % nbh;
+    hd = r % p.nh;
+    b = r / p.nh;
+  };
 
   if (threadIdx.x == 0) {
     ptx::tma_prefetch_desc(&tm);
@@ -469,6 +518,8 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
     ptx::mbar_init(dq_empty, 8);
     ptx::mbar_init(st_empty, 8);
     ptx::mbar_init(pt_free, 1);
+    ptx::mbar_init(kv_empty, 1);
+    ptx::mbar_init(acc_empty, 8);
     ptx::fence_mbar_init();
   }
   if (warp == 1) ptx::tmem_alloc<512>(tmem_slot);
@@ -480,29 +531,40 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
   const uint32_t T_S = tmem, T_DP = tmem + 128, T_DV = tmem + 256;
   const uint32_t T_DQ = C::DQ_OWN ? tmem + 384 : tmem;
   const uint32_t T_PT = tmem + 448;  // PT_TMEM only
-  const int64_t ld_base = ((int64_t)b * p.nh + hd) * p.s;
 
   if (warp == 0) {
     if (lane == 0) {
-      ptx::mbar_arrive_expect_tx(kv_full, 2 * C::T_BYTES);
+      int g = 0, n = 0;  // global tile / item counters of this CTA
+      for (int pass = 0; pass * ncta < n_items; ++pass) {
+        const int item = bwd_item_of(pass, ncta, cta);
+        if (item >= n_items) continue;
+        int kt, hd, b;
+        decode(item, kt, hd, b);
+        const int nq = n_t - kt;
+        const int64_t ld_base = ((int64_t)b * p.nh + hd) * p.s;
+        auto load_q = [&](int it) {
+          const int gg = g + it, st = gg % QS, ph = (gg / QS) & 1, qi = kt + it;
+          ptx::mbar_wait(&q_empty[st], ph ^ 1);
+          ptx::mbar_arrive_expect_tx(&q_full[st], 2 * C::T_BYTES + 1024);
 #pragma unroll
-      for (int c = 0; c < DH / 64; ++c) {
-        ptx::tma_load_4d(sK + c * 16384, &tm, kv_full, 64 * c, kt * 128, p.nh + hd, b);
-        ptx::tma_load_4d(sV + c * 16384, &tm, kv_full, 64 * c, kt * 128, 2 * p.nh + hd, b);
-      }
-      for (int it = 0; it < nq; ++it) {
-        const int st = it % QS;
-        const int ph = (it / QS) & 1;
-        const int qi = i0 + it;
-        ptx::mbar_wait(&q_empty[st], ph ^ 1);
-        ptx::mbar_arrive_expect_tx(&q_full[st], 2 * C::T_BYTES + 1024);
+          for (int c = 0; c < DH / 64; ++c) {
+            ptx::tma_load_4d(sQ + st * C::T_BYTES + c * 16384, &tm, &q_full[st], 64 * c, qi * 128, hd, b);
+            ptx::tma_load_4d(sdO + st * C::T_BYTES + c * 16384, &tdo, &q_full[st], 64 * c, qi * 128, hd, b);
+          }
+          bulk_g2s(sLD + st * 256, p.lse + ld_base + qi * 128, 512, &q_full[st]);
+          bulk_g2s(sLD + st * 256 + 128, p.Dsum + ld_base + qi * 128, 512, &q_full[st]);
+        };
+        load_q(0);  // its ring slot frees before the previous item's K/V do
+        if (n >= 1) ptx::mbar_wait(kv_empty, (n - 1) & 1);
+        ptx::mbar_arrive_expect_tx(kv_full, 2 * C::T_BYTES);
 #pragma unroll
         for (int c = 0; c < DH / 64; ++c) {
-          ptx::tma_load_4d(sQ + st * C::T_BYTES + c * 16384, &tm, &q_full[st], 64 * c, qi * 128, hd, b);
-          ptx::tma_load_4d(sdO + st * C::T_BYTES + c * 16384, &tdo, &q_full[st], 64 * c, qi * 128, hd, b);
+          ptx::tma_load_4d(sK + c * 16384, &tm, kv_full, 64 * c, kt * 128, p.nh + hd, b);
+          ptx::tma_load_4d(sV + c * 16384, &tm, kv_full, 64 * c, kt * 128, 2 * p.nh + hd, b);
         }
-        bulk_g2s(sLD + st * 256, p.lse + ld_base + qi * 128, 512, &q_full[st]);
-        bulk_g2s(sLD + st * 256 + 128, p.Dsum + ld_base + qi * 128, 512, &q_full[st]);
+        for (int it = 1; it < nq; ++it) load_q(it);
+        g += nq;
+        ++n;
       }
     }
   } else if (warp == 1) {
@@ -512,11 +574,11 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
       constexpr uint32_t ID_DQ = ptx::idesc_bf16(128, DH, 1, 1);   // dQ
       const uint32_t ak = ptx::smem_u32(sK), av = ptx::smem_u32(sV);
       const uint32_t apt = ptx::smem_u32(sPT), adst = ptx::smem_u32(sdST);
-      auto issue_st = [&](int it) {
-        const int st = it % QS, ph = (it / QS) & 1;
+      auto issue_st = [&](int gg) {
+        const int st = gg % QS, ph = (gg / QS) & 1;
         const uint32_t aq = ptx::smem_u32(sQ + st * C::T_BYTES), ado = ptx::smem_u32(sdO + st * C::T_BYTES);
         ptx::mbar_wait(&q_full[st], ph);
-        if (!C::DQ_OWN && it >= 1) ptx::mbar_wait(dq_empty, (it - 1) & 1);  // S^T region holds dQ(it-1)
+        if (!C::DQ_OWN && gg >= 1) ptx::mbar_wait(dq_empty, (gg - 1) & 1);  // S^T region holds dQ(gg-1)
         ptx::tc_fence_after();
 #pragma unroll
         for (int t = 0; t < DH / 16; ++t) {
@@ -531,53 +593,65 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
         }
         ptx::mma_commit(s_full);
       };
-      ptx::mbar_wait(kv_full, 0);
-      issue_st(0);
-      for (int it = 0; it < nq; ++it) {
-        const int st = it % QS;
-        const uint32_t aq = ptx::smem_u32(sQ + st * C::T_BYTES), ado = ptx::smem_u32(sdO + st * C::T_BYTES);
-        if (C::DQ_OWN && it + 1 < nq) {  // scores of the next query tile overlap this tile's softmax-gradient
-          ptx::mbar_wait(st_empty, it & 1);
-          issue_st(it + 1);
-        }
-        ptx::mbar_wait(p_full, it & 1);
-        ptx::tc_fence_after();
-        if (C::PT_TMEM) {
-          const uint32_t ads = ptx::smem_u32(sdS_buf[it & 1]);
-#pragma unroll
-          for (int t = 0; t < 128 / 16; ++t)  // dV += P^T dO, P^T from TMEM (8 columns per 16 queries)
-            ptx::mma_bf16_ts(T_DV, T_PT + 8 * t, ptx::sdesc_sw128(ado + t * 2048, 16384, 1024), ID_DV,
-                             (it > 0 || t > 0) ? 1u : 0u);
-          ptx::mma_commit(pt_free);
-#pragma unroll
-          for (int t = 0; t < 128 / 16; ++t) {  // dK += dS^T Q
-            const uint32_t offa = (t >> 2) * 16384 + (t & 3) * 32;
-            ptx::mma_bf16(T_DV + DH, ptx::sdesc_sw128(ads + offa, 16, 1024), ptx::sdesc_sw128(aq + t * 2048, 16384, 1024),
-                          ID_DV, (it > 0 || t > 0) ? 1u : 0u);
+      int g = 0, n = 0;
+      for (int pass = 0; pass * ncta < n_items; ++pass) {
+        const int item = bwd_item_of(pass, ncta, cta);
+        if (item >= n_items) continue;
+        const int nq = n_t - item / nbh;
+        ptx::mbar_wait(kv_full, n & 1);
+        // S^T / dP^T TMEM must have been read (dh 64; dh 128: issue_st waits dq_empty)
+        if (C::DQ_OWN && g >= 1) ptx::mbar_wait(st_empty, (g - 1) & 1);
+        issue_st(g);
+        for (int it = 0; it < nq; ++it) {
+          const int gg = g + it, st = gg % QS;
+          const uint32_t aq = ptx::smem_u32(sQ + st * C::T_BYTES), ado = ptx::smem_u32(sdO + st * C::T_BYTES);
+          if (C::DQ_OWN && it + 1 < nq) {  // scores of the next query tile overlap this tile's softmax-gradient
+            ptx::mbar_wait(st_empty, gg & 1);
+            issue_st(gg + 1);
           }
-          if (it >= 1) ptx::mbar_wait(dq_empty, (it - 1) & 1);  // dQ(it-1) read out
+          ptx::mbar_wait(p_full, gg & 1);
+          if (it == 0 && n >= 1) ptx::mbar_wait(acc_empty, (n - 1) & 1);  // previous item's dV/dK read out
+          ptx::tc_fence_after();
+          if (C::PT_TMEM) {
+            const uint32_t ads = ptx::smem_u32(sdS_buf[gg & 1]);
 #pragma unroll
-          for (int t = 0; t < 128 / 16; ++t)  // K = 128 keys: dQ = dS K
-            ptx::mma_bf16(T_DQ, ptx::sdesc_sw128(ads + t * 2048, 16384, 1024),
-                          ptx::sdesc_sw128(ak + t * 2048, 16384, 1024), ID_DQ, t > 0);
-        } else {
+            for (int t = 0; t < 128 / 16; ++t)  // dV += P^T dO, P^T from TMEM (8 columns per 16 queries)
+              ptx::mma_bf16_ts(T_DV, T_PT + 8 * t, ptx::sdesc_sw128(ado + t * 2048, 16384, 1024), ID_DV,
+                               (it > 0 || t > 0) ? 1u : 0u);
+            ptx::mma_commit(pt_free);
 #pragma unroll
-          for (int t = 0; t < 128 / 16; ++t) {  // K = 128 queries
-            const uint32_t offa = (t >> 2) * 16384 + (t & 3) * 32;
-            ptx::mma_bf16(T_DV, ptx::sdesc_sw128(apt + offa, 16, 1024), ptx::sdesc_sw128(ado + t * 2048, 16384, 1024),
-                          ID_DV, (it > 0 || t > 0) ? 1u : 0u);  // dV += P^T dO
-            ptx::mma_bf16(T_DV + DH, ptx::sdesc_sw128(adst + offa, 16, 1024),
-                          ptx::sdesc_sw128(aq + t * 2048, 16384, 1024), ID_DV, (it > 0 || t > 0) ? 1u : 0u);  // dK += dS^T Q
+            for (int t = 0; t < 128 / 16; ++t) {  // dK += dS^T Q
+              const uint32_t offa = (t >> 2) * 16384 + (t & 3) * 32;
+              ptx::mma_bf16(T_DV + DH, ptx::sdesc_sw128(ads + offa, 16, 1024), ptx::sdesc_sw128(aq + t * 2048, 16384, 1024),
+                            ID_DV, (it > 0 || t > 0) ? 1u : 0u);
+            }
+            if (gg >= 1) ptx::mbar_wait(dq_empty, (gg - 1) & 1);  // dQ(gg-1) read out
+#pragma unroll
+            for (int t = 0; t < 128 / 16; ++t)  // K = 128 keys: dQ = dS K
+              ptx::mma_bf16(T_DQ, ptx::sdesc_sw128(ads + t * 2048, 16384, 1024),
+                            ptx::sdesc_sw128(ak + t * 2048, 16384, 1024), ID_DQ, t > 0);
+          } else {
+#pragma unroll
+            for (int t = 0; t < 128 / 16; ++t) {  // K = 128 queries
+              const uint32_t offa = (t >> 2) * 16384 + (t & 3) * 32;
+              ptx::mma_bf16(T_DV, ptx::sdesc_sw128(apt + offa, 16, 1024), ptx::sdesc_sw128(ado + t * 2048, 16384, 1024),
+                            ID_DV, (it > 0 || t > 0) ? 1u : 0u);  // dV += P^T dO
+              ptx::mma_bf16(T_DV + DH, ptx::sdesc_sw128(adst + offa, 16, 1024),
+                            ptx::sdesc_sw128(aq + t * 2048, 16384, 1024), ID_DV, (it > 0 || t > 0) ? 1u : 0u);  // dK += dS^T Q
+            }
+            if (C::DQ_OWN && gg >= 1) ptx::mbar_wait(dq_empty, (gg - 1) & 1);  // dQ(gg-1) read out
+#pragma unroll
+            for (int t = 0; t < 128 / 16; ++t)  // K = 128 keys: dQ = dS K
+              ptx::mma_bf16(T_DQ, ptx::sdesc_sw128(adst + t * 2048, 16384, 1024),
+                            ptx::sdesc_sw128(ak + t * 2048, 16384, 1024), ID_DQ, t > 0);
           }
-          if (C::DQ_OWN && it >= 1) ptx::mbar_wait(dq_empty, (it - 1) & 1);  // dQ(it-1) read out
-#pragma unroll
-          for (int t = 0; t < 128 / 16; ++t)  // K = 128 keys: dQ = dS K
-            ptx::mma_bf16(T_DQ, ptx::sdesc_sw128(adst + t * 2048, 16384, 1024),
-                          ptx::sdesc_sw128(ak + t * 2048, 16384, 1024), ID_DQ, t > 0);
+          ptx::mma_commit(mm_done);
+          ptx::mma_commit(&q_empty[st]);
+          if (!C::DQ_OWN && it + 1 < nq) issue_st(gg + 1);
         }
-        ptx::mma_commit(mm_done);
-        ptx::mma_commit(&q_empty[st]);
-        if (!C::DQ_OWN && it + 1 < nq) issue_st(it + 1);
+        ptx::mma_commit(kv_empty);
+        g += nq;
+        ++n;
       }
     }
   } else {
@@ -589,7 +663,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
     const int r = q4 * 32 + lane;  // key row of this thread (TMEM lane)
     const uint32_t lane_base = (uint32_t)(q4 * 32) << 16;
     const uint32_t spt = ptx::smem_u32(sPT);
-    // dQ(it) (TMEM lane = query row) -> fp32 staging [DH/32 slabs][128 rows][128 B],
+    // dQ (TMEM lane = query row) -> fp32 staging [DH/32 slabs][128 rows][128 B],
     // 16-byte chunks XOR-swizzled by row (TMA SWIZZLE_128B, conflict-free
     // stores) -> one TMA reduce-add per 32-column slab into the dQ buffer
     // The reduce is not waited for here: the staging memory is next written
@@ -599,8 +673,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
       if (warp == 2 && lane == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
       named_bar(1, 256);
     };
-    auto dq_drain = [&](int itq, uint32_t stg) {
-      const int qiq = i0 + itq;
+    auto dq_drain = [&](int qiq, int hd, int b, uint32_t stg) {
       uint32_t v[DH / 64][32];
 #pragma unroll
       for (int cc = 0; cc < DH / 64; ++cc) {
@@ -634,114 +707,119 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
         asm volatile("cp.async.bulk.commit_group;" ::: "memory");
       }
     };
-    for (int it = 0; it < nq; ++it) {
-      const int st = it % QS;
-      const int qi = i0 + it;
-      const bool diag = (qi == kt);
-      ptx::mbar_wait(&q_full[st], (it / QS) & 1);  // lse / D of this query tile in smem
-      ptx::mbar_wait(s_full, it & 1);
-      ptx::tc_fence_after();
-      uint32_t vs[2][32], vd[2][32];
-      __syncwarp();
-      ptx::tmem_ld32(T_S + hf * 64 + lane_base, vs[0]);
-      ptx::tmem_ld32(T_S + hf * 64 + 32 + lane_base, vs[1]);
-      ptx::tmem_ld32(T_DP + hf * 64 + lane_base, vd[0]);
-      ptx::tmem_ld32(T_DP + hf * 64 + 32 + lane_base, vd[1]);
-      ptx::tmem_ld_wait();
-      ptx::tc_fence_before();
-      __syncwarp();
-      if (lane == 0) ptx::mbar_arrive(st_empty);  // S^T / dP^T TMEM may be overwritten
-      // P^T / dS^T smem must be free: dh 128 - the previous tile's dQ drain
-      // (staged there) completed; dh 64 - the previous tile's MMAs completed
-      if (C::PT_TMEM) {
-        // P^T (TMEM) free once the dV MMAs of the previous tile completed;
-        // dS^T buffer it&1 was last read by the MMAs of tile it-2, whose
-        // completion the dQ drain of tile it-2 already waited for
-        if (it >= 1) {
-          ptx::mbar_wait(pt_free, (it - 1) & 1);
+    int g = 0, n = 0;
+    for (int pass = 0; pass * ncta < n_items; ++pass) {
+      const int item = bwd_item_of(pass, ncta, cta);
+      if (item >= n_items) continue;
+      int kt, hd, b;
+      decode(item, kt, hd, b);
+      const int nq = n_t - kt;
+      for (int it = 0; it < nq; ++it) {
+        const int gg = g + it, st = gg % QS;
+        const int qi = kt + it;
+        const bool diag = (it == 0);
+        ptx::mbar_wait(&q_full[st], (gg / QS) & 1);  // lse / D of this query tile in smem
+        ptx::mbar_wait(s_full, gg & 1);
+        ptx::tc_fence_after();
+        uint32_t vs[2][32], vd[2][32];
+        __syncwarp();
+        ptx::tmem_ld32(T_S + hf * 64 + lane_base, vs[0]);
+        ptx::tmem_ld32(T_S + hf * 64 + 32 + lane_base, vs[1]);
+        ptx::tmem_ld32(T_DP + hf * 64 + lane_base, vd[0]);
+        ptx::tmem_ld32(T_DP + hf * 64 + 32 + lane_base, vd[1]);
+        ptx::tmem_ld_wait();
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(st_empty);  // S^T / dP^T TMEM may be overwritten
+        // P^T / dS^T smem must be free: dh 128 - the previous tile's dQ drain
+        // (staged there) completed; dh 64 - the previous tile's MMAs completed
+        if (C::PT_TMEM) {
+          // P^T (TMEM) free once the dV MMAs of the previous tile completed;
+          // dS^T buffer gg&1 was last read by the MMAs of tile gg-2, whose
+          // completion the dQ drain of tile gg-2 already waited for
+          if (gg >= 1) {
+            ptx::mbar_wait(pt_free, (gg - 1) & 1);
+            ptx::tc_fence_after();
+          }
+        } else if (C::DQ_OWN && gg >= 1) {
+          ptx::mbar_wait(mm_done, (gg - 1) & 1);
           ptx::tc_fence_after();
         }
-      } else if (C::DQ_OWN && it >= 1) {
-        ptx::mbar_wait(mm_done, (it - 1) & 1);
-        ptx::tc_fence_after();
-      }
-      if (!C::DQ_OWN && it >= 1) stage_free();  // dQ(it-1) staged in P^T / dS^T: reduce must have read it
-      const uint32_t sds = ptx::smem_u32(sdS_buf[C::PT_TMEM ? (it & 1) : 0]);
+        if (!C::DQ_OWN && gg >= 1) stage_free();  // dQ(gg-1) staged in P^T / dS^T: reduce must have read it
+        const uint32_t sds = ptx::smem_u32(sdS_buf[C::PT_TMEM ? (gg & 1) : 0]);
 #pragma unroll
-      for (int cc = 0; cc < 2; ++cc) {
-        const int c = hf * 2 + cc;
-        uint32_t ppk[16], dpk[16];
-        const uint32_t aL = ptx::smem_u32(sLD + st * 256 + c * 32), aD = aL + 512;
+        for (int cc = 0; cc < 2; ++cc) {
+          const int c = hf * 2 + cc;
+          uint32_t ppk[16], dpk[16];
+          const uint32_t aL = ptx::smem_u32(sLD + st * 256 + c * 32);
+          if (diag)
+            bwd_slab_math<true>(vs[cc], vd[cc], aL, c * 32, r, p.scale_log2, ppk, dpk);
+          else
+            bwd_slab_math<false>(vs[cc], vd[cc], aL, c * 32, r, p.scale_log2, ppk, dpk);
+          if (C::PT_TMEM) {  // P^T row r, queries c*32.. -> TMEM columns (2 bf16 per column)
+            ptx::tmem_st16(T_PT + c * 16 + lane_base, ppk);
 #pragma unroll
-        for (int e = 0; e < 32; e += 2) {
-          const int q = c * 32 + e;
-          const float2 L = lds_f32x2(aL + e * 4), Dd = lds_f32x2(aD + e * 4);  // broadcast reads
-          float p0 = ex2(fmaf(__uint_as_float(vs[cc][e]), p.scale_log2, -L.x));
-          float p1 = ex2(fmaf(__uint_as_float(vs[cc][e + 1]), p.scale_log2, -L.y));
-          if (diag) {  // key r attends only from queries >= r
-            if (q < r) p0 = 0.f;
-            if (q + 1 < r) p1 = 0.f;
+            for (int k = 0; k < 4; ++k)
+              st_shared_v4(sds + sw128_off(r, c * 4 + k), dpk[4 * k], dpk[4 * k + 1], dpk[4 * k + 2], dpk[4 * k + 3]);
+          } else {
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+              const uint32_t o = sw128_off(r, c * 4 + k);
+              st_shared_v4(spt + o, ppk[4 * k], ppk[4 * k + 1], ppk[4 * k + 2], ppk[4 * k + 3]);
+              st_shared_v4(sds + o, dpk[4 * k], dpk[4 * k + 1], dpk[4 * k + 2], dpk[4 * k + 3]);
+            }
           }
-          const float d0 = p0 * (__uint_as_float(vd[cc][e]) - Dd.x) * p.scale;
-          const float d1 = p1 * (__uint_as_float(vd[cc][e + 1]) - Dd.y) * p.scale;
-          ppk[e >> 1] = pack_bf16(p0, p1);
-          dpk[e >> 1] = pack_bf16(d0, d1);
         }
-        if (C::PT_TMEM) {  // P^T row r, queries c*32.. -> TMEM columns (2 bf16 per column)
-          ptx::tmem_st16(T_PT + c * 16 + lane_base, ppk);
-#pragma unroll
-          for (int k = 0; k < 4; ++k)
-            st_shared_v4(sds + sw128_off(r, c * 4 + k), dpk[4 * k], dpk[4 * k + 1], dpk[4 * k + 2], dpk[4 * k + 3]);
+        if (C::PT_TMEM) ptx::tmem_st_wait();
+        ptx::tc_fence_before();
+        ptx::fence_proxy_async();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(p_full);
+        if (C::DQ_OWN) {
+          // drain dQ of the previous query tile of this item while this tile's MMAs run
+          if (it >= 1) {
+            if (C::PT_TMEM) {
+              ptx::mbar_wait(mm_done, (gg - 1) & 1);
+              ptx::tc_fence_after();
+            }
+            dq_drain(qi - 1, hd, b, ptx::smem_u32(sSTG));
+          }
         } else {
-#pragma unroll
-          for (int k = 0; k < 4; ++k) {
-            const uint32_t o = sw128_off(r, c * 4 + k);
-            st_shared_v4(spt + o, ppk[4 * k], ppk[4 * k + 1], ppk[4 * k + 2], ppk[4 * k + 3]);
-            st_shared_v4(sds + o, dpk[4 * k], dpk[4 * k + 1], dpk[4 * k + 2], dpk[4 * k + 3]);
-          }
-        }
-      }
-      if (C::PT_TMEM) ptx::tmem_st_wait();
-      ptx::tc_fence_before();
-      ptx::fence_proxy_async();
-      __syncwarp();
-      if (lane == 0) ptx::mbar_arrive(p_full);
-      if (C::DQ_OWN) {
-        // drain dQ of the previous query tile while this tile's MMAs run
-        if (C::PT_TMEM && it >= 1) {
-          ptx::mbar_wait(mm_done, (it - 1) & 1);
+          ptx::mbar_wait(mm_done, gg & 1);
           ptx::tc_fence_after();
+          dq_drain(qi, hd, b, spt);  // staged in the (now free) P^T / dS^T tiles
         }
-        if (it >= 1) dq_drain(it - 1, ptx::smem_u32(sSTG));
-      } else {
-        ptx::mbar_wait(mm_done, it & 1);
-        ptx::tc_fence_after();
-        dq_drain(it, spt);  // staged in the (now free) P^T / dS^T tiles
       }
-    }
-    if (C::DQ_OWN) {
-      ptx::mbar_wait(mm_done, (nq - 1) & 1);
+      const int glast = g + nq - 1;
+      ptx::mbar_wait(mm_done, glast & 1);
       ptx::tc_fence_after();
-      dq_drain(nq - 1, ptx::smem_u32(sSTG));
+      if (C::DQ_OWN) dq_drain(kt + nq - 1, hd, b, ptx::smem_u32(sSTG));
+      // dV (half 0) / dK (half 1) of this key tile (rows = keys)
+      __nv_bfloat16* out = (hf == 0 ? p.dV : p.dK) + ((int64_t)b * p.s + kt * 128 + r) * p.ldd + hd * DH;
+#pragma unroll
+      for (int c = 0; c < DH / 32; ++c) {
+        uint32_t v[32];
+        __syncwarp();
+        ptx::tmem_ld32(T_DV + hf * DH + c * 32 + lane_base, v);
+        ptx::tmem_ld_wait();
+        if (c == DH / 32 - 1) {  // last TMEM read of this item's accumulators
+          ptx::tc_fence_before();
+          __syncwarp();
+          if (lane == 0) ptx::mbar_arrive(acc_empty);
+        }
+        uint32_t pk[16];
+        const float f = hf == 0 ? 1.f : p.scale;  // dK = scale * sum dS^T Q (dS^T was stored unscaled)
+#pragma unroll
+        for (int e = 0; e < 32; e += 2)
+          pk[e / 2] = pack_bf16x2(__fmul2_rn(make_float2(__uint_as_float(v[e]), __uint_as_float(v[e + 1])), make_float2(f, f)));
+#pragma unroll
+        for (int k = 0; k < 4; ++k)
+          *reinterpret_cast<uint4*>(out + c * 32 + k * 8) = make_uint4(pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
+      }
+      g += nq;
+      ++n;
     }
     if (warp == 2 && lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");  // last dQ reduce
-    // dV (half 0) / dK (half 1) of this key tile (rows = keys)
-    ptx::mbar_wait(mm_done, (nq - 1) & 1);
-    ptx::tc_fence_after();
-    __nv_bfloat16* out = (hf == 0 ? p.dV : p.dK) + ((int64_t)b * p.s + kt * 128 + r) * p.ldd + hd * DH;
-#pragma unroll
-    for (int c = 0; c < DH / 32; ++c) {
-      uint32_t v[32];
-      __syncwarp();
-      ptx::tmem_ld32(T_DV + hf * DH + c * 32 + lane_base, v);
-      ptx::tmem_ld_wait();
-      uint32_t pk[16];
-#pragma unroll
-      for (int e = 0; e < 32; e += 2) pk[e / 2] = pack_bf16(__uint_as_float(v[e]), __uint_as_float(v[e + 1]));
-#pragma unroll
-      for (int k = 0; k < 4; ++k)
-        *reinterpret_cast<uint4*>(out + c * 32 + k * 8) = make_uint4(pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
-    }
     ptx::tc_fence_before();
   }
   __syncthreads();
@@ -751,45 +829,55 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
   }
 }
 
-// D[b, h, q] = sum_d dO[q, d] * O[q, d]; 8 lanes per (row, head) for dh=64
-// (16 for dh=128), 16-byte loads
-__global__ void flash_dsum_kernel(const __nv_bfloat16* dO, const __nv_bfloat16* O, float* D, int rows, int nh, int dh,
-                                  int h, int s) {
-  const int lanes = dh / 8;
-  const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  const int64_t item = t / lanes;  // (row, head)
-  const int sub = (int)(t % lanes);
-  float acc = 0.f;
-  if (item < (int64_t)rows * nh) {
-    const int row = (int)(item / nh), hd = (int)(item % nh);
-    const int64_t off = (int64_t)row * h + hd * dh + sub * 8;
-    const uint4 a = *reinterpret_cast<const uint4*>(dO + off);
-    const uint4 o = *reinterpret_cast<const uint4*>(O + off);
-    const __nv_bfloat162* a2 = reinterpret_cast<const __nv_bfloat162*>(&a);
-    const __nv_bfloat162* o2 = reinterpret_cast<const __nv_bfloat162*>(&o);
+// Pre-pass of the flash backward, one warp per token row: negD[b, head, q] =
+// -sum_d dO[q, d] O[q, d] (stored negated so the softmax-gradient loop adds
+// it with FADD2), and the row's fp32 dQ accumulator zeroed (the kernel
+// reduce-adds into it).  16-byte loads; DH/8 lanes per head.
+template <int DH>
+__global__ void __launch_bounds__(256) flash_dsum_kernel(const __nv_bfloat16* __restrict__ dO,
+                                                         const __nv_bfloat16* __restrict__ O, float* __restrict__ negD,
+                                                         float* __restrict__ dQacc, int rows, int nh, int s) {
+  constexpr int LPH = DH / 8;  // lanes per head
+  const int lane = threadIdx.x % 32;
+  const int row = blockIdx.x * 8 + threadIdx.x / 32;
+  if (row >= rows) return;
+  const int h = nh * DH, nvec = h / 8;
+  const int b = row / s, q = row % s;
+  const __nv_bfloat16* dr = dO + (int64_t)row * h;
+  const __nv_bfloat16* orow = O + (int64_t)row * h;
+  float4* zr = reinterpret_cast<float4*>(dQacc + (int64_t)row * h);
+  for (int v0 = 0; v0 < nvec; v0 += 32) {  // nvec is a multiple of LPH; a head never straddles iterations
+    const int v = v0 + lane;
+    float acc = 0.f;
+    if (v < nvec) {
+      const uint4 a = *reinterpret_cast<const uint4*>(dr + v * 8);
+      const uint4 o = *reinterpret_cast<const uint4*>(orow + v * 8);
+      const __nv_bfloat162* a2 = reinterpret_cast<const __nv_bfloat162*>(&a);
+      const __nv_bfloat162* o2 = reinterpret_cast<const __nv_bfloat162*>(&o);
 #pragma unroll
-    for (int k = 0; k < 4; ++k) {
-      const float2 x = __bfloat1622float2(a2[k]), y = __bfloat1622float2(o2[k]);
-      acc += x.x * y.x + x.y * y.y;
+      for (int k = 0; k < 4; ++k) {
+        const float2 x = __bfloat1622float2(a2[k]), y = __bfloat1622float2(o2[k]);
+        acc += x.x * y.x + x.y * y.y;
+      }
+      zr[2 * v] = make_float4(0.f, 0.f, 0.f, 0.f);
+      zr[2 * v + 1] = make_float4(0.f, 0.f, 0.f, 0.f);
     }
-  }
-  for (int k = lanes / 2; k; k >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, k);
-  if (sub == 0 && item < (int64_t)rows * nh) {
-    const int row = (int)(item / nh), hd = (int)(item % nh);
-    const int b = row / s, q = row % s;
-    D[((int64_t)b * nh + hd) * s + q] = acc;
+#pragma unroll
+    for (int k = LPH / 2; k; k >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, k);
+    if (v < nvec && (v % LPH) == 0) negD[((int64_t)b * nh + v / LPH) * s + q] = -acc;
   }
 }
 
-// dqkv q-part (bf16, row stride 3h) = dQacc (fp32, row stride h)
-__global__ void flash_dq_cast_kernel(const float* dQacc, __nv_bfloat16* dq, int64_t rows, int h, int64_t ldd) {
+// dqkv q-part (bf16, row stride 3h) = scale * dQacc (fp32, row stride h)
+__global__ void flash_dq_cast_kernel(const float* dQacc, __nv_bfloat16* dq, int64_t rows, int h, int64_t ldd,
+                                     float scale) {
   const int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 4;
   if (i >= rows * h) return;
   const int64_t r = i / h, c = i % h;
   float4 v = *reinterpret_cast<const float4*>(dQacc + i);
   __nv_bfloat162* o = reinterpret_cast<__nv_bfloat162*>(dq + r * ldd + c);
-  o[0] = __floats2bfloat162_rn(v.x, v.y);
-  o[1] = __floats2bfloat162_rn(v.z, v.w);
+  o[0] = __floats2bfloat162_rn(v.x * scale, v.y * scale);
+  o[1] = __floats2bfloat162_rn(v.z * scale, v.w * scale);
 }
 
 typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
@@ -900,12 +988,11 @@ int flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* o, const __nv_
   if (rc) return rc;
   rc = dq_map(&tdq, dq_ws, h, dh, s, nh, mbs);
   if (rc) return rc;
-  {
-    const int64_t threads = rows * nh * (dh / 8);
-    flash_dsum_kernel<<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(dout, o, dsum_ws, (int)rows, nh, dh, h, s);
-  }
-  cudaError_t e = cudaMemsetAsync(dq_ws, 0, rows * h * sizeof(float), st);
-  if (e != cudaSuccess) MOBIUS_FAIL(MOBIUS_ECUDA, "flash dq memset");
+  if (dh == 64)
+    flash_dsum_kernel<64><<<(unsigned)((rows + 7) / 8), 256, 0, st>>>(dout, o, dsum_ws, dq_ws, (int)rows, nh, s);
+  else
+    flash_dsum_kernel<128><<<(unsigned)((rows + 7) / 8), 256, 0, st>>>(dout, o, dsum_ws, dq_ws, (int)rows, nh, s);
+  cudaError_t e;
   BwdParams p;
   p.lse = lse;
   p.Dsum = dsum_ws;
@@ -918,7 +1005,15 @@ int flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* o, const __nv_
   p.h = h;
   p.scale_log2 = 1.4426950408889634f / sqrtf((float)dh);
   p.scale = 1.0f / sqrtf((float)dh);
-  dim3 grid((s / 128) * nh * mbs);
+  p.mbs = mbs;
+  const int n_items = (s / 128) * nh * mbs;
+  int sms = 148;
+  {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  }
+  dim3 grid(n_items < sms ? n_items : sms);  // persistent
   if (dh == 64) {
     static bool once = false;
     if (!once) { rc = set_smem(flash_bwd_kernel<64>, BwdCfg<64>::SMEM); if (rc) return rc; once = true; }
@@ -930,7 +1025,7 @@ int flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* o, const __nv_
   }
   {
     const int64_t n = rows * h / 4;
-    flash_dq_cast_kernel<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(dq_ws, dqkv, rows, h, 3 * h);
+    flash_dq_cast_kernel<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(dq_ws, dqkv, rows, h, 3 * h, p.scale);
   }
   e = cudaGetLastError();
   if (e != cudaSuccess) MOBIUS_FAIL(MOBIUS_ECUDA, "flash_bwd launch: %s", cudaGetErrorString(e));

@@ -370,7 +370,11 @@ __global__ void __launch_bounds__(NUM_THREADS2, 1)
       while (sc.next(p, total, w)) {
         int mt, nt;
         tile_of(w.t, mt, nt);
-        const int m0 = mt * BM2 + (int)r2 * 128, n0 = nt * BN + (int)r2 * (BN / 2);
+        // a ragged last tile column of <= BN/2 columns runs as an N = BN/2
+        // MMA: each CTA then supplies BN/4 rows of B (the rest of its box is
+        // loaded but not read)
+        const int nhalf = (p.N - nt * BN <= BN / 2) ? BN / 4 : BN / 2;
+        const int m0 = mt * BM2 + (int)r2 * 128, n0 = nt * BN + (int)r2 * nhalf;
         for (int kb = w.k0; kb < w.k1; ++kb) {
           ptx::mbar_wait_cluster(&empty[stage], phase ^ 1);
           if (leader) ptx::mbar_arrive_expect_tx(&full[stage], 2 * C::STAGE_BYTES);
@@ -408,6 +412,7 @@ __global__ void __launch_bounds__(NUM_THREADS2, 1)
   } else if (warp == 1) {
     if (leader && lane == 0) {  // MMA issuer (pair leader)
       constexpr uint32_t IDESC = ptx::idesc_bf16(BM2, BN, A_MN ? 1 : 0, B_MN ? 1 : 0);
+      constexpr uint32_t IDESC_NARROW = ptx::idesc_bf16(BM2, BN / 2, A_MN ? 1 : 0, B_MN ? 1 : 0);
       const uint16_t all_mask = (uint16_t)((1u << (2 * NP)) - 1);
       const uint16_t pair_mask = (uint16_t)(3u << (2 * pair));
       int stage = 0;
@@ -417,6 +422,9 @@ __global__ void __launch_bounds__(NUM_THREADS2, 1)
       Sched sc(p, cl, ncl);
       Work w;
       while (sc.next(p, total, w)) {
+        int mt_, nt_;
+        tile_of(w.t, mt_, nt_);
+        const uint32_t idesc = (p.N - nt_ * BN <= BN / 2) ? IDESC_NARROW : IDESC;  // ragged last column
         ptx::mbar_wait_cluster(&tempty[acc], aphase ^ 1);
         ptx::tc_fence_after();
         const uint32_t tmem_d = tmem_base + acc * BN;
@@ -431,7 +439,7 @@ __global__ void __launch_bounds__(NUM_THREADS2, 1)
                                : ptx::sdesc_sw128(a_base + k * 32, 16, 1024);
             uint64_t bd = B_MN ? ptx::sdesc_sw128(b_base + k * 2048, 8192, 1024)
                                : ptx::sdesc_sw128(b_base + k * 32, 16, 1024);
-            ptx::mma_bf16_2sm(tmem_d, ad, bd, IDESC, (kb > w.k0 || k > 0) ? 1u : 0u);
+            ptx::mma_bf16_2sm(tmem_d, ad, bd, idesc, (kb > w.k0 || k > 0) ? 1u : 0u);
           }
           // the slot may be refilled by this pair's producers and (A halves)
           // by the other pair's: free it in every CTA of the cluster

@@ -54,8 +54,10 @@ def randn(*shape, scale=1.0):
 
 # ------------------------------------------------------------------ GEMM
 # all dims multiples of 8 (TMA: 16-byte row strides), none a multiple of every tile size
+# (512, 1600, 320) / (520, 384, 136): 2-CTA tiles whose ragged last column
+# (64 / 128 wide) runs as an N = 128 MMA; (640, 392, 256): a 136-wide one (full width)
 GEMM_SHAPES = [(256, 256, 256), (200, 320, 192), (136, 64, 64), (384, 96, 1000), (128, 512, 128),
-               (344, 264, 136), (1024, 1024, 512)]
+               (344, 264, 136), (1024, 1024, 512), (512, 1600, 320), (520, 384, 136), (640, 392, 256)]
 
 
 @pytest.mark.parametrize("dtype", [BF16, F32])
@@ -168,6 +170,33 @@ def test_gemm_epilogues(dtype):
     kt.gemm(dtype, M, N, K, tA, K, False, tB, N, True, tC, N, c_f32=True, epi=5, accumulate=True)
     torch.cuda.synchronize()
     assert rel(from_dev(tC), C0 + acc) < (1e-4 if dtype == BF16 else 1e-5)
+
+
+@pytest.mark.parametrize("shape", [(300, 520, 200), (200, 192, 64), (2000, 1000, 4104)])
+def test_gemm_gelu_bwd_aux(shape):
+    """EPI_GELU_BWD with AUX (compact kept activations): C = acc * gelu'(u)
+    and AUX = gelu(u), where gelu(u) must be bit-identical to what the
+    forward epilogue (EPI_BIAS_GELU) stored for the same bf16 u.  Shapes:
+    2-CTA TMA epilogue, 1-CTA epilogue, 2-CTA Stream-K fixup."""
+    M, N, K = shape
+    g = torch.Generator(device=DEV).manual_seed(11)
+    A = (torch.randn(M, K, device=DEV, generator=g) * 0.5).to(torch.bfloat16)
+    B = (torch.randn(K, N, device=DEV, generator=g) * 0.1).to(torch.bfloat16)
+    bias = (torch.randn(N, device=DEV, generator=g) * 0.5).to(torch.bfloat16)
+    # forward: u = A B + bias (AUX), g = gelu(u) (C)
+    u = torch.zeros(M, N, device=DEV, dtype=torch.bfloat16)
+    g_fwd = torch.zeros(M, N, device=DEV, dtype=torch.bfloat16)
+    kt.gemm(BF16, M, N, K, A, K, False, B, N, True, g_fwd, N, epi=2, bias=bias, AUX=u, ldx=N)
+    # backward: dU = dY W^T * gelu'(u), g recomputed from u into AUX
+    dY = (torch.randn(M, K, device=DEV, generator=g)).to(torch.bfloat16)
+    W = (torch.randn(N, K, device=DEV, generator=g) * 0.1).to(torch.bfloat16)
+    du = torch.zeros(M, N, device=DEV, dtype=torch.bfloat16)
+    g_bwd = torch.zeros(M, N, device=DEV, dtype=torch.bfloat16)
+    kt.gemm(BF16, M, N, K, dY, K, False, W, K, False, du, N, epi=4, R=u, ldr=N, AUX=g_bwd, ldx=N)
+    torch.cuda.synchronize()
+    assert torch.equal(g_bwd, g_fwd)
+    ref = (dY.double() @ W.double().T).cpu().numpy() * om.gelu_grad(u.double().cpu().numpy())
+    assert rel(from_dev(du), ref) < 1e-2
 
 
 @pytest.mark.parametrize("dtype", [BF16, F32])
