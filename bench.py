@@ -47,12 +47,16 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="1.5b")
     ap.add_argument("--layers", type=int, default=0, help="override the block count (shape checks only)")
-    ap.add_argument("--microbatches", type=int, default=0, help="M per GPU (default 16 for 1.5b)")
+    ap.add_argument("--microbatches", type=int, default=0, help="M per GPU (default 8 for 1.5b)")
     ap.add_argument("--cap-gib", type=float, default=1.0, help="HBM stage-ring cap G per GPU")
+    ap.add_argument("--micro-batch", type=int, default=0,
+                    help="micro-batch size mbs (default 16 for 1.5b: 8 x 16 x 1024 = 131072 tokens per GPU-step)")
     ap.add_argument("--impl", default="mobius", choices=["mobius", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-keep", action="store_true", help="always recompute (no kept activations)")
+    ap.add_argument("--host-tail-update", action="store_true",
+                    help="update the last-in-backward stage on the host too (default: GPU AdamW for it)")
     ap.add_argument("--partition", default="mip", choices=["mip", "max", "min"],
                     help="MIP (paper) or the Fig 9 max-stage / min-stage baselines")
     return ap.parse_args()
@@ -158,11 +162,23 @@ def cpu_oracle_sample(c: synth.GPTConfig, tokens_per_step: int, budget_s: float 
                       f"(host AdamW and transfers not included)"}
 
 
+def bench_workload(args, world):
+    """(config, M): the bench's GPT config (mbs overridable) and microbatch
+    count.  1.5b default: M = 8 per GPU of mbs 16 (131072 tokens per GPU per
+    step; measured 83k vs 79.5k tokens/s for 16 x mbs 8 - larger GEMMs
+    quantise better over the 74 SM pairs)."""
+    import dataclasses
+    c = synth.CONFIGS[args.config]
+    mbs = args.micro_batch or (16 if args.config == "1.5b" else c.micro_batch)
+    c = dataclasses.replace(c, n_layers=args.layers or c.n_layers, micro_batch=mbs)
+    M = (args.microbatches or (8 if args.config == "1.5b" else 16)) * world
+    return c, M
+
+
 def run_reference(args, rank, world):
     if rank != 0:
         return
-    c = synth.CONFIGS[args.config]
-    M = (args.microbatches or 16) * args.gpus
+    c, M = bench_workload(args, args.gpus)
     tps = M * c.micro_batch * c.seq_len
     vals = []
     for _ in range(args.warmup):
@@ -203,9 +219,9 @@ def measure_h2d_GBps(torch, nbytes=512 << 20):
 def run_mobius(args, rank, world, local):
     import torch
     import torch.distributed as dist
-    from paper_conf_asplos_fengxtwls23_b200 import (BF16, FLAG_KEEP_ACTS, FLAG_TIMING, MobiusContext, make_topology,
-                                                    mobius_discover_topology, mobius_plan, mobius_profile,
-                                                    model_cfg)
+    from paper_conf_asplos_fengxtwls23_b200 import (BF16, FLAG_DEVICE_TAIL_UPDATE, FLAG_KEEP_ACTS, FLAG_TIMING,
+                                                    MobiusContext, make_topology, mobius_discover_topology,
+                                                    mobius_plan, mobius_profile, model_cfg)
     # MOBIUS_BENCH_SAME_GPU=1: every rank on device 0 (checks the N>1 code
     # path on a 1-GPU box; ranks time-slice the GPU, numbers are not scaling
     # numbers).  Plumbing then uses gloo (NCCL rejects duplicate GPUs).
@@ -219,11 +235,7 @@ def run_mobius(args, rank, world, local):
         else:
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     pg_dev = "cpu" if same_gpu else "cuda"
-    c = synth.CONFIGS[args.config]
-    if args.layers:
-        import dataclasses
-        c = dataclasses.replace(c, n_layers=args.layers)
-    M = (args.microbatches or 16) * world
+    c, M = bench_workload(args, world)
     cfg = model_cfg(c.n_layers, c.hidden, c.n_heads, c.seq_len, c.vocab, c.micro_batch, dtype=BF16)
     G = int(args.cap_gib * GiB)
     # profile (layer similarity) and plan (MIP + cross mapping)
@@ -259,7 +271,8 @@ def run_mobius(args, rank, world, local):
         from paper_conf_asplos_fengxtwls23_b200 import dist as mdist
         assert mdist.check_same_plan(plan), "ranks derived different plans"
     timing = os.environ.get("MOBIUS_BENCH_TIMING", "1") != "0"  # per-kernel CUDA events (roofline)
-    flags = (FLAG_TIMING if timing else 0) | (0 if args.no_keep else FLAG_KEEP_ACTS)
+    flags = (FLAG_TIMING if timing else 0) | (0 if args.no_keep else FLAG_KEEP_ACTS) | \
+        (0 if args.host_tail_update else FLAG_DEVICE_TAIL_UPDATE)
     ctx = MobiusContext(cfg, plan, rank=rank, world=world, device=local, seed=1234, flags=flags)
     if world > 1:
         blobs = [None] * world
@@ -357,6 +370,8 @@ def run_mobius(args, rank, world, local):
                        "gpu_perm": [plan.gpu_perm[g] for g in range(world)], "plan_s": plan_s,
                        "profile_s": prof_s, "plan_exhaustive": bool(plan.exhaustive),
                        "partition": args.partition, "plan_makespan_ms": plan.makespan_ns / 1e6,
+                       "tail_stage_update": "host AdamW" if args.host_tail_update else
+                       "GPU AdamW (first stage, last in backward; optimizer state in HBM)",
                        "l2": "inputs larger than L2: every stage (3.1 GB bf16 total) streams from host DRAM each step"},
             "loss": loss,
             "e2e": e2e,

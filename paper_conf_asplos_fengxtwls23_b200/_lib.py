@@ -69,6 +69,7 @@ class StepStats(C.Structure):
 
 FLAG_TIMING = 1
 FLAG_KEEP_ACTS = 2
+FLAG_DEVICE_TAIL_UPDATE = 4
 
 P = C.c_void_p
 I = C.c_int

@@ -9,11 +9,11 @@ from typing import Optional, Sequence
 import numpy as np
 
 from . import _lib as L
-from ._lib import BF16, F32, FLAG_KEEP_ACTS, FLAG_TIMING, MobiusError, check, lib  # noqa: F401
+from ._lib import BF16, F32, FLAG_DEVICE_TAIL_UPDATE, FLAG_KEEP_ACTS, FLAG_TIMING, MobiusError, check, lib  # noqa: F401
 
 __all__ = ["mobius_plan", "mobius_plan_partition", "PARTITION_MIP", "PARTITION_MAX_STAGE", "PARTITION_MIN_STAGE", "mobius_plan_cost", "mobius_cross_map", "mobius_mapping_contention",
            "mobius_discover_topology", "mobius_layer_sizes", "mobius_profile", "MobiusContext", "model_cfg",
-           "make_topology", "plan_from_sizes", "kt", "BF16", "F32", "FLAG_TIMING", "FLAG_KEEP_ACTS", "MobiusError",
+           "make_topology", "plan_from_sizes", "kt", "BF16", "F32", "FLAG_TIMING", "FLAG_KEEP_ACTS", "FLAG_DEVICE_TAIL_UPDATE", "MobiusError",
            "build_info"]
 
 

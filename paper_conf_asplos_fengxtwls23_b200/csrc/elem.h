@@ -54,6 +54,12 @@ int gelu_fwd_bf16(const __nv_bfloat16* u, __nv_bfloat16* g, int64_t n, cudaStrea
 // dst = (T) src
 template <typename T>
 int cast_from_f32(const float* src, T* dst, int64_t n, cudaStream_t st);
+// AdamW on device-resident fp32 master/m/v (the host update's formula,
+// host.cpp adamw_chunk): g is the stage gradient in transfer precision T,
+// w_out the new weights in T.  bc1 = 1 - b1^t, bc2 = 1 - b2^t.
+template <typename T>
+int adamw_device(float* w, float* m, float* v, const T* g, T* w_out, int64_t n, float lr, float b1, float b2,
+                 float eps, float wd, float bc1, float bc2, cudaStream_t st);
 
 // device-side flag wait / set (inter-rank arrival flags, release/acquire at system scope)
 int flag_wait(const volatile int* flag, int value, cudaStream_t st);

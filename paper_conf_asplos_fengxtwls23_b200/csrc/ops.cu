@@ -429,7 +429,7 @@ int block_bwd(const Shape& sh, const T* w, const BlockActs<T>& A_in, const T* dy
   }
   T* dx1 = sc.t2;
   {
-    ElemScope es(st, 1);
+    ElemScope es(st, 2);
     RC(layernorm_bwd<T>(sc.t1, A.x1, w + L.ln2_g, A.mu2, A.rs2, dy, dx1, G + L.ln2_g, G + L.ln2_b, Tn, h, st));
   }
   {  // dWo += o^T dx1
@@ -478,7 +478,7 @@ int block_bwd(const Shape& sh, const T* w, const BlockActs<T>& A_in, const T* dy
     RC(run_gemm<T>(d, st, KCLS_GEMM));
   }
   {
-    ElemScope es(st, 1);
+    ElemScope es(st, 2);
     RC(layernorm_bwd<T>(sc.t1, A.x, w + L.ln1_g, A.mu1, A.rs1, dx1, dx, G + L.ln1_g, G + L.ln1_b, Tn, h, st));
   }
   return MOBIUS_OK;
@@ -538,7 +538,7 @@ int head_layer_fwd_bwd(const Shape& sh, const T* w, const T* x, const int32_t* t
     RC(run_gemm<T>(d, st, KCLS_GEMM));
   }
   {
-    ElemScope es(st, 1);
+    ElemScope es(st, 2);
     RC(layernorm_bwd<T>(sc.t2, x, w + L.lnf_g, sc.mu, sc.rs, (const T*)nullptr, dx, G + L.lnf_g, G + L.lnf_b, Tn,
                         h, st));
   }

@@ -192,6 +192,11 @@ struct mobius_ctx {
   uint8_t* tok_dev = nullptr;
   double* loss_dev = nullptr;
   int64_t off_ckpt = 0, off_gslot = 0, off_fflag = 0, off_bflag = 0;
+  // MOBIUS_FLAG_DEVICE_TAIL_UPDATE: optimizer state of local stage 0 in HBM
+  bool dev_tail = false;
+  float* d_opt = nullptr;         // master | m | v, each al256(np0 * 4) bytes
+  int64_t d_opt_stride = 0;       // floats between the three
+  uint8_t* d_wstage = nullptr;    // new stage-0 weights (transfer precision) for the D2H
 
   // peers
   std::vector<uint8_t*> peer_base;  // opened IPC bases (nullptr for me)
@@ -595,12 +600,24 @@ struct StepRunner {
     if (ls + 1 < (int)ctx->mine.size()) CU(cudaStreamWaitEvent(s, ctx->ev_d2h[ls + 1], 0));
     RC(cast_from_f32<T>(ctx->grad_acc, tptr<T>(ctx->grad_stage), st.n_params, s));
     ++ctx->launches_step;
+    const bool dev_upd = ctx->dev_tail && ls == 0;
+    if (dev_upd) {  // AdamW on the GPU; the new weights go to the pinned store instead of the gradient
+      const AdamWArgs a{ctx->cfg.lr, ctx->cfg.beta1, ctx->cfg.beta2, ctx->cfg.eps, ctx->cfg.weight_decay,
+                        ctx->step_count + 1};
+      const float bc1 = (float)(1.0 - std::pow((double)a.beta1, (double)a.step));
+      const float bc2 = (float)(1.0 - std::pow((double)a.beta2, (double)a.step));
+      float* w = ctx->d_opt;
+      RC(adamw_device<T>(w, w + ctx->d_opt_stride, w + 2 * ctx->d_opt_stride, tptr<T>(ctx->grad_stage),
+                         tptr<T>(ctx->d_wstage), st.n_params, a.lr, a.beta1, a.beta2, a.eps, a.wd, bc1, bc2, s));
+      ++ctx->launches_step;
+    }
     CU(cudaEventRecord(ctx->ev_gready[ls], s));
     CU(cudaStreamWaitEvent(ctx->s_d2h, ctx->ev_gready[ls], 0));
-    CU(cudaMemcpyAsync(ctx->h_grads[ls], ctx->grad_stage, st.n_params * sizeof(T), cudaMemcpyDeviceToHost,
-                       ctx->s_d2h));
+    CU(cudaMemcpyAsync(dev_upd ? ctx->h_weights[ls] : ctx->h_grads[ls], dev_upd ? ctx->d_wstage : ctx->grad_stage,
+                       st.n_params * sizeof(T), cudaMemcpyDeviceToHost, ctx->s_d2h));
     CU(cudaEventRecord(ctx->ev_d2h[ls], ctx->s_d2h));
     ctx->stats.d2h_bytes += st.n_params * sizeof(T);
+    if (dev_upd) return MOBIUS_OK;
     {
       std::lock_guard<std::mutex> g(ctx->upd_mu);
       ctx->upd_queue.push_back(ls);
@@ -888,6 +905,13 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
     CU(cudaMalloc(&ctx->arena, ctx->arena_bytes));
     CU(cudaMemset(ctx->arena + o_gacc, 0, max_params * 4));
     ctx->ring = ctx->arena;
+    ctx->dev_tail = (dist->flags & MOBIUS_FLAG_DEVICE_TAIL_UPDATE) && n > 0;
+    if (ctx->dev_tail) {  // before the keep pool takes the free HBM
+      const int64_t np0 = ctx->all[ctx->mine[0]].n_params;
+      ctx->d_opt_stride = al256(np0 * 4) / 4;
+      CU(cudaMalloc(&ctx->d_opt, ctx->d_opt_stride * 4 * 3));
+      CU(cudaMalloc(&ctx->d_wstage, al256(np0 * esz)));
+    }
     // kept activations (reading #17: keep instead of recompute when they fit):
     // whole local stages, latest first, within the free HBM minus a margin
     ctx->keep_off.assign(n, -1);
@@ -993,6 +1017,11 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
           std::memcpy((float*)ctx->h_weights[k] + b, mst + b, (e - b) * 4);
         }
       });
+    }
+    if (ctx->dev_tail) {  // stage 0's optimizer state moves to HBM (m = v = 0)
+      const int64_t np0 = ctx->all[ctx->mine[0]].n_params;
+      CU(cudaMemcpy(ctx->d_opt, ctx->h_master[0], np0 * 4, cudaMemcpyHostToDevice));
+      CU(cudaMemset(ctx->d_opt + ctx->d_opt_stride, 0, ctx->d_opt_stride * 4 * 2));
     }
     CU(cudaHostAlloc(&ctx->h_loss, sizeof(double), cudaHostAllocDefault));
     ctx->h_tokens_cap = (int64_t)M * sh.mbs * (sh.s + 1);
@@ -1136,11 +1165,19 @@ extern "C" int mobius_read_grads(mobius_ctx* ctx, float* out, size_t n) {
   for (int ls = 0; ls < (int)ctx->mine.size(); ++ls) {
     const StageDesc& st = ctx->all[ctx->mine[ls]];
     MOBIUS_CHECK_ARG((size_t)(st.param_off + st.n_params) <= n, "output too small");
+    const void* src = ctx->h_grads[ls];
+    std::vector<uint8_t> tmp;
+    if (ctx->dev_tail && ls == 0) {  // never offloaded: the staging buffer still holds it (last stage in backward)
+      tmp.resize(st.n_params * ctx->esz);
+      if (cudaMemcpy(tmp.data(), ctx->grad_stage, tmp.size(), cudaMemcpyDeviceToHost) != cudaSuccess)
+        MOBIUS_FAIL(MOBIUS_ECUDA, "read_grads: device copy");
+      src = tmp.data();
+    }
     if (ctx->esz == 2) {
-      const uint16_t* g = (const uint16_t*)ctx->h_grads[ls];
+      const uint16_t* g = (const uint16_t*)src;
       for (int64_t i = 0; i < st.n_params; ++i) out[st.param_off + i] = bf16_to_f32(g[i]);
     } else {
-      std::memcpy(out + st.param_off, ctx->h_grads[ls], st.n_params * 4);
+      std::memcpy(out + st.param_off, src, st.n_params * 4);
     }
   }
   return MOBIUS_OK;
@@ -1153,7 +1190,12 @@ extern "C" int mobius_read_params(mobius_ctx* ctx, float* out, size_t n) {
   for (int ls = 0; ls < (int)ctx->mine.size(); ++ls) {
     const StageDesc& st = ctx->all[ctx->mine[ls]];
     MOBIUS_CHECK_ARG((size_t)(st.param_off + st.n_params) <= n, "output too small");
-    std::memcpy(out + st.param_off, ctx->h_master[ls], st.n_params * 4);
+    if (ctx->dev_tail && ls == 0) {
+      if (cudaMemcpy(out + st.param_off, ctx->d_opt, st.n_params * 4, cudaMemcpyDeviceToHost) != cudaSuccess)
+        MOBIUS_FAIL(MOBIUS_ECUDA, "read_params: device copy");
+    } else {
+      std::memcpy(out + st.param_off, ctx->h_master[ls], st.n_params * 4);
+    }
   }
   return MOBIUS_OK;
 }
@@ -1200,6 +1242,8 @@ extern "C" void mobius_destroy(mobius_ctx* ctx) {
   if (ctx->h_tokens) cudaFreeHost(ctx->h_tokens);
   if (ctx->arena) cudaFree(ctx->arena);
   if (ctx->keep_pool) cudaFree(ctx->keep_pool);
+  if (ctx->d_opt) cudaFree(ctx->d_opt);
+  if (ctx->d_wstage) cudaFree(ctx->d_wstage);
   if (ctx->s_comp) cudaStreamDestroy(ctx->s_comp);
   if (ctx->s_h2d) cudaStreamDestroy(ctx->s_h2d);
   if (ctx->s_d2h) cudaStreamDestroy(ctx->s_d2h);

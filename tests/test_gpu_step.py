@@ -21,8 +21,8 @@ from oracle import adamw as oa  # noqa: E402
 from oracle import model as om  # noqa: E402
 from oracle import planner as op  # noqa: E402
 from oracle import schedule as osch  # noqa: E402
-from paper_conf_asplos_fengxtwls23_b200 import (BF16, F32, MobiusContext, mobius_layer_sizes,  # noqa: E402
-                                                model_cfg, plan_from_sizes)
+from paper_conf_asplos_fengxtwls23_b200 import (BF16, F32, FLAG_DEVICE_TAIL_UPDATE, MobiusContext,  # noqa: E402
+                                                mobius_layer_sizes, model_cfg, plan_from_sizes)
 
 MiB = 1 << 20
 
@@ -95,6 +95,45 @@ def test_tiny_step_parity(dtype, tol, cap, sizes):
     w1, _, _ = oa.adamw_step(w, np.zeros_like(w), np.zeros_like(w), g, 1)
     assert rel(p1 - w, w1 - w) < 1e-5
     assert np.max(np.abs(p1 - w1)) < 1e-6
+
+
+@pytest.mark.parametrize("dtype", [BF16, F32])
+@pytest.mark.parametrize("sizes", [(3, 3), (1, 2, 1, 2)])
+def test_device_tail_update(dtype, sizes):
+    """MOBIUS_FLAG_DEVICE_TAIL_UPDATE: the first stage (last in backward)
+    is updated by the GPU AdamW on HBM-resident optimizer state; the result
+    must be the oracle's AdamW on the offloaded-precision gradient (as the
+    host update is), byte counters unchanged, and a 3-step run must track
+    the host-update run."""
+    c = synth.TINY
+    M = 2
+    w = synth.perturb_norm_params(c, synth.gen_params(c), scale=0.1)
+    if dtype == BF16:
+        w = synth.round_bf16(w)
+    cap = 4 * MiB if dtype == BF16 else 8 * MiB
+    toks = [synth.gen_tokens(c, M, seed=20 + i) for i in range(3)]
+    plan = plan_from_sizes(sizes, 1, M, hbm_cap_bytes=cap)
+    runs = {}
+    for flags in (0, FLAG_DEVICE_TAIL_UPDATE):
+        ctx = MobiusContext(mk_cfg(c, dtype), plan, init_params=w, flags=flags)
+        losses = [ctx.step(toks[0])]
+        g = ctx.read_grads(c.n_params)
+        p1 = ctx.read_params(c.n_params)
+        st = ctx.stats()
+        losses += [ctx.step(t) for t in toks[1:]]
+        p3 = ctx.read_params(c.n_params)
+        ctx.close()
+        runs[flags] = (losses, g, p1, p3, st)
+    (lh, gh, p1h, p3h, sth), (ld, gd, p1d, p3d, std) = runs[0], runs[FLAG_DEVICE_TAIL_UPDATE]
+    # same first step up to the update (bias-gradient column sums use fp32
+    # atomics, so equal to rounding, not bitwise)
+    assert rel(gd, gh) < 1e-6 and abs(ld[0] - lh[0]) <= 1e-6 * abs(lh[0])
+    assert (std.h2d_bytes, std.d2h_bytes) == (sth.h2d_bytes, sth.d2h_bytes)
+    w1, _, _ = oa.adamw_step(w, np.zeros_like(w), np.zeros_like(w), gd, 1)
+    assert np.max(np.abs(p1d - w1)) < 1e-6
+    assert rel(p1d - w, p1h - w) < 1e-3
+    assert max(abs(a - b) / abs(b) for a, b in zip(ld, lh)) < 1e-3
+    assert rel(p3d - w, p3h - w) < 1e-2
 
 
 def test_tiny_two_steps_bf16():
