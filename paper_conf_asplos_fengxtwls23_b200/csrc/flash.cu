@@ -127,6 +127,13 @@ struct FwdParams {
   float scale_log2;  // log2(e) / sqrt(dh)
 };
 
+// Persistent item order: pass k visits CTAs left-to-right for even k and
+// right-to-left for odd k over a list sorted heaviest first, so per-CTA
+// work balances (static round robin leaves the first CTAs ~9% heavier)
+__device__ __forceinline__ int snake_item(int pass, int ncta, int cta) {
+  return pass * ncta + ((pass & 1) ? ncta - 1 - cta : cta);
+}
+
 __device__ __forceinline__ void fwd_item(const FwdParams& p, int i, int& qt, int& hd, int& b) {
   const int n_qt = p.s / BQ, nb = p.nh * p.mbs;
   qt = n_qt - 1 - i / nb;  // heaviest (most kv tiles) first
@@ -199,7 +206,9 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
   if (warp == 0) {
     if (lane == 0) {
       int g = 0, it = 0;
-      for (int i = blockIdx.x; i < n_items; i += gridDim.x, ++it) {
+      for (int pass = 0; pass * (int)gridDim.x < n_items; ++pass) {
+        const int i = snake_item(pass, (int)gridDim.x, (int)blockIdx.x);
+        if (i >= n_items) continue;
         int qt, hd, b;
         fwd_item(p, i, qt, hd, b);
         const int qb = it & 1;
@@ -221,6 +230,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
           for (int c = 0; c < DH / 64; ++c)
             ptx::tma_load_4d(sV + st * C::KV_BYTES + c * 16384, &tm, &v_full[st], 64 * c, j * BKV, 2 * p.nh + hd, b);
         }
+        ++it;
       }
     }
   } else if (warp == 1) {
@@ -228,7 +238,9 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
       constexpr uint32_t ID_S = ptx::idesc_bf16(BQ, BKV, 0, 0);
       constexpr uint32_t ID_O = ptx::idesc_bf16(BQ, DH, 0, 1);
       int gs = 0, gp = 0, it = 0;  // global S-issue step, global PV step, local item count
-      for (int i = blockIdx.x; i < n_items; i += gridDim.x, ++it) {
+      for (int pass = 0; pass * (int)gridDim.x < n_items; ++pass) {
+        const int i = snake_item(pass, (int)gridDim.x, (int)blockIdx.x);
+        if (i >= n_items) continue;
         int qt, hd, b;
         fwd_item(p, i, qt, hd, b);
         const int nkv = qt + 1, ob = it & 1;
@@ -271,6 +283,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
           ++gp;
         }
         ptx::mma_commit(&o_ready[ob]);
+        ++it;
       }
     }
   } else {
@@ -281,7 +294,9 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
     const uint32_t lb = (uint32_t)(q4 * 32) << 16;
     const float sc = p.scale_log2;
     int g = 0, it = 0;
-    for (int i = blockIdx.x; i < n_items; i += gridDim.x, ++it) {
+    for (int pass = 0; pass * (int)gridDim.x < n_items; ++pass) {
+      const int i = snake_item(pass, (int)gridDim.x, (int)blockIdx.x);
+      if (i >= n_items) continue;
       int qt, hd, b;
       fwd_item(p, i, qt, hd, b);
       const int nkv = qt + 1, ob = it & 1;
@@ -401,6 +416,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(&o_empty[ob]);
       named_bar(2 + q4, 64);  // partner read sSum before the next item overwrites it
+      ++it;
     }
   }
   __syncthreads();
@@ -453,9 +469,6 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
 // MMA order per query tile: [S^T, dP^T](i) ... wait P^T/dS^T(i) ... dV, dK,
 // dQ(i), then [S^T, dP^T](i+1) right away (the softmax-gradient warps are
 // done with S^T(i)), so the next scores overlap the dQ read-out.
-__device__ __forceinline__ int bwd_item_of(int pass, int ncta, int cta) {
-  return pass * ncta + ((pass & 1) ? ncta - 1 - cta : cta);
-}
 
 template <int DH>
 __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_constant__ CUtensorMap tm,
@@ -536,7 +549,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
     if (lane == 0) {
       int g = 0, n = 0;  // global tile / item counters of this CTA
       for (int pass = 0; pass * ncta < n_items; ++pass) {
-        const int item = bwd_item_of(pass, ncta, cta);
+        const int item = snake_item(pass, ncta, cta);
         if (item >= n_items) continue;
         int kt, hd, b;
         decode(item, kt, hd, b);
@@ -595,7 +608,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
       };
       int g = 0, n = 0;
       for (int pass = 0; pass * ncta < n_items; ++pass) {
-        const int item = bwd_item_of(pass, ncta, cta);
+        const int item = snake_item(pass, ncta, cta);
         if (item >= n_items) continue;
         const int nq = n_t - item / nbh;
         ptx::mbar_wait(kv_full, n & 1);
@@ -605,9 +618,17 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
         for (int it = 0; it < nq; ++it) {
           const int gg = g + it, st = gg % QS;
           const uint32_t aq = ptx::smem_u32(sQ + st * C::T_BYTES), ado = ptx::smem_u32(sdO + st * C::T_BYTES);
-          if (C::DQ_OWN && it + 1 < nq) {  // scores of the next query tile overlap this tile's softmax-gradient
+          // scores of the next query tile overlap this tile's softmax-gradient -
+          // if its Q / dO tile has landed; otherwise this tile's dV/dK/dQ go first
+          // (blocking on the load here would stall the whole chain)
+          bool st_next = false;
+          if (C::DQ_OWN && it + 1 < nq) {
             ptx::mbar_wait(st_empty, gg & 1);
-            issue_st(gg + 1);
+            const int sn = (gg + 1) % QS;
+            if (ptx::mbar_test(&q_full[sn], ((gg + 1) / QS) & 1)) {
+              issue_st(gg + 1);
+              st_next = true;
+            }
           }
           ptx::mbar_wait(p_full, gg & 1);
           if (it == 0 && n >= 1) ptx::mbar_wait(acc_empty, (n - 1) & 1);  // previous item's dV/dK read out
@@ -625,6 +646,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
               ptx::mma_bf16(T_DV + DH, ptx::sdesc_sw128(ads + offa, 16, 1024), ptx::sdesc_sw128(aq + t * 2048, 16384, 1024),
                             ID_DV, (it > 0 || t > 0) ? 1u : 0u);
             }
+            ptx::mma_commit(&q_empty[st]);  // last reads of Q / dO (dQ needs only dS and K): refill the slot now
             if (gg >= 1) ptx::mbar_wait(dq_empty, (gg - 1) & 1);  // dQ(gg-1) read out
 #pragma unroll
             for (int t = 0; t < 128 / 16; ++t)  // K = 128 keys: dQ = dS K
@@ -639,6 +661,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
               ptx::mma_bf16(T_DV + DH, ptx::sdesc_sw128(adst + offa, 16, 1024),
                             ptx::sdesc_sw128(aq + t * 2048, 16384, 1024), ID_DV, (it > 0 || t > 0) ? 1u : 0u);  // dK += dS^T Q
             }
+            ptx::mma_commit(&q_empty[st]);  // last reads of Q / dO
             if (C::DQ_OWN && gg >= 1) ptx::mbar_wait(dq_empty, (gg - 1) & 1);  // dQ(gg-1) read out
 #pragma unroll
             for (int t = 0; t < 128 / 16; ++t)  // K = 128 keys: dQ = dS K
@@ -646,7 +669,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
                             ptx::sdesc_sw128(ak + t * 2048, 16384, 1024), ID_DQ, t > 0);
           }
           ptx::mma_commit(mm_done);
-          ptx::mma_commit(&q_empty[st]);
+          if (C::DQ_OWN && it + 1 < nq && !st_next) issue_st(gg + 1);
           if (!C::DQ_OWN && it + 1 < nq) issue_st(gg + 1);
         }
         ptx::mma_commit(kv_empty);
@@ -709,7 +732,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
     };
     int g = 0, n = 0;
     for (int pass = 0; pass * ncta < n_items; ++pass) {
-      const int item = bwd_item_of(pass, ncta, cta);
+      const int item = snake_item(pass, ncta, cta);
       if (item >= n_items) continue;
       int kt, hd, b;
       decode(item, kt, hd, b);
