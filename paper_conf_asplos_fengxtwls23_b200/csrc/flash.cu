@@ -294,6 +294,39 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
     const uint32_t lb = (uint32_t)(q4 * 32) << 16;
     const float sc = p.scale_log2;
     int g = 0, it = 0;
+    // deferred O epilogue of the previous item
+    bool pend = false;
+    int pd_ob = 0;
+    uint32_t pd_ph = 0;
+    float pd_l = 1.f, pd_m = 0.f;
+    __nv_bfloat16* pd_orow = nullptr;
+    float* pd_lse = nullptr;
+    auto store_o = [&]() {
+      if (!pend) return;
+      pend = false;
+      ptx::mbar_wait(&o_ready[pd_ob], pd_ph);
+      ptx::tc_fence_after();
+      const float inv_l = 1.f / pd_l;
+#pragma unroll
+      for (int c = 0; c < DH / 64; ++c) {
+        uint32_t v[32];
+        __syncwarp();
+        ptx::tmem_ld32(tmem + 256 + pd_ob * DH + hf * (DH / 2) + c * 32 + lb, v);
+        ptx::tmem_ld_wait();
+        uint32_t pk[16];
+#pragma unroll
+        for (int e = 0; e < 32; e += 2)
+          pk[e / 2] = pack_bf16(__uint_as_float(v[e]) * inv_l, __uint_as_float(v[e + 1]) * inv_l);
+#pragma unroll
+        for (int k = 0; k < 4; ++k)
+          *reinterpret_cast<uint4*>(pd_orow + c * 32 + k * 8) =
+              make_uint4(pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
+      }
+      if (hf == 0) *pd_lse = pd_m + __log2f(pd_l);
+      ptx::tc_fence_before();
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(&o_empty[pd_ob]);
+    };
     for (int pass = 0; pass * (int)gridDim.x < n_items; ++pass) {
       const int i = snake_item(pass, (int)gridDim.x, (int)blockIdx.x);
       if (i >= n_items) continue;
@@ -387,37 +420,25 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
         ptx::fence_proxy_async();
         __syncwarp();
         if (lane == 0) ptx::mbar_arrive(&p_full[sb]);
+        if (j == 0) store_o();  // previous item's O while this tile's PV runs
       }
-      // output: O / l  (l = sum of both halves)
+      // output: O / l  (l = sum of both halves).  The O read-out waits for
+      // the item's last PV, so it is deferred until the next item's first P
+      // tile is handed to the tensor core (O is double-buffered in TMEM)
       sts_f32(ptx::smem_u32(sSum + hf * 128 + row), l_run);
       named_bar(2 + q4, 64);
       const float l_tot = l_run + lds_f32(ptx::smem_u32(sSum + (1 - hf) * 128 + row));
-      ptx::mbar_wait(&o_ready[ob], (it >> 1) & 1);
-      ptx::tc_fence_after();
-      const float inv_l = 1.f / l_tot;
-      __nv_bfloat16* orow = p.O + ((int64_t)b * p.s + qrow) * p.h + hd * DH + hf * (DH / 2);
-#pragma unroll
-      for (int c = 0; c < DH / 64; ++c) {
-        uint32_t v[32];
-        __syncwarp();
-        ptx::tmem_ld32(tmem + 256 + ob * DH + hf * (DH / 2) + c * 32 + lb, v);
-        ptx::tmem_ld_wait();
-        uint32_t pk[16];
-#pragma unroll
-        for (int e = 0; e < 32; e += 2)
-          pk[e / 2] = pack_bf16(__uint_as_float(v[e]) * inv_l, __uint_as_float(v[e + 1]) * inv_l);
-#pragma unroll
-        for (int k = 0; k < 4; ++k)
-          *reinterpret_cast<uint4*>(orow + c * 32 + k * 8) =
-              make_uint4(pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
-      }
-      if (hf == 0) p.lse[((int64_t)b * p.nh + hd) * p.s + qrow] = m_run + __log2f(l_tot);
-      ptx::tc_fence_before();
-      __syncwarp();
-      if (lane == 0) ptx::mbar_arrive(&o_empty[ob]);
       named_bar(2 + q4, 64);  // partner read sSum before the next item overwrites it
+      pend = true;
+      pd_ob = ob;
+      pd_ph = (it >> 1) & 1;
+      pd_l = l_tot;
+      pd_m = m_run;
+      pd_orow = p.O + ((int64_t)b * p.s + qrow) * p.h + hd * DH + hf * (DH / 2);
+      pd_lse = p.lse + ((int64_t)b * p.nh + hd) * p.s + qrow;
       ++it;
     }
+    store_o();
   }
   __syncthreads();
   if (warp == 1) {
