@@ -344,12 +344,16 @@ def run_mobius(args, rank, world, local):
     achieved_tf = gemm_flops / (gemm_ns * 1e-9) / 1e12 if gemm_ns else 0.0
     peak_tf = peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops"))
     traffic = traffic_alg = None
-    tr_path = os.path.join(ROOT, "profiles", "r1_gemm_traffic_v3.json")
-    if os.path.exists(tr_path):  # ncu --set full capture of the block GEMM shapes (per launch)
+    # ncu --set full capture of the block GEMM shapes (per launch) at this T
+    tr_name = {16384: "r1_gemm_traffic_v4.json", 8192: "r1_gemm_traffic_v3.json"}.get(c.micro_batch * c.seq_len)
+    tr_path = os.path.join(ROOT, "profiles", tr_name) if tr_name else ""
+    tr_n = 0
+    if tr_path and os.path.exists(tr_path):
         with open(tr_path) as f:
             tr = json.load(f)
         traffic = float(np.mean([t["dram_bytes"] for t in tr]))
         traffic_alg = float(np.mean([t["algorithmic_bytes"] for t in tr]))
+        tr_n = len(tr)
     # step roofline (north_star): max(FLOP / P_tc, H2D bytes / host link), per GPU
     flop_step = model_flops_per_token(c) * tokens_per_step / world
     t_tc = flop_step / (peak_tf * 1e12)
@@ -379,9 +383,9 @@ def run_mobius(args, rank, world, local):
                          "achieved": achieved_tf, "peak": peak_tf, "unit": "TFLOP/s",
                          "frac": achieved_tf / peak_tf if peak_tf else None, "traffic": traffic,
                          "traffic_algorithmic_bytes": traffic_alg,
-                         "traffic_source": "profiles/r1_gemm_traffic_v3.json: dram__bytes_read+write per launch, mean "
-                                           "over the 8 captured 1.5B block GEMM shapes (ncu --set full, cold L2; "
-                                           "tools/gemm_traffic.py)",
+                         "traffic_source": f"profiles/{tr_name}: dram__bytes_read+write per launch, mean over the "
+                                           f"{tr_n} captured 1.5B block GEMM shapes at T={c.micro_batch * c.seq_len} "
+                                           "(ncu --set full, cold L2; tools/gemm_prof.py + tools/gemm_traffic.py)",
                          "peak_source": f"MEASURED_PEAKS.json bf16_tflops_sustained ({peak_src})"},
             "step_roofline": {"t_tensor_ms": t_tc * 1e3, "t_link_ms": t_link * 1e3, "t_roofline_ms": t_roof * 1e3,
                               "frac": t_roof / (ms * 1e-3), "h2d_GBps_link": h2d_gbps,
