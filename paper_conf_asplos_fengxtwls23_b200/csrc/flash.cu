@@ -494,7 +494,8 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
 template <int DH>
 __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_constant__ CUtensorMap tm,
                                                               const __grid_constant__ CUtensorMap tdo,
-                                                              const __grid_constant__ CUtensorMap tdq, const BwdParams p) {
+                                                              const __grid_constant__ CUtensorMap tdq,
+                                                              const __grid_constant__ CUtensorMap tdkv, const BwdParams p) {
   using C = BwdCfg<DH>;
   constexpr int QS = C::QS;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -541,6 +542,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
     ptx::tma_prefetch_desc(&tm);
     ptx::tma_prefetch_desc(&tdo);
     ptx::tma_prefetch_desc(&tdq);
+    ptx::tma_prefetch_desc(&tdkv);
     ptx::mbar_init(kv_full, 1);
     for (int i = 0; i < 2; ++i) {
       ptx::mbar_init(&q_full[i], 1);
@@ -790,6 +792,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
           ptx::tc_fence_after();
         }
         if (!C::DQ_OWN && gg >= 1) stage_free();  // dQ(gg-1) staged in P^T / dS^T: reduce must have read it
+        if (C::DQ_OWN && it == 0 && gg >= 1) stage_free();  // previous item's dV/dK stores read the P^T / dS^T tiles
         const uint32_t sds = ptx::smem_u32(sdS_buf[C::PT_TMEM ? (gg & 1) : 0]);
 #pragma unroll
         for (int cc = 0; cc < 2; ++cc) {
@@ -837,9 +840,16 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
       const int glast = g + nq - 1;
       ptx::mbar_wait(mm_done, glast & 1);
       ptx::tc_fence_after();
-      if (C::DQ_OWN) dq_drain(kt + nq - 1, hd, b, ptx::smem_u32(sSTG));
-      // dV (half 0) / dK (half 1) of this key tile (rows = keys)
-      __nv_bfloat16* out = (hf == 0 ? p.dV : p.dK) + ((int64_t)b * p.s + kt * 128 + r) * p.ldd + hd * DH;
+      if (C::DQ_OWN)
+        dq_drain(kt + nq - 1, hd, b, ptx::smem_u32(sSTG));
+      else
+        stage_free();  // dh 128: the last dQ was staged in the P^T / dS^T tiles
+      // dV (half 0) / dK (half 1) of this key tile (rows = keys), bf16, staged
+      // 128B-swizzled in the (now idle) P^T / dS^T tiles and written by two
+      // TMA stores per tensor atom (row-per-thread global stores are 64 B
+      // pieces 3h apart); the next item's first P^T / dS^T write waits for
+      // the stores' smem reads (stage_free)
+      const uint32_t stg = ptx::smem_u32(sPT) + hf * (DH / 64) * 16384;
 #pragma unroll
       for (int c = 0; c < DH / 32; ++c) {
         uint32_t v[32];
@@ -858,7 +868,21 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
           pk[e / 2] = pack_bf16x2(__fmul2_rn(make_float2(__uint_as_float(v[e]), __uint_as_float(v[e + 1])), make_float2(f, f)));
 #pragma unroll
         for (int k = 0; k < 4; ++k)
-          *reinterpret_cast<uint4*>(out + c * 32 + k * 8) = make_uint4(pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
+          st_shared_v4(stg + sw128_off(r, c * 4 + k), pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
+      }
+      ptx::fence_proxy_async();
+      named_bar(1, 256);
+      if (warp == 2 && lane == 0) {
+#pragma unroll
+        for (int t = 0; t < 2; ++t)
+#pragma unroll
+          for (int a = 0; a < DH / 64; ++a)
+            asm volatile("cp.async.bulk.tensor.4d.global.shared::cta.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
+                             reinterpret_cast<uint64_t>(&tdkv)),
+                         "r"(ptx::smem_u32(sPT) + (t * (DH / 64) + a) * 16384), "r"(64 * a), "r"(kt * 128),
+                         "r"((t == 0 ? 2 * p.nh : p.nh) + hd), "r"(b)
+                         : "memory");
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
       }
       g += nq;
       ++n;
@@ -1032,6 +1056,9 @@ int flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* o, const __nv_
   if (rc) return rc;
   rc = dq_map(&tdq, dq_ws, h, dh, s, nh, mbs);
   if (rc) return rc;
+  CUtensorMap tdkv;  // TMA-store view of dqkv (dK / dV head slots)
+  rc = head_map(&tdkv, dqkv, 3 * h, dh, s, 3 * nh, mbs);
+  if (rc) return rc;
   if (dh == 64)
     flash_dsum_kernel<64><<<(unsigned)((rows + 7) / 8), 256, 0, st>>>(dout, o, dsum_ws, dq_ws, (int)rows, nh, s);
   else
@@ -1061,11 +1088,11 @@ int flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* o, const __nv_
   if (dh == 64) {
     static bool once = false;
     if (!once) { rc = set_smem(flash_bwd_kernel<64>, BwdCfg<64>::SMEM); if (rc) return rc; once = true; }
-    flash_bwd_kernel<64><<<grid, NT_FWD, BwdCfg<64>::SMEM, st>>>(tm, tdo, tdq, p);
+    flash_bwd_kernel<64><<<grid, NT_FWD, BwdCfg<64>::SMEM, st>>>(tm, tdo, tdq, tdkv, p);
   } else {
     static bool once = false;
     if (!once) { rc = set_smem(flash_bwd_kernel<128>, BwdCfg<128>::SMEM); if (rc) return rc; once = true; }
-    flash_bwd_kernel<128><<<grid, NT_FWD, BwdCfg<128>::SMEM, st>>>(tm, tdo, tdq, p);
+    flash_bwd_kernel<128><<<grid, NT_FWD, BwdCfg<128>::SMEM, st>>>(tm, tdo, tdq, tdkv, p);
   }
   {
     const int64_t n = rows * h / 4;
