@@ -117,7 +117,10 @@ struct FwdCfg {
   static constexpr int KV_BYTES = BKV * DH * 2;
   static constexpr int P_BYTES = BQ * BKV * 2;
   static constexpr int KVS = DH == 64 ? 2 : 1;  // K/V ring depth (smem budget)
-  static constexpr int SMEM = 1024 + 2 * Q_BYTES + 2 * KVS * KV_BYTES + 2 * P_BYTES + 4096;
+  // dh 64: O leaves through a staging tile (4 KB per 32-row quadrant) and
+  // TMA stores; dh 128 has no smem left for it and stores row per thread
+  static constexpr int O_STG = DH == 64 ? 128 * 128 : 0;
+  static constexpr int SMEM = 1024 + 2 * Q_BYTES + 2 * KVS * KV_BYTES + 2 * P_BYTES + O_STG + 4096;
 };
 
 struct FwdParams {
@@ -150,7 +153,8 @@ __device__ __forceinline__ void fwd_item(const FwdParams& p, int i, int& qt, int
 // (column halves) that exchange only the row max.  All barrier phases run on
 // global step counters across items.
 template <int DH>
-__global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_constant__ CUtensorMap tm, const FwdParams p) {
+__global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_constant__ CUtensorMap tm,
+                                                              const __grid_constant__ CUtensorMap tmo, const FwdParams p) {
   using C = FwdCfg<DH>;
   constexpr int KVS = C::KVS;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -159,7 +163,8 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
   uint8_t* sK = sQ + 2 * C::Q_BYTES;      // [KVS]
   uint8_t* sV = sK + KVS * C::KV_BYTES;   // [KVS]
   uint8_t* sP = sV + KVS * C::KV_BYTES;   // [2]
-  float* sMax = reinterpret_cast<float*>(sP + 2 * C::P_BYTES);  // [2 iters][2 halves][128]
+  uint8_t* sO = sP + 2 * C::P_BYTES;      // O staging (dh 64)
+  float* sMax = reinterpret_cast<float*>(sO + C::O_STG);  // [2 iters][2 halves][128]
   float* sSum = sMax + 512;                                       // [2 halves][128]
   uint64_t* bars = reinterpret_cast<uint64_t*>(sSum + 256);
   uint64_t* q_full = bars;          // [2]
@@ -301,12 +306,19 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
     float pd_l = 1.f, pd_m = 0.f;
     __nv_bfloat16* pd_orow = nullptr;
     float* pd_lse = nullptr;
+    int pd_qt = 0, pd_hd = 0, pd_b = 0;
+    const bool o_issuer = hf == 0 && lane == 0;  // issues this quadrant's O TMA stores (dh 64)
+    const uint32_t o_slab = ptx::smem_u32(sO) + q4 * 4096;
     auto store_o = [&]() {
       if (!pend) return;
       pend = false;
       ptx::mbar_wait(&o_ready[pd_ob], pd_ph);
       ptx::tc_fence_after();
       const float inv_l = 1.f / pd_l;
+      if constexpr (DH == 64) {
+        if (o_issuer) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // previous store read the slab
+        named_bar(2 + q4, 64);
+      }
 #pragma unroll
       for (int c = 0; c < DH / 64; ++c) {
         uint32_t v[32];
@@ -317,10 +329,28 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
 #pragma unroll
         for (int e = 0; e < 32; e += 2)
           pk[e / 2] = pack_bf16(__uint_as_float(v[e]) * inv_l, __uint_as_float(v[e + 1]) * inv_l);
+        if constexpr (DH == 64) {  // row `lane` of the quadrant's 32-row slab, 16-byte chunks hf*4.., SW128
 #pragma unroll
-        for (int k = 0; k < 4; ++k)
-          *reinterpret_cast<uint4*>(pd_orow + c * 32 + k * 8) =
-              make_uint4(pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
+          for (int k = 0; k < 4; ++k)
+            st_shared_v4(o_slab + lane * 128 + (((hf * 4 + k) ^ (lane & 7)) << 4), pk[4 * k], pk[4 * k + 1],
+                         pk[4 * k + 2], pk[4 * k + 3]);
+        } else {
+#pragma unroll
+          for (int k = 0; k < 4; ++k)
+            *reinterpret_cast<uint4*>(pd_orow + c * 32 + k * 8) =
+                make_uint4(pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
+        }
+      }
+      if constexpr (DH == 64) {
+        ptx::fence_proxy_async();
+        named_bar(2 + q4, 64);
+        if (o_issuer) {
+          asm volatile("cp.async.bulk.tensor.4d.global.shared::cta.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
+                           reinterpret_cast<uint64_t>(&tmo)),
+                       "r"(o_slab), "r"(0), "r"(pd_qt * BQ + q4 * 32), "r"(pd_hd), "r"(pd_b)
+                       : "memory");
+          asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        }
       }
       if (hf == 0) *pd_lse = pd_m + __log2f(pd_l);
       ptx::tc_fence_before();
@@ -436,9 +466,13 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
       pd_m = m_run;
       pd_orow = p.O + ((int64_t)b * p.s + qrow) * p.h + hd * DH + hf * (DH / 2);
       pd_lse = p.lse + ((int64_t)b * p.nh + hd) * p.s + qrow;
+      pd_qt = qt;
+      pd_hd = hd;
+      pd_b = b;
       ++it;
     }
     store_o();
+    if (DH == 64 && o_issuer) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");  // O stores complete
   }
   __syncthreads();
   if (warp == 1) {
@@ -966,12 +1000,12 @@ EncodeTiledFn encode_fn() {
 
 // {d, token, head-slot, batch} map over a [mbs*s, ld] bf16 buffer whose head
 // slots are dh apart; box {64, 128, 1, 1}
-int head_map(CUtensorMap* m, const void* base, int64_t ld, int dh, int s, int n_slots, int mbs) {
+int head_map(CUtensorMap* m, const void* base, int64_t ld, int dh, int s, int n_slots, int mbs, int box_rows = 128) {
   EncodeTiledFn enc = encode_fn();
   if (!enc) MOBIUS_FAIL(MOBIUS_ECUDA, "cuTensorMapEncodeTiled unavailable");
   cuuint64_t dims[4] = {(cuuint64_t)dh, (cuuint64_t)s, (cuuint64_t)n_slots, (cuuint64_t)mbs};
   cuuint64_t strides[3] = {(cuuint64_t)(ld * 2), (cuuint64_t)(dh * 2), (cuuint64_t)(s * ld * 2)};
-  cuuint32_t box[4] = {64, 128, 1, 1};
+  cuuint32_t box[4] = {64, (cuuint32_t)box_rows, 1, 1};
   cuuint32_t es[4] = {1, 1, 1, 1};
   CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void*>(base), dims, strides, box, es,
                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
@@ -1013,6 +1047,9 @@ int flash_attn_fwd(const __nv_bfloat16* qkv, __nv_bfloat16* o, float* lse, int m
   CUtensorMap tm;
   int rc = head_map(&tm, qkv, 3 * h, dh, s, 3 * nh, mbs);
   if (rc) return rc;
+  CUtensorMap tmo;  // TMA-store view of O, 32-row boxes (one per softmax lane quadrant)
+  rc = head_map(&tmo, o, h, dh, s, nh, mbs, 32);
+  if (rc) return rc;
   FwdParams p;
   p.O = o;
   p.lse = lse;
@@ -1032,11 +1069,11 @@ int flash_attn_fwd(const __nv_bfloat16* qkv, __nv_bfloat16* o, float* lse, int m
   if (dh == 64) {
     static bool once = false;
     if (!once) { rc = set_smem(flash_fwd_kernel<64>, FwdCfg<64>::SMEM); if (rc) return rc; once = true; }
-    flash_fwd_kernel<64><<<grid, NT_FWD, FwdCfg<64>::SMEM, st>>>(tm, p);
+    flash_fwd_kernel<64><<<grid, NT_FWD, FwdCfg<64>::SMEM, st>>>(tm, tmo, p);
   } else {
     static bool once = false;
     if (!once) { rc = set_smem(flash_fwd_kernel<128>, FwdCfg<128>::SMEM); if (rc) return rc; once = true; }
-    flash_fwd_kernel<128><<<grid, NT_FWD, FwdCfg<128>::SMEM, st>>>(tm, p);
+    flash_fwd_kernel<128><<<grid, NT_FWD, FwdCfg<128>::SMEM, st>>>(tm, tm, p);
   }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) MOBIUS_FAIL(MOBIUS_ECUDA, "flash_fwd launch: %s", cudaGetErrorString(e));
