@@ -53,7 +53,12 @@ struct Params {
   // sk_tiles tiles' k-blocks are split evenly over all clusters; partial
   // accumulators go to sk_ws, the last-arriving segment reduces them in
   // segment order (deterministic) and runs the fused epilogue.
-  int sk_tiles, sk_maxseg;
+  // sk_slices > 0 selects the k-aligned variant: the sk_tiles remainder
+  // tiles are cut into sk_slices equal k-slices, unit u = (slice u / sk_tiles,
+  // tile u % sk_tiles) goes to cluster u % clusters, so all clusters of the
+  // Stream-K round stream the same k range of their panels (L2 reuse); the
+  // contiguous variant gives each cluster a different k phase.
+  int sk_tiles, sk_maxseg, sk_slices;
   int64_t sk_units;
   float* sk_ws;
   int* sk_cnt;

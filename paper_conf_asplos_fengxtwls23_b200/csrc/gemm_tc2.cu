@@ -266,12 +266,27 @@ struct Sched {
   int64_t g, gend;
   int t, cl, ncl;
   __device__ __forceinline__ Sched(const Params& p, int cl_, int ncl_) : cl(cl_), ncl(ncl_) {
-    g = p.sk_tiles ? sk_start(p, cl, ncl) : 0;
-    gend = p.sk_tiles ? sk_start(p, cl + 1, ncl) : 0;
+    if (p.sk_slices) {  // k-aligned: units cl, cl + ncl, ... of sk_tiles * sk_slices
+      g = cl;
+      gend = (int64_t)p.sk_tiles * p.sk_slices;
+    } else {
+      g = p.sk_tiles ? sk_start(p, cl, ncl) : 0;
+      gend = p.sk_tiles ? sk_start(p, cl + 1, ncl) : 0;
+    }
     t = p.sk_tiles + cl;
   }
   __device__ __forceinline__ bool next(const Params& p, int total, Work& w) {
-    if (g < gend) {
+    if (p.sk_slices && g < gend) {
+      const int sl = (int)(g / p.sk_tiles), kbs = (p.num_kb + p.sk_slices - 1) / p.sk_slices;
+      w.t = (int)(g % p.sk_tiles);
+      w.k0 = sl * kbs;
+      w.k1 = min(p.num_kb, w.k0 + kbs);
+      w.seg = sl;
+      w.nseg = p.sk_slices;
+      g += ncl;
+      return true;
+    }
+    if (!p.sk_slices && g < gend) {
       const int nkb = p.num_kb;
       const int tt = (int)(g / nkb);
       w.t = tt;
@@ -700,17 +715,36 @@ static int sk_owner_h(int64_t units, int64_t g, int ncl) {
 // Stream-K keeps floor(T/P)-1 whole waves and spreads the remaining tiles'
 // k-blocks evenly (cost ~ T/P + fixup); used when that saves >= 5% of a
 // wave and every cluster gets a reasonable k-range.
+static int g_gemm_skmode = -1;  // MOBIUS_GEMM_SKMODE: 0 auto, 1 contiguous only, 2 k-aligned when possible
+
 static void plan_stream_k(Params& p, int P) {
   p.sk_tiles = 0;
   p.sk_units = 0;
   p.sk_maxseg = 0;
+  p.sk_slices = 0;
   if (g_gemm_sk < 0) {
     const char* e = getenv("MOBIUS_GEMM_SK");
     g_gemm_sk = (e && e[0] == '0') ? 0 : 1;
   }
   if (!g_gemm_sk) return;
+  if (g_gemm_skmode < 0) {
+    const char* e = getenv("MOBIUS_GEMM_SKMODE");
+    g_gemm_skmode = e ? atoi(e) : 0;
+  }
   const int T = p.tiles_m * p.tiles_n, nkb = p.num_kb;
   if (T % P == 0) return;
+  if (g_gemm_skmode != 1 && T > P && nkb >= 64) {
+    // k-aligned: every full wave data-parallel, the R remainder tiles in S
+    // slices, one round (R * S <= P); cost T/P rounded to 1/S of a wave
+    const int R = T % P, S = std::min(P / R, nkb / 16);
+    if (S >= 2) {
+      p.sk_tiles = R;
+      p.sk_slices = S;
+      p.sk_maxseg = S;
+      p.sk_units = (int64_t)R * S;
+      return;
+    }
+  }
   const int waves = (T + P - 1) / P;
   const int dp_waves = T / P >= 1 ? T / P - 1 : 0;
   const int sk_tiles = T - dp_waves * P;
