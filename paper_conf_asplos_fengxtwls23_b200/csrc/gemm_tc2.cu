@@ -733,15 +733,31 @@ static void plan_stream_k(Params& p, int P) {
   }
   const int T = p.tiles_m * p.tiles_n, nkb = p.num_kb;
   if (T % P == 0) return;
-  if (g_gemm_skmode != 1 && T > P && nkb >= 64) {
+  if (g_gemm_skmode != 1 && nkb >= 64) {
     // k-aligned: every full wave data-parallel, the R remainder tiles in S
-    // slices, one round (R * S <= P); cost T/P rounded to 1/S of a wave
-    const int R = T % P, S = std::min(P / R, nkb / 16);
-    if (S >= 2) {
+    // slices of >= 16 k-blocks dealt round-robin (slice-major) over the P
+    // clusters; the tail then costs ceil(R*S/P)/S of a wave instead of 1.
+    // S minimises that (ties: fewer slices = fewer partials to reduce).
+    static double pen = -1.0;  // per-slice cost (partials written and reduced), in waves
+    if (pen < 0) {
+      const char* e = getenv("MOBIUS_GEMM_SKPEN");
+      pen = e ? atof(e) : 0.04;
+    }
+    const int R = T % P;
+    int best_s = 0;
+    double best = 1.0;
+    for (int S = 2; S <= std::min(16, nkb / 16); ++S) {
+      const double c = (double)((R * S + P - 1) / P) / S + pen * S;
+      if (c < best - 1e-9) {
+        best = c;
+        best_s = S;
+      }
+    }
+    if (best_s && best <= 0.92) {
       p.sk_tiles = R;
-      p.sk_slices = S;
-      p.sk_maxseg = S;
-      p.sk_units = (int64_t)R * S;
+      p.sk_slices = best_s;
+      p.sk_maxseg = best_s;
+      p.sk_units = (int64_t)R * best_s;
       return;
     }
   }
