@@ -733,7 +733,12 @@ static void plan_stream_k(Params& p, int P) {
   }
   const int T = p.tiles_m * p.tiles_n, nkb = p.num_kb;
   if (T % P == 0) return;
-  if (g_gemm_skmode != 1 && nkb >= 64) {
+  static int min_slice = -1;  // k-blocks per slice (MOBIUS_GEMM_SKSLICE, default 16)
+  if (min_slice < 0) {
+    const char* e = getenv("MOBIUS_GEMM_SKSLICE");
+    min_slice = e ? std::max(4, atoi(e)) : 16;
+  }
+  if (g_gemm_skmode != 1 && nkb >= 2 * min_slice) {
     // k-aligned: every full wave data-parallel, the R remainder tiles in S
     // slices of >= 16 k-blocks dealt round-robin (slice-major) over the P
     // clusters; the tail then costs ceil(R*S/P)/S of a wave instead of 1.
@@ -746,7 +751,7 @@ static void plan_stream_k(Params& p, int P) {
     const int R = T % P;
     int best_s = 0;
     double best = 1.0;
-    for (int S = 2; S <= std::min(16, nkb / 16); ++S) {
+    for (int S = 2; S <= std::min(16, nkb / min_slice); ++S) {
       const double c = (double)((R * S + P - 1) / P) / S + pen * S;
       if (c < best - 1e-9) {
         best = c;
