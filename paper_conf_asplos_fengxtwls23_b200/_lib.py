@@ -56,6 +56,13 @@ class Dist(C.Structure):
     _fields_ = [("rank", C.c_int), ("world", C.c_int), ("device", C.c_int), ("flags", C.c_int)]
 
 
+class TimelineEvent(C.Structure):
+    _fields_ = [("kind", C.c_int32), ("stage", C.c_int32), ("t0_ms", C.c_double), ("t1_ms", C.c_double)]
+
+
+TL_KINDS = {0: "h2d", 1: "fwd", 2: "bwd", 3: "d2h"}
+
+
 class StepStats(C.Structure):
     _fields_ = [("step_ns", C.c_int64), ("device_step_ns", C.c_int64), ("h2d_bytes", C.c_int64),
                 ("d2h_bytes", C.c_int64), ("p2p_bytes", C.c_int64), ("n_h2d_copies", C.c_int64),
@@ -98,6 +105,7 @@ SIGNATURES = {
     "mobius_read_params": (I, [P, P, C.c_size_t]),
     "mobius_read_trace": (I, [P, P, C.c_size_t, C.POINTER(C.c_size_t)]),
     "mobius_stats": (I, [P, C.POINTER(StepStats)]),
+    "mobius_read_timeline": (I, [P, P, C.c_size_t, C.POINTER(C.c_size_t)]),
     "mobius_destroy": (None, [P]),
     "mobius_last_error": (C.c_char_p, []),
     "mobius_build_info": (C.c_char_p, []),

@@ -202,6 +202,15 @@ class MobiusContext:
         check(lib.mobius_read_trace(self._ctx, buf, cap, C.byref(n)))
         return [("F" if buf[3 * i] == 0 else "B", buf[3 * i + 1], buf[3 * i + 2]) for i in range(n.value)]
 
+    def read_timeline(self):
+        """Device timeline of the last step: list of (kind, stage, t0_ms, t1_ms),
+        kind in h2d / fwd / bwd / d2h (include/mobius.h mobius_read_timeline)."""
+        n = C.c_size_t()
+        check(lib.mobius_read_timeline(self._ctx, None, 0, C.byref(n)))
+        buf = (L.TimelineEvent * max(1, n.value))()
+        check(lib.mobius_read_timeline(self._ctx, buf, n.value, C.byref(n)))
+        return [(L.TL_KINDS[e.kind], e.stage, e.t0_ms, e.t1_ms) for e in buf[:n.value]]
+
     def stats(self) -> L.StepStats:
         s = L.StepStats()
         check(lib.mobius_stats(self._ctx, C.byref(s)))

@@ -211,6 +211,11 @@ struct mobius_ctx {
   std::vector<cudaEvent_t> ev_gready, ev_d2h;      // per local stage
   cudaEvent_t ev_step0 = nullptr, ev_step1 = nullptr;
   std::vector<cudaEvent_t> ev_wait_a, ev_wait_b;   // exposed load waits
+  // timeline (mobius_read_timeline): compute passes and offloads of the last step
+  std::vector<cudaEvent_t> ev_pass_a, ev_pass_b;   // per exec entry (2 per local stage)
+  std::vector<cudaEvent_t> ev_off_a, ev_off_b;     // per local stage
+  std::vector<int> part_stage;                     // global stage of each copy part
+  int n_parts_last = 0;
 
   // update worker
   std::thread upd_thread;
@@ -410,6 +415,7 @@ struct StepRunner {
     CU(cudaMemcpyAsync(dst, src, b1 - b0, cudaMemcpyHostToDevice, ctx->s_h2d));
     CU(cudaEventRecord(b, ctx->s_h2d));
     ctx->part_bytes[n_parts] = b1 - b0;
+    ctx->part_stage[n_parts] = ctx->mine[L.stage_local];
     ++n_parts;
     h2d_bytes += b1 - b0;
     return MOBIUS_OK;
@@ -613,8 +619,10 @@ struct StepRunner {
     }
     CU(cudaEventRecord(ctx->ev_gready[ls], s));
     CU(cudaStreamWaitEvent(ctx->s_d2h, ctx->ev_gready[ls], 0));
+    CU(cudaEventRecord(ctx->ev_off_a[ls], ctx->s_d2h));
     CU(cudaMemcpyAsync(dev_upd ? ctx->h_weights[ls] : ctx->h_grads[ls], dev_upd ? ctx->d_wstage : ctx->grad_stage,
                        st.n_params * sizeof(T), cudaMemcpyDeviceToHost, ctx->s_d2h));
+    CU(cudaEventRecord(ctx->ev_off_b[ls], ctx->s_d2h));
     CU(cudaEventRecord(ctx->ev_d2h[ls], ctx->s_d2h));
     ctx->stats.d2h_bytes += st.n_params * sizeof(T);
     if (dev_upd) return MOBIUS_OK;
@@ -640,11 +648,13 @@ struct StepRunner {
     for (int k = n - 1; k >= 0; --k) ex.push_back({0, k, ctx->res_b[k], k != n - 1, true});
     RC(load_first_part(0));
     RC(load_second_part(0));
-    for (const Exec& e : ex) {
+    for (size_t xi = 0; xi < ex.size(); ++xi) {
+      const Exec& e = ex[xi];
       if (e.first_of_res) {
         RC(wait_loaded(e.res));
         RC(load_first_part(e.res + 1));  // prefetch of the next residence starts with this one
       }
+      CU(cudaEventRecord(ctx->ev_pass_a[xi], s));
       if (!e.fwd) CU(cudaMemsetAsync(ctx->grad_acc, 0, ctx->all[ctx->mine[e.ls]].n_params * 4, s));
       for (int m = 0; m < M; ++m) {
         if (e.fwd)
@@ -652,6 +662,7 @@ struct StepRunner {
         else
           RC(backward(e.ls, e.res, m));
       }
+      CU(cudaEventRecord(ctx->ev_pass_b[xi], s));
       if (e.last_of_res) {
         CU(cudaEventRecord(ctx->ev_release[e.res], s));
         RC(load_second_part(e.res + 1));
@@ -719,6 +730,7 @@ int do_step(mobius_ctx* ctx, const int32_t* tok_dev, int M, float* loss_out) {
   S.device_step_ns = (int64_t)(ms * 1e6);
   S.h2d_bytes = R.h2d_bytes;
   S.n_h2d_copies = R.n_parts;
+  ctx->n_parts_last = R.n_parts;
   std::vector<double> gbps;
   for (int i = 0; i < R.n_parts; ++i) {
     float pm = 0.f;
@@ -969,6 +981,11 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
     RC(mk(ctx->ev_gready, n, cudaEventDisableTiming));
     RC(mk(ctx->ev_d2h, n, cudaEventDisableTiming));
     RC(mk(ctx->ev_wait_a, R, cudaEventDefault));
+    RC(mk(ctx->ev_pass_a, 2 * n, cudaEventDefault));
+    RC(mk(ctx->ev_pass_b, 2 * n, cudaEventDefault));
+    RC(mk(ctx->ev_off_a, n, cudaEventDefault));
+    RC(mk(ctx->ev_off_b, n, cudaEventDefault));
+    ctx->part_stage.assign(2 * R + 2, 0);
     RC(mk(ctx->ev_wait_b, R, cudaEventDefault));
     CU(cudaEventCreate(&ctx->ev_step0));
     CU(cudaEventCreate(&ctx->ev_step1));
@@ -1208,6 +1225,37 @@ extern "C" int mobius_read_trace(mobius_ctx* ctx, int32_t* out, size_t cap, size
   return MOBIUS_OK;
 }
 
+extern "C" int mobius_read_timeline(mobius_ctx* ctx, mobius_timeline_event* out, size_t cap, size_t* n) {
+  MOBIUS_CHECK_ARG(ctx && n && (out || cap == 0), "null argument");
+  if (ctx->step_count == 0) MOBIUS_FAIL(MOBIUS_ESTATE, "read_timeline: no step has run");
+  std::vector<mobius_timeline_event> v;
+  auto rel = [&](cudaEvent_t a, double* t) {
+    float ms = 0.f;
+    if (cudaEventElapsedTime(&ms, ctx->ev_step0, a) != cudaSuccess) return false;
+    *t = ms;
+    return true;
+  };
+  auto add = [&](int kind, int stage, cudaEvent_t a, cudaEvent_t b) {
+    mobius_timeline_event e;
+    e.kind = kind;
+    e.stage = stage + 1;
+    if (rel(a, &e.t0_ms) && rel(b, &e.t1_ms)) v.push_back(e);
+  };
+  for (int i = 0; i < ctx->n_parts_last; ++i)
+    add(MOBIUS_TL_H2D, ctx->part_stage[i], ctx->ev_part_a[i], ctx->ev_part_b[i]);
+  const int nl = (int)ctx->mine.size();
+  for (int xi = 0; xi < 2 * nl; ++xi) {  // exec order: F of local stages ascending, then B descending
+    const bool fwd = xi < nl;
+    const int ls = fwd ? xi : 2 * nl - 1 - xi;
+    add(fwd ? MOBIUS_TL_FWD : MOBIUS_TL_BWD, ctx->mine[ls], ctx->ev_pass_a[xi], ctx->ev_pass_b[xi]);
+  }
+  for (int ls = nl - 1; ls >= 0; --ls) add(MOBIUS_TL_D2H, ctx->mine[ls], ctx->ev_off_a[ls], ctx->ev_off_b[ls]);
+  cudaGetLastError();  // clear a not-ready / unrecorded event status
+  *n = v.size();
+  if (out) std::memcpy(out, v.data(), std::min(cap, v.size()) * sizeof(mobius_timeline_event));
+  return MOBIUS_OK;
+}
+
 extern "C" int mobius_stats(mobius_ctx* ctx, mobius_step_stats* out) {
   MOBIUS_CHECK_ARG(ctx && out, "null argument");
   *out = ctx->stats;
@@ -1229,7 +1277,8 @@ extern "C" void mobius_destroy(mobius_ctx* ctx) {
   for (auto p : ctx->peer_base)
     if (p) cudaIpcCloseMemHandle(p);
   for (auto* v : {&ctx->ev_release, &ctx->ev_loaded, &ctx->ev_part_a, &ctx->ev_part_b, &ctx->ev_gready,
-                  &ctx->ev_d2h, &ctx->ev_wait_a, &ctx->ev_wait_b})
+                  &ctx->ev_d2h, &ctx->ev_wait_a, &ctx->ev_wait_b, &ctx->ev_pass_a, &ctx->ev_pass_b,
+                  &ctx->ev_off_a, &ctx->ev_off_b})
     for (auto e : *v) cudaEventDestroy(e);
   if (ctx->ev_step0) cudaEventDestroy(ctx->ev_step0);
   if (ctx->ev_step1) cudaEventDestroy(ctx->ev_step1);

@@ -136,6 +136,43 @@ def test_device_tail_update(dtype, sizes):
     assert rel(p3d - w, p3h - w) < 1e-2
 
 
+@pytest.mark.parametrize("sizes", [(3, 3), (1, 2, 1, 2)])
+def test_step_timeline(sizes):
+    """mobius_read_timeline: one record per H2D copy part (== the copy count
+    in the stats), one forward and one backward pass per stage, one D2H
+    offload per stage; every pass starts after its stage's load completed
+    (the compute stream waits for it), backward passes in descending stage
+    order after all forward passes (Fig 4 at N = 1)."""
+    from paper_conf_asplos_fengxtwls23_b200.timeline import overlap_summary
+    c = synth.TINY
+    M = 2
+    w = synth.round_bf16(synth.gen_params(c))
+    ctx = MobiusContext(mk_cfg(c, BF16), plan_from_sizes(sizes, 1, M, hbm_cap_bytes=4 * MiB), init_params=w)
+    ctx.step(synth.gen_tokens(c, M))
+    tl = ctx.read_timeline()
+    st = ctx.stats()
+    ctx.close()
+    K = len(sizes)
+    h2d = [x for x in tl if x[0] == "h2d"]
+    fwd = [x for x in tl if x[0] == "fwd"]
+    bwd = [x for x in tl if x[0] == "bwd"]
+    d2h = [x for x in tl if x[0] == "d2h"]
+    assert len(h2d) == st.n_h2d_copies
+    assert [x[1] for x in fwd] == list(range(1, K + 1)) and [x[1] for x in bwd] == list(range(K, 0, -1))
+    assert sorted(x[1] for x in d2h) == list(range(1, K + 1))
+    for k, j, t0, t1 in tl:
+        assert 0.0 <= t0 <= t1
+    eps = 1e-3
+    for a, b in zip(fwd + bwd, (fwd + bwd)[1:]):
+        assert b[2] >= a[3] - eps  # passes run back to back on one stream
+    # the forward pass of stage j starts after every copy of stage j issued so far has finished
+    for k, j, t0, _ in fwd:
+        loads = [x for x in h2d if x[1] == j and x[2] <= t0 + eps]
+        assert loads and all(x[3] <= t0 + eps for x in loads)
+    s = overlap_summary(tl)
+    assert 0.0 <= s["h2d_hidden_ms"] <= s["h2d_ms"] + 1e-9
+
+
 def test_tiny_two_steps_bf16():
     """Second step runs on the host-updated stages (swap-in of the new
     weights) and matches the oracle's second step."""
