@@ -115,7 +115,12 @@ template <int DH>
 struct FwdCfg {
   static constexpr int Q_BYTES = BQ * DH * 2;
   static constexpr int KV_BYTES = BKV * DH * 2;
-  static constexpr int P_BYTES = BQ * BKV * 2;
+  // dh 64: P (bf16, 64 packed columns per buffer) lives in TMEM columns
+  // 384 / 448 and feeds O += P V as the A operand of a TS-MMA, so PV reads
+  // only V from smem and the softmax warps write P with tcgen05.st; dh 128
+  // has no TMEM left (O[2] takes 256 columns) and stages P in smem
+  static constexpr bool P_TMEM = DH == 64;
+  static constexpr int P_BYTES = P_TMEM ? 0 : BQ * BKV * 2;
   static constexpr int KVS = DH == 64 ? 2 : 1;  // K/V ring depth (smem budget)
   // dh 64: O leaves through a staging tile (4 KB per 32-row quadrant) and
   // TMA stores; dh 128 has no smem left for it and stores row per thread
@@ -207,7 +212,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_slot;
-  // TMEM: S[2] at 0 / 128, O[2] at 256 / 256 + DH
+  // TMEM: S[2] at 0 / 128, O[2] at 256 / 256 + DH, P[2] at 384 / 448 (dh 64)
   if (warp == 0) {
     if (lane == 0) {
       int g = 0, it = 0;
@@ -277,11 +282,18 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
           ptx::mbar_wait(&v_full[st], kph);
           ptx::tc_fence_after();
           const uint32_t ap = ptx::smem_u32(sP + pb * C::P_BYTES), av = ptx::smem_u32(sV + st * C::KV_BYTES);
+          if constexpr (C::P_TMEM) {
 #pragma unroll
-          for (int k = 0; k < BKV / 16; ++k) {
-            const uint32_t offp = (k >> 2) * 16384 + (k & 3) * 32;
-            ptx::mma_bf16(tmem + 256 + ob * DH, ptx::sdesc_sw128(ap + offp, 16, 1024),
-                          ptx::sdesc_sw128(av + k * 2048, 16384, 1024), ID_O, (j > 0 || k > 0) ? 1u : 0u);
+            for (int k = 0; k < BKV / 16; ++k)  // 16 keys = 8 packed TMEM columns of P
+              ptx::mma_bf16_ts(tmem + 256 + ob * DH, tmem + 384 + pb * 64 + 8 * k,
+                               ptx::sdesc_sw128(av + k * 2048, 16384, 1024), ID_O, (j > 0 || k > 0) ? 1u : 0u);
+          } else {
+#pragma unroll
+            for (int k = 0; k < BKV / 16; ++k) {
+              const uint32_t offp = (k >> 2) * 16384 + (k & 3) * 32;
+              ptx::mma_bf16(tmem + 256 + ob * DH, ptx::sdesc_sw128(ap + offp, 16, 1024),
+                            ptx::sdesc_sw128(av + k * 2048, 16384, 1024), ID_O, (j > 0 || k > 0) ? 1u : 0u);
+            }
           }
           ptx::mma_commit(&pv_done[pb]);
           ptx::mma_commit(&v_empty[st]);
@@ -430,9 +442,13 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
             rs += p0 + p1;
             pk[e >> 1] = pack_bf16(p0, p1);
           }
+          if constexpr (C::P_TMEM) {  // keys hf*64 .. +31 -> packed columns hf*32 .. +15
+            ptx::tmem_st16(tmem + 384 + sb * 64 + hf * 32 + lb, pk);
+          } else {
 #pragma unroll
-          for (int k = 0; k < 4; ++k)
-            st_shared_v4(sp + sw128_off(row, hf * 8 + k), pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
+            for (int k = 0; k < 4; ++k)
+              st_shared_v4(sp + sw128_off(row, hf * 8 + k), pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
+          }
 #pragma unroll
           for (int e = 0; e < 32; e += 2) {
             const float p0 = ex2(fmaf(__uint_as_float(v1[e]), sc, -m_new));
@@ -440,9 +456,14 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
             rs += p0 + p1;
             pk[e >> 1] = pack_bf16(p0, p1);
           }
+          if constexpr (C::P_TMEM) {
+            ptx::tmem_st16(tmem + 384 + sb * 64 + hf * 32 + 16 + lb, pk);
+            ptx::tmem_st_wait();
+          } else {
 #pragma unroll
-          for (int k = 0; k < 4; ++k)
-            st_shared_v4(sp + sw128_off(row, hf * 8 + 4 + k), pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
+            for (int k = 0; k < 4; ++k)
+              st_shared_v4(sp + sw128_off(row, hf * 8 + 4 + k), pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
+          }
         }
         l_run = l_run * alpha + rs;
         m_run = m_new;
