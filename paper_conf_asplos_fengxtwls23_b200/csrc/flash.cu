@@ -121,7 +121,7 @@ struct FwdCfg {
   // has no TMEM left (O[2] takes 256 columns) and stages P in smem
   static constexpr bool P_TMEM = DH == 64;
   static constexpr int P_BYTES = P_TMEM ? 0 : BQ * BKV * 2;
-  static constexpr int KVS = DH == 64 ? 2 : 1;  // K/V ring depth (smem budget)
+  static constexpr int KVS = DH == 64 ? 4 : 1;  // K/V ring depth (smem budget)
   // dh 64: O leaves through a staging tile (4 KB per 32-row quadrant) and
   // TMA stores; dh 128 has no smem left for it and stores row per thread
   static constexpr int O_STG = DH == 64 ? 128 * 128 : 0;
@@ -172,32 +172,34 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
   float* sMax = reinterpret_cast<float*>(sO + C::O_STG);  // [2 iters][2 halves][128]
   float* sSum = sMax + 512;                                       // [2 halves][128]
   uint64_t* bars = reinterpret_cast<uint64_t*>(sSum + 256);
-  uint64_t* q_full = bars;          // [2]
-  uint64_t* q_empty = bars + 2;     // [2]
-  uint64_t* k_full = bars + 4;      // [2]
-  uint64_t* k_empty = bars + 6;     // [2]
-  uint64_t* v_full = bars + 8;      // [2]
-  uint64_t* v_empty = bars + 10;    // [2]
-  uint64_t* s_full = bars + 12;     // [2]
-  uint64_t* s_empty = bars + 14;    // [2] (count 8)
-  uint64_t* p_full = bars + 16;     // [2] (count 8)
-  uint64_t* pv_done = bars + 18;    // [2] PV of global step g commits pv_done[g & 1]
-  uint64_t* o_ready = bars + 20;    // [2] all PVs of an item done
-  uint64_t* o_empty = bars + 22;    // [2] (count 8) O read out
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 24);
+  uint64_t* q_full = bars;                  // [2]
+  uint64_t* q_empty = bars + 2;             // [2]
+  uint64_t* s_full = bars + 4;              // [2]
+  uint64_t* s_empty = bars + 6;             // [2] (count 8)
+  uint64_t* p_full = bars + 8;              // [2] (count 8)
+  uint64_t* pv_done = bars + 10;            // [2] PV of global step g commits pv_done[g & 1]
+  uint64_t* o_ready = bars + 12;            // [2] all PVs of an item done
+  uint64_t* o_empty = bars + 14;            // [2] (count 8) O read out
+  uint64_t* k_full = bars + 16;             // [KVS]
+  uint64_t* k_empty = k_full + KVS;         // [KVS]
+  uint64_t* v_full = k_empty + KVS;         // [KVS]
+  uint64_t* v_empty = v_full + KVS;         // [KVS]
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(v_empty + KVS);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const int n_items = (p.s / BQ) * p.nh * p.mbs;
 
   if (threadIdx.x == 0) {
     ptx::tma_prefetch_desc(&tm);
-    for (int i = 0; i < 2; ++i) {
-      ptx::mbar_init(&q_full[i], 1);
-      ptx::mbar_init(&q_empty[i], 1);
+    for (int i = 0; i < KVS; ++i) {
       ptx::mbar_init(&k_full[i], 1);
       ptx::mbar_init(&k_empty[i], 1);
       ptx::mbar_init(&v_full[i], 1);
       ptx::mbar_init(&v_empty[i], 1);
+    }
+    for (int i = 0; i < 2; ++i) {
+      ptx::mbar_init(&q_full[i], 1);
+      ptx::mbar_init(&q_empty[i], 1);
       ptx::mbar_init(&s_full[i], 1);
       ptx::mbar_init(&s_empty[i], 8);
       ptx::mbar_init(&p_full[i], 8);
