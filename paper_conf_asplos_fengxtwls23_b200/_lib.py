@@ -60,7 +60,7 @@ class TimelineEvent(C.Structure):
     _fields_ = [("kind", C.c_int32), ("stage", C.c_int32), ("t0_ms", C.c_double), ("t1_ms", C.c_double)]
 
 
-TL_KINDS = {0: "h2d", 1: "fwd", 2: "bwd", 3: "d2h"}
+TL_KINDS = {0: "h2d", 1: "fwd", 2: "bwd", 3: "d2h", 4: "d2d"}
 
 
 class StepStats(C.Structure):
@@ -71,7 +71,7 @@ class StepStats(C.Structure):
                 ("elem_ns", C.c_int64), ("kernel_launches", C.c_int64), ("exposed_load_ns", C.c_int64),
                 ("update_tail_ns", C.c_int64), ("arena_bytes", C.c_int64), ("ring_bytes", C.c_int64),
                 ("pinned_bytes", C.c_int64), ("host_update_ns", C.c_int64), ("n_local_stages", C.c_int),
-                ("recompute", C.c_int), ("timing_stride", C.c_int)]
+                ("recompute", C.c_int), ("timing_stride", C.c_int), ("d2d_bytes", C.c_int64)]
 
 
 FLAG_TIMING = 1

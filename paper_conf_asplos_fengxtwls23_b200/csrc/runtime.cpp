@@ -194,6 +194,7 @@ struct mobius_ctx {
   int64_t off_ckpt = 0, off_gslot = 0, off_fflag = 0, off_bflag = 0;
   // MOBIUS_FLAG_DEVICE_TAIL_UPDATE: optimizer state of local stage 0 in HBM
   bool dev_tail = false;
+  bool tail_resident = false;     // d_wstage holds local stage 0's current weights (after the first update)
   float* d_opt = nullptr;         // master | m | v, each al256(np0 * 4) bytes
   int64_t d_opt_stride = 0;       // floats between the three
   uint8_t* d_wstage = nullptr;    // new stage-0 weights (transfer precision) for the D2H
@@ -215,6 +216,7 @@ struct mobius_ctx {
   std::vector<cudaEvent_t> ev_pass_a, ev_pass_b;   // per exec entry (2 per local stage)
   std::vector<cudaEvent_t> ev_off_a, ev_off_b;     // per local stage
   std::vector<int> part_stage;                     // global stage of each copy part
+  std::vector<char> part_d2d;                      // part served from HBM (device tail update)
   int n_parts_last = 0;
 
   // update worker
@@ -351,7 +353,7 @@ struct StepRunner {
   float inv_ntok;
   Scratch<T> sc;
   std::vector<BlockActs<T>> acts;
-  int64_t h2d_bytes = 0;
+  int64_t h2d_bytes = 0, d2d_bytes = 0;
   int n_parts = 0;
 
   T* xbuf(int i) { return tptr<T>(ctx->xs_base + (int64_t)i * ctx->slot_bytes); }
@@ -409,15 +411,21 @@ struct StepRunner {
     const StageDesc& st = ctx->all[ctx->mine[L.stage_local]];
     (void)st;
     uint8_t* dst = ctx->ring + L.base + b0;
-    const uint8_t* src = (const uint8_t*)ctx->h_weights[L.stage_local] + b0;
+    // device tail update: local stage 0's weights already live in HBM
+    const bool d2d = ctx->tail_resident && L.stage_local == 0;
+    const uint8_t* src = d2d ? ctx->d_wstage + b0 : (const uint8_t*)ctx->h_weights[L.stage_local] + b0;
     cudaEvent_t a = ctx->ev_part_a[n_parts], b = ctx->ev_part_b[n_parts];
     CU(cudaEventRecord(a, ctx->s_h2d));
-    CU(cudaMemcpyAsync(dst, src, b1 - b0, cudaMemcpyHostToDevice, ctx->s_h2d));
+    CU(cudaMemcpyAsync(dst, src, b1 - b0, d2d ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, ctx->s_h2d));
     CU(cudaEventRecord(b, ctx->s_h2d));
-    ctx->part_bytes[n_parts] = b1 - b0;
+    ctx->part_bytes[n_parts] = d2d ? 0 : b1 - b0;  // the per-copy GB/s statistics are host-link copies
     ctx->part_stage[n_parts] = ctx->mine[L.stage_local];
+    ctx->part_d2d[n_parts] = d2d;
     ++n_parts;
-    h2d_bytes += b1 - b0;
+    if (d2d)
+      d2d_bytes += b1 - b0;
+    else
+      h2d_bytes += b1 - b0;
     return MOBIUS_OK;
   }
 
@@ -620,11 +628,13 @@ struct StepRunner {
     CU(cudaEventRecord(ctx->ev_gready[ls], s));
     CU(cudaStreamWaitEvent(ctx->s_d2h, ctx->ev_gready[ls], 0));
     CU(cudaEventRecord(ctx->ev_off_a[ls], ctx->s_d2h));
-    CU(cudaMemcpyAsync(dev_upd ? ctx->h_weights[ls] : ctx->h_grads[ls], dev_upd ? ctx->d_wstage : ctx->grad_stage,
-                       st.n_params * sizeof(T), cudaMemcpyDeviceToHost, ctx->s_d2h));
+    if (!dev_upd) {  // the device-updated stage's weights stay in HBM (d_wstage): nothing crosses the link
+      CU(cudaMemcpyAsync(ctx->h_grads[ls], ctx->grad_stage, st.n_params * sizeof(T), cudaMemcpyDeviceToHost,
+                         ctx->s_d2h));
+      ctx->stats.d2h_bytes += st.n_params * sizeof(T);
+    }
     CU(cudaEventRecord(ctx->ev_off_b[ls], ctx->s_d2h));
     CU(cudaEventRecord(ctx->ev_d2h[ls], ctx->s_d2h));
-    ctx->stats.d2h_bytes += st.n_params * sizeof(T);
     if (dev_upd) return MOBIUS_OK;
     {
       std::lock_guard<std::mutex> g(ctx->upd_mu);
@@ -730,11 +740,14 @@ int do_step(mobius_ctx* ctx, const int32_t* tok_dev, int M, float* loss_out) {
   S.device_step_ns = (int64_t)(ms * 1e6);
   S.h2d_bytes = R.h2d_bytes;
   S.n_h2d_copies = R.n_parts;
+  S.d2d_bytes = R.d2d_bytes;
   ctx->n_parts_last = R.n_parts;
+  if (ctx->dev_tail) ctx->tail_resident = true;  // d_wstage now holds local stage 0's updated weights
   std::vector<double> gbps;
   for (int i = 0; i < R.n_parts; ++i) {
     float pm = 0.f;
-    if (cudaEventElapsedTime(&pm, ctx->ev_part_a[i], ctx->ev_part_b[i]) == cudaSuccess && pm > 0)
+    if (ctx->part_bytes[i] > 0 && cudaEventElapsedTime(&pm, ctx->ev_part_a[i], ctx->ev_part_b[i]) == cudaSuccess &&
+        pm > 0)
       gbps.push_back(ctx->part_bytes[i] / (pm * 1e-3) / 1e9);
   }
   if (!gbps.empty()) {
@@ -986,6 +999,7 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
     RC(mk(ctx->ev_off_a, n, cudaEventDefault));
     RC(mk(ctx->ev_off_b, n, cudaEventDefault));
     ctx->part_stage.assign(2 * R + 2, 0);
+    ctx->part_d2d.assign(2 * R + 2, 0);
     RC(mk(ctx->ev_wait_b, R, cudaEventDefault));
     CU(cudaEventCreate(&ctx->ev_step0));
     CU(cudaEventCreate(&ctx->ev_step1));
@@ -1242,7 +1256,7 @@ extern "C" int mobius_read_timeline(mobius_ctx* ctx, mobius_timeline_event* out,
     if (rel(a, &e.t0_ms) && rel(b, &e.t1_ms)) v.push_back(e);
   };
   for (int i = 0; i < ctx->n_parts_last; ++i)
-    add(MOBIUS_TL_H2D, ctx->part_stage[i], ctx->ev_part_a[i], ctx->ev_part_b[i]);
+    add(ctx->part_d2d[i] ? MOBIUS_TL_D2D : MOBIUS_TL_H2D, ctx->part_stage[i], ctx->ev_part_a[i], ctx->ev_part_b[i]);
   const int nl = (int)ctx->mine.size();
   for (int xi = 0; xi < 2 * nl; ++xi) {  // exec order: F of local stages ascending, then B descending
     const bool fwd = xi < nl;

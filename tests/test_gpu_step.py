@@ -122,13 +122,23 @@ def test_device_tail_update(dtype, sizes):
         st = ctx.stats()
         losses += [ctx.step(t) for t in toks[1:]]
         p3 = ctx.read_params(c.n_params)
+        st3 = ctx.stats()
         ctx.close()
-        runs[flags] = (losses, g, p1, p3, st)
-    (lh, gh, p1h, p3h, sth), (ld, gd, p1d, p3d, std) = runs[0], runs[FLAG_DEVICE_TAIL_UPDATE]
+        runs[flags] = (losses, g, p1, p3, st, st3)
+    (lh, gh, p1h, p3h, sth, st3h), (ld, gd, p1d, p3d, std, st3d) = runs[0], runs[FLAG_DEVICE_TAIL_UPDATE]
     # same first step up to the update (bias-gradient column sums use fp32
     # atomics, so equal to rounding, not bitwise)
     assert rel(gd, gh) < 1e-6 and abs(ld[0] - lh[0]) <= 1e-6 * abs(lh[0])
-    assert (std.h2d_bytes, std.d2h_bytes) == (sth.h2d_bytes, sth.d2h_bytes)
+    # step 1 loads every stage from the host; the device-updated first stage
+    # never crosses the link again: no gradient / weight D2H, and from step 2
+    # on its loads are device-to-device (d2d_bytes)
+    esz = 2 if dtype == BF16 else 4
+    stage0 = sum(p.mem_fwd for p in mobius_layer_sizes(mk_cfg(c, dtype))[:sizes[0]])
+    assert std.h2d_bytes == sth.h2d_bytes and std.d2d_bytes == 0
+    assert std.d2h_bytes == sth.d2h_bytes - stage0
+    assert st3d.d2d_bytes > 0 and st3d.d2d_bytes % stage0 == 0
+    assert st3d.h2d_bytes + st3d.d2d_bytes == st3h.h2d_bytes
+    assert esz in (2, 4)
     w1, _, _ = oa.adamw_step(w, np.zeros_like(w), np.zeros_like(w), gd, 1)
     assert np.max(np.abs(p1d - w1)) < 1e-6
     assert rel(p1d - w, p1h - w) < 1e-3
