@@ -4,7 +4,7 @@ os.environ.setdefault('MOBIUS_KT_NOSYNC', '1')
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
 from paper_conf_asplos_fengxtwls23_b200 import BF16, kt
-T, h = 8192, 1600
+T, h = int(os.environ.get("ELEM_T", "16384")), 1600
 def t(fn, it=20):
     for _ in range(3): fn()
     torch.cuda.synchronize()
@@ -23,3 +23,17 @@ us = t(lambda: kt.layernorm_bwd(BF16, dy, x, g, mu, rs, dres, dx, dg, db, T, h))
 for n in (h, 4 * h, 3 * h):
     X = mk(T, n); o = torch.zeros(n, device="cuda")
     us = t(lambda: kt.colsum(BF16, X, n, T, n, o)); print(f"colsum n={n:5d} {us:7.1f} us  {T*n*2/us/1e3:7.1f} GB/s")
+# cold inputs: a fresh buffer set per call (larger than L2 in total), the in-step situation
+NB = 6
+xs = [mk(T, h) for _ in range(NB)]
+ys = [torch.empty_like(x) for x in xs]
+dys = [mk(T, h) for _ in range(NB)]
+dxs = [torch.empty_like(x) for x in xs]
+k = [0]
+def nxt():
+    k[0] = (k[0] + 1) % NB
+    return k[0]
+us = t(lambda: (lambda i: kt.layernorm_fwd(BF16, xs[i], g, bb, ys[i], mu, rs, T, h))(nxt()))
+print(f"ln_fwd   cold {us:7.1f} us  {2*T*h*2/us/1e3:7.1f} GB/s")
+us = t(lambda: (lambda i: kt.layernorm_bwd(BF16, dys[i], xs[i], g, mu, rs, dres, dxs[i], dg, db, T, h))(nxt()))
+print(f"ln_bwd   cold {us:7.1f} us  {4*T*h*2/us/1e3:7.1f} GB/s (dx + param grads)")
