@@ -250,7 +250,7 @@ __device__ __forceinline__ uint4 pack8(const float* f) {
 }
 
 template <int NV>
-__global__ void __launch_bounds__(256, 3) ln_fwd_bf16_k(const __nv_bfloat16* __restrict__ x,
+__global__ void __launch_bounds__(256, 4) ln_fwd_bf16_k(const __nv_bfloat16* __restrict__ x,
                                                      const __nv_bfloat16* __restrict__ g,
                                                      const __nv_bfloat16* __restrict__ b, __nv_bfloat16* __restrict__ y,
                                                      float* mu_out, float* rstd_out, int rows, int h) {
