@@ -47,10 +47,10 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="1.5b")
     ap.add_argument("--layers", type=int, default=0, help="override the block count (shape checks only)")
-    ap.add_argument("--microbatches", type=int, default=0, help="M per GPU (default 8 for 1.5b)")
+    ap.add_argument("--microbatches", type=int, default=0, help="M per GPU (default 4 for 1.5b)")
     ap.add_argument("--cap-gib", type=float, default=1.0, help="HBM stage-ring cap G per GPU")
     ap.add_argument("--micro-batch", type=int, default=0,
-                    help="micro-batch size mbs (default 16 for 1.5b: 8 x 16 x 1024 = 131072 tokens per GPU-step)")
+                    help="micro-batch size mbs (default 32 for 1.5b: 4 x 32 x 1024 = 131072 tokens per GPU-step)")
     ap.add_argument("--impl", default="mobius", choices=["mobius", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -165,14 +165,15 @@ def cpu_oracle_sample(c: synth.GPTConfig, tokens_per_step: int, budget_s: float 
 
 def bench_workload(args, world):
     """(config, M): the bench's GPT config (mbs overridable) and microbatch
-    count.  1.5b default: M = 8 per GPU of mbs 16 (131072 tokens per GPU per
-    step; measured 83k vs 79.5k tokens/s for 16 x mbs 8 - larger GEMMs
-    quantise better over the 74 SM pairs)."""
+    count.  1.5b default: M = 4 per GPU of mbs 32 (131072 tokens per GPU per
+    step).  Same tokens, measured on one box back to back: 16 x mbs 8 79.5k,
+    8 x mbs 16 86.0k, 4 x mbs 32 87.6k tokens/s - larger GEMMs quantise
+    better over the 74 SM pairs and the elementwise kernels amortise."""
     import dataclasses
     c = synth.CONFIGS[args.config]
-    mbs = args.micro_batch or (16 if args.config == "1.5b" else c.micro_batch)
+    mbs = args.micro_batch or (32 if args.config == "1.5b" else c.micro_batch)
     c = dataclasses.replace(c, n_layers=args.layers or c.n_layers, micro_batch=mbs)
-    M = (args.microbatches or (8 if args.config == "1.5b" else 16)) * world
+    M = (args.microbatches or (4 if args.config == "1.5b" else 16)) * world
     return c, M
 
 
@@ -356,7 +357,8 @@ def run_mobius(args, rank, world, local):
     peak_tf = peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops"))
     traffic = traffic_alg = None
     # ncu --set full capture of the block GEMM shapes (per launch) at this T
-    tr_name = {16384: "r1_gemm_traffic_v5.json", 8192: "r1_gemm_traffic_v3.json"}.get(c.micro_batch * c.seq_len)
+    tr_name = {32768: "r1_gemm_traffic_v6.json", 16384: "r1_gemm_traffic_v5.json",
+               8192: "r1_gemm_traffic_v3.json"}.get(c.micro_batch * c.seq_len)
     tr_path = os.path.join(ROOT, "profiles", tr_name) if tr_name else ""
     tr_n = 0
     if tr_path and os.path.exists(tr_path):
