@@ -37,3 +37,11 @@ us = t(lambda: (lambda i: kt.layernorm_fwd(BF16, xs[i], g, bb, ys[i], mu, rs, T,
 print(f"ln_fwd   cold {us:7.1f} us  {2*T*h*2/us/1e3:7.1f} GB/s")
 us = t(lambda: (lambda i: kt.layernorm_bwd(BF16, dys[i], xs[i], g, mu, rs, dres, dxs[i], dg, db, T, h))(nxt()))
 print(f"ln_bwd   cold {us:7.1f} us  {4*T*h*2/us/1e3:7.1f} GB/s (dx + param grads)")
+# cross entropy over the LM-head logits of one microbatch (in place)
+Vv, s_ = 50304, 1024
+rows_ce = T
+z = mk(rows_ce, Vv)
+tok = torch.randint(0, Vv, (rows_ce // s_, s_ + 1), device="cuda", dtype=torch.int32)
+lr_ = torch.empty(rows_ce, device="cuda")
+us = t(lambda: kt.cross_entropy(BF16, z, tok, lr_, rows_ce, Vv, s_, 1.0 / rows_ce), it=5)
+print(f"cross_entropy {us:7.1f} us  {2*rows_ce*Vv*2/us/1e3:7.1f} GB/s (1 read + 1 write of the logits)")
