@@ -183,6 +183,7 @@ struct mobius_ctx {
   uint8_t* keep_pool = nullptr;   // kept activations (no recompute) for some stages
   int64_t keep_bytes = 0;
   std::vector<int64_t> keep_off;  // per local stage: offset into keep_pool, -1 if not kept
+  std::vector<int> keep_nb;       // per local stage: kept blocks (its LAST keep_nb blocks; the rest recomputed)
   int64_t acts_bytes = 0;
   int64_t keep_acts_bytes = 0;  // per kept block-microbatch (compact layout on the bf16 flash path)
   bool keep_compact = false;
@@ -387,11 +388,13 @@ struct StepRunner {
     return tptr<T>(b + pi.off_gslot + ((int64_t)pv.ord * pi.M + m) * pi.slot_bytes);
   }
 
+  // a stage keeps the activations of its last keep_nb blocks (all of them
+  // when the budget allows, reading #17); blocks before kf(ls) are recomputed
   bool kept(int ls) const { return ctx->keep_off[ls] >= 0; }
+  int kf(int ls) const { return ctx->all[ctx->mine[ls]].n_blocks - ctx->keep_nb[ls]; }
   uint8_t* keep_entry(int ls, int m, int bi) {
-    const StageDesc& st = ctx->all[ctx->mine[ls]];
     const int64_t e = ctx->keep_acts_bytes + ctx->slot_bytes;
-    return ctx->keep_pool + ctx->keep_off[ls] + ((int64_t)m * st.n_blocks + bi) * e;
+    return ctx->keep_pool + ctx->keep_off[ls] + ((int64_t)m * ctx->keep_nb[ls] + (bi - kf(ls))) * e;
   }
   // input x of block bi of a kept stage (block 0 of an embed stage too)
   T* keep_x(int ls, int m, int bi) { return tptr<T>(keep_entry(ls, m, bi) + ctx->keep_acts_bytes); }
@@ -493,7 +496,7 @@ struct StepRunner {
       if (st.n_blocks == 0 && !last_stage)
         out = fwd_dest(st.j, m, &flag);
       else
-        out = kept(ls) ? keep_x(ls, m, 0) : xbuf(0);
+        out = (kept(ls) && kf(ls) == 0) ? keep_x(ls, m, 0) : xbuf(0);
       RC(embed_layer_fwd<T>(sh, stage_w(res, st, 0), tok(m), out, s));
       if (flag) { RC(flag_set(flag, (int)seq, s)); ++ctx->launches_step; }
       x = out;
@@ -508,7 +511,7 @@ struct StepRunner {
       if (li == 0) continue;
       const bool last_block = (bi == st.n_blocks - 1);
       int* flag = nullptr;
-      if (kept(ls)) {  // keep every activation of this stage for its backward (no recompute)
+      if (kept(ls) && bi >= kf(ls)) {  // keep this block's activations for its backward (no recompute)
         T* y = last_block ? fwd_dest(st.j, m, &flag) : keep_x(ls, m, bi + 1);
         BlockActs<T> ka = keep_acts(ls, m, bi);
         ka.x = x;
@@ -518,7 +521,8 @@ struct StepRunner {
         ++bi;
         continue;
       }
-      T* y = last_block ? fwd_dest(st.j, m, &flag) : xbuf(1 + (bi % 2));
+      T* y = last_block ? fwd_dest(st.j, m, &flag)
+                        : (kept(ls) && bi + 1 == kf(ls)) ? keep_x(ls, m, bi + 1) : xbuf(1 + (bi % 2));
       acts[0].x = x;
       RC(block_fwd<T>(sh, stage_w(res, st, li), acts[0], y, sc, s));
       if (flag) { RC(flag_set(flag, (int)seq, s)); ++ctx->launches_step; }
@@ -537,10 +541,28 @@ struct StepRunner {
     const T* x;
     int bi = 0;
     std::vector<BlockActs<T>> kacts;
-    if (kept(ls)) {  // activations kept from F_{j,m}: no recompute
-      for (int b = 0; b < st.n_blocks; ++b) {
+    if (kept(ls)) {  // activations of blocks >= kf kept from F_{j,m}: no recompute for them
+      const int k0 = kf(ls);
+      for (int b = k0; b < st.n_blocks; ++b) {
         kacts.push_back(keep_acts(ls, m, b));
         kacts.back().x = (b == 0) ? (st.has_embed ? keep_x(ls, m, 0) : ckpt_slot(ls, m)) : keep_x(ls, m, b);
+      }
+      if (k0 > 0) {  // recompute blocks [0, k0) from the stage input (their outputs match the kept inputs)
+        if (st.has_embed) {
+          RC(embed_layer_fwd<T>(sh, stage_w(res, st, 0), tok(m), xbuf(0), s));
+          x = xbuf(0);
+        } else {
+          x = ckpt_slot(ls, m);
+        }
+        int b = 0;
+        for (int li = st.first; li < st.last && b < k0; ++li) {
+          if (li == 0 || li == ctx->cfg.n_layers + 1) continue;
+          T* y = xbuf(b + 1);
+          acts[b].x = x;
+          RC(block_fwd<T>(sh, stage_w(res, st, li), acts[b], y, sc, s));
+          x = y;
+          ++b;
+        }
       }
       bi = st.n_blocks;
       x = nullptr;  // the head is never in a kept stage
@@ -591,7 +613,8 @@ struct StepRunner {
         pp ^= 1;
       }
       float* G = ctx->grad_acc + st.layer_off[li - st.first];
-      RC(block_bwd<T>(sh, stage_w(res, st, li), kept(ls) ? kacts[bi] : acts[bi], dy, dx, G, sc, s));
+      RC(block_bwd<T>(sh, stage_w(res, st, li), (kept(ls) && bi >= kf(ls)) ? kacts[bi - kf(ls)] : acts[bi], dy, dx,
+                      G, sc, s));
       if (flag) { RC(flag_set(flag, (int)seq, s)); ++ctx->launches_step; }
       dy = dx;
     }
@@ -788,8 +811,8 @@ int do_step(mobius_ctx* ctx, const int32_t* tok_dev, int M, float* loss_out) {
   S.n_local_stages = (int)ctx->mine.size();
   S.recompute = 0;
   for (int ls = 0; ls < (int)ctx->mine.size(); ++ls)
-    if (ctx->keep_off[ls] < 0 && ctx->mine[ls] != ctx->plan.n_stages - 1 && ctx->all[ctx->mine[ls]].n_blocks > 0)
-      S.recompute += ctx->all[ctx->mine[ls]].n_blocks;  // this stage's blocks are recomputed in backward
+    if (ctx->mine[ls] != ctx->plan.n_stages - 1 && ctx->all[ctx->mine[ls]].n_blocks > 0)
+      S.recompute += ctx->all[ctx->mine[ls]].n_blocks - ctx->keep_nb[ls];  // blocks recomputed in backward
   ctx->upd_ns = 0;
   ctx->step_count++;
   return MOBIUS_OK;
@@ -940,6 +963,7 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
     // kept activations (reading #17: keep instead of recompute when they fit):
     // whole local stages, latest first, within the free HBM minus a margin
     ctx->keep_off.assign(n, -1);
+    ctx->keep_nb.assign(n, 0);
     if (dist->flags & MOBIUS_FLAG_KEEP_ACTS) {
       size_t fr = 0, tot = 0;
       CU(cudaMemGetInfo(&fr, &tot));
@@ -950,10 +974,13 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
       for (int k = n - 1; k >= 0; --k) {
         const StageDesc& st = ctx->all[ctx->mine[k]];
         if (st.j == plan->n_stages - 1 || st.n_blocks == 0) continue;  // last stage: F is folded into B
-        const int64_t need = al256((int64_t)M * st.n_blocks * entry);
-        if (off + need > budget) continue;
+        // whole stage if it fits, else its last blocks (the rest is recomputed)
+        int nb = st.n_blocks;
+        while (nb > 0 && off + al256((int64_t)M * nb * entry) > budget) --nb;
+        if (nb == 0) continue;
         ctx->keep_off[k] = off;
-        off += need;
+        ctx->keep_nb[k] = nb;
+        off += al256((int64_t)M * nb * entry);
       }
       if (off > 0) {
         CU(cudaMalloc(&ctx->keep_pool, off));

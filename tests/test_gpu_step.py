@@ -257,6 +257,33 @@ def test_tiny_step_keep_acts(dtype, tol, sizes, layout, monkeypatch):
     assert np.isfinite(loss2)
 
 
+def test_partial_keep(monkeypatch):
+    """Keep budget between whole stages: a stage keeps its LAST blocks and
+    recomputes the first ones from its checkpoint (sizes (2, 3, 1): keepable
+    stages [embed, b1] and [b2, b3, b4]; with whole-stage keeping the
+    recompute count can only be 4, 3, 1 or 0 - 2 needs a partial stage).
+    Loss and gradients stay the oracle's for every budget."""
+    from paper_conf_asplos_fengxtwls23_b200 import FLAG_KEEP_ACTS
+    monkeypatch.delenv("MOBIUS_KEEP_FULL", raising=False)
+    c = synth.TINY
+    M = 2
+    w = synth.round_bf16(synth.perturb_norm_params(c, synth.gen_params(c), scale=0.1))
+    tok = synth.gen_tokens(c, M)
+    ref_loss, ref_g = om.reference_loss_and_grads(c, w, tok)
+    seen = set()
+    for gib in (0.001, 0.0035, 0.0065, 0.0095, 0.0125, 0.0155, 0.0185, 1.0):
+        monkeypatch.setenv("MOBIUS_KEEP_GIB", str(gib))
+        ctx = MobiusContext(mk_cfg(c, BF16), plan_from_sizes((2, 3, 1), 1, M, hbm_cap_bytes=8 * MiB), init_params=w,
+                            flags=FLAG_KEEP_ACTS)
+        loss = ctx.step(tok)
+        g = ctx.read_grads(c.n_params)
+        seen.add(ctx.stats().recompute)
+        ctx.close()
+        assert abs(loss - ref_loss) / abs(ref_loss) < 2e-2
+        assert max(tensor_errs(c, g, ref_g).values()) < 2e-2
+    assert 2 in seen and 0 in seen and 4 in seen, seen
+
+
 @pytest.mark.parametrize("dtype,tol", [(F32, 1e-5), (BF16, 2e-2)])
 def test_multistep_mobius_vs_gpipe_mode(dtype, tol):
     """SURVEY f4 / P:L596-602, Fig 13 analog without a dataset: four
