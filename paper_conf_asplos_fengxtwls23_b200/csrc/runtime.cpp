@@ -967,7 +967,12 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
     if (dist->flags & MOBIUS_FLAG_KEEP_ACTS) {
       size_t fr = 0, tot = 0;
       CU(cudaMemGetInfo(&fr, &tot));
-      int64_t budget = (int64_t)fr - (int64_t)6 * (1LL << 30);
+      // margin for what is allocated after create (Stream-K workspaces, the
+      // caller's buffers: tens of MB); MOBIUS_KEEP_MARGIN_GIB overrides the
+      // default 2.5 GiB (6 GiB cost one more recomputed block at 1.5B / mbs 32)
+      double margin_gib = 2.5;
+      if (const char* e = getenv("MOBIUS_KEEP_MARGIN_GIB")) margin_gib = std::max(0.5, atof(e));
+      int64_t budget = (int64_t)fr - (int64_t)(margin_gib * (1LL << 30));
       if (const char* e = getenv("MOBIUS_KEEP_GIB")) budget = std::min<int64_t>(budget, (int64_t)(atof(e) * (1LL << 30)));
       const int64_t entry = ctx->keep_acts_bytes + ctx->slot_bytes;
       int64_t off = 0;
