@@ -188,6 +188,7 @@ struct mobius_ctx {
   int64_t keep_acts_bytes = 0;  // per kept block-microbatch (compact layout on the bf16 flash path)
   bool keep_compact = false;
   int max_blocks = 0;
+  int ws_blocks = 0;              // recompute workspace entries (acts_base)
   uint8_t* xs_base = nullptr;     // [max_blocks+1] x buffers [T,h]
   uint8_t* scratch_base = nullptr;
   uint8_t* tok_dev = nullptr;
@@ -723,7 +724,7 @@ int do_step(mobius_ctx* ctx, const int32_t* tok_dev, int M, float* loss_out) {
   R.seq = ctx->step_count + 1;
   R.inv_ntok = 1.0f / ((float)M * sh.mbs * sh.s);
   carve_scratch<T>(sh, ctx->scratch_base, true, R.sc);
-  R.acts.resize(std::max(1, ctx->max_blocks));
+  R.acts.resize(std::max(1, ctx->ws_blocks));
   for (int i = 0; i < (int)R.acts.size(); ++i) carve_block_acts<T>(sh, ctx->acts_base + i * ctx->acts_bytes, R.acts[i]);
   ctx->trace.clear();
   ctx->timer.reset();
@@ -938,18 +939,69 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
   ctx->off_gslot = take((int64_t)n * M * ctx->slot_bytes);
   ctx->off_fflag = take((int64_t)n * M * 4);
   ctx->off_bflag = take((int64_t)n * M * 4);
-  int64_t o_acts = take(ctx->acts_bytes * std::max(1, ctx->max_blocks));
   int64_t o_xs = take(ctx->slot_bytes * (ctx->max_blocks + 3));
   int64_t o_scr = take(scratch_bytes(sh, esz, true, fl));
   int64_t o_tok = take((int64_t)M * sh.mbs * (sh.s + 1) * 4);
   int64_t o_loss = take(8);
-  ctx->arena_bytes = off;
+  const int64_t o_acts = off;  // recompute workspace last: its size depends on the keep plan
 
   int cu_dev = dist->device;
   {
     mobius_ctx* ctxp = ctx.get();
     mobius_ctx* ctx = ctxp;  // for CU()
     CU(cudaSetDevice(cu_dev));
+    // kept activations (reading #17: keep instead of recompute when they fit):
+    // whole local stages, latest first, else a stage's last blocks, within the
+    // free HBM minus a margin.  The recompute workspace (acts, full layout) is
+    // then sized by what is still recomputed - the last stage (forward folded
+    // into backward) and the non-kept blocks - instead of the largest stage;
+    // the two are solved together (the workspace only grows, a few rounds).
+    ctx->keep_off.assign(n, -1);
+    ctx->keep_nb.assign(n, 0);
+    const int64_t dev_tail_bytes = (dist->flags & MOBIUS_FLAG_DEVICE_TAIL_UPDATE) && n > 0
+        ? al256(ctx->all[ctx->mine[0]].n_params * 4) * 3 + al256(ctx->all[ctx->mine[0]].n_params * esz) : 0;
+    int ws = std::max(1, ctx->max_blocks);
+    int64_t keep_total = 0;
+    if (dist->flags & MOBIUS_FLAG_KEEP_ACTS) {
+      size_t fr = 0, tot = 0;
+      CU(cudaMemGetInfo(&fr, &tot));
+      // margin for what is allocated after create (Stream-K workspaces, the
+      // caller's buffers: tens of MB); MOBIUS_KEEP_MARGIN_GIB overrides the
+      // default 2.5 GiB (6 GiB cost one more recomputed block at 1.5B / mbs 32)
+      double margin_gib = 2.5;
+      if (const char* e = getenv("MOBIUS_KEEP_MARGIN_GIB")) margin_gib = std::max(0.5, atof(e));
+      const int64_t entry = ctx->keep_acts_bytes + ctx->slot_bytes;
+      ws = 1;
+      for (int k = 0; k < n; ++k)
+        if (ctx->all[ctx->mine[k]].j == plan->n_stages - 1) ws = std::max(ws, ctx->all[ctx->mine[k]].n_blocks);
+      for (int round = 0; round < 8; ++round) {
+        int64_t budget = (int64_t)fr - o_acts - al256(ctx->acts_bytes * ws) - dev_tail_bytes -
+                         (int64_t)(margin_gib * (1LL << 30));
+        if (const char* e = getenv("MOBIUS_KEEP_GIB"))
+          budget = std::min<int64_t>(budget, (int64_t)(atof(e) * (1LL << 30)));
+        int64_t koff = 0;
+        int need_ws = ws;
+        for (int k = n - 1; k >= 0; --k) {
+          const StageDesc& st = ctx->all[ctx->mine[k]];
+          ctx->keep_off[k] = -1;
+          ctx->keep_nb[k] = 0;
+          if (st.j == plan->n_stages - 1 || st.n_blocks == 0) continue;  // last stage: F is folded into B
+          // whole stage if it fits, else its last blocks (the rest is recomputed)
+          int nb = st.n_blocks;
+          while (nb > 0 && koff + al256((int64_t)M * nb * entry) > budget) --nb;
+          need_ws = std::max(need_ws, st.n_blocks - nb);
+          if (nb == 0) continue;
+          ctx->keep_off[k] = koff;
+          ctx->keep_nb[k] = nb;
+          koff += al256((int64_t)M * nb * entry);
+        }
+        keep_total = koff;
+        if (need_ws <= ws) break;
+        ws = need_ws;
+      }
+    }
+    ctx->ws_blocks = ws;
+    ctx->arena_bytes = o_acts + al256(ctx->acts_bytes * ws);
     CU(cudaMalloc(&ctx->arena, ctx->arena_bytes));
     CU(cudaMemset(ctx->arena + o_gacc, 0, max_params * 4));
     ctx->ring = ctx->arena;
@@ -960,37 +1012,9 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
       CU(cudaMalloc(&ctx->d_opt, ctx->d_opt_stride * 4 * 3));
       CU(cudaMalloc(&ctx->d_wstage, al256(np0 * esz)));
     }
-    // kept activations (reading #17: keep instead of recompute when they fit):
-    // whole local stages, latest first, within the free HBM minus a margin
-    ctx->keep_off.assign(n, -1);
-    ctx->keep_nb.assign(n, 0);
-    if (dist->flags & MOBIUS_FLAG_KEEP_ACTS) {
-      size_t fr = 0, tot = 0;
-      CU(cudaMemGetInfo(&fr, &tot));
-      // margin for what is allocated after create (Stream-K workspaces, the
-      // caller's buffers: tens of MB); MOBIUS_KEEP_MARGIN_GIB overrides the
-      // default 2.5 GiB (6 GiB cost one more recomputed block at 1.5B / mbs 32)
-      double margin_gib = 2.5;
-      if (const char* e = getenv("MOBIUS_KEEP_MARGIN_GIB")) margin_gib = std::max(0.5, atof(e));
-      int64_t budget = (int64_t)fr - (int64_t)(margin_gib * (1LL << 30));
-      if (const char* e = getenv("MOBIUS_KEEP_GIB")) budget = std::min<int64_t>(budget, (int64_t)(atof(e) * (1LL << 30)));
-      const int64_t entry = ctx->keep_acts_bytes + ctx->slot_bytes;
-      int64_t off = 0;
-      for (int k = n - 1; k >= 0; --k) {
-        const StageDesc& st = ctx->all[ctx->mine[k]];
-        if (st.j == plan->n_stages - 1 || st.n_blocks == 0) continue;  // last stage: F is folded into B
-        // whole stage if it fits, else its last blocks (the rest is recomputed)
-        int nb = st.n_blocks;
-        while (nb > 0 && off + al256((int64_t)M * nb * entry) > budget) --nb;
-        if (nb == 0) continue;
-        ctx->keep_off[k] = off;
-        ctx->keep_nb[k] = nb;
-        off += al256((int64_t)M * nb * entry);
-      }
-      if (off > 0) {
-        CU(cudaMalloc(&ctx->keep_pool, off));
-        ctx->keep_bytes = off;
-      }
+    if (keep_total > 0) {
+      CU(cudaMalloc(&ctx->keep_pool, keep_total));
+      ctx->keep_bytes = keep_total;
     }
     ctx->grad_acc = reinterpret_cast<float*>(ctx->arena + o_gacc);
     ctx->grad_stage = ctx->arena + o_gstage;
