@@ -1,21 +1,30 @@
 // Fused causal attention (flash-style) on tcgen05 for sm_100a (SURVEY
 // §8(f) f1; replaces the materialised S / P of K3/K4).
 //
-// Forward, one CTA per (batch, head, 128-query tile):
-//   warp 0     TMA producer: Q once, then K_j / V_j tiles (2-stage ring)
-//   warp 1     MMA issuer:   S_j = Q K_j^T  -> TMEM (double buffered)
-//                            O_j = P_j V_j  -> TMEM (double buffered, fresh per tile)
-//   warps 2-5  softmax:      thread = query row; online max / sum in the log2
-//                            domain, P_j (bf16) -> smem (UMMA K-major SW128
-//                            layout), O_reg = O_reg * 2^(a_{j-2}-a_{j-1}) + O_{j-1}
-//                            merged from TMEM; writes O (bf16) and lse (log2).
-// Backward, one CTA per (batch, head, 128-key tile), loop over query tiles
-// i >= j:  S^T = K Q_i^T, dP^T = V dO_i^T (TMEM); thread = key row computes
-// P^T = 2^(S^T*c - lse_q), dS^T = P^T (dP^T - D_q) into smem; then
-// dV += P^T dO_i, dK += dS^T Q_i (TMEM accumulators), dQ_i = dS K_j (TMEM,
-// TMA reduce-add into an fp32 dQ buffer); the 1/sqrt(dh) of dS is applied to
-// dK at its store and to dQ in the final cast.  The same smem tiles serve as
-// K-major and MN-major UMMA operands, so no transposes are materialised.
+// Both kernels are persistent (one CTA per SM walking a heaviest-first item
+// list in snake order) with warp-specialised roles and mbarrier hand-offs.
+//
+// Forward, item = (batch, head, 128-query tile):
+//   warp 0     TMA producer: Q (double buffered across items), K_j / V_j
+//              tiles through a 4-deep ring (dh 64)
+//   warp 1     MMA issuer:   S_j = Q K_j^T -> TMEM (double buffered);
+//                            O += P_j V_j  -> TMEM (O double buffered across
+//                            items; dh 64: P_j from TMEM as a TS-MMA operand)
+//   warps 2-9  softmax:      (lane quadrant x column half) per S row; online
+//                            max / sum in the log2 domain, lazy O rescale,
+//                            P_j (bf16) -> TMEM (dh 64) or smem (dh 128); the
+//                            O / l read-out of an item is deferred until the
+//                            next item's first P tile is issued and leaves
+//                            through smem + TMA stores (dh 64); writes lse.
+// Backward, item = (batch, head, 128-key tile kt), query tiles i >= kt:
+//   S^T = K Q_i^T, dP^T = V dO_i^T (TMEM); thread = key row computes
+//   P^T = 2^(S^T*c - lse_q) (-> TMEM, dh 64) and dS^T = P^T (dP^T - D_q)
+//   (-> smem); then dV += P^T dO_i, dK += dS^T Q_i (TMEM accumulators),
+//   dQ_i = dS K_j (TMEM, drained one tile behind by TMA reduce-add into an
+//   fp32 buffer); the 1/sqrt(dh) of dS is applied to dK at its store and to
+//   dQ in the final cast; dV / dK leave through smem + TMA stores.  The same
+//   smem tiles serve as K-major and MN-major UMMA operands, so no transposes
+//   are materialised.
 #include <cuda.h>
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
@@ -523,10 +532,7 @@ struct BwdCfg {
 struct BwdParams {
   const float* lse;     // [mbs, nh, s] log2 domain
   const float* Dsum;    // [mbs, nh, s] -rowsum(dO * O) (negated)
-  float* dQacc;         // [mbs*s, h] fp32 (head view), accumulated with red.add
-  __nv_bfloat16* dK;    // head view into dqkv (k part)
-  __nv_bfloat16* dV;    // head view into dqkv (v part)
-  int64_t ldd;          // row stride of dK/dV (3h)
+  float* dQacc;         // [mbs*s, h] fp32 (head view), accumulated by TMA reduce-add
   int s, nh, h, mbs;
   float scale_log2, scale;
 };
@@ -1128,9 +1134,6 @@ int flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* o, const __nv_
   p.lse = lse;
   p.Dsum = dsum_ws;
   p.dQacc = dq_ws;
-  p.dK = dqkv + h;
-  p.dV = dqkv + 2 * h;
-  p.ldd = 3 * h;
   p.s = s;
   p.nh = nh;
   p.h = h;
