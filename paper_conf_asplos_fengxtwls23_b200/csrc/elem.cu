@@ -836,11 +836,12 @@ int cast_from_f32(const float* src, T* dst, int64_t n, cudaStream_t st) {
 }
 
 namespace {
-__device__ __forceinline__ float gelu_tanh_approx(float u) {  // == gemm_common.cuh gelu_f
-  const float c = 0.7978845608028654f, a = 0.044715f;
+__device__ __forceinline__ float gelu_tanh_approx(float u) {  // == gemm_common.cuh gelu_f (same ops)
+  const float c = 0.7978845608028654f, ca = 0.7978845608028654f * 0.044715f;
   float t;
-  asm("tanh.approx.f32 %0, %1;" : "=f"(t) : "f"(c * (u + a * u * u * u)));
-  return 0.5f * u * (1.f + t);
+  asm("tanh.approx.f32 %0, %1;" : "=f"(t) : "f"(u * fmaf(ca, u * u, c)));
+  const float hu = 0.5f * u;
+  return fmaf(hu, t, hu);
 }
 __global__ void gelu_fwd_k(const uint4* __restrict__ u, uint4* __restrict__ g, int64_t n8) {
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n8; i += (int64_t)gridDim.x * blockDim.x) {

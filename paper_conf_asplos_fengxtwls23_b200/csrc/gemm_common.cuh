@@ -69,10 +69,14 @@ __device__ __forceinline__ float tanh_fast(float x) {
   asm("tanh.approx.f32 %0, %1;" : "=f"(y) : "f"(x));
   return y;
 }
+// tanh GeLU, 0.5 u (1 + tanh(c (u + a u^3))), in FMA form: u (c + c a u^2)
+// then 0.5u + 0.5u t (5 FP32 ops + one MUFU.TANH per element; the epilogue
+// of the bias+GeLU forward GEMM evaluates it for every output element)
 __device__ __forceinline__ float gelu_f(float u) {
-  const float c = 0.7978845608028654f, a = 0.044715f;
-  float t = tanh_fast(c * (u + a * u * u * u));
-  return 0.5f * u * (1.f + t);
+  const float c = 0.7978845608028654f, ca = 0.7978845608028654f * 0.044715f;
+  const float t = tanh_fast(u * fmaf(ca, u * u, c));
+  const float hu = 0.5f * u;
+  return fmaf(hu, t, hu);
 }
 __device__ __forceinline__ float gelu_grad_f(float u) {
   const float c = 0.7978845608028654f, a = 0.044715f;
