@@ -250,7 +250,7 @@ __device__ __forceinline__ uint4 pack8(const float* f) {
 }
 
 template <int NV>
-__global__ void __launch_bounds__(256, 4) ln_fwd_bf16_k(const __nv_bfloat16* __restrict__ x,
+__global__ void __launch_bounds__(256, 3) ln_fwd_bf16_k(const __nv_bfloat16* __restrict__ x,
                                                      const __nv_bfloat16* __restrict__ g,
                                                      const __nv_bfloat16* __restrict__ b, __nv_bfloat16* __restrict__ y,
                                                      float* mu_out, float* rstd_out, int rows, int h) {
@@ -263,44 +263,53 @@ __global__ void __launch_bounds__(256, 4) ln_fwd_bf16_k(const __nv_bfloat16* __r
 #pragma unroll
   for (int k = 0; k < NV; ++k)
     if (lane + 32 * k < nvec) xv[k] = xr[lane + 32 * k];
-  float sum = 0.f;
+  // packed f32x2 arithmetic (FADD2 / FFMA2 / FMUL2): the kernel is
+  // instruction-issue bound (25.5 us warm vs 27 us cold at 16384 x 1600)
+  float2 s2 = make_float2(0.f, 0.f);
 #pragma unroll
   for (int k = 0; k < NV; ++k)
     if (lane + 32 * k < nvec) {
-      float f[8];
-      unpack8(xv[k], f);
+      const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&xv[k]);
 #pragma unroll
-      for (int e = 0; e < 8; ++e) sum += f[e];
+      for (int i = 0; i < 4; ++i) s2 = __fadd2_rn(s2, __bfloat1622float2(h2[i]));
     }
-  const float m = warp_sum(sum) / h;
-  float q = 0.f;
+  const float m = warp_sum(s2.x + s2.y) / h;
+  const float2 nm2 = make_float2(-m, -m);
+  float2 q2 = make_float2(0.f, 0.f);
 #pragma unroll
   for (int k = 0; k < NV; ++k)
     if (lane + 32 * k < nvec) {
-      float f[8];
-      unpack8(xv[k], f);
+      const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&xv[k]);
 #pragma unroll
-      for (int e = 0; e < 8; ++e) {
-        const float d = f[e] - m;
-        q += d * d;
+      for (int i = 0; i < 4; ++i) {
+        const float2 d = __fadd2_rn(__bfloat1622float2(h2[i]), nm2);
+        q2 = __ffma2_rn(d, d, q2);
       }
     }
-  const float rs = rsqrtf(warp_sum(q) / h + 1e-5f);
+  const float rs = rsqrtf(warp_sum(q2.x + q2.y) / h + 1e-5f);
   if (lane == 0) {
     mu_out[r] = m;
     rstd_out[r] = rs;
   }
+  const float2 rs2 = make_float2(rs, rs);
   uint4* yr = reinterpret_cast<uint4*>(y + (int64_t)r * h);
 #pragma unroll
   for (int k = 0; k < NV; ++k)
     if (lane + 32 * k < nvec) {
-      float f[8], gg[8], bb[8], o[8];
-      unpack8(xv[k], f);
-      unpack8(__ldg(reinterpret_cast<const uint4*>(g) + lane + 32 * k), gg);
-      unpack8(__ldg(reinterpret_cast<const uint4*>(b) + lane + 32 * k), bb);
+      const uint4 gu = __ldg(reinterpret_cast<const uint4*>(g) + lane + 32 * k);
+      const uint4 bu = __ldg(reinterpret_cast<const uint4*>(b) + lane + 32 * k);
+      const __nv_bfloat162* x2 = reinterpret_cast<const __nv_bfloat162*>(&xv[k]);
+      const __nv_bfloat162* g2 = reinterpret_cast<const __nv_bfloat162*>(&gu);
+      const __nv_bfloat162* b2 = reinterpret_cast<const __nv_bfloat162*>(&bu);
+      uint4 ov;
+      __nv_bfloat162* o2 = reinterpret_cast<__nv_bfloat162*>(&ov);
 #pragma unroll
-      for (int e = 0; e < 8; ++e) o[e] = (f[e] - m) * rs * gg[e] + bb[e];
-      yr[lane + 32 * k] = pack8(o);
+      for (int i = 0; i < 4; ++i) {
+        const float2 t = __fmul2_rn(__fadd2_rn(__bfloat1622float2(x2[i]), nm2), rs2);
+        const float2 o = __ffma2_rn(t, __bfloat1622float2(g2[i]), __bfloat1622float2(b2[i]));
+        o2[i] = __floats2bfloat162_rn(o.x, o.y);
+      }
+      yr[lane + 32 * k] = ov;
     }
 }
 
