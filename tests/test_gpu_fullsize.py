@@ -135,3 +135,41 @@ def test_full_1p5b_step_properties():
     h2d, d2h, _ = osch.byte_counts(ss, sg, M, [s["Xf"] for s in ss], n_gpus=1)
     assert st.h2d_bytes == h2d[0] == plan.h2d_bytes[0]
     assert st.d2h_bytes == d2h[0]
+
+
+def test_bench_launch_config_step_properties():
+    """The bench's launch configuration (BASELINE configs[1], bench.py
+    defaults): GPT-1.5B, mbs 32 x M 4, 1 GiB stage ring, kept activations
+    and the device tail update.  Properties that hold at this size: the init
+    loss equals its closed form, the loss falls, the schedule trace is Fig 4's,
+    and every stage byte the paper's O-10 count moves over the host link
+    either still does or (first stage, from step 2) is served device-to-device."""
+    import dataclasses
+    from paper_conf_asplos_fengxtwls23_b200 import FLAG_DEVICE_TAIL_UPDATE, FLAG_KEEP_ACTS
+    c = dataclasses.replace(synth.GPT_1_5B, micro_batch=32)
+    M = 4
+    cfg = model_cfg(c.n_layers, c.hidden, c.n_heads, c.seq_len, c.vocab, c.micro_batch, dtype=BF16)
+    prof = mobius_profile(cfg, 0)
+    plan = mobius_plan(prof, 1, 1 << 30, M, make_topology([0], 55 * 10 ** 9, 0))
+    K = plan.n_stages
+    ctx = MobiusContext(cfg, plan, seed=1234, flags=FLAG_KEEP_ACTS | FLAG_DEVICE_TAIL_UPDATE)
+    tok = synth.gen_tokens(c, M)
+    l1 = ctx.step(tok)
+    trace = ctx.read_trace()
+    st1 = ctx.stats()
+    l2 = ctx.step(tok)
+    st2 = ctx.stats()
+    l3 = ctx.step(tok)
+    ctx.close()
+    expect = math.log(c.vocab) + c.hidden * 0.02 ** 2 / 2
+    assert abs(l1 - expect) < 0.05, (l1, expect)
+    assert l2 < l1 and np.isfinite(l3), (l1, l2, l3)
+    assert trace == osch.per_gpu_ops([0] * K, M)[0]
+    sizes = [plan.stage_first_layer[j + 1] - plan.stage_first_layer[j] for j in range(K)]
+    sz = mobius_layer_sizes(cfg)
+    layers = [op.LayerProfile(0, 0, p.mem_fwd, p.mem_bwd, p.xfer_fwd, p.xfer_bwd, p.act_out) for p in sz]
+    ss = op.stage_sums(layers, sizes)
+    h2d, d2h, _ = osch.byte_counts(ss, [0] * K, M, [s["Xf"] for s in ss], n_gpus=1)
+    assert st1.h2d_bytes == h2d[0] and st1.d2d_bytes == 0
+    assert st2.h2d_bytes + st2.d2d_bytes == h2d[0] and st2.d2d_bytes > 0
+    assert st1.recompute <= 2  # nearly every block's activations kept (reading #17)
