@@ -222,7 +222,8 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
-  const uint32_t tmem = *tmem_slot;
+  const uint32_t tmem_k = *tmem_slot;
+  const uint32_t tmem = tmem_k;
   // TMEM: S[2] at 0 / 128, O[2] at 256 / 256 + DH, P[2] at 384 / 448 (dh 64)
   if (warp == 0) {
     if (lane == 0) {
@@ -255,7 +256,8 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
       }
     }
   } else if (warp == 1) {
-    if (lane == 0) {
+    {  // whole warp, converged: every MMA / commit is issued by one elected lane (ptx::*_w)
+      const uint32_t tmem = __shfl_sync(0xffffffffu, tmem_k, 0);  // warp-uniform TMEM base
       constexpr uint32_t ID_S = ptx::idesc_bf16(BQ, BKV, 0, 0);
       constexpr uint32_t ID_O = ptx::idesc_bf16(BQ, DH, 0, 1);
       int gs = 0, gp = 0, it = 0;  // global S-issue step, global PV step, local item count
@@ -276,12 +278,12 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
 #pragma unroll
           for (int k = 0; k < DH / 16; ++k) {
             const uint32_t off = (k >> 2) * 16384 + (k & 3) * 32;
-            ptx::mma_bf16(tmem + sb * 128, ptx::sdesc_sw128(aq + off, 16, 1024), ptx::sdesc_sw128(ak + off, 16, 1024),
+            ptx::mma_bf16_w(tmem + sb * 128, ptx::sdesc_sw128(aq + off, 16, 1024), ptx::sdesc_sw128(ak + off, 16, 1024),
                           ID_S, k > 0);
           }
-          ptx::mma_commit(&s_full[sb]);
-          ptx::mma_commit(&k_empty[st]);
-          if (last) ptx::mma_commit(&q_empty[ob]);
+          ptx::mma_commit_w(&s_full[sb]);
+          ptx::mma_commit_w(&k_empty[st]);
+          if (last) ptx::mma_commit_w(&q_empty[ob]);
           ++gs;
         };
         issue_s(nkv == 1);
@@ -296,21 +298,21 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
           if constexpr (C::P_TMEM) {
 #pragma unroll
             for (int k = 0; k < BKV / 16; ++k)  // 16 keys = 8 packed TMEM columns of P
-              ptx::mma_bf16_ts(tmem + 256 + ob * DH, tmem + 384 + pb * 64 + 8 * k,
+              ptx::mma_bf16_ts_w(tmem + 256 + ob * DH, tmem + 384 + pb * 64 + 8 * k,
                                ptx::sdesc_sw128(av + k * 2048, 16384, 1024), ID_O, (j > 0 || k > 0) ? 1u : 0u);
           } else {
 #pragma unroll
             for (int k = 0; k < BKV / 16; ++k) {
               const uint32_t offp = (k >> 2) * 16384 + (k & 3) * 32;
-              ptx::mma_bf16(tmem + 256 + ob * DH, ptx::sdesc_sw128(ap + offp, 16, 1024),
+              ptx::mma_bf16_w(tmem + 256 + ob * DH, ptx::sdesc_sw128(ap + offp, 16, 1024),
                             ptx::sdesc_sw128(av + k * 2048, 16384, 1024), ID_O, (j > 0 || k > 0) ? 1u : 0u);
             }
           }
-          ptx::mma_commit(&pv_done[pb]);
-          ptx::mma_commit(&v_empty[st]);
+          ptx::mma_commit_w(&pv_done[pb]);
+          ptx::mma_commit_w(&v_empty[st]);
           ++gp;
         }
-        ptx::mma_commit(&o_ready[ob]);
+        ptx::mma_commit_w(&o_ready[ob]);
         ++it;
       }
     }
@@ -667,7 +669,12 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
       }
     }
   } else if (warp == 1) {
-    if (lane == 0) {
+    {  // whole warp, converged: every MMA / commit is issued by one elected lane (ptx::*_w)
+      // TMEM addresses re-derived from a shuffled (provably warp-uniform) base so
+      // the MMA operands live in uniform registers (no per-MMA waterfall loop)
+      const uint32_t T_S = __shfl_sync(0xffffffffu, tmem, 0), T_DP = T_S + 128, T_DV = T_S + 256;
+      const uint32_t T_DQ = C::DQ_OWN ? T_S + 384 : T_S;
+      const uint32_t T_PT = T_S + 448;
       constexpr uint32_t ID_ST = ptx::idesc_bf16(128, 128, 0, 0);  // S^T, dP^T
       constexpr uint32_t ID_DV = ptx::idesc_bf16(128, DH, 0, 1);   // dV, dK
       constexpr uint32_t ID_DQ = ptx::idesc_bf16(128, DH, 1, 1);   // dQ
@@ -682,15 +689,15 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
 #pragma unroll
         for (int t = 0; t < DH / 16; ++t) {
           const uint32_t off = (t >> 2) * 16384 + (t & 3) * 32;
-          ptx::mma_bf16(T_S, ptx::sdesc_sw128(ak + off, 16, 1024), ptx::sdesc_sw128(aq + off, 16, 1024), ID_ST, t > 0);
+          ptx::mma_bf16_w(T_S, ptx::sdesc_sw128(ak + off, 16, 1024), ptx::sdesc_sw128(aq + off, 16, 1024), ID_ST, t > 0);
         }
 #pragma unroll
         for (int t = 0; t < DH / 16; ++t) {
           const uint32_t off = (t >> 2) * 16384 + (t & 3) * 32;
-          ptx::mma_bf16(T_DP, ptx::sdesc_sw128(av + off, 16, 1024), ptx::sdesc_sw128(ado + off, 16, 1024), ID_ST,
+          ptx::mma_bf16_w(T_DP, ptx::sdesc_sw128(av + off, 16, 1024), ptx::sdesc_sw128(ado + off, 16, 1024), ID_ST,
                         t > 0);
         }
-        ptx::mma_commit(s_full);
+        ptx::mma_commit_w(s_full);
       };
       int g = 0, n = 0;
       for (int pass = 0; pass * ncta < n_items; ++pass) {
@@ -711,7 +718,8 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
           if (C::DQ_OWN && it + 1 < nq) {
             ptx::mbar_wait(st_empty, gg & 1);
             const int sn = (gg + 1) % QS;
-            if (ptx::mbar_test(&q_full[sn], ((gg + 1) / QS) & 1)) {
+            const bool landed = __shfl_sync(0xffffffffu, (int)ptx::mbar_test(&q_full[sn], ((gg + 1) / QS) & 1), 0);
+            if (landed) {  // warp-uniform decision
               issue_st(gg + 1);
               st_next = true;
             }
@@ -723,42 +731,42 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
             const uint32_t ads = ptx::smem_u32(sdS_buf[gg & 1]);
 #pragma unroll
             for (int t = 0; t < 128 / 16; ++t)  // dV += P^T dO, P^T from TMEM (8 columns per 16 queries)
-              ptx::mma_bf16_ts(T_DV, T_PT + 8 * t, ptx::sdesc_sw128(ado + t * 2048, 16384, 1024), ID_DV,
+              ptx::mma_bf16_ts_w(T_DV, T_PT + 8 * t, ptx::sdesc_sw128(ado + t * 2048, 16384, 1024), ID_DV,
                                (it > 0 || t > 0) ? 1u : 0u);
-            ptx::mma_commit(pt_free);
+            ptx::mma_commit_w(pt_free);
 #pragma unroll
             for (int t = 0; t < 128 / 16; ++t) {  // dK += dS^T Q
               const uint32_t offa = (t >> 2) * 16384 + (t & 3) * 32;
-              ptx::mma_bf16(T_DV + DH, ptx::sdesc_sw128(ads + offa, 16, 1024), ptx::sdesc_sw128(aq + t * 2048, 16384, 1024),
+              ptx::mma_bf16_w(T_DV + DH, ptx::sdesc_sw128(ads + offa, 16, 1024), ptx::sdesc_sw128(aq + t * 2048, 16384, 1024),
                             ID_DV, (it > 0 || t > 0) ? 1u : 0u);
             }
-            ptx::mma_commit(&q_empty[st]);  // last reads of Q / dO (dQ needs only dS and K): refill the slot now
+            ptx::mma_commit_w(&q_empty[st]);  // last reads of Q / dO (dQ needs only dS and K): refill the slot now
             if (gg >= 1) ptx::mbar_wait(dq_empty, (gg - 1) & 1);  // dQ(gg-1) read out
 #pragma unroll
             for (int t = 0; t < 128 / 16; ++t)  // K = 128 keys: dQ = dS K
-              ptx::mma_bf16(T_DQ, ptx::sdesc_sw128(ads + t * 2048, 16384, 1024),
+              ptx::mma_bf16_w(T_DQ, ptx::sdesc_sw128(ads + t * 2048, 16384, 1024),
                             ptx::sdesc_sw128(ak + t * 2048, 16384, 1024), ID_DQ, t > 0);
           } else {
 #pragma unroll
             for (int t = 0; t < 128 / 16; ++t) {  // K = 128 queries
               const uint32_t offa = (t >> 2) * 16384 + (t & 3) * 32;
-              ptx::mma_bf16(T_DV, ptx::sdesc_sw128(apt + offa, 16, 1024), ptx::sdesc_sw128(ado + t * 2048, 16384, 1024),
+              ptx::mma_bf16_w(T_DV, ptx::sdesc_sw128(apt + offa, 16, 1024), ptx::sdesc_sw128(ado + t * 2048, 16384, 1024),
                             ID_DV, (it > 0 || t > 0) ? 1u : 0u);  // dV += P^T dO
-              ptx::mma_bf16(T_DV + DH, ptx::sdesc_sw128(adst + offa, 16, 1024),
+              ptx::mma_bf16_w(T_DV + DH, ptx::sdesc_sw128(adst + offa, 16, 1024),
                             ptx::sdesc_sw128(aq + t * 2048, 16384, 1024), ID_DV, (it > 0 || t > 0) ? 1u : 0u);  // dK += dS^T Q
             }
-            ptx::mma_commit(&q_empty[st]);  // last reads of Q / dO
+            ptx::mma_commit_w(&q_empty[st]);  // last reads of Q / dO
             if (C::DQ_OWN && gg >= 1) ptx::mbar_wait(dq_empty, (gg - 1) & 1);  // dQ(gg-1) read out
 #pragma unroll
             for (int t = 0; t < 128 / 16; ++t)  // K = 128 keys: dQ = dS K
-              ptx::mma_bf16(T_DQ, ptx::sdesc_sw128(adst + t * 2048, 16384, 1024),
+              ptx::mma_bf16_w(T_DQ, ptx::sdesc_sw128(adst + t * 2048, 16384, 1024),
                             ptx::sdesc_sw128(ak + t * 2048, 16384, 1024), ID_DQ, t > 0);
           }
-          ptx::mma_commit(mm_done);
+          ptx::mma_commit_w(mm_done);
           if (C::DQ_OWN && it + 1 < nq && !st_next) issue_st(gg + 1);
           if (!C::DQ_OWN && it + 1 < nq) issue_st(gg + 1);
         }
-        ptx::mma_commit(kv_empty);
+        ptx::mma_commit_w(kv_empty);
         g += nq;
         ++n;
       }
