@@ -425,7 +425,8 @@ __global__ void __launch_bounds__(NUM_THREADS2, 1)
       }
     }
   } else if (warp == 1) {
-    if (leader && lane == 0) {  // MMA issuer (pair leader)
+    if (leader) {  // MMA issuer (pair leader): the whole warp, converged; one elected lane issues (ptx::*_w)
+      const uint32_t tmem_base_u = __shfl_sync(0xffffffffu, tmem_base, 0);  // warp-uniform
       constexpr uint32_t IDESC = ptx::idesc_bf16(BM2, BN, A_MN ? 1 : 0, B_MN ? 1 : 0);
       constexpr uint32_t IDESC_NARROW = ptx::idesc_bf16(BM2, BN / 2, A_MN ? 1 : 0, B_MN ? 1 : 0);
       const uint16_t all_mask = (uint16_t)((1u << (2 * NP)) - 1);
@@ -442,7 +443,7 @@ __global__ void __launch_bounds__(NUM_THREADS2, 1)
         const uint32_t idesc = (p.N - nt_ * BN <= BN / 2) ? IDESC_NARROW : IDESC;  // ragged last column
         ptx::mbar_wait_cluster(&tempty[acc], aphase ^ 1);
         ptx::tc_fence_after();
-        const uint32_t tmem_d = tmem_base + acc * BN;
+        const uint32_t tmem_d = tmem_base_u + acc * BN;
         for (int kb = w.k0; kb < w.k1; ++kb) {
           ptx::mbar_wait_cluster(&full[stage], phase);
           ptx::tc_fence_after();
@@ -454,17 +455,17 @@ __global__ void __launch_bounds__(NUM_THREADS2, 1)
                                : ptx::sdesc_sw128(a_base + k * 32, 16, 1024);
             uint64_t bd = B_MN ? ptx::sdesc_sw128(b_base + k * 2048, 8192, 1024)
                                : ptx::sdesc_sw128(b_base + k * 32, 16, 1024);
-            ptx::mma_bf16_2sm(tmem_d, ad, bd, idesc, (kb > w.k0 || k > 0) ? 1u : 0u);
+            ptx::mma_bf16_2sm_w(tmem_d, ad, bd, idesc, (kb > w.k0 || k > 0) ? 1u : 0u);
           }
           // the slot may be refilled by this pair's producers and (A halves)
           // by the other pair's: free it in every CTA of the cluster
-          ptx::mma_commit_2sm(&empty[stage], all_mask);
+          ptx::mma_commit_2sm_w(&empty[stage], all_mask);
           if (++stage == C::STAGES) {
             stage = 0;
             phase ^= 1;
           }
         }
-        ptx::mma_commit_2sm(&tfull[acc], pair_mask);  // accumulator ready in both CTAs of the pair
+        ptx::mma_commit_2sm_w(&tfull[acc], pair_mask);  // accumulator ready in both CTAs of the pair
         if (++acc == 2) {
           acc = 0;
           aphase ^= 1;
