@@ -97,6 +97,37 @@ def test_tiny_step_parity(dtype, tol, cap, sizes):
     assert np.max(np.abs(p1 - w1)) < 1e-6
 
 
+@pytest.mark.parametrize("M", [1, 3])
+@pytest.mark.parametrize("sizes,cap", [((1, 1, 1, 1, 1, 1), 4 * MiB), ((2, 4), 12 * MiB)])
+def test_edge_microbatches_and_max_stages(M, sizes, cap):
+    """Degenerate schedules: one microbatch (no pipelining inside a stage),
+    an odd M, and K = 6 one-layer stages (the most stages the tiny profile
+    allows; every stage swaps).  Loss, gradients, Fig 4 trace and byte
+    counters against the oracle, as in test_tiny_step_parity."""
+    c = synth.TINY
+    w = synth.round_bf16(synth.perturb_norm_params(c, synth.gen_params(c), scale=0.1))
+    tok = synth.gen_tokens(c, M)
+    plan = plan_from_sizes(sizes, 1, M, hbm_cap_bytes=cap)
+    ctx = MobiusContext(mk_cfg(c, BF16), plan, init_params=w)
+    loss = ctx.step(tok)
+    g = ctx.read_grads(c.n_params)
+    trace = ctx.read_trace()
+    st = ctx.stats()
+    ctx.close()
+    ref_loss, ref_g = om.reference_loss_and_grads(c, w, tok)
+    assert abs(loss - ref_loss) / abs(ref_loss) < 2e-2
+    errs = tensor_errs(c, g, ref_g)
+    assert rel(g, ref_g) < 2e-2 and max(errs.values()) < 2e-2, errs
+    sg = op.sequential_stage_gpu(len(sizes), 1)
+    assert trace == osch.per_gpu_ops(sg, M)[0]
+    prof = mobius_layer_sizes(mk_cfg(c, BF16))
+    layers = [op.LayerProfile(0, 0, p.mem_fwd, p.mem_bwd, p.xfer_fwd, p.xfer_bwd, p.act_out) for p in prof]
+    ss = op.stage_sums(layers, sizes)
+    h2d, d2h, _ = osch.byte_counts(ss, sg, M, [s["Xf"] for s in ss])
+    assert st.h2d_bytes == h2d[0]
+    assert st.d2h_bytes == d2h[0]
+
+
 @pytest.mark.parametrize("dtype", [BF16, F32])
 @pytest.mark.parametrize("sizes", [(3, 3), (1, 2, 1, 2)])
 def test_device_tail_update(dtype, sizes):
