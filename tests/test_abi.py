@@ -191,3 +191,20 @@ def test_fig9_baseline_partitions(mb, seed):
         r = op.stage_cost(layers, ref, N, M, G, W, W)
         assert pl.makespan_ns == r[0]
         assert mip.makespan_ns <= pl.makespan_ns
+
+
+def test_package_fails_loudly_without_library(tmp_path):
+    """No CPU or Python fallback: a copy of the package without
+    libmobius.so must refuse to import (the product path is the CUDA
+    library or nothing)."""
+    import shutil
+    import subprocess
+    import sys
+    pkg = os.path.join(ROOT, "paper_conf_asplos_fengxtwls23_b200")
+    dst = tmp_path / "paper_conf_asplos_fengxtwls23_b200"
+    shutil.copytree(pkg, dst, ignore=shutil.ignore_patterns("*.so", "csrc", "__pycache__"))
+    r = subprocess.run([sys.executable, "-c", "import paper_conf_asplos_fengxtwls23_b200"], cwd=tmp_path,
+                       capture_output=True, text=True, timeout=300,
+                       env={**os.environ, "PYTHONPATH": str(tmp_path)})
+    assert r.returncode != 0
+    assert "libmobius.so not built" in r.stderr
