@@ -139,3 +139,86 @@ def test_adamw_first_step_closed_form():
     # a constant gradient keeps m_hat = g, v_hat = g^2 -> identical steps
     w2, _, _ = oa.adamw_step(w1, m1, v1, g, 2)
     assert np.allclose(w2.astype(np.float64) - w1, expect, rtol=1e-3, atol=1e-9)
+
+
+# --- max_stage_sizes pins (Fig 9 "max-stage": "as many Transformer blocks as
+# possible without running out of memory") -------------------
+
+def _mem_layers(pairs):
+    """Profile layers with only (mem_fwd, mem_bwd) set."""
+    return [op.LayerProfile(1, 1, mf, mb, mf, mf, 1) for mf, mb in pairs]
+
+
+@pytest.mark.parametrize("pairs,G,expect", [
+    # hand-worked: forward and backward memory equal, greedy fills to G
+    ([(4, 4)] * 5, 10, (2, 2, 1)),
+    ([(3, 3), (3, 3), (4, 4), (6, 6), (1, 1)], 10, (3, 2)),
+    # mem_bwd binds, mem_fwd does not: forward sums are 2+2+2 = 6 <= 10, but
+    # backward sums 4+4 = 8, 8+4 = 12 > 10 -> the stage closes after 2 layers
+    ([(2, 4), (2, 4), (2, 4), (2, 4), (2, 4)], 10, (2, 2, 1)),
+    # mem_fwd binds, mem_bwd does not
+    ([(5, 1), (5, 1), (5, 1)], 10, (2, 1)),
+    # a stage exactly at the cap is allowed (Eq 4 is <=)
+    ([(5, 5), (5, 5), (5, 5), (5, 5)], 10, (2, 2)),
+    # every layer alone at the cap -> one layer per stage
+    ([(10, 10)] * 3, 10, (1, 1, 1)),
+])
+def test_max_stage_sizes_hand_worked(pairs, G, expect):
+    assert op.max_stage_sizes(_mem_layers(pairs), G) == expect
+
+
+@pytest.mark.parametrize("seed", range(25))
+def test_max_stage_sizes_is_fewest_stages_largest_first(seed):
+    """Brute force over all compositions: the max-stage partition is a
+    feasible partition with the fewest stages, and among those the one
+    whose stages are filled earliest (lexicographically largest sizes) -
+    what packing each stage 'as many blocks as possible' in layer order
+    means.  Independent of the greedy loop."""
+    rng = random.Random(900 + seed)
+    Lp = rng.randint(1, 9)
+    pairs = [(rng.randint(1, 9), rng.randint(1, 12)) for _ in range(Lp)]
+    G = max(max(p) for p in pairs) + rng.randint(0, 20)
+    layers = _mem_layers(pairs)
+    best = None
+    for sizes in op.compositions(Lp):
+        pos, ok = 0, True
+        for n in sizes:
+            ok &= sum(p[0] for p in pairs[pos:pos + n]) <= G and sum(p[1] for p in pairs[pos:pos + n]) <= G
+            pos += n
+        if ok:
+            key = (-len(sizes), sizes)
+            if best is None or key > best:
+                best = key
+    assert op.max_stage_sizes(layers, G) == best[1]
+
+
+# --- AdamW weight-decay pins (decoupled decay, O-4) ------------------------
+
+def test_adamw_weight_decay_zero_grad_is_pure_decay():
+    """g = 0 at step 1: m = v = 0, the Adam term is 0/(0 + eps) = 0, so the
+    step is exactly the decoupled decay w <- w - lr*wd*w."""
+    rng = np.random.default_rng(3)
+    w = rng.standard_normal(512).astype(np.float32)
+    z = np.zeros_like(w)
+    w1, m1, v1 = oa.adamw_step(w, z, z, z, 1, lr=1e-2, wd=0.1)
+    expect = w.astype(np.float64) * (1 - 1e-2 * 0.1)
+    assert np.allclose(w1, expect, rtol=1e-6, atol=0)
+    assert not m1.any() and not v1.any()
+
+
+def test_adamw_weight_decay_first_step_closed_form():
+    """Step 1 with wd != 0: dw = -lr*wd*w - lr*g/(|g| + eps) (Loshchilov &
+    Hutter's decoupled decay; the decay uses the pre-step weight)."""
+    rng = np.random.default_rng(4)
+    w = rng.standard_normal(1000).astype(np.float32)
+    g = (rng.standard_normal(1000) * 1e-3).astype(np.float32)
+    z = np.zeros_like(w)
+    lr, wd = 1e-3, 0.05
+    w1, _, _ = oa.adamw_step(w, z, z, g, 1, lr=lr, wd=wd)
+    w64, g64 = w.astype(np.float64), g.astype(np.float64)
+    expect = -lr * wd * w64 - lr * g64 / (np.abs(g64) + oa.EPS)
+    # fp32 rounding of w (|w| ~ 1) is ~6e-8 absolute; the step is ~1e-3
+    assert np.allclose(w1.astype(np.float64) - w64, expect, rtol=1e-3, atol=3e-7)
+    # and the decay term is really there: without it the result differs
+    w1_nowd, _, _ = oa.adamw_step(w, z, z, g, 1, lr=lr, wd=0.0)
+    assert np.abs(w1 - w1_nowd).max() > 10 * 3e-7
