@@ -60,6 +60,12 @@ def parse():
                     help="update the last-in-backward stage on the host too (default: GPU AdamW for it)")
     ap.add_argument("--partition", default="mip", choices=["mip", "max", "min"],
                     help="MIP (paper) or the Fig 9 max-stage / min-stage baselines")
+    ap.add_argument("--arena-cap-gib", type=float, default=0.0,
+                    help="Table 2's G as the WHOLE per-GPU memory (ring + checkpoints + workspaces): "
+                         "MOBIUS_FLAG_ARENA_CAP, planner fed G_eff = G - fixed bytes (SURVEY O-11), the paper's "
+                         "recompute and host update; survey C2 = --micro-batch 8 --arena-cap-gib 2")
+    ap.add_argument("--no-offload", action="store_true",
+                    help="with --arena-cap-gib: keep every stage-input checkpoint in HBM (no A_Mobius offload)")
     return ap.parse_args()
 
 
@@ -240,10 +246,27 @@ def run_mobius(args, rank, world, local):
     c, M = bench_workload(args, world)
     cfg = model_cfg(c.n_layers, c.hidden, c.n_heads, c.seq_len, c.vocab, c.micro_batch, dtype=BF16)
     G = int(args.cap_gib * GiB)
+    arena = args.arena_cap_gib > 0
+    arena_flags = 0
+    if arena:
+        from paper_conf_asplos_fengxtwls23_b200 import (FLAG_ARENA_CAP, FLAG_CKPT_OFFLOAD, mobius_arena_fixed_bytes,
+                                                        mobius_arena_layer_sizes)
+        arena_flags = FLAG_ARENA_CAP | (0 if (args.no_offload or world > 1) else FLAG_CKPT_OFFLOAD)
+        # G_eff = G - everything outside the ring (upper bound on the local
+        # stage count for the per-stage slot / flag arrays)
+        fixed = mobius_arena_fixed_bytes(cfg, M, c.n_layers + 2, arena_flags)
+        G = int(args.arena_cap_gib * GiB) - fixed
+        if G <= 0:
+            sys.exit(f"bench.py: --arena-cap-gib {args.arena_cap_gib}: the fixed workspaces alone need "
+                     f"{fixed / GiB:.2f} GiB")
     # profile (layer similarity) and plan (MIP + cross mapping)
     t_prof0 = time.perf_counter()
     prof = mobius_profile(cfg, local)
     prof_s = time.perf_counter() - t_prof0
+    if arena:  # whole-memory mem_fwd / mem_bwd, measured times (SURVEY O-11)
+        mem = mobius_arena_layer_sizes(cfg)
+        for p, q in zip(prof, mem):
+            p.mem_fwd, p.mem_bwd, p.xfer_fwd, p.xfer_bwd = q.mem_fwd, q.mem_bwd, q.xfer_fwd, q.xfer_bwd
     h2d_gbps = measure_h2d_GBps(torch)
     topo = mobius_discover_topology()
     groups = [topo.group[i] for i in range(topo.n_gpus)][:world]
@@ -275,6 +298,8 @@ def run_mobius(args, rank, world, local):
     timing = os.environ.get("MOBIUS_BENCH_TIMING", "1") != "0"  # per-kernel CUDA events (roofline)
     flags = (FLAG_TIMING if timing else 0) | (0 if args.no_keep else FLAG_KEEP_ACTS) | \
         (0 if args.host_tail_update else FLAG_DEVICE_TAIL_UPDATE)
+    if arena:  # the paper's regime: everything inside G, recompute, host update
+        flags = (FLAG_TIMING if timing else 0) | arena_flags
     ctx = MobiusContext(cfg, plan, rank=rank, world=world, device=local, seed=1234, flags=flags)
     if world > 1:
         blobs = [None] * world
@@ -370,7 +395,7 @@ def run_mobius(args, rank, world, local):
     # step roofline (north_star): max(FLOP / P_tc, H2D bytes / host link), per GPU
     flop_step = model_flops_per_token(c) * tokens_per_step / world
     t_tc = flop_step / (peak_tf * 1e12)
-    t_link = max(st.h2d_bytes, st.d2h_bytes) / (h2d_gbps * 1e9)
+    t_link = max(st.h2d_bytes + st.ckpt_h2d_bytes, st.d2h_bytes + st.ckpt_d2h_bytes) / (h2d_gbps * 1e9)
     t_roof = max(t_tc, t_link)
     line = None
     if rank == 0:
@@ -379,7 +404,10 @@ def run_mobius(args, rank, world, local):
             "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "bf16", "data": "synthetic (seeded GPT-shaped tokens, random-init weights)",
             "config": {"workload": f"GPT {args.config} (configs[1]): L={c.n_layers} h={c.hidden} heads={c.n_heads} "
-                                   f"s={c.seq_len} V={c.vocab}, stage ring capped at {args.cap_gib} GiB per GPU",
+                                   f"s={c.seq_len} V={c.vocab}, " +
+                                   (f"whole HBM arena capped at {args.arena_cap_gib} GiB per GPU (Table 2 G: ring + "
+                                    f"checkpoints + workspaces{', checkpoint offload' if arena_flags & 16 else ''})"
+                                    if arena else f"stage ring capped at {args.cap_gib} GiB per GPU"),
                        "model": f"gpt-{args.config}", "global_batch": M * c.micro_batch, "seq_len": c.seq_len,
                        "microbatches": M, "micro_batch": c.micro_batch, "parallelism": f"mobius-pp{world}",
                        "n_stages": plan.n_stages, "stage_layers": [plan.stage_first_layer[j + 1] - plan.stage_first_layer[j]
@@ -387,7 +415,8 @@ def run_mobius(args, rank, world, local):
                        "gpu_perm": [plan.gpu_perm[g] for g in range(world)], "plan_s": plan_s,
                        "profile_s": prof_s, "plan_exhaustive": bool(plan.exhaustive),
                        "partition": args.partition, "plan_makespan_ms": plan.makespan_ns / 1e6,
-                       "tail_stage_update": "host AdamW" if args.host_tail_update else
+                       "arena_cap_GB": args.arena_cap_gib * GiB / 1e9 if arena else None,
+                       "tail_stage_update": "host AdamW" if (args.host_tail_update or arena) else
                        "GPU AdamW (first stage, last in backward; optimizer state in HBM)",
                        "l2": "inputs larger than L2: every stage (3.1 GB bf16 total) streams from host DRAM each step"},
             "loss": loss,
@@ -417,7 +446,10 @@ def run_mobius(args, rank, world, local):
                              "update_tail": st.update_tail_ns / 1e6},
             "memory": {"arena_GB": st.arena_bytes / 1e9, "ring_GB": st.ring_bytes / 1e9,
                        "pinned_host_GB": st.pinned_bytes / 1e9, "recompute_blocks": int(st.recompute),
-                       "kept_layout": "compact (x, qkv, o, x1, u, lse, LN stats)"},
+                       "kept_layout": "none (recompute)" if (arena or args.no_keep) else
+                       "compact (x, qkv, o, x1, u, lse, LN stats)",
+                       "ckpt_offload_GB_per_step": (st.ckpt_d2h_bytes + st.ckpt_h2d_bytes) / 1e9,
+                       "exposed_ckpt_ms": st.exposed_ckpt_ns / 1e6},
             "gpu_launches": int(sum(s.kernel_launches for s in stats)),
             "clocks": clocks,
         }
@@ -431,11 +463,35 @@ def run_mobius(args, rank, world, local):
         dist.destroy_process_group()
 
 
+def spawn_ranks(n):
+    """`--gpus N` without a launcher: re-exec this command under
+    torch.distributed.run with one rank per GPU (127.0.0.1 rendezvous), or
+    fail loudly if the box has fewer than N GPUs - never silently benchmark
+    one rank and label it N."""
+    import socket
+    same_gpu = os.environ.get("MOBIUS_BENCH_SAME_GPU") == "1"
+    if not same_gpu:
+        import torch
+        have = torch.cuda.device_count()
+        if have < n:
+            sys.exit(f"bench.py: --gpus {n} needs {n} GPUs, this box has {have} "
+                     f"(set MOBIUS_BENCH_SAME_GPU=1 to run {n} ranks on one GPU as a code-path check)")
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+    print(f"bench.py: launching {n} ranks: {' '.join(cmd)}", file=sys.stderr, flush=True)
+    sys.exit(subprocess.call(cmd))
+
+
 def main():
     args = parse()
     rank, world, local = dist_env()
     if world != args.gpus and world > 1:
-        print(f"warning: WORLD_SIZE={world} != --gpus {args.gpus}", file=sys.stderr)
+        sys.exit(f"bench.py: WORLD_SIZE={world} != --gpus {args.gpus}")
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ and args.impl != "reference":
+        spawn_ranks(args.gpus)
     if args.impl == "reference":
         run_reference(args, rank, world)
         return

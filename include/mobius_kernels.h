@@ -54,7 +54,7 @@ int mobius_kt_cross_entropy(int dtype, void* logits, const int32_t* tok, float* 
 int mobius_kt_embed_fwd(int dtype, const int32_t* tok, const void* wte, const void* wpe, void* x, int mbs, int s,
                         int h);
 int mobius_kt_embed_bwd(int dtype, const int32_t* tok, const void* dx, float* dwte, float* dwpe, int mbs, int s,
-                        int h);
+                        int h, int V);
 int mobius_kt_colsum(int dtype, const void* X, int64_t ld, int rows, int n, float* out);
 /* Causal attention core of a block (the path the block uses: fused tcgen05
  * flash kernels on the bf16 path when head_dim in {64,128} and s % 128 == 0,

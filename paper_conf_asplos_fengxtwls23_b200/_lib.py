@@ -60,7 +60,7 @@ class TimelineEvent(C.Structure):
     _fields_ = [("kind", C.c_int32), ("stage", C.c_int32), ("t0_ms", C.c_double), ("t1_ms", C.c_double)]
 
 
-TL_KINDS = {0: "h2d", 1: "fwd", 2: "bwd", 3: "d2h", 4: "d2d"}
+TL_KINDS = {0: "h2d", 1: "fwd", 2: "bwd", 3: "d2h", 4: "d2d", 5: "ckpt_d2h", 6: "ckpt_h2d"}
 
 
 class StepStats(C.Structure):
@@ -71,12 +71,15 @@ class StepStats(C.Structure):
                 ("elem_ns", C.c_int64), ("kernel_launches", C.c_int64), ("exposed_load_ns", C.c_int64),
                 ("update_tail_ns", C.c_int64), ("arena_bytes", C.c_int64), ("ring_bytes", C.c_int64),
                 ("pinned_bytes", C.c_int64), ("host_update_ns", C.c_int64), ("n_local_stages", C.c_int),
-                ("recompute", C.c_int), ("timing_stride", C.c_int), ("d2d_bytes", C.c_int64)]
+                ("recompute", C.c_int), ("timing_stride", C.c_int), ("d2d_bytes", C.c_int64),
+                ("ckpt_d2h_bytes", C.c_int64), ("ckpt_h2d_bytes", C.c_int64), ("exposed_ckpt_ns", C.c_int64)]
 
 
 FLAG_TIMING = 1
 FLAG_KEEP_ACTS = 2
 FLAG_DEVICE_TAIL_UPDATE = 4
+FLAG_ARENA_CAP = 8
+FLAG_CKPT_OFFLOAD = 16
 
 P = C.c_void_p
 I = C.c_int
@@ -87,6 +90,7 @@ F = C.c_float
 SIGNATURES = {
     "mobius_plan": (I, [C.POINTER(LayerProfile), I, I, I64, I, C.POINTER(Topology), C.POINTER(Plan)]),
     "mobius_plan_partition": (I, [C.POINTER(LayerProfile), I, I, I64, I, C.POINTER(Topology), I, C.POINTER(Plan)]),
+    "mobius_plan_search_nodes": (I64, []),
     "mobius_plan_cost": (I, [C.POINTER(LayerProfile), I, C.POINTER(C.c_int), I, I, I64, I, I64, I64,
                              C.POINTER(I64), C.POINTER(I64), C.POINTER(I64)]),
     "mobius_cross_map": (I, [I, I, C.POINTER(C.c_int), C.POINTER(C.c_int), C.POINTER(C.c_double),
@@ -96,6 +100,8 @@ SIGNATURES = {
     "mobius_discover_topology": (I, [C.POINTER(Topology)]),
     "mobius_layer_sizes": (I, [C.POINTER(ModelCfg), C.POINTER(LayerProfile), C.POINTER(C.c_int)]),
     "mobius_profile": (I, [C.POINTER(ModelCfg), I, C.POINTER(LayerProfile), C.POINTER(C.c_int)]),
+    "mobius_arena_layer_sizes": (I, [C.POINTER(ModelCfg), C.POINTER(LayerProfile), C.POINTER(C.c_int)]),
+    "mobius_arena_fixed_bytes": (I, [C.POINTER(ModelCfg), I, I, I, C.POINTER(I64)]),
     "mobius_create": (I, [C.POINTER(ModelCfg), C.POINTER(Plan), C.POINTER(Dist), P, C.c_uint64, C.POINTER(P)]),
     "mobius_dist_export": (I, [P, P, C.c_size_t, C.POINTER(C.c_size_t)]),
     "mobius_dist_connect": (I, [P, P, C.c_size_t]),
@@ -118,7 +124,7 @@ SIGNATURES = {
     "mobius_kt_softmax_bwd": (I, [I, P, P, P, I, I, F]),
     "mobius_kt_cross_entropy": (I, [I, P, P, P, I, I, I, F]),
     "mobius_kt_embed_fwd": (I, [I, P, P, P, P, I, I, I]),
-    "mobius_kt_embed_bwd": (I, [I, P, P, P, P, I, I, I]),
+    "mobius_kt_embed_bwd": (I, [I, P, P, P, P, I, I, I, I]),
     "mobius_kt_colsum": (I, [I, P, I64, I, I, P]),
     "mobius_kt_block": (I, [I, I, I, I, I, P, P, P, P, P, P]),
     "mobius_kt_attention": (I, [I, I, I, I, I, P, P, P, P]),

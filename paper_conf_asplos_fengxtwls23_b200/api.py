@@ -9,11 +9,13 @@ from typing import Optional, Sequence
 import numpy as np
 
 from . import _lib as L
-from ._lib import BF16, F32, FLAG_DEVICE_TAIL_UPDATE, FLAG_KEEP_ACTS, FLAG_TIMING, MobiusError, check, lib  # noqa: F401
+from ._lib import (BF16, F32, FLAG_ARENA_CAP, FLAG_CKPT_OFFLOAD, FLAG_DEVICE_TAIL_UPDATE, FLAG_KEEP_ACTS,  # noqa: F401
+                   FLAG_TIMING, MobiusError, check, lib)
 
 __all__ = ["mobius_plan", "mobius_plan_partition", "PARTITION_MIP", "PARTITION_MAX_STAGE", "PARTITION_MIN_STAGE", "mobius_plan_cost", "mobius_cross_map", "mobius_mapping_contention",
            "mobius_discover_topology", "mobius_layer_sizes", "mobius_profile", "MobiusContext", "model_cfg",
-           "make_topology", "plan_from_sizes", "kt", "BF16", "F32", "FLAG_TIMING", "FLAG_KEEP_ACTS", "FLAG_DEVICE_TAIL_UPDATE", "MobiusError",
+           "make_topology", "plan_from_sizes", "kt", "BF16", "F32", "FLAG_TIMING", "FLAG_KEEP_ACTS", "FLAG_DEVICE_TAIL_UPDATE", "FLAG_ARENA_CAP", "FLAG_CKPT_OFFLOAD",
+           "mobius_arena_layer_sizes", "mobius_arena_fixed_bytes", "MobiusError",
            "build_info"]
 
 
@@ -114,6 +116,19 @@ def mobius_layer_sizes(cfg: L.ModelCfg):
     n = C.c_int()
     check(lib.mobius_layer_sizes(C.byref(cfg), out, C.byref(n)))
     return [out[i] for i in range(n.value)]
+
+
+def mobius_arena_layer_sizes(cfg: L.ModelCfg):
+    out = (L.LayerProfile * L.MAX_LAYERS)()
+    n = C.c_int()
+    check(lib.mobius_arena_layer_sizes(C.byref(cfg), out, C.byref(n)))
+    return [out[i] for i in range(n.value)]
+
+
+def mobius_arena_fixed_bytes(cfg: L.ModelCfg, n_microbatches: int, n_local_stages: int, flags: int) -> int:
+    b = C.c_int64()
+    check(lib.mobius_arena_fixed_bytes(C.byref(cfg), n_microbatches, n_local_stages, flags, C.byref(b)))
+    return b.value
 
 
 def mobius_profile(cfg: L.ModelCfg, device: int = 0):
@@ -269,8 +284,9 @@ class _KT:
     def embed_fwd(self, dtype, tok, wte, wpe, x, mbs, s, h):
         check(lib.mobius_kt_embed_fwd(dtype, *map(self._p, (tok, wte, wpe, x)), mbs, s, h))
 
-    def embed_bwd(self, dtype, tok, dx, dwte, dwpe, mbs, s, h):
-        check(lib.mobius_kt_embed_bwd(dtype, *map(self._p, (tok, dx, dwte, dwpe)), mbs, s, h))
+    def embed_bwd(self, dtype, tok, dx, dwte, dwpe, mbs, s, h, V=None):
+        V = dwte.shape[0] if V is None else V
+        check(lib.mobius_kt_embed_bwd(dtype, *map(self._p, (tok, dx, dwte, dwpe)), mbs, s, h, V))
 
     def colsum(self, dtype, X, ld, rows, n, out):
         check(lib.mobius_kt_colsum(dtype, self._p(X), ld, rows, n, self._p(out)))

@@ -4,6 +4,10 @@
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
+#include <algorithm>
+
+#include <cooperative_groups.h>
+
 #include "common.h"
 #include "elem.h"
 
@@ -142,8 +146,12 @@ __global__ void embed_fwd_k(const int32_t* tok, const T* wte, const T* wpe, T* x
   }
 }
 
+// dWte scatter, bf16 path: vector reductions (red.global.add.v4.f32) of
+// each dx row into its token's fp32 row - one pass over dx, L2 resolves
+// repeated tokens (the bf16 path is not bitwise reproducible anyway: the
+// flash backward reduces dQ with TMA reduce-adds).
 template <typename T>
-__global__ void embed_bwd_wte_k(const int32_t* tok, const T* dx, float* dwte, int s, int h) {
+__global__ void embed_bwd_wte_red_k(const int32_t* tok, const T* dx, float* dwte, int s, int h) {
   constexpr int V = Vec<T>::N;
   const int r = blockIdx.x;
   const int b = r / s, i = r % s;
@@ -153,12 +161,82 @@ __global__ void embed_bwd_wte_k(const int32_t* tok, const T* dx, float* dwte, in
   for (int c = threadIdx.x * V; c < h; c += blockDim.x * V) {
     float a[V];
     Vec<T>::load(g + c, a);
-    // vector reductions (sm_90+): a quarter of the atomic operations
 #pragma unroll
     for (int k = 0; k < V; k += 4)
       asm volatile("red.relaxed.gpu.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(o + c + k), "f"(a[k]),
                    "f"(a[k + 1]), "f"(a[k + 2]), "f"(a[k + 3])
                    : "memory");
+  }
+}
+
+// dWte scatter, fp32 debug path: no float atomics, bitwise reproducible
+// (the synchronous-update equivalence of P:L596-602 is checked bit for bit
+// on this path).  CTA b owns the vocabulary rows [b*ids, (b+1)*ids).  It
+// scans the microbatch's token ids in position order, EB_CHUNK at a time
+// (each warp compacts a contiguous run of positions with ballots, so the
+// per-warp lists concatenated in warp order are in position order), then
+// every thread adds the dx rows of the matches into its own columns of the
+// owned rows, in list order; a run of equal ids is summed in registers
+// first.  Same-address read-modify-writes of one thread are program
+// ordered, so the sums are in position order.
+constexpr int EB_THREADS = 256;
+constexpr int EB_CHUNK = 4096;                      // positions per scan round
+constexpr int EB_PER_WARP = EB_CHUNK / (EB_THREADS / 32);
+template <typename T>
+__global__ void __launch_bounds__(EB_THREADS) embed_bwd_wte_det_k(const int32_t* __restrict__ tok,
+                                                                  const T* __restrict__ dx, float* __restrict__ dwte,
+                                                                  int mbs, int s, int h, int ids) {
+  constexpr int V = Vec<T>::N;
+  __shared__ int2 list[EB_CHUNK];                   // (row r, token id)
+  __shared__ int wcount[EB_THREADS / 32];
+  const int v0 = blockIdx.x * ids, v1 = v0 + ids;
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int T_ = mbs * s;
+  for (int base = 0; base < T_; base += EB_CHUNK) {
+    int n = 0;
+    const int p0 = base + warp * EB_PER_WARP;
+#pragma unroll 4
+    for (int i = 0; i < EB_PER_WARP; i += 32) {
+      const int r = p0 + i + lane;
+      int t = -1;
+      if (r < T_) t = __ldg(tok + (int64_t)(r / s) * (s + 1) + (r % s));
+      const bool hit = t >= v0 && t < v1;
+      const unsigned b = __ballot_sync(0xffffffffu, hit);
+      if (hit) list[warp * EB_PER_WARP + n + __popc(b & ((1u << lane) - 1))] = make_int2(r, t);
+      n += __popc(b);
+    }
+    if (lane == 0) wcount[warp] = n;
+    __syncthreads();
+    for (int c = threadIdx.x * V; c < h; c += EB_THREADS * V) {
+      float acc[V];
+      int prev = -1;
+      for (int w = 0; w < EB_THREADS / 32; ++w) {
+        const int nw = wcount[w];
+        for (int k = 0; k < nw; ++k) {
+          const int2 e = list[w * EB_PER_WARP + k];
+          if (e.y != prev) {
+            if (prev >= 0) {
+              float* o = dwte + (int64_t)prev * h + c;
+#pragma unroll
+              for (int q = 0; q < V; ++q) o[q] += acc[q];
+            }
+#pragma unroll
+            for (int q = 0; q < V; ++q) acc[q] = 0.f;
+            prev = e.y;
+          }
+          float a[V];
+          Vec<T>::load(dx + (int64_t)e.x * h + c, a);
+#pragma unroll
+          for (int q = 0; q < V; ++q) acc[q] += a[q];
+        }
+      }
+      if (prev >= 0) {
+        float* o = dwte + (int64_t)prev * h + c;
+#pragma unroll
+        for (int q = 0; q < V; ++q) o[q] += acc[q];
+      }
+    }
+    __syncthreads();
   }
 }
 
@@ -527,19 +605,28 @@ __global__ void __launch_bounds__(256) ln_bwd_dx_k(const T* __restrict__ dy, con
 }
 
 // Column reductions over `rows` rows, 16-byte vectors per thread, partial
-// sums in registers, CTA-level smem reduction, one atomic per column per
-// CTA.  mode 0: out0[c] += sum_r X[r,c].  mode 1 (LayerNorm parameters):
-// out0[c] += sum_r X[r,c] * (Y[r,c] - mu[r]) * rstd[r] (dgamma), out1[c] +=
-// sum_r X[r,c] (dbeta).
+// sums in registers, CTA-level smem reduction.  mode 0: out0[c] += sum_r
+// X[r,c].  mode 1 (LayerNorm parameters): out0[c] += sum_r X[r,c] *
+// (Y[r,c] - mu[r]) * rstd[r] (dgamma), out1[c] += sum_r X[r,c] (dbeta).
+// Deterministic, no float atomics: the CS_CL CTAs of a cluster (stacked
+// along the rows) add their column totals through distributed shared memory
+// in rank order; each cluster leader writes one partial row; the last
+// leader of a column slab to arrive (arrival counter, reset by it) adds the
+// gridDim.y / CS_CL partials to out in order.
 constexpr int CS_THREADS = 256;
 constexpr int CS_COLV = 32;  // column vectors (of 8/4 elements) per CTA
+constexpr int CS_CL = 8;     // CTAs per cluster (rows direction)
 template <typename T, int MODE>
-__global__ void __launch_bounds__(CS_THREADS) colsum2_k(const T* __restrict__ X, int64_t ld, const T* __restrict__ Y,
-                                                        const float* __restrict__ mu, const float* __restrict__ rstd,
-                                                        int rows, int n, float* out0, float* out1, int rows_per_cta) {
+__global__ void __cluster_dims__(1, CS_CL, 1) __launch_bounds__(CS_THREADS)
+    colsum2_k(const T* __restrict__ X, int64_t ld, const T* __restrict__ Y, const float* __restrict__ mu,
+              const float* __restrict__ rstd, int rows, int n, float* out0, float* out1, int rows_per_cta,
+              float* part, unsigned* cnt) {
   constexpr int V = Vec<T>::N;
-  __shared__ float red0[CS_THREADS / CS_COLV][CS_COLV * V];
-  __shared__ float red1[MODE == 1 ? CS_THREADS / CS_COLV : 1][MODE == 1 ? CS_COLV * V : 1];
+  constexpr int W = CS_COLV * V;  // columns per CTA
+  __shared__ float red0[CS_THREADS / CS_COLV][W];
+  __shared__ float red1[MODE == 1 ? CS_THREADS / CS_COLV : 1][MODE == 1 ? W : 1];
+  __shared__ float tot[MODE == 1 ? 2 : 1][W];
+  __shared__ bool last;
   const int cv = threadIdx.x % CS_COLV;  // column vector within the CTA's slab
   const int rg = threadIdx.x / CS_COLV;  // row group (CS_THREADS / CS_COLV groups)
   const int c = (blockIdx.x * CS_COLV + cv) * V;
@@ -573,29 +660,69 @@ __global__ void __launch_bounds__(CS_THREADS) colsum2_k(const T* __restrict__ X,
     if (MODE == 1) red1[rg][cv * V + e] = a1[e];
   }
   __syncthreads();
-  for (int i = threadIdx.x; i < CS_COLV * V; i += CS_THREADS) {
-    const int col = blockIdx.x * CS_COLV * V + i;
-    if (col >= n) continue;
+  for (int i = threadIdx.x; i < W; i += CS_THREADS) {
     float t0 = 0.f, t1 = 0.f;
 #pragma unroll
     for (int g2 = 0; g2 < CS_THREADS / CS_COLV; ++g2) {
       t0 += red0[g2][i];
       if (MODE == 1) t1 += red1[g2][i];
     }
-    atomicAdd(out0 + col, t0);
-    if (MODE == 1) atomicAdd(out1 + col, t1);
+    tot[0][i] = t0;
+    if (MODE == 1) tot[MODE][i] = t1;
+  }
+  // cluster: the leader adds the CS_CL CTA totals in rank order (DSMEM)
+  namespace cg = cooperative_groups;
+  cg::cluster_group cluster = cg::this_cluster();
+  cluster.sync();
+  const bool leader = cluster.block_rank() == 0;
+  const int64_t nparts = gridDim.y / CS_CL;
+  const int64_t prow = blockIdx.y / CS_CL;
+  if (leader) {
+    for (int i = threadIdx.x; i < W; i += CS_THREADS) {
+      const int col = blockIdx.x * W + i;
+      float t0 = 0.f, t1 = 0.f;
+#pragma unroll
+      for (int r = 0; r < CS_CL; ++r) {
+        const float* rt = cluster.map_shared_rank(&tot[0][0], r);
+        t0 += rt[i];
+        if (MODE == 1) t1 += rt[W + i];
+      }
+      if (col < n) {
+        part[prow * n + col] = t0;
+        if (MODE == 1) part[(nparts + prow) * n + col] = t1;
+      }
+    }
+  }
+  cluster.sync();  // remote reads done before any CTA of the cluster exits
+  if (!leader) return;
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) last = atomicInc(cnt + blockIdx.x, (unsigned)nparts - 1) == (unsigned)nparts - 1;  // wraps to 0
+  __syncthreads();
+  if (!last) return;
+  __threadfence();
+  for (int i = threadIdx.x; i < W; i += CS_THREADS) {
+    const int col = blockIdx.x * W + i;
+    if (col >= n) continue;
+    float t0 = 0.f, t1 = 0.f;
+    for (int64_t g2 = 0; g2 < nparts; ++g2) {
+      t0 += __ldcg(part + g2 * n + col);
+      if (MODE == 1) t1 += __ldcg(part + (nparts + g2) * n + col);
+    }
+    out0[col] += t0;
+    if (MODE == 1) out1[col] += t1;
   }
 }
 
+// generic fallback (unaligned / odd widths): one thread per column sums all
+// rows in order (deterministic; never on the hot path)
 template <typename T>
-__global__ void colsum_k(const T* X, int64_t ld, int rows, int n, float* out, int rows_per_block) {
+__global__ void colsum_k(const T* X, int64_t ld, int rows, int n, float* out) {
   const int c = blockIdx.x * blockDim.x + threadIdx.x;
   if (c >= n) return;
-  const int r0 = blockIdx.y * rows_per_block;
-  const int r1 = min(rows, r0 + rows_per_block);
   float acc = 0.f;
-  for (int r = r0; r < r1; ++r) acc += to_f(X[(int64_t)r * ld + c]);
-  atomicAdd(out + c, acc);
+  for (int r = 0; r < rows; ++r) acc += to_f(X[(int64_t)r * ld + c]);
+  out[c] += acc;
 }
 
 template <typename T>
@@ -613,6 +740,18 @@ __global__ void cast_k(const float* src, T* dst, int64_t n) {
       for (int64_t k = i; k < n; ++k) dst[k] = from_f<T>(src[k]);
     }
   }
+}
+
+__global__ void tokens_check_k(const int32_t* __restrict__ src, int32_t* __restrict__ dst, int64_t n, int V,
+                               int* bad) {
+  int cnt = 0;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t t = src[i];
+    cnt += (uint32_t)t >= (uint32_t)V;
+    dst[i] = t;
+  }
+  cnt = __reduce_add_sync(0xffffffffu, cnt);
+  if (cnt && threadIdx.x % 32 == 0) atomicAdd(bad, cnt);  // integer count: order-independent
 }
 
 __global__ void flag_wait_k(const volatile int* flag, int value) {
@@ -639,6 +778,13 @@ int colsum_rows_per_cta(int col_ctas, int rows) {
   while (rpc > 32 && (int64_t)col_ctas * ((rows + rpc - 1) / rpc) < 4 * 148) rpc /= 2;
   return rpc;
 }
+// grid of colsum2_k for n columns of vector width vw (gy a multiple of the
+// cluster size; trailing CTAs of a short last cluster have no rows)
+void colsum_grid(int rows, int n, int vw, int* gx, int* gy, int* rpc) {
+  *gx = (n / vw + CS_COLV - 1) / CS_COLV;
+  *rpc = colsum_rows_per_cta(*gx, rows);
+  *gy = ((rows + *rpc - 1) / *rpc + CS_CL - 1) / CS_CL * CS_CL;
+}
 
 template <typename T>
 bool aligned16(const T* p) {
@@ -654,10 +800,18 @@ int embed_fwd(const int32_t* tok, const T* wte, const T* wpe, T* x, int mbs, int
   return check_launch("embed_fwd");
 }
 template <typename T>
-int embed_bwd(const int32_t* tok, const T* dx, float* dwte, float* dwpe, int mbs, int s, int h, cudaStream_t st) {
-  MOBIUS_CHECK_ARG(h % 8 == 0 && (reinterpret_cast<uintptr_t>(dwte) & 15) == 0,
-                   "embed_bwd: h %% 8 and a 16-byte aligned dWte are required (vector reductions)");
-  embed_bwd_wte_k<T><<<mbs * s, 128, 0, st>>>(tok, dx, dwte, s, h);
+int embed_bwd(const int32_t* tok, const T* dx, float* dwte, float* dwpe, int mbs, int s, int h, int V,
+              cudaStream_t st) {
+  MOBIUS_CHECK_ARG(h % 8 == 0 && (reinterpret_cast<uintptr_t>(dwte) & 15) == 0 && V > 0,
+                   "embed_bwd: h %% 8 and a 16-byte aligned dWte are required");
+  if constexpr (sizeof(T) == 2) {
+    embed_bwd_wte_red_k<T><<<mbs * s, 128, 0, st>>>(tok, dx, dwte, s, h);
+  } else {
+    // ~4 CTAs per SM, each owning ceil(V / grid) vocabulary rows
+    const int grid = std::min(V, 148 * 4);
+    const int ids = (V + grid - 1) / grid;
+    embed_bwd_wte_det_k<T><<<(V + ids - 1) / ids, EB_THREADS, 0, st>>>(tok, dx, dwte, mbs, s, h, ids);
+  }
   int rc = check_launch("embed_bwd_wte");
   if (rc) return rc;
   embed_bwd_wpe_k<T><<<s, 256, 0, st>>>(dx, dwpe, mbs, s, h);
@@ -713,7 +867,7 @@ int layernorm_fwd(const T* x, const T* g, const T* b, T* y, float* mu, float* rs
 }
 template <typename T>
 int layernorm_bwd(const T* dy, const T* x, const T* g, const float* mu, const float* rstd, const T* dres, T* dx,
-                  float* dg, float* db, int rows, int h, cudaStream_t st) {
+                  float* dg, float* db, int rows, int h, const RedWs& ws, cudaStream_t st) {
   MOBIUS_CHECK_ARG(h % Vec<T>::N == 0, "layernorm: unsupported h=%d", h);
   // dx, then gamma / beta grads by a column-reduction pass.  Fusing the
   // param grads into the dx pass was measured slower at 8192 x 1600 (42 us
@@ -727,10 +881,10 @@ int layernorm_bwd(const T* dy, const T* x, const T* g, const float* mu, const fl
   int rc = check_launch("layernorm_bwd_dx");
   if (rc) return rc;
   {
-    const int gx = (h / Vec<T>::N + CS_COLV - 1) / CS_COLV;
-    const int rpc = colsum_rows_per_cta(gx, rows);
-    dim3 grid(gx, (rows + rpc - 1) / rpc);
-    colsum2_k<T, 1><<<grid, CS_THREADS, 0, st>>>(dy, h, x, mu, rstd, rows, h, dg, db, rpc);
+    int gx, gy, rpc;
+    colsum_grid(rows, h, Vec<T>::N, &gx, &gy, &rpc);
+    MOBIUS_CHECK_ARG(ws.part && ws.cnt && gx <= RED_WS_COUNTERS, "layernorm_bwd: reduction workspace");
+    colsum2_k<T, 1><<<dim3(gx, gy), CS_THREADS, 0, st>>>(dy, h, x, mu, rstd, rows, h, dg, db, rpc, ws.part, ws.cnt);
   }
   return check_launch("layernorm_param_grad");
 }
@@ -761,18 +915,28 @@ int loss_accumulate(const float* loss_rows, int rows, double* acc, cudaStream_t 
   return check_launch("loss_accumulate");
 }
 
+int64_t colsum_ws_floats(int rows, int n, int planes) {
+  // the bf16 grid (8-wide vectors) has fewer column CTAs, hence more row CTAs
+  int64_t best = 0;
+  for (int vw : {4, 8}) {
+    int gx, gy, rpc;
+    colsum_grid(rows, n, vw, &gx, &gy, &rpc);
+    best = std::max<int64_t>(best, (int64_t)(gy / CS_CL) * n * planes);
+  }
+  return best;
+}
+
 template <typename T>
-int colsum_accum(const T* X, int64_t ld, int rows, int n, float* out, cudaStream_t st) {
+int colsum_accum(const T* X, int64_t ld, int rows, int n, float* out, const RedWs& ws, cudaStream_t st) {
   if (n % Vec<T>::N == 0 && ld % Vec<T>::N == 0 && aligned16(X)) {
-    const int gx = (n / Vec<T>::N + CS_COLV - 1) / CS_COLV;
-    const int rpc = colsum_rows_per_cta(gx, rows);
-    dim3 grid(gx, (rows + rpc - 1) / rpc);
-    colsum2_k<T, 0><<<grid, CS_THREADS, 0, st>>>(X, ld, (const T*)nullptr, nullptr, nullptr, rows, n, out, nullptr, rpc);
+    int gx, gy, rpc;
+    colsum_grid(rows, n, Vec<T>::N, &gx, &gy, &rpc);
+    MOBIUS_CHECK_ARG(ws.part && ws.cnt && gx <= RED_WS_COUNTERS, "colsum: reduction workspace");
+    colsum2_k<T, 0><<<dim3(gx, gy), CS_THREADS, 0, st>>>(X, ld, (const T*)nullptr, nullptr, nullptr, rows, n, out,
+                                                         nullptr, rpc, ws.part, ws.cnt);
     return check_launch("colsum");
   }
-  const int rpb = 128;
-  dim3 grid((n + 255) / 256, (rows + rpb - 1) / rpb);
-  colsum_k<T><<<grid, 256, 0, st>>>(X, ld, rows, n, out, rpb);
+  colsum_k<T><<<(n + 255) / 256, 256, 0, st>>>(X, ld, rows, n, out);
   return check_launch("colsum");
 }
 
@@ -877,6 +1041,13 @@ int gelu_fwd_bf16(const __nv_bfloat16* u, __nv_bfloat16* g, int64_t n, cudaStrea
   return check_launch("gelu_fwd");
 }
 
+int tokens_check_copy(const int32_t* src, int32_t* dst, int64_t n, int V, int* bad_dev, cudaStream_t st) {
+  if (cudaMemsetAsync(bad_dev, 0, sizeof(int), st) != cudaSuccess) MOBIUS_FAIL(MOBIUS_ECUDA, "tokens_check: memset");
+  const int grid = (int)std::min<int64_t>(148 * 2, (n + 255) / 256);
+  tokens_check_k<<<std::max(grid, 1), 256, 0, st>>>(src, dst, n, V, bad_dev);
+  return check_launch("tokens_check");
+}
+
 int flag_wait(const volatile int* flag, int value, cudaStream_t st) {
   flag_wait_k<<<1, 1, 0, st>>>(flag, value);
   return check_launch("flag_wait");
@@ -888,14 +1059,14 @@ int flag_set(int* flag, int value, cudaStream_t st) {
 
 #define INST(T)                                                                                                  \
   template int embed_fwd<T>(const int32_t*, const T*, const T*, T*, int, int, int, cudaStream_t);               \
-  template int embed_bwd<T>(const int32_t*, const T*, float*, float*, int, int, int, cudaStream_t);             \
+  template int embed_bwd<T>(const int32_t*, const T*, float*, float*, int, int, int, int, cudaStream_t);        \
   template int layernorm_fwd<T>(const T*, const T*, const T*, T*, float*, float*, int, int, cudaStream_t);      \
   template int layernorm_bwd<T>(const T*, const T*, const T*, const float*, const float*, const T*, T*, float*, \
-                                float*, int, int, cudaStream_t);                                                \
+                                float*, int, int, const RedWs&, cudaStream_t);                                  \
   template int softmax_causal_fwd<T>(const float*, T*, int, int, float, cudaStream_t);                          \
   template int softmax_causal_bwd<T>(const T*, const float*, T*, int, int, float, cudaStream_t);                \
   template int cross_entropy_fwd_bwd<T>(T*, const int32_t*, float*, int, int, int, float, cudaStream_t);        \
-  template int colsum_accum<T>(const T*, int64_t, int, int, float*, cudaStream_t);                              \
+  template int colsum_accum<T>(const T*, int64_t, int, int, float*, const RedWs&, cudaStream_t);               \
   template int cast_from_f32<T>(const float*, T*, int64_t, cudaStream_t);                                       \
   template int adamw_device<T>(float*, float*, float*, const T*, T*, int64_t, float, float, float, float, float,   \
                                float, float, cudaStream_t);

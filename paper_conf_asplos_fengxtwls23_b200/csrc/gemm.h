@@ -60,6 +60,11 @@ int gemm_f32(const GemmDesc& d, cudaStream_t s);
 
 int num_sms();
 
+// Stream-K workspaces are kept per (device, stream); the owner of a stream
+// frees its entry before destroying the stream.
+void gemm_release_stream(cudaStream_t s);
+size_t gemm_workspace_entries();
+
 // Kernel selection knobs (tests / perf A-B): -1 = environment default
 // (MOBIUS_GEMM_2CTA, MOBIUS_GEMM_SK), 0 = off, 1 = on.
 void gemm_set_config(int two_cta, int stream_k);

@@ -4,6 +4,8 @@
 // wave of long-K shapes.  Shared epilogue and parameters: gemm_common.cuh.
 #include "gemm_common.cuh"
 
+#include <vector>
+
 namespace mobius {
 namespace gemm_detail {
 
@@ -652,10 +654,13 @@ using namespace gemm_detail;
 
 static int g_gemm_sk = -1;  // Stream-K tail: env MOBIUS_GEMM_SK=0 disables
 
-// Stream-K workspace, one per stream (GEMMs on different streams may run
-// concurrently).  Grows on demand; counters start at zero and are reset by
-// the reducing warp, so consecutive launches on one stream reuse them.
+// Stream-K workspace, one per (device, stream): GEMMs on different streams
+// may run concurrently.  Grows on demand; counters start at zero and are
+// reset by the reducing warp, so consecutive launches on one stream reuse
+// them.  The owner of a stream releases its entry (gemm_release_stream,
+// called by mobius_destroy for the context's compute stream).
 struct SkWs {
+  int dev;
   cudaStream_t s;
   float* ws;
   size_t ws_bytes;
@@ -663,19 +668,18 @@ struct SkWs {
   size_t cnt_n;
 };
 static std::mutex g_sk_mu;
-static SkWs g_sk[16];
-static int g_sk_n = 0;
+static std::vector<SkWs> g_sk;
 
 static int sk_workspace(cudaStream_t s, size_t ws_bytes, size_t cnt_n, float** ws, int** cnt) {
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) MOBIUS_FAIL(MOBIUS_ECUDA, "gemm: cudaGetDevice");
   std::lock_guard<std::mutex> lk(g_sk_mu);
   SkWs* e = nullptr;
-  for (int i = 0; i < g_sk_n; ++i)
-    if (g_sk[i].s == s) e = &g_sk[i];
+  for (auto& x : g_sk)
+    if (x.s == s && x.dev == dev) e = &x;
   if (!e) {
-    if (g_sk_n == 16) MOBIUS_FAIL(MOBIUS_ENOMEM, "gemm: too many streams for Stream-K workspaces");
-    e = &g_sk[g_sk_n++];
-    std::memset(e, 0, sizeof(*e));
-    e->s = s;
+    g_sk.push_back(SkWs{dev, s, nullptr, 0, nullptr, 0});
+    e = &g_sk.back();
   }
   if (e->ws_bytes < ws_bytes) {
     if (e->ws) {
@@ -701,6 +705,25 @@ static int sk_workspace(cudaStream_t s, size_t ws_bytes, size_t cnt_n, float** w
   *ws = e->ws;
   *cnt = e->cnt;
   return MOBIUS_OK;
+}
+
+// free the Stream-K workspace of stream s on the current device (the stream
+// must be idle; no-op when it never ran a Stream-K GEMM)
+void gemm_release_stream(cudaStream_t s) {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  std::lock_guard<std::mutex> lk(g_sk_mu);
+  for (size_t i = 0; i < g_sk.size(); ++i) {
+    if (g_sk[i].s != s || g_sk[i].dev != dev) continue;
+    if (g_sk[i].ws) cudaFree(g_sk[i].ws);
+    if (g_sk[i].cnt) cudaFree(g_sk[i].cnt);
+    g_sk.erase(g_sk.begin() + i);
+    return;
+  }
+}
+size_t gemm_workspace_entries() {
+  std::lock_guard<std::mutex> lk(g_sk_mu);
+  return g_sk.size();
 }
 
 // host copy of the device owner function (same integer arithmetic)

@@ -34,6 +34,21 @@ uint8_t* ws_get(int64_t bytes) {
   }
   return buf;
 }
+// reduction workspace of the kt column sums (counters zeroed once; the
+// reduction kernels leave them zero)
+RedWs red_ws_get(int64_t floats) {
+  static RedWs w;
+  static int64_t cap = -1;
+  if (floats > cap) {
+    if (w.part) cudaFree(w.part);
+    if (!w.cnt && cudaMalloc(&w.cnt, RED_WS_COUNTERS * 4) == cudaSuccess) cudaMemset(w.cnt, 0, RED_WS_COUNTERS * 4);
+    w.part = nullptr;
+    cap = -1;
+    if (cudaMalloc(&w.part, floats * 4 + 16) != cudaSuccess) return RedWs{};
+    cap = floats;
+  }
+  return w;
+}
 int sync_rc(int rc) {
   if (rc) return rc;
   static int nosync = -1;  // MOBIUS_KT_NOSYNC=1: timing loops (launch-only, errors via cudaGetLastError)
@@ -88,11 +103,12 @@ extern "C" int mobius_kt_layernorm_fwd(int dtype, const void* x, const void* g, 
 extern "C" int mobius_kt_layernorm_bwd(int dtype, const void* dy, const void* x, const void* g, const float* mu,
                                        const float* rstd, const void* dres, void* dx, float* dg, float* db, int rows,
                                        int h) {
+  const RedWs ws = red_ws_get(colsum_ws_floats(rows, h, 2));
   if (dtype == MOBIUS_BF16)
     return sync_rc(layernorm_bwd<bf16>((const bf16*)dy, (const bf16*)x, (const bf16*)g, mu, rstd, (const bf16*)dres,
-                                       (bf16*)dx, dg, db, rows, h, 0));
+                                       (bf16*)dx, dg, db, rows, h, ws, 0));
   return sync_rc(layernorm_bwd<float>((const float*)dy, (const float*)x, (const float*)g, mu, rstd,
-                                      (const float*)dres, (float*)dx, dg, db, rows, h, 0));
+                                      (const float*)dres, (float*)dx, dg, db, rows, h, ws, 0));
 }
 
 extern "C" int mobius_kt_softmax_fwd(int dtype, const float* S, void* P, int B, int s, float scale) {
@@ -120,14 +136,15 @@ extern "C" int mobius_kt_embed_fwd(int dtype, const int32_t* tok, const void* wt
 }
 
 extern "C" int mobius_kt_embed_bwd(int dtype, const int32_t* tok, const void* dx, float* dwte, float* dwpe, int mbs,
-                                   int s, int h) {
-  if (dtype == MOBIUS_BF16) return sync_rc(embed_bwd<bf16>(tok, (const bf16*)dx, dwte, dwpe, mbs, s, h, 0));
-  return sync_rc(embed_bwd<float>(tok, (const float*)dx, dwte, dwpe, mbs, s, h, 0));
+                                   int s, int h, int V) {
+  if (dtype == MOBIUS_BF16) return sync_rc(embed_bwd<bf16>(tok, (const bf16*)dx, dwte, dwpe, mbs, s, h, V, 0));
+  return sync_rc(embed_bwd<float>(tok, (const float*)dx, dwte, dwpe, mbs, s, h, V, 0));
 }
 
 extern "C" int mobius_kt_colsum(int dtype, const void* X, int64_t ld, int rows, int n, float* out) {
-  if (dtype == MOBIUS_BF16) return sync_rc(colsum_accum<bf16>((const bf16*)X, ld, rows, n, out, 0));
-  return sync_rc(colsum_accum<float>((const float*)X, ld, rows, n, out, 0));
+  const RedWs ws = red_ws_get(colsum_ws_floats(rows, n, 1));
+  if (dtype == MOBIUS_BF16) return sync_rc(colsum_accum<bf16>((const bf16*)X, ld, rows, n, out, ws, 0));
+  return sync_rc(colsum_accum<float>((const float*)X, ld, rows, n, out, ws, 0));
 }
 
 namespace {
@@ -144,6 +161,7 @@ int kt_block(int hidden, int nh, int s, int mbs, const void* w, const void* x, v
   Scratch<T> sc;
   carve_block_acts<T>(sh, buf, acts);
   carve_scratch<T>(sh, buf + ab, false, sc);
+  if (int rz = scratch_zero<T>(sc, 0)) return rz;
   acts.x = (const T*)x;
   int rc = block_fwd<T>(sh, (const T*)w, acts, (T*)y, sc, 0);
   if (!rc && dy) rc = block_bwd<T>(sh, (const T*)w, acts, (const T*)dy, (T*)dx, grads, sc, 0);
@@ -170,6 +188,7 @@ int kt_attn(int mbs, int s, int nh, int dh, const void* qkv, void* o, const void
   Scratch<T> sc;
   carve_block_acts<T>(sh, buf, acts);
   carve_scratch<T>(sh, buf + ab, false, sc);
+  if (int rz = scratch_zero<T>(sc, 0)) return rz;
   int rc = attention_fwd<T>(sh, (const T*)qkv, (T*)o, acts.P, acts.lse, sc, 0);
   if (!rc && dout) rc = attention_bwd<T>(sh, (const T*)qkv, (const T*)o, acts.P, acts.lse, (const T*)dout, (T*)dqkv, sc, 0);
   return sync_rc(rc);

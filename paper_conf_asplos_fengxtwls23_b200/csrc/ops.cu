@@ -2,6 +2,7 @@
 // the SIMT GEMM (fp32 debug path) and the fused HBM-bound kernels.
 // Equations: SURVEY §8(c) O-2 (reading #1 of the paper's "GPT-like"
 // blocks).
+#include <algorithm>
 #include <cmath>
 
 #include "common.h"
@@ -161,6 +162,12 @@ void carve_block_acts(const Shape& sh, uint8_t* base, BlockActs<T>& a, bool comp
   (void)full;
 }
 
+// partial sums of the widest column reduction of a block / head backward
+static int64_t red_ws_floats(const Shape& sh) {
+  const int T = sh.T(), h = sh.h;
+  return std::max({colsum_ws_floats(T, 4 * h, 1), colsum_ws_floats(T, 3 * h, 1), colsum_ws_floats(T, h, 2)});
+}
+
 int64_t scratch_bytes(const Shape& sh, int e, bool with_head, bool flash) {
   const int64_t T = sh.T(), h = sh.h, B = (int64_t)sh.mbs * sh.nh, s = sh.s;
   Carver c{nullptr};
@@ -173,13 +180,15 @@ int64_t scratch_bytes(const Shape& sh, int e, bool with_head, bool flash) {
   c.take<char>(T * h * e);
   c.take<char>(T * h * e);
   c.take<char>(T * 3 * h * e);
-  c.take<char>(with_head ? T * (int64_t)sh.V * e : 0);
+  c.take<char>(with_head ? (int64_t)sh.head_chunk() * sh.V * e : 0);
   c.take<char>(T * 4);
   c.take<char>(T * 4);
   c.take<char>(T * 4);
   c.take<char>(T * h * e);      // ra
   c.take<char>(T * h * e);      // ra2
   c.take<char>(T * 4 * h * e);  // rg
+  c.take<char>(red_ws_floats(sh) * 4);
+  c.take<char>(RED_WS_COUNTERS * 4);
   return c.off;
 }
 
@@ -197,13 +206,22 @@ void carve_scratch(const Shape& sh, uint8_t* base, bool with_head, Scratch<T>& s
   sc.t2 = c.take<T>(Tn * h * e);
   sc.t3 = c.take<T>(Tn * h * e);
   sc.qkv_g = c.take<T>(Tn * 3 * h * e);
-  sc.logits = c.take<T>(with_head ? Tn * (int64_t)sh.V * e : 0);
+  sc.logits = c.take<T>(with_head ? (int64_t)sh.head_chunk() * sh.V * e : 0);
   sc.loss_rows = c.take<float>(Tn * 4);
   sc.mu = c.take<float>(Tn * 4);
   sc.rs = c.take<float>(Tn * 4);
   sc.ra = c.take<T>(Tn * h * e);
   sc.ra2 = c.take<T>(Tn * h * e);
   sc.rg = c.take<T>(Tn * 4 * h * e);
+  sc.red.part = c.take<float>(red_ws_floats(sh) * 4);
+  sc.red.cnt = c.take<unsigned>(RED_WS_COUNTERS * 4);
+}
+
+template <typename T>
+int scratch_zero(const Scratch<T>& sc, cudaStream_t st) {
+  if (cudaMemsetAsync(sc.red.cnt, 0, RED_WS_COUNTERS * 4, st) != cudaSuccess)
+    MOBIUS_FAIL(MOBIUS_ECUDA, "scratch_zero");
+  return MOBIUS_OK;
 }
 
 // ------------------------------------------------------------ attention
@@ -407,8 +425,8 @@ int block_bwd(const Shape& sh, const T* w, const BlockActs<T>& A_in, const T* dy
   }
   {
     ElemScope es(st, 2);
-    RC(colsum_accum<T>(dy, h, Tn, h, G + L.b_2, st));
-    RC(colsum_accum<T>(du, 4 * h, Tn, 4 * h, G + L.b_1, st));
+    RC(colsum_accum<T>(dy, h, Tn, h, G + L.b_2, sc.red, st));
+    RC(colsum_accum<T>(du, 4 * h, Tn, 4 * h, G + L.b_1, sc.red, st));
   }
   {  // dW1 += a2^T du
     GemmDesc d;
@@ -430,7 +448,7 @@ int block_bwd(const Shape& sh, const T* w, const BlockActs<T>& A_in, const T* dy
   T* dx1 = sc.t2;
   {
     ElemScope es(st, 2);
-    RC(layernorm_bwd<T>(sc.t1, A.x1, w + L.ln2_g, A.mu2, A.rs2, dy, dx1, G + L.ln2_g, G + L.ln2_b, Tn, h, st));
+    RC(layernorm_bwd<T>(sc.t1, A.x1, w + L.ln2_g, A.mu2, A.rs2, dy, dx1, G + L.ln2_g, G + L.ln2_b, Tn, h, sc.red, st));
   }
   {  // dWo += o^T dx1
     GemmDesc d;
@@ -443,7 +461,7 @@ int block_bwd(const Shape& sh, const T* w, const BlockActs<T>& A_in, const T* dy
   }
   {
     ElemScope es(st, 1);
-    RC(colsum_accum<T>(dx1, h, Tn, h, G + L.b_o, st));
+    RC(colsum_accum<T>(dx1, h, Tn, h, G + L.b_o, sc.red, st));
   }
   T* dO = sc.t3;
   {  // do = dx1 Wo^T
@@ -467,7 +485,7 @@ int block_bwd(const Shape& sh, const T* w, const BlockActs<T>& A_in, const T* dy
   }
   {
     ElemScope es(st, 1);
-    RC(colsum_accum<T>(dqkv, 3 * h, Tn, 3 * h, G + L.b_qkv, st));
+    RC(colsum_accum<T>(dqkv, 3 * h, Tn, 3 * h, G + L.b_qkv, sc.red, st));
   }
   {  // da = dqkv Wqkv^T
     GemmDesc d;
@@ -479,7 +497,7 @@ int block_bwd(const Shape& sh, const T* w, const BlockActs<T>& A_in, const T* dy
   }
   {
     ElemScope es(st, 2);
-    RC(layernorm_bwd<T>(sc.t1, A.x, w + L.ln1_g, A.mu1, A.rs1, dx1, dx, G + L.ln1_g, G + L.ln1_b, Tn, h, st));
+    RC(layernorm_bwd<T>(sc.t1, A.x, w + L.ln1_g, A.mu1, A.rs1, dx1, dx, G + L.ln1_g, G + L.ln1_b, Tn, h, sc.red, st));
   }
   return MOBIUS_OK;
 }
@@ -495,7 +513,7 @@ template <typename T>
 int embed_layer_bwd(const Shape& sh, const T* w, const int32_t* tok, const T* dx, float* G, cudaStream_t st) {
   const EmbedLayout L(sh.h, sh.V, sh.s);
   ElemScope es(st, 2);
-  return embed_bwd<T>(tok, dx, G + L.wte, G + L.wpe, sh.mbs, sh.s, sh.h, st);
+  return embed_bwd<T>(tok, dx, G + L.wte, G + L.wpe, sh.mbs, sh.s, sh.h, sh.V, st);
 }
 
 template <typename T>
@@ -507,40 +525,48 @@ int head_layer_fwd_bwd(const Shape& sh, const T* w, const T* x, const int32_t* t
     ElemScope es(st, 1);
     RC(layernorm_fwd<T>(x, w + L.lnf_g, w + L.lnf_b, sc.t1, sc.mu, sc.rs, Tn, h, st));
   }
-  {  // logits = a Whead
-    GemmDesc d;
-    d.M = Tn; d.N = V; d.K = h;
-    d.A = mv(sc.t1, h);
-    d.B = mv(w + L.w_head, V); d.b_mn = true;
-    d.C = mv(sc.logits, V);
-    RC(run_gemm<T>(d, st, KCLS_GEMM));
-  }
-  {
-    ElemScope es(st, 2);
-    RC(cross_entropy_fwd_bwd<T>(sc.logits, tok, sc.loss_rows, Tn, V, sh.s, inv_ntok, st));
-    RC(loss_accumulate(sc.loss_rows, Tn, loss_acc, st));
-  }
-  {  // dWhead += a^T dlogits
-    GemmDesc d;
-    d.M = h; d.N = V; d.K = Tn;
-    d.A = mv(sc.t1, h); d.a_mn = true;
-    d.B = mv(sc.logits, V); d.b_mn = true;
-    d.C = mv(G + L.w_head, V); d.c_f32 = true;
-    d.epi = EPI_ACCUM; d.accumulate = true;
-    RC(run_gemm<T>(d, st, KCLS_GEMM));
-  }
-  {  // da = dlogits Whead^T
-    GemmDesc d;
-    d.M = Tn; d.N = h; d.K = V;
-    d.A = mv(sc.logits, V);
-    d.B = mv(w + L.w_head, V);
-    d.C = mv(sc.t2, h);
-    RC(run_gemm<T>(d, st, KCLS_GEMM));
+  // row chunks of hc rows (whole sequences): logits [hc, V] live in scratch,
+  // CE in place, dW accumulated chunk by chunk (fp32), da chunk into t2
+  const int hc = sh.head_chunk();
+  for (int r0 = 0; r0 < Tn; r0 += hc) {
+    const int rows = std::min(hc, Tn - r0);
+    const T* a = sc.t1 + (int64_t)r0 * h;
+    const int32_t* tk = tok + (int64_t)(r0 / sh.s) * (sh.s + 1);
+    {  // logits = a Whead
+      GemmDesc d;
+      d.M = rows; d.N = V; d.K = h;
+      d.A = mv(a, h);
+      d.B = mv(w + L.w_head, V); d.b_mn = true;
+      d.C = mv(sc.logits, V);
+      RC(run_gemm<T>(d, st, KCLS_GEMM));
+    }
+    {
+      ElemScope es(st, 2);
+      RC(cross_entropy_fwd_bwd<T>(sc.logits, tk, sc.loss_rows, rows, V, sh.s, inv_ntok, st));
+      RC(loss_accumulate(sc.loss_rows, rows, loss_acc, st));
+    }
+    {  // dWhead += a^T dlogits
+      GemmDesc d;
+      d.M = h; d.N = V; d.K = rows;
+      d.A = mv(a, h); d.a_mn = true;
+      d.B = mv(sc.logits, V); d.b_mn = true;
+      d.C = mv(G + L.w_head, V); d.c_f32 = true;
+      d.epi = EPI_ACCUM; d.accumulate = true;
+      RC(run_gemm<T>(d, st, KCLS_GEMM));
+    }
+    {  // da = dlogits Whead^T
+      GemmDesc d;
+      d.M = rows; d.N = h; d.K = V;
+      d.A = mv(sc.logits, V);
+      d.B = mv(w + L.w_head, V);
+      d.C = mv(sc.t2 + (int64_t)r0 * h, h);
+      RC(run_gemm<T>(d, st, KCLS_GEMM));
+    }
   }
   {
     ElemScope es(st, 2);
     RC(layernorm_bwd<T>(sc.t2, x, w + L.lnf_g, sc.mu, sc.rs, (const T*)nullptr, dx, G + L.lnf_g, G + L.lnf_b, Tn,
-                        h, st));
+                        h, sc.red, st));
   }
   return MOBIUS_OK;
 }
@@ -548,6 +574,7 @@ int head_layer_fwd_bwd(const Shape& sh, const T* w, const T* x, const int32_t* t
 #define INST(T)                                                                                                   \
   template void carve_block_acts<T>(const Shape&, uint8_t*, BlockActs<T>&, bool);                                      \
   template void carve_scratch<T>(const Shape&, uint8_t*, bool, Scratch<T>&);                                     \
+  template int scratch_zero<T>(const Scratch<T>&, cudaStream_t);                                                  \
   template int block_fwd<T>(const Shape&, const T*, BlockActs<T>&, T*, Scratch<T>&, cudaStream_t);               \
   template int block_bwd<T>(const Shape&, const T*, const BlockActs<T>&, const T*, T*, float*, Scratch<T>&,      \
                             cudaStream_t);                                                                       \

@@ -9,13 +9,16 @@
 #include <cuda_runtime.h>
 
 #include "../../include/mobius.h"
+#include "elem.h"
 
 namespace mobius {
 
 struct Shape {
   int h, nh, s, mbs, V;
+  int head_rows = 0;  // LM head row chunk (multiple of s; 0 = all T rows at once)
   int T() const { return mbs * s; }
   int dh() const { return h / nh; }
+  int head_chunk() const { return head_rows > 0 && head_rows < T() ? head_rows : T(); }
 };
 
 // element offsets of the block tensors inside one packed block (oracle order)
@@ -64,7 +67,11 @@ struct Scratch {
   float* loss_rows;  // [T]
   float *mu, *rs;  // [T] (head LN)
   T *ra, *ra2, *rg;  // recompute targets of a compact BlockActs: [T, h], [T, h], [T, 4h]
+  RedWs red;       // deterministic column-reduction workspace (counters zeroed by scratch_zero)
 };
+// zero the reduction counters of a freshly carved Scratch (once per arena)
+template <typename T>
+int scratch_zero(const Scratch<T>& sc, cudaStream_t st);
 
 // true when the fused tcgen05 attention is used (bf16, dh in {64,128}, s % 128 == 0)
 template <typename T>

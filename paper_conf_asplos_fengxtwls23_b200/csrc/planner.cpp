@@ -26,6 +26,8 @@ struct StageSum {
   int64_t Tf, Tb, Sf, Sb, Xf, Xb, A;
 };
 
+thread_local int64_t g_last_plan_nodes = 0;  // branch-and-bound nodes of the last mobius_plan (L' > 20)
+
 int64_t ceil_xfer_ns(int64_t bytes, int64_t bw) {
   if (bw <= 0 || bytes <= 0) return 0;
   __int128 num = (__int128)bytes * 1000000000LL;
@@ -307,6 +309,145 @@ extern "C" int mobius_cross_map(int K, int N, const int* group, int* perm_out, d
   return MOBIUS_OK;
 }
 
+// Exact partition search for L' > 20 (branch and bound over stage
+// boundaries, left to right).  For a prefix ending with stage j (first layer
+// a_j) the forward start times t^f of the prefix are final (Eq 8-10 only look
+// at earlier stages), and the dependency chain F_{j,M} -> ... -> F_{K,M} ->
+// B_{K,1} (Eq 11) -> ... -> B_{1,1} -> ... -> B_{1,M} (Eq 8 / 10) bounds the
+// makespan of every completion from below:
+//   LB = t^f_{j,M} + sum_{i >= a_j} t_f(i) + sum_i t_b(i) + (M - 1) T^b_1
+// (transfer terms >= 0 dropped; the sums are partition independent).  Ties
+// of the key (makespan, K, sizes) prune through the fewest stages any
+// completion needs (greedy packing from a_j) and the lexicographic order of
+// the prefix.  The local-search result seeds the incumbent; a node budget
+// (MOBIUS_PLAN_BNB_NODES, default 1M at N = 1, 200k otherwise) bounds the work - when it is hit the
+// search is not a certificate and the incumbent is returned.
+struct BnB {
+  const mobius_layer_profile* L;
+  int n, N, M;
+  int64_t G, Wh, Wp;
+  std::vector<int64_t> sf_suffix;   // sum t_f over layers >= i
+  int64_t sb_all = 0;
+  std::vector<int> min_stages;      // fewest stages covering layers >= i
+  std::vector<int> sizes;           // current prefix
+  std::vector<StageSum> st;         // prefix stage sums
+  std::vector<std::vector<int64_t>> tf;  // prefix forward start rows
+  std::vector<int> best;
+  int64_t best_mk = -1;
+  int64_t nodes = 0, node_limit = 0;
+  bool aborted = false;
+  std::vector<int64_t> wa, wb;
+
+  int64_t p2p(int64_t b) const { return N == 1 ? 0 : ceil_xfer_ns(b, Wp); }
+
+  void init() {
+    sf_suffix.assign(n + 1, 0);
+    for (int i = n - 1; i >= 0; --i) sf_suffix[i] = sf_suffix[i + 1] + L[i].t_fwd_ns;
+    for (int i = 0; i < n; ++i) sb_all += L[i].t_bwd_ns;
+    min_stages.assign(n + 1, 0);
+    for (int i = n - 1; i >= 0; --i) {  // greedy packing from i is the fewest contiguous stages
+      int cnt = 0, pos = i;
+      while (pos < n) {
+        int64_t a = 0, b = 0;
+        int q = pos;
+        while (q < n && a + L[q].mem_fwd <= G && b + L[q].mem_bwd <= G) {
+          a += L[q].mem_fwd;
+          b += L[q].mem_bwd;
+          ++q;
+        }
+        if (q == pos) {
+          cnt = INT_MAX / 2;
+          break;
+        }
+        ++cnt;
+        pos = q;
+      }
+      min_stages[i] = cnt;
+    }
+  }
+  // forward row of stage j = sizes.size()-1 (its sums in st.back())
+  void push_row() {
+    const int j = (int)st.size() - 1;
+    std::vector<int64_t> row(M, 0);
+    for (int m = 0; m < M; ++m) {
+      int64_t t = 0;
+      if (m > 0) t = std::max(t, row[m - 1] + st[j].Tf);
+      if (j > 0) t = std::max(t, tf[j - 1][m] + st[j - 1].Tf + p2p(st[j - 1].A));
+      if (m == 0 && j >= N) {
+        const int q = j - N;
+        const int64_t B = tf[q][0], E = tf[q][M - 1] + st[q].Tf;
+        t = std::max(t, std::max(E, std::max(E + ceil_xfer_ns(std::max<int64_t>(0, st[j].Xf - (G - st[q].Sf)), Wh),
+                                             B + ceil_xfer_ns(st[j].Xf, Wh))));
+      }
+      row[m] = t;
+    }
+    tf.push_back(row);
+  }
+  // false: no completion of the prefix can beat the incumbent's key
+  bool may_improve(int pos) const {
+    if (best_mk < 0) return true;
+    const int j = (int)st.size() - 1;
+    int64_t lb = tf[j][M - 1] + sf_suffix[pos - sizes.back()] + sb_all + (int64_t)(M - 1) * st[0].Tb;
+    // one GPU runs everything serially: after F_{j,M} it still runs M
+    // forwards of every later layer and M backwards of every layer
+    if (N == 1) lb = std::max(lb, tf[j][M - 1] + st[j].Tf + (int64_t)M * (sf_suffix[pos] + sb_all));
+    if (lb > best_mk) return false;
+    if (lb < best_mk) return true;
+    const int k_lb = (int)sizes.size() + (pos < n ? min_stages[pos] : 0);
+    if (k_lb > (int)best.size()) return false;
+    if (k_lb < (int)best.size()) return true;
+    // same K possible: the completion's sizes start with the prefix
+    for (size_t i = 0; i < sizes.size() && i < best.size(); ++i) {
+      if (sizes[i] != best[i]) return sizes[i] < best[i];
+    }
+    return true;
+  }
+  void dfs(int pos) {
+    if (aborted) return;
+    if (++nodes > node_limit) {
+      aborted = true;
+      return;
+    }
+    if (pos == n) {
+      const int64_t mk = cost(L, sizes.data(), (int)sizes.size(), N, G, M, Wh, Wp, nullptr, nullptr, wa, wb);
+      if (mk >= 0 && better(mk, sizes, best_mk, best)) {
+        best_mk = mk;
+        best = sizes;
+      }
+      return;
+    }
+    StageSum s{0, 0, 0, 0, 0, 0, 0};
+    for (int len = 1; pos + len <= n; ++len) {
+      const mobius_layer_profile& l = L[pos + len - 1];
+      s.Tf += l.t_fwd_ns;
+      s.Tb += l.t_bwd_ns;
+      s.Sf += l.mem_fwd;
+      s.Sb += l.mem_bwd;
+      s.Xf += l.xfer_fwd;
+      s.Xb += l.xfer_bwd;
+      s.A = l.act_out;
+      if (s.Sf > G || s.Sb > G) break;  // longer stages only grow (Eq 4)
+      sizes.push_back(len);
+      st.push_back(s);
+      push_row();
+      if (may_improve(pos + len)) dfs(pos + len);
+      tf.pop_back();
+      st.pop_back();
+      sizes.pop_back();
+      if (aborted) return;
+    }
+  }
+};
+
+// brute force over all 2^(L'-1) compositions up to this many profile layers
+// (MOBIUS_PLAN_EXHAUSTIVE_MAX, default 20, at most 26: tests compare it with
+// the branch and bound just above 20)
+static int exhaustive_limit() {
+  int v = 20;
+  if (const char* e = getenv("MOBIUS_PLAN_EXHAUSTIVE_MAX")) v = std::min(26, std::max(1, atoi(e)));
+  return v;
+}
+
 static int plan_impl(const mobius_layer_profile* layers, int n_layers, int N, int64_t G, int M,
                      const mobius_topology* topo_in, int algo, mobius_plan_t* out) {
   int rc = validate_profile(layers, n_layers);
@@ -325,6 +466,7 @@ static int plan_impl(const mobius_layer_profile* layers, int n_layers, int N, in
       MOBIUS_FAIL(MOBIUS_EINFEASIBLE, "layer %d needs %lld bytes > cap %lld", i,
                   (long long)std::max(layers[i].mem_fwd, layers[i].mem_bwd), (long long)G);
   const int64_t Wh = topo.host_bw_Bps, Wp = topo.p2p_bw_Bps;
+  g_last_plan_nodes = 0;
 
   std::vector<int> best;
   int64_t best_mk = -1;
@@ -352,7 +494,7 @@ static int plan_impl(const mobius_layer_profile* layers, int n_layers, int N, in
     }
     best_mk = cost(layers, best.data(), (int)best.size(), N, G, M, Wh, Wp, nullptr, nullptr, a, b);
     if (best_mk < 0) best.clear();
-  } else if (n_layers <= 20) {
+  } else if (n_layers <= exhaustive_limit()) {
     exhaustive = 1;
     std::vector<int> sizes;
     sizes.reserve(n_layers);
@@ -406,6 +548,27 @@ static int plan_impl(const mobius_layer_profile* layers, int n_layers, int N, in
         best = sizes;
       }
     }
+    // certify (or improve) the local-search result by branch and bound
+    BnB bb;
+    bb.L = layers;
+    bb.n = n_layers;
+    bb.N = N;
+    bb.M = M;
+    bb.G = G;
+    bb.Wh = Wh;
+    bb.Wp = Wp;
+    bb.node_limit = N == 1 ? 1000000 : 200000;  // the N > 1 bounds are weaker: best found
+    if (const char* e = getenv("MOBIUS_PLAN_BNB_NODES")) bb.node_limit = atoll(e);
+    bb.best = best;
+    bb.best_mk = best_mk;
+    bb.init();
+    if (bb.node_limit > 0) bb.dfs(0);
+    if (!bb.best.empty()) {
+      best = bb.best;
+      best_mk = bb.best_mk;
+    }
+    exhaustive = (!bb.aborted && bb.node_limit > 0) ? 1 : 0;
+    g_last_plan_nodes = bb.nodes;
   }
   if (best.empty()) MOBIUS_FAIL(MOBIUS_EINFEASIBLE, "no feasible partition under cap %lld", (long long)G);
 
@@ -486,6 +649,8 @@ extern "C" int mobius_discover_topology(mobius_topology* out) {
   }
   return MOBIUS_OK;
 }
+
+extern "C" int64_t mobius_plan_search_nodes(void) { return g_last_plan_nodes; }
 
 extern "C" int mobius_plan(const mobius_layer_profile* layers, int n_layers, int N, int64_t G, int M,
                            const mobius_topology* topo_in, mobius_plan_t* out) {

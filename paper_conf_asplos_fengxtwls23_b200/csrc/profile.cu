@@ -50,6 +50,12 @@ int profile_impl(const mobius_model_cfg& c, mobius_layer_profile* out, int Lp) {
   Scratch<T> sc;
   carve_block_acts<T>(sh, actb, acts);
   carve_scratch<T>(sh, scb, true, sc);
+  scratch_zero<T>(sc, 0);
+  {  // token ids spread over the vocabulary (a multiplicative hash of the position)
+    std::vector<int32_t> ht((size_t)sh.mbs * (sh.s + 1));
+    for (size_t i = 0; i < ht.size(); ++i) ht[i] = (int32_t)((i * 2654435761ull) % (uint64_t)sh.V);
+    cudaMemcpy(tok, ht.data(), ht.size() * 4, cudaMemcpyHostToDevice);
+  }
   acts.x = x0;
   cudaStream_t st;
   cudaStreamCreate(&st);

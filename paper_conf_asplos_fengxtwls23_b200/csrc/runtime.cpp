@@ -40,6 +40,7 @@
 #include "elem.h"
 #include "host.h"
 #include "flash.h"
+#include "gemm.h"
 #include "ops.h"
 
 namespace mobius {
@@ -78,8 +79,77 @@ struct Load {           // one residence of a stage in the ring
   int stage_local;      // index into mine
   int end;              // 0 bottom, 1 top
   int64_t base;         // byte offset in the ring
-  int64_t bytes;
+  int64_t bytes;        // footprint in the ring (weights; + dW / staging / recompute workspace, arena mode bwd)
+  int64_t copy;         // bytes copied in (the stage weights, at the start of the footprint)
+  bool bwd;             // the residence runs the stage's backward
 };
+
+// byte layout of a backward residence in MOBIUS_FLAG_ARENA_CAP mode:
+// [weights | fp32 dW | gradient staging | nb recompute activation sets |
+//  (has_embed + nb) activation buffers]
+struct BwdFootprint {
+  int64_t w, gacc, gst, acts, xs, total;
+};
+inline BwdFootprint bwd_footprint(int64_t np, int esz, int nb, bool has_embed, int64_t acts_bytes,
+                                  int64_t slot_bytes) {
+  auto al = [](int64_t x) { return (x + 255) & ~int64_t(255); };
+  BwdFootprint f;
+  f.w = 0;
+  f.gacc = al(np * esz);
+  f.gst = f.gacc + al(np * 4);
+  f.acts = f.gst + al(np * esz);
+  f.xs = f.acts + nb * acts_bytes;
+  f.total = f.xs + (nb + (has_embed ? 1 : 0)) * slot_bytes;
+  return f;
+}
+
+// The arena behind the ring: offsets of every fixed region (shared by
+// mobius_create and mobius_arena_fixed_bytes, so the planner's G_eff and the
+// runtime's layout agree by construction).  Arena mode keeps no dW /
+// staging here (they live in the backward residences), 5 activation buffers
+// (embedding output, forward pingpong, backward pingpong) and one forward
+// activation set; with checkpoint offload the checkpoint and gradient slots
+// are two banks of M.
+struct FixedLayout {
+  int64_t gacc, gstage, ckpt, gslot, fflag, bflag, xs, scr, tok, loss, bad, acts, end;
+  int xs_slots, slot_sets;
+};
+inline FixedLayout fixed_layout(const Shape& sh, int esz, bool flash, int M, int n, int max_blocks,
+                                int64_t max_params, bool arena, bool offload, int64_t slot, int64_t ring) {
+  auto al = [](int64_t x) { return (x + 255) & ~int64_t(255); };
+  FixedLayout f;
+  int64_t off = al(ring);
+  auto take = [&](int64_t bytes) {
+    int64_t o = off;
+    off += al(bytes);
+    return o;
+  };
+  f.slot_sets = offload ? 2 : n;
+  f.xs_slots = arena ? 5 : max_blocks + 3;
+  f.gacc = take(arena ? 0 : max_params * 4);
+  f.gstage = take(arena ? 0 : max_params * esz);
+  f.ckpt = take((int64_t)f.slot_sets * M * slot);
+  f.gslot = take((int64_t)f.slot_sets * M * slot);
+  f.fflag = take((int64_t)n * M * 4);
+  f.bflag = take((int64_t)n * M * 4);
+  f.xs = take(slot * f.xs_slots);
+  f.scr = take(scratch_bytes(sh, esz, true, flash));
+  f.tok = take((int64_t)M * sh.mbs * (sh.s + 1) * 4);
+  f.loss = take(8);
+  f.bad = take(4);
+  f.acts = off;  // recompute workspace last (non-arena: its size depends on the keep plan)
+  f.end = arena ? f.acts + al(block_acts_bytes(sh, esz, flash)) : f.acts;
+  return f;
+}
+
+// LM head row chunk in arena mode: MOBIUS_HEAD_ROWS (default 2048) rounded
+// down to whole sequences
+inline int arena_head_rows(const Shape& sh) {
+  int r = 2048;
+  if (const char* e = getenv("MOBIUS_HEAD_ROWS")) r = atoi(e);
+  r = std::max(sh.s, r / sh.s * sh.s);
+  return std::min(r, sh.T());
+}
 
 struct EventTimer : KernelTimer {
   struct Rec {
@@ -236,7 +306,90 @@ struct mobius_ctx {
   EventTimer timer;
   mobius_step_stats stats;
   int64_t launches_step = 0;
+  int* h_bad_tok = nullptr;       // pinned: out-of-range token count (mobius_step_device check)
+  // MOBIUS_FLAG_ARENA_CAP / MOBIUS_FLAG_CKPT_OFFLOAD
+  bool arena_mode = false, offload = false;
+  int xs_fixed = 0;               // fixed activation buffers (pingpong of backward at xs_fixed-2, -1)
+  std::vector<void*> h_ckpt;      // pinned, per local stage: its M offloaded checkpoints (nullptr if resident)
+  std::vector<char> ck_off;       // per local stage: checkpoint offloaded in forward / uploaded in backward
+  std::vector<cudaEvent_t> ev_ckoff;              // [2][M]: last offload of bank slot done (s_d2h)
+  std::vector<cudaEvent_t> ev_ckprod;             // [M]: a stage input produced (s_comp)
+  std::vector<cudaEvent_t> ev_ckup;               // per local stage: its upload done (s_ckup)
+  std::vector<cudaEvent_t> ev_ck_a, ev_ck_b;      // per local stage x {offload, upload}: timeline
+  std::vector<cudaEvent_t> ev_ckw_a, ev_ckw_b;    // per local stage: compute waiting on its upload
+  cudaEvent_t ev_fwd_off = nullptr;               // all forward offloads issued so far done (s_d2h)
+  cudaStream_t s_ckup = nullptr;
+  int* bad_tok_dev = nullptr;     // its device counter (arena)
+
+  // Releases everything owned so far: mobius_destroy, and any early return
+  // of mobius_create (partially built context held by a unique_ptr).
+  ~mobius_ctx() { teardown(); }
+  void teardown();
 };
+
+void mobius_ctx::teardown() {
+  cudaSetDevice(dist.device);
+  {
+    std::lock_guard<std::mutex> g(upd_mu);
+    upd_stop = true;
+  }
+  upd_cv.notify_all();
+  if (upd_thread.joinable()) upd_thread.join();
+  if (s_comp) cudaStreamSynchronize(s_comp);
+  if (s_h2d) cudaStreamSynchronize(s_h2d);
+  if (s_d2h) cudaStreamSynchronize(s_d2h);
+  for (auto p : peer_base)
+    if (p) cudaIpcCloseMemHandle(p);
+  peer_base.clear();
+  if (s_ckup) cudaStreamSynchronize(s_ckup);
+  for (auto* v : {&ev_release, &ev_loaded, &ev_part_a, &ev_part_b, &ev_gready, &ev_d2h, &ev_wait_a, &ev_wait_b,
+                  &ev_pass_a, &ev_pass_b, &ev_off_a, &ev_off_b, &ev_ckoff, &ev_ckprod, &ev_ckup, &ev_ck_a,
+                  &ev_ck_b, &ev_ckw_a, &ev_ckw_b}) {
+    for (auto e : *v)
+      if (e) cudaEventDestroy(e);
+    v->clear();
+  }
+  if (ev_step0) cudaEventDestroy(ev_step0);
+  if (ev_step1) cudaEventDestroy(ev_step1);
+  if (ev_fwd_off) cudaEventDestroy(ev_fwd_off);
+  ev_step0 = ev_step1 = ev_fwd_off = nullptr;
+  for (auto p : h_ckpt)
+    if (p) cudaFreeHost(p);
+  h_ckpt.clear();
+  for (auto p : h_weights)
+    if (p) cudaFreeHost(p);
+  for (auto p : h_grads)
+    if (p) cudaFreeHost(p);
+  for (auto p : h_master) std::free(p);
+  for (auto p : h_m) std::free(p);
+  for (auto p : h_v) std::free(p);
+  h_weights.clear();
+  h_grads.clear();
+  h_master.clear();
+  h_m.clear();
+  h_v.clear();
+  if (h_loss) cudaFreeHost(h_loss);
+  if (h_tokens) cudaFreeHost(h_tokens);
+  if (h_bad_tok) cudaFreeHost(h_bad_tok);
+  h_loss = nullptr;
+  h_tokens = nullptr;
+  h_bad_tok = nullptr;
+  if (arena) cudaFree(arena);
+  if (keep_pool) cudaFree(keep_pool);
+  if (d_opt) cudaFree(d_opt);
+  if (d_wstage) cudaFree(d_wstage);
+  arena = keep_pool = d_wstage = nullptr;
+  d_opt = nullptr;
+  if (s_comp) {
+    gemm_release_stream(s_comp);
+    cudaStreamDestroy(s_comp);
+  }
+  if (s_h2d) cudaStreamDestroy(s_h2d);
+  if (s_d2h) cudaStreamDestroy(s_d2h);
+  if (s_ckup) cudaStreamDestroy(s_ckup);
+  s_comp = s_h2d = s_d2h = s_ckup = nullptr;
+  cudaGetLastError();  // a failed create must not leave a stale error for the caller's next CUDA call
+}
 
 namespace {
 
@@ -358,9 +511,17 @@ struct StepRunner {
   int64_t h2d_bytes = 0, d2d_bytes = 0;
   int n_parts = 0;
 
+  int64_t ckpt_d2h = 0, ckpt_h2d = 0;
+  uint8_t* xrec_base = nullptr;      // backward recompute buffers: xrec(0) embedding output, xrec(b+1) block b output
+  std::vector<BlockActs<T>> racts;   // backward recompute activation sets (acts, or the residence's in arena mode)
+
   T* xbuf(int i) { return tptr<T>(ctx->xs_base + (int64_t)i * ctx->slot_bytes); }
-  T* ckpt_slot(int ls, int m) { return tptr<T>(ctx->ckpt + ((int64_t)ls * M + m) * ctx->slot_bytes); }
-  T* grad_slot(int ls, int m) { return tptr<T>(ctx->gslot + ((int64_t)ls * M + m) * ctx->slot_bytes); }
+  T* xrec(int i) { return tptr<T>(xrec_base + (int64_t)i * ctx->slot_bytes); }
+  // checkpoint / activation-gradient slots: one set of M per local stage, or
+  // with checkpoint offload two banks of M (local stage ord uses bank ord % 2)
+  int64_t slot_index(int ls, int m) const { return (int64_t)(ctx->offload ? ls % 2 : ls) * M + m; }
+  T* ckpt_slot(int ls, int m) { return tptr<T>(ctx->ckpt + slot_index(ls, m) * ctx->slot_bytes); }
+  T* grad_slot(int ls, int m) { return tptr<T>(ctx->gslot + slot_index(ls, m) * ctx->slot_bytes); }
   const int32_t* tok(int m) { return tok_dev + (int64_t)m * ctx->sh.mbs * (ctx->sh.s + 1); }
 
   // destination slot of stage j's output for microbatch m (the input of j+1)
@@ -437,7 +598,7 @@ struct StepRunner {
   // bottom load; for a top load the non-overlapping bytes are [split, S)
   void split_of(int r, int64_t& first0, int64_t& first1, int64_t& second0, int64_t& second1) {
     const Load& L = ctx->loads[r];
-    const int64_t S = L.bytes, G = ctx->ring_bytes;
+    const int64_t S = L.copy, G = ctx->ring_bytes;  // the copied bytes vs the previous footprint
     if (r == 0) {
       first0 = 0, first1 = S, second0 = second1 = 0;
       return;
@@ -453,9 +614,19 @@ struct StepRunner {
     (void)G;
   }
 
+  // arena mode: a backward residence holds its stage's gradient staging,
+  // read by the D2H offload after the release - overwrite only after it
+  int wait_offload_of(int r) {
+    const Load& P = ctx->loads[r];
+    if (ctx->arena_mode && P.bwd) CU(cudaStreamWaitEvent(ctx->s_h2d, ctx->ev_d2h[P.stage_local], 0));
+    return MOBIUS_OK;
+  }
   int load_first_part(int r) {  // issued when residence r-1 starts computing
     if (r >= (int)ctx->loads.size()) return MOBIUS_OK;
-    if (r >= 2) CU(cudaStreamWaitEvent(ctx->s_h2d, ctx->ev_release[r - 2], 0));
+    if (r >= 2) {
+      CU(cudaStreamWaitEvent(ctx->s_h2d, ctx->ev_release[r - 2], 0));
+      RC(wait_offload_of(r - 2));
+    }
     int64_t a0, a1, b0, b1;
     split_of(r, a0, a1, b0, b1);
     return issue_part(r, a0, a1);
@@ -464,7 +635,10 @@ struct StepRunner {
     if (r >= (int)ctx->loads.size()) return MOBIUS_OK;
     int64_t a0, a1, b0, b1;
     split_of(r, a0, a1, b0, b1);
-    if (r >= 1 && b1 > b0) CU(cudaStreamWaitEvent(ctx->s_h2d, ctx->ev_release[r - 1], 0));
+    if (r >= 1 && b1 > b0) {
+      CU(cudaStreamWaitEvent(ctx->s_h2d, ctx->ev_release[r - 1], 0));
+      RC(wait_offload_of(r - 1));
+    }
     RC(issue_part(r, b0, b1));
     CU(cudaEventRecord(ctx->ev_loaded[r], ctx->s_h2d));
     return MOBIUS_OK;
@@ -550,17 +724,17 @@ struct StepRunner {
       }
       if (k0 > 0) {  // recompute blocks [0, k0) from the stage input (their outputs match the kept inputs)
         if (st.has_embed) {
-          RC(embed_layer_fwd<T>(sh, stage_w(res, st, 0), tok(m), xbuf(0), s));
-          x = xbuf(0);
+          RC(embed_layer_fwd<T>(sh, stage_w(res, st, 0), tok(m), xrec(0), s));
+          x = xrec(0);
         } else {
           x = ckpt_slot(ls, m);
         }
         int b = 0;
         for (int li = st.first; li < st.last && b < k0; ++li) {
           if (li == 0 || li == ctx->cfg.n_layers + 1) continue;
-          T* y = xbuf(b + 1);
-          acts[b].x = x;
-          RC(block_fwd<T>(sh, stage_w(res, st, li), acts[b], y, sc, s));
+          T* y = xrec(b + 1);
+          racts[b].x = x;
+          RC(block_fwd<T>(sh, stage_w(res, st, li), racts[b], y, sc, s));
           x = y;
           ++b;
         }
@@ -570,23 +744,23 @@ struct StepRunner {
     } else {
       // recompute the stage forward from the checkpoint (a5/a7)
       if (st.has_embed) {
-        RC(embed_layer_fwd<T>(sh, stage_w(res, st, 0), tok(m), xbuf(0), s));
-        x = xbuf(0);
+        RC(embed_layer_fwd<T>(sh, stage_w(res, st, 0), tok(m), xrec(0), s));
+        x = xrec(0);
       } else {
         x = ckpt_slot(ls, m);
       }
       for (int li = st.first; li < st.last; ++li) {
         if (li == 0 || li == ctx->cfg.n_layers + 1) continue;
-        T* y = xbuf(bi + 1);
-        acts[bi].x = x;
-        RC(block_fwd<T>(sh, stage_w(res, st, li), acts[bi], y, sc, s));
+        T* y = xrec(bi + 1);
+        racts[bi].x = x;
+        RC(block_fwd<T>(sh, stage_w(res, st, li), racts[bi], y, sc, s));
         x = y;
         ++bi;
       }
     }
     // gradient w.r.t. the stage output
     const T* dy;
-    T* pingpong[2] = {xbuf(ctx->max_blocks + 1), xbuf(ctx->max_blocks + 2)};
+    T* pingpong[2] = {xbuf(ctx->xs_fixed - 2), xbuf(ctx->xs_fixed - 1)};
     int pp = 0;
     if (st.has_head) {
       const int hl = ctx->cfg.n_layers + 1;
@@ -614,7 +788,7 @@ struct StepRunner {
         pp ^= 1;
       }
       float* G = ctx->grad_acc + st.layer_off[li - st.first];
-      RC(block_bwd<T>(sh, stage_w(res, st, li), (kept(ls) && bi >= kf(ls)) ? kacts[bi - kf(ls)] : acts[bi], dy, dx,
+      RC(block_bwd<T>(sh, stage_w(res, st, li), (kept(ls) && bi >= kf(ls)) ? kacts[bi - kf(ls)] : racts[bi], dy, dx,
                       G, sc, s));
       if (flag) { RC(flag_set(flag, (int)seq, s)); ++ctx->launches_step; }
       dy = dx;
@@ -669,6 +843,58 @@ struct StepRunner {
     return MOBIUS_OK;
   }
 
+  // backward buffers of local stage ls in residence res: the fixed
+  // workspace, or (arena mode) the residence's own dW / staging / recompute
+  // region behind the weights
+  void prepare_bwd(int ls, int res) {
+    if (!ctx->arena_mode) {
+      xrec_base = ctx->xs_base;
+      racts = acts;
+      return;
+    }
+    const StageDesc& st = ctx->all[ctx->mine[ls]];
+    const BwdFootprint f = bwd_footprint(st.n_params, ctx->esz, st.n_blocks, st.has_embed, ctx->acts_bytes,
+                                         ctx->slot_bytes);
+    uint8_t* base = ctx->ring + ctx->loads[res].base;
+    ctx->grad_acc = reinterpret_cast<float*>(base + f.gacc);
+    ctx->grad_stage = base + f.gst;
+    racts.resize(std::max(1, st.n_blocks));
+    for (int b = 0; b < st.n_blocks; ++b) carve_block_acts<T>(ctx->sh, base + f.acts + b * ctx->acts_bytes, racts[b]);
+    // xrec(0) is the embedding output (embedding stages only)
+    xrec_base = base + f.xs - (st.has_embed ? 0 : ctx->slot_bytes);
+  }
+
+  // ---- checkpoint offload (A_Mobius), world size 1
+  // stage k's input slot (bank k % 2) is overwritten by stage k+2's input:
+  // offloaded right after F_{k-1,m} produced it, uploaded after B_{k+2}
+  int ckpt_offload(int k, int m) {
+    const int64_t sb = ctx->slot_bytes;
+    CU(cudaEventRecord(ctx->ev_ckprod[m], ctx->s_comp));
+    CU(cudaStreamWaitEvent(ctx->s_d2h, ctx->ev_ckprod[m], 0));
+    if (m == 0) CU(cudaEventRecord(ctx->ev_ck_a[2 * k], ctx->s_d2h));
+    CU(cudaMemcpyAsync((uint8_t*)ctx->h_ckpt[k] + m * sb, ckpt_slot(k, m), sb, cudaMemcpyDeviceToHost, ctx->s_d2h));
+    CU(cudaEventRecord(ctx->ev_ckoff[slot_index(k, m)], ctx->s_d2h));
+    if (m == M - 1) {
+      CU(cudaEventRecord(ctx->ev_ck_b[2 * k], ctx->s_d2h));
+      CU(cudaEventRecord(ctx->ev_fwd_off, ctx->s_d2h));
+    }
+    ckpt_d2h += sb;
+    return MOBIUS_OK;
+  }
+  int ckpt_upload(int k, cudaEvent_t after) {
+    const int64_t sb = ctx->slot_bytes;
+    CU(cudaStreamWaitEvent(ctx->s_ckup, after, 0));
+    CU(cudaStreamWaitEvent(ctx->s_ckup, ctx->ev_fwd_off, 0));
+    CU(cudaEventRecord(ctx->ev_ck_a[2 * k + 1], ctx->s_ckup));
+    for (int m = 0; m < M; ++m)
+      CU(cudaMemcpyAsync(ckpt_slot(k, m), (uint8_t*)ctx->h_ckpt[k] + m * sb, sb, cudaMemcpyHostToDevice,
+                         ctx->s_ckup));
+    CU(cudaEventRecord(ctx->ev_ck_b[2 * k + 1], ctx->s_ckup));
+    CU(cudaEventRecord(ctx->ev_ckup[k], ctx->s_ckup));
+    ckpt_h2d += M * sb;
+    return MOBIUS_OK;
+  }
+
   int run() {
     const int n = (int)ctx->mine.size();
     cudaStream_t s = ctx->s_comp;
@@ -682,6 +908,7 @@ struct StepRunner {
     for (int k = n - 1; k >= 0; --k) ex.push_back({0, k, ctx->res_b[k], k != n - 1, true});
     RC(load_first_part(0));
     RC(load_second_part(0));
+    std::vector<int> bwd_xi(n, -1);
     for (size_t xi = 0; xi < ex.size(); ++xi) {
       const Exec& e = ex[xi];
       if (e.first_of_res) {
@@ -689,19 +916,39 @@ struct StepRunner {
         RC(load_first_part(e.res + 1));  // prefetch of the next residence starts with this one
       }
       CU(cudaEventRecord(ctx->ev_pass_a[xi], s));
-      if (!e.fwd) CU(cudaMemsetAsync(ctx->grad_acc, 0, ctx->all[ctx->mine[e.ls]].n_params * 4, s));
+      if (!e.fwd) {
+        prepare_bwd(e.ls, e.res);
+        if (ctx->ck_off[e.ls]) {  // this stage's checkpoints come back from DRAM
+          CU(cudaEventRecord(ctx->ev_ckw_a[e.ls], s));
+          CU(cudaStreamWaitEvent(s, ctx->ev_ckup[e.ls], 0));
+          CU(cudaEventRecord(ctx->ev_ckw_b[e.ls], s));
+        }
+        CU(cudaMemsetAsync(ctx->grad_acc, 0, ctx->all[ctx->mine[e.ls]].n_params * 4, s));
+      }
       for (int m = 0; m < M; ++m) {
-        if (e.fwd)
+        if (e.fwd) {
+          // the output slot (input of stage ls+1) last held stage ls-1's input:
+          // its offload must have finished
+          if (e.ls + 1 < n && e.ls >= 1 && ctx->ck_off[e.ls - 1])
+            CU(cudaStreamWaitEvent(s, ctx->ev_ckoff[slot_index(e.ls + 1, m)], 0));
           RC(forward(e.ls, e.res, m));
-        else
+          if (e.ls + 1 < n && ctx->ck_off[e.ls + 1]) RC(ckpt_offload(e.ls + 1, m));
+        } else {
           RC(backward(e.ls, e.res, m));
+        }
       }
       CU(cudaEventRecord(ctx->ev_pass_b[xi], s));
+      if (!e.fwd) {
+        bwd_xi[e.ls] = (int)xi;
+        // stage ls-2's checkpoints go back into the bank slots B_{ls} just freed
+        if (e.ls >= 2 && ctx->ck_off[e.ls - 2]) RC(ckpt_upload(e.ls - 2, ctx->ev_pass_b[xi]));
+      }
+      if (!e.fwd && ctx->arena_mode) RC(finish_stage_grads(e.ls));  // D2H recorded before the release waits on it
       if (e.last_of_res) {
         CU(cudaEventRecord(ctx->ev_release[e.res], s));
         RC(load_second_part(e.res + 1));
       }
-      if (!e.fwd) RC(finish_stage_grads(e.ls));
+      if (!e.fwd && !ctx->arena_mode) RC(finish_stage_grads(e.ls));
     }
     ctx->last_bwd_host_ns = 0;
     return MOBIUS_OK;
@@ -724,6 +971,7 @@ int do_step(mobius_ctx* ctx, const int32_t* tok_dev, int M, float* loss_out) {
   R.seq = ctx->step_count + 1;
   R.inv_ntok = 1.0f / ((float)M * sh.mbs * sh.s);
   carve_scratch<T>(sh, ctx->scratch_base, true, R.sc);
+  if (ctx->step_count == 0) RC(scratch_zero<T>(R.sc, ctx->s_comp));
   R.acts.resize(std::max(1, ctx->ws_blocks));
   for (int i = 0; i < (int)R.acts.size(); ++i) carve_block_acts<T>(sh, ctx->acts_base + i * ctx->acts_bytes, R.acts[i]);
   ctx->trace.clear();
@@ -736,6 +984,8 @@ int do_step(mobius_ctx* ctx, const int32_t* tok_dev, int M, float* loss_out) {
   int64_t t0 = now_ns();
   CU(cudaEventRecord(ctx->ev_step0, ctx->s_comp));
   CU(cudaMemsetAsync(ctx->loss_dev, 0, sizeof(double), ctx->s_comp));
+  if (getenv("MOBIUS_INJECT_CUDA_FAULT"))  // test hook: a (non-sticky) CUDA API failure inside the step
+    CU(cudaMemcpyAsync(ctx->tok_dev, nullptr, 4, cudaMemcpyDeviceToDevice, ctx->s_comp));
   int rc = R.run();
   set_kernel_timer(nullptr);
   if (rc) {
@@ -763,6 +1013,8 @@ int do_step(mobius_ctx* ctx, const int32_t* tok_dev, int M, float* loss_out) {
   cudaEventElapsedTime(&ms, ctx->ev_step0, ctx->ev_step1);
   S.device_step_ns = (int64_t)(ms * 1e6);
   S.h2d_bytes = R.h2d_bytes;
+  S.ckpt_d2h_bytes = R.ckpt_d2h;
+  S.ckpt_h2d_bytes = R.ckpt_h2d;
   S.n_h2d_copies = R.n_parts;
   S.d2d_bytes = R.d2d_bytes;
   ctx->n_parts_last = R.n_parts;
@@ -785,6 +1037,13 @@ int do_step(mobius_ctx* ctx, const int32_t* tok_dev, int M, float* loss_out) {
     if (cudaEventElapsedTime(&wm, ctx->ev_wait_a[r], ctx->ev_wait_b[r]) == cudaSuccess) exposed += (int64_t)(wm * 1e6);
   }
   S.exposed_load_ns = exposed;
+  int64_t exposed_ck = 0;
+  for (int ls = 0; ls < (int)ctx->mine.size(); ++ls) {
+    float wm = 0.f;
+    if (ctx->ck_off[ls] && cudaEventElapsedTime(&wm, ctx->ev_ckw_a[ls], ctx->ev_ckw_b[ls]) == cudaSuccess)
+      exposed_ck += (int64_t)(wm * 1e6);
+  }
+  S.exposed_ckpt_ns = exposed_ck;
   for (auto& rec : ctx->timer.recs) {
     float km = 0.f;
     if (cudaEventElapsedTime(&km, rec.a, rec.b) != cudaSuccess) continue;
@@ -805,7 +1064,10 @@ int do_step(mobius_ctx* ctx, const int32_t* tok_dev, int M, float* loss_out) {
   S.arena_bytes = ctx->arena_bytes + ctx->keep_bytes;
   S.ring_bytes = ctx->ring_bytes;
   int64_t pinned = 0;
-  for (int ls = 0; ls < (int)ctx->mine.size(); ++ls) pinned += 2 * ctx->all[ctx->mine[ls]].n_params * ctx->esz;
+  for (int ls = 0; ls < (int)ctx->mine.size(); ++ls) {
+    pinned += 2 * ctx->all[ctx->mine[ls]].n_params * ctx->esz;
+    if (ctx->h_ckpt[ls]) pinned += (int64_t)ctx->max_M * ctx->slot_bytes;
+  }
   S.pinned_bytes = pinned;
   S.host_update_ns = ctx->upd_ns;
   S.update_tail_ns = t1 - t_gpu_done;
@@ -822,6 +1084,57 @@ int do_step(mobius_ctx* ctx, const int32_t* tok_dev, int M, float* loss_out) {
 }  // namespace
 
 // ======================================================================
+static int arena_shape(const mobius_model_cfg* c, Shape* sh, int* esz, bool* flash) {
+  MOBIUS_CHECK_ARG(c && c->n_layers >= 1 && c->hidden > 0 && c->n_heads > 0 && c->hidden % c->n_heads == 0 &&
+                       c->seq_len > 0 && c->vocab > 0 && c->micro_batch > 0 && c->n_layers + 2 <= MOBIUS_MAX_LAYERS,
+                   "bad model config");
+  *sh = Shape{c->hidden, c->n_heads, c->seq_len, c->micro_batch, c->vocab};
+  sh->head_rows = arena_head_rows(*sh);
+  *esz = c->dtype == MOBIUS_F32 ? 4 : 2;
+  *flash = *esz == 2 && flash_supported(sh->dh(), sh->s);
+  return MOBIUS_OK;
+}
+
+extern "C" int mobius_arena_layer_sizes(const mobius_model_cfg* c, mobius_layer_profile* out, int* n_out) {
+  MOBIUS_CHECK_ARG(out && n_out, "null argument");
+  Shape sh;
+  int esz;
+  bool fl;
+  if (int rc = arena_shape(c, &sh, &esz, &fl)) return rc;
+  const int64_t slot = al256((int64_t)sh.T() * sh.h * esz);
+  const int64_t acts = al256(block_acts_bytes(sh, esz, fl));
+  const int Lp = c->n_layers + 2;
+  for (int i = 0; i < Lp; ++i) {
+    const int64_t np = layer_numel(*c, i);
+    const bool block = i > 0 && i < Lp - 1;
+    // a stage's footprint is the sum over its layers of these (each region
+    // rounded up per layer: >= the runtime's per-stage rounding)
+    const BwdFootprint f = bwd_footprint(np, esz, block ? 1 : 0, i == 0, acts, slot);
+    mobius_layer_profile& p = out[i];
+    std::memset(&p, 0, sizeof(p));
+    p.mem_fwd = al256(np * esz);
+    p.mem_bwd = f.total;
+    p.xfer_fwd = p.xfer_bwd = np * esz;
+    p.act_out = (int64_t)sh.T() * sh.h * esz;
+  }
+  *n_out = Lp;
+  return MOBIUS_OK;
+}
+
+extern "C" int mobius_arena_fixed_bytes(const mobius_model_cfg* c, int n_microbatches, int n_local_stages, int flags,
+                                        int64_t* bytes) {
+  MOBIUS_CHECK_ARG(bytes && n_microbatches >= 1 && n_local_stages >= 1, "bad arguments");
+  Shape sh;
+  int esz;
+  bool fl;
+  if (int rc = arena_shape(c, &sh, &esz, &fl)) return rc;
+  const int64_t slot = al256((int64_t)sh.T() * sh.h * esz);
+  const FixedLayout f = fixed_layout(sh, esz, fl, n_microbatches, n_local_stages, 0, 0, true,
+                                     (flags & MOBIUS_FLAG_CKPT_OFFLOAD) != 0, slot, 0);
+  *bytes = f.end;
+  return MOBIUS_OK;
+}
+
 extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* plan, const mobius_dist* dist,
                              const float* init_params, uint64_t seed, mobius_ctx** out) {
   MOBIUS_CHECK_ARG(cfg && plan && dist && out, "null argument");
@@ -887,6 +1200,28 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
   MOBIUS_CHECK_ARG(!ctx->mine.empty(), "rank %d owns no stage", dist->rank);
   const int n = (int)ctx->mine.size();
 
+  const bool arena = (dist->flags & MOBIUS_FLAG_ARENA_CAP) != 0;
+  const bool offload = (dist->flags & MOBIUS_FLAG_CKPT_OFFLOAD) != 0;
+  MOBIUS_CHECK_ARG(!offload || dist->world == 1, "MOBIUS_FLAG_CKPT_OFFLOAD needs world size 1 (banked slots are "
+                                                 "written by a peer at N > 1)");
+  MOBIUS_CHECK_ARG(!(arena && (dist->flags & MOBIUS_FLAG_DEVICE_TAIL_UPDATE)),
+                   "MOBIUS_FLAG_ARENA_CAP excludes MOBIUS_FLAG_DEVICE_TAIL_UPDATE (its optimizer state is outside "
+                   "the capped memory)");
+  MOBIUS_CHECK_ARG(!arena || plan->hbm_cap_bytes > 0, "MOBIUS_FLAG_ARENA_CAP needs a cap");
+  ctx->arena_mode = arena;
+  ctx->offload = offload;
+  if (arena) ctx->sh.head_rows = arena_head_rows(ctx->sh);
+
+  // per-microbatch sizes
+  const Shape& sh = ctx->sh;
+  const int M = plan->n_microbatches > 0 ? plan->n_microbatches : dist->world;
+  ctx->max_M = M;
+  ctx->slot_bytes = al256((int64_t)sh.T() * sh.h * esz);
+  const bool fl = esz == 2 && flash_supported(sh.dh(), sh.s);
+  ctx->acts_bytes = al256(block_acts_bytes(sh, esz, fl));
+  ctx->keep_compact = fl && !getenv("MOBIUS_KEEP_FULL");
+  ctx->keep_acts_bytes = al256(block_acts_bytes(sh, esz, fl, ctx->keep_compact));
+
   // ring: cap G (plan) or double-buffer default
   int64_t max_stage = 0, max_params = 0;
   for (int ls = 0; ls < n; ++ls) {
@@ -896,54 +1231,55 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
     ctx->max_blocks = std::max(ctx->max_blocks, st.n_blocks);
   }
   int64_t G = plan->hbm_cap_bytes > 0 ? (plan->hbm_cap_bytes & ~int64_t(255)) : 2 * al256(max_stage);
-  if (c.dtype == MOBIUS_F32 && plan->hbm_cap_bytes > 0) G = G;  // cap given in the path precision by the caller
-  if (max_stage > G) MOBIUS_FAIL(MOBIUS_EINFEASIBLE, "stage of %lld bytes exceeds the cap %lld", (long long)max_stage, (long long)G);
   ctx->ring_bytes = G;
 
   // residences: fwd loads ascending, bwd reloads descending except the last
+  // (which stays resident: its forward residence is its backward one)
+  auto footprint = [&](int k, bool bwd) -> int64_t {
+    const StageDesc& st = ctx->all[ctx->mine[k]];
+    if (!arena || !bwd) return st.n_params * esz;
+    return bwd_footprint(st.n_params, esz, st.n_blocks, st.has_embed, ctx->acts_bytes, ctx->slot_bytes).total;
+  };
   ctx->res_f.assign(n, -1);
   ctx->res_b.assign(n, -1);
   for (int k = 0; k < n; ++k) {
     ctx->res_f[k] = (int)ctx->loads.size();
-    ctx->loads.push_back({k, 0, 0, ctx->all[ctx->mine[k]].n_params * esz});
+    const bool last = k == n - 1;
+    ctx->loads.push_back({k, 0, 0, footprint(k, last), ctx->all[ctx->mine[k]].n_params * esz, last});
   }
   ctx->res_b[n - 1] = ctx->res_f[n - 1];
   for (int k = n - 2; k >= 0; --k) {
     ctx->res_b[k] = (int)ctx->loads.size();
-    ctx->loads.push_back({k, 0, 0, ctx->all[ctx->mine[k]].n_params * esz});
+    ctx->loads.push_back({k, 0, 0, footprint(k, true), ctx->all[ctx->mine[k]].n_params * esz, true});
   }
+  int64_t max_fp = 0;
+  for (const Load& L : ctx->loads) max_fp = std::max(max_fp, L.bytes);
+  if (max_fp > G)
+    MOBIUS_FAIL(MOBIUS_EINFEASIBLE, "stage %s of %lld bytes exceeds the cap %lld", arena ? "footprint" : "",
+                (long long)max_fp, (long long)G);
   for (size_t r = 0; r < ctx->loads.size(); ++r) {
     Load& L = ctx->loads[r];
     L.end = (int)(r % 2);
     L.base = L.end == 0 ? 0 : ((G - L.bytes) & ~int64_t(255));
   }
 
-  // arena layout
-  const Shape& sh = ctx->sh;
-  const int M = plan->n_microbatches > 0 ? plan->n_microbatches : dist->world;
-  ctx->max_M = M;
-  ctx->slot_bytes = al256((int64_t)sh.T() * sh.h * esz);
-  const bool fl = esz == 2 && flash_supported(sh.dh(), sh.s);
-  ctx->acts_bytes = al256(block_acts_bytes(sh, esz, fl));
-  ctx->keep_compact = fl && !getenv("MOBIUS_KEEP_FULL");
-  ctx->keep_acts_bytes = al256(block_acts_bytes(sh, esz, fl, ctx->keep_compact));
-  int64_t off = al256(G);
-  auto take = [&](int64_t bytes) {
-    int64_t o = off;
-    off += al256(bytes);
-    return o;
-  };
-  int64_t o_gacc = take(max_params * 4);
-  int64_t o_gstage = take(max_params * esz);
-  ctx->off_ckpt = take((int64_t)n * M * ctx->slot_bytes);
-  ctx->off_gslot = take((int64_t)n * M * ctx->slot_bytes);
-  ctx->off_fflag = take((int64_t)n * M * 4);
-  ctx->off_bflag = take((int64_t)n * M * 4);
-  int64_t o_xs = take(ctx->slot_bytes * (ctx->max_blocks + 3));
-  int64_t o_scr = take(scratch_bytes(sh, esz, true, fl));
-  int64_t o_tok = take((int64_t)M * sh.mbs * (sh.s + 1) * 4);
-  int64_t o_loss = take(8);
-  const int64_t o_acts = off;  // recompute workspace last: its size depends on the keep plan
+  // arena layout behind the ring
+  const FixedLayout FL = fixed_layout(sh, esz, fl, M, n, ctx->max_blocks, max_params, arena, offload,
+                                      ctx->slot_bytes, G);
+  ctx->xs_fixed = FL.xs_slots;
+  int64_t o_gacc = FL.gacc;
+  int64_t o_gstage = FL.gstage;
+  ctx->off_ckpt = FL.ckpt;
+  ctx->off_gslot = FL.gslot;
+  ctx->off_fflag = FL.fflag;
+  ctx->off_bflag = FL.bflag;
+  int64_t o_xs = FL.xs;
+  int64_t o_scr = FL.scr;
+  int64_t o_tok = FL.tok;
+  int64_t o_loss = FL.loss;
+  int64_t o_bad = FL.bad;
+  const int64_t o_acts = FL.acts;
+  (void)o_xs;
 
   int cu_dev = dist->device;
   {
@@ -960,9 +1296,9 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
     ctx->keep_nb.assign(n, 0);
     const int64_t dev_tail_bytes = (dist->flags & MOBIUS_FLAG_DEVICE_TAIL_UPDATE) && n > 0
         ? al256(ctx->all[ctx->mine[0]].n_params * 4) * 3 + al256(ctx->all[ctx->mine[0]].n_params * esz) : 0;
-    int ws = std::max(1, ctx->max_blocks);
+    int ws = arena ? 1 : std::max(1, ctx->max_blocks);  // arena: the recompute sets live in the residences
     int64_t keep_total = 0;
-    if (dist->flags & MOBIUS_FLAG_KEEP_ACTS) {
+    if ((dist->flags & MOBIUS_FLAG_KEEP_ACTS) && !arena) {
       size_t fr = 0, tot = 0;
       CU(cudaMemGetInfo(&fr, &tot));
       // margin for what is allocated after create (Stream-K workspaces, the
@@ -1001,9 +1337,9 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
       }
     }
     ctx->ws_blocks = ws;
-    ctx->arena_bytes = o_acts + al256(ctx->acts_bytes * ws);
+    ctx->arena_bytes = arena ? FL.end : o_acts + al256(ctx->acts_bytes * ws);
     CU(cudaMalloc(&ctx->arena, ctx->arena_bytes));
-    CU(cudaMemset(ctx->arena + o_gacc, 0, max_params * 4));
+    if (!arena) CU(cudaMemset(ctx->arena + o_gacc, 0, max_params * 4));
     ctx->ring = ctx->arena;
     ctx->dev_tail = (dist->flags & MOBIUS_FLAG_DEVICE_TAIL_UPDATE) && n > 0;
     if (ctx->dev_tail) {  // before the keep pool takes the free HBM
@@ -1016,8 +1352,8 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
       CU(cudaMalloc(&ctx->keep_pool, keep_total));
       ctx->keep_bytes = keep_total;
     }
-    ctx->grad_acc = reinterpret_cast<float*>(ctx->arena + o_gacc);
-    ctx->grad_stage = ctx->arena + o_gstage;
+    ctx->grad_acc = arena ? nullptr : reinterpret_cast<float*>(ctx->arena + o_gacc);  // arena: per residence
+    ctx->grad_stage = arena ? nullptr : ctx->arena + o_gstage;
     ctx->ckpt = ctx->arena + ctx->off_ckpt;
     ctx->gslot = ctx->arena + ctx->off_gslot;
     ctx->fflag = reinterpret_cast<int*>(ctx->arena + ctx->off_fflag);
@@ -1027,6 +1363,7 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
     ctx->scratch_base = ctx->arena + o_scr;
     ctx->tok_dev = ctx->arena + o_tok;
     ctx->loss_dev = reinterpret_cast<double*>(ctx->arena + o_loss);
+    ctx->bad_tok_dev = reinterpret_cast<int*>(ctx->arena + o_bad);
     CU(cudaMemset(ctx->fflag, 0, (int64_t)n * M * 4));
     CU(cudaMemset(ctx->bflag, 0, (int64_t)n * M * 4));
 
@@ -1060,6 +1397,26 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
     CU(cudaEventCreate(&ctx->ev_step0));
     CU(cudaEventCreate(&ctx->ev_step1));
     for (int k = 0; k < n; ++k) CU(cudaEventRecord(ctx->ev_d2h[k], ctx->s_d2h));
+    // checkpoint offload: stage k (1 <= k <= n-3) has its input slot reused
+    // by stage k+2's input, so its checkpoints round-trip through DRAM
+    ctx->ck_off.assign(n, 0);
+    ctx->h_ckpt.assign(n, nullptr);
+    if (offload) {
+      CU(cudaStreamCreateWithPriority(&ctx->s_ckup, cudaStreamNonBlocking, hi));
+      RC(mk(ctx->ev_ckoff, 2 * M, cudaEventDisableTiming));
+      RC(mk(ctx->ev_ckprod, M, cudaEventDisableTiming));
+      RC(mk(ctx->ev_ckup, n, cudaEventDisableTiming));
+      RC(mk(ctx->ev_ck_a, 2 * n, cudaEventDefault));
+      RC(mk(ctx->ev_ck_b, 2 * n, cudaEventDefault));
+      RC(mk(ctx->ev_ckw_a, n, cudaEventDefault));
+      RC(mk(ctx->ev_ckw_b, n, cudaEventDefault));
+      CU(cudaEventCreateWithFlags(&ctx->ev_fwd_off, cudaEventDisableTiming));
+      CU(cudaEventRecord(ctx->ev_fwd_off, ctx->s_d2h));
+      for (int k = 1; k + 2 < n; ++k) {
+        ctx->ck_off[k] = 1;
+        CU(cudaHostAlloc(&ctx->h_ckpt[k], (size_t)M * ctx->slot_bytes, cudaHostAllocDefault));
+      }
+    }
 
     // host stage store
     unsigned hw = std::thread::hardware_concurrency();
@@ -1113,10 +1470,11 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
     CU(cudaHostAlloc(&ctx->h_loss, sizeof(double), cudaHostAllocDefault));
     ctx->h_tokens_cap = (int64_t)M * sh.mbs * (sh.s + 1);
     CU(cudaHostAlloc(&ctx->h_tokens, ctx->h_tokens_cap * 4, cudaHostAllocDefault));
+    CU(cudaHostAlloc(&ctx->h_bad_tok, sizeof(int), cudaHostAllocDefault));
     ctx->peer_base.assign(dist->world, nullptr);
     ctx->connected = dist->world == 1;
-    ctx->upd_thread = std::thread(update_worker, ctxp);
     CU(cudaDeviceSynchronize());
+    ctx->upd_thread = std::thread(update_worker, ctxp);  // last: nothing after it can fail
   }
   *out = ctx.release();
   return MOBIUS_OK;
@@ -1231,6 +1589,12 @@ extern "C" int mobius_step(mobius_ctx* ctx, const int32_t* tokens, int M, float*
   if (!ctx->connected) MOBIUS_FAIL(MOBIUS_ESTATE, "world > 1: call mobius_dist_connect first");
   CU(cudaSetDevice(ctx->dist.device));
   const int64_t n = (int64_t)M * ctx->sh.mbs * (ctx->sh.s + 1);
+  // token ids index wte rows and the logits (embedding gather / scatter, CE):
+  // an id outside [0, V) is rejected before anything runs
+  const int32_t V = ctx->cfg.vocab;
+  for (int64_t i = 0; i < n; ++i)
+    if ((uint32_t)tokens[i] >= (uint32_t)V)
+      MOBIUS_FAIL(MOBIUS_EINVAL, "token %lld = %d outside [0, %d)", (long long)i, tokens[i], V);
   std::memcpy(ctx->h_tokens, tokens, n * 4);
   CU(cudaMemcpyAsync(ctx->tok_dev, ctx->h_tokens, n * 4, cudaMemcpyHostToDevice, ctx->s_comp));
   return step_common(ctx, reinterpret_cast<const int32_t*>(ctx->tok_dev), M, loss_out);
@@ -1242,7 +1606,16 @@ extern "C" int mobius_step_device(mobius_ctx* ctx, const int32_t* tokens_dev, in
   MOBIUS_CHECK_ARG(tokens_dev && loss_out && M == ctx->max_M, "bad arguments");
   if (!ctx->connected) MOBIUS_FAIL(MOBIUS_ESTATE, "world > 1: call mobius_dist_connect first");
   CU(cudaSetDevice(ctx->dist.device));
-  return step_common(ctx, tokens_dev, M, loss_out);
+  // copy into the context's token buffer while counting ids outside [0, V)
+  // (one small kernel + a sync before the step: a bad id would otherwise
+  // scatter into arbitrary arena memory in the embedding backward)
+  const int64_t n = (int64_t)M * ctx->sh.mbs * (ctx->sh.s + 1);
+  RC(tokens_check_copy(tokens_dev, reinterpret_cast<int32_t*>(ctx->tok_dev), n, ctx->cfg.vocab, ctx->bad_tok_dev,
+                       ctx->s_comp));
+  CU(cudaMemcpyAsync(ctx->h_bad_tok, ctx->bad_tok_dev, sizeof(int), cudaMemcpyDeviceToHost, ctx->s_comp));
+  CU(cudaStreamSynchronize(ctx->s_comp));
+  if (*ctx->h_bad_tok) MOBIUS_FAIL(MOBIUS_EINVAL, "%d token ids outside [0, %d)", *ctx->h_bad_tok, ctx->cfg.vocab);
+  return step_common(ctx, reinterpret_cast<const int32_t*>(ctx->tok_dev), M, loss_out);
 }
 
 extern "C" int mobius_read_grads(mobius_ctx* ctx, float* out, size_t n) {
@@ -1320,6 +1693,11 @@ extern "C" int mobius_read_timeline(mobius_ctx* ctx, mobius_timeline_event* out,
     add(fwd ? MOBIUS_TL_FWD : MOBIUS_TL_BWD, ctx->mine[ls], ctx->ev_pass_a[xi], ctx->ev_pass_b[xi]);
   }
   for (int ls = nl - 1; ls >= 0; --ls) add(MOBIUS_TL_D2H, ctx->mine[ls], ctx->ev_off_a[ls], ctx->ev_off_b[ls]);
+  for (int ls = 0; ls < nl; ++ls)
+    if (ctx->ck_off[ls]) {
+      add(MOBIUS_TL_CKPT_D2H, ctx->mine[ls], ctx->ev_ck_a[2 * ls], ctx->ev_ck_b[2 * ls]);
+      add(MOBIUS_TL_CKPT_H2D, ctx->mine[ls], ctx->ev_ck_a[2 * ls + 1], ctx->ev_ck_b[2 * ls + 1]);
+    }
   cudaGetLastError();  // clear a not-ready / unrecorded event status
   *n = v.size();
   if (out) std::memcpy(out, v.data(), std::min(cap, v.size()) * sizeof(mobius_timeline_event));
@@ -1333,38 +1711,5 @@ extern "C" int mobius_stats(mobius_ctx* ctx, mobius_step_stats* out) {
 }
 
 extern "C" void mobius_destroy(mobius_ctx* ctx) {
-  if (!ctx) return;
-  cudaSetDevice(ctx->dist.device);
-  {
-    std::lock_guard<std::mutex> g(ctx->upd_mu);
-    ctx->upd_stop = true;
-  }
-  ctx->upd_cv.notify_all();
-  if (ctx->upd_thread.joinable()) ctx->upd_thread.join();
-  if (ctx->s_comp) cudaStreamSynchronize(ctx->s_comp);
-  if (ctx->s_h2d) cudaStreamSynchronize(ctx->s_h2d);
-  if (ctx->s_d2h) cudaStreamSynchronize(ctx->s_d2h);
-  for (auto p : ctx->peer_base)
-    if (p) cudaIpcCloseMemHandle(p);
-  for (auto* v : {&ctx->ev_release, &ctx->ev_loaded, &ctx->ev_part_a, &ctx->ev_part_b, &ctx->ev_gready,
-                  &ctx->ev_d2h, &ctx->ev_wait_a, &ctx->ev_wait_b, &ctx->ev_pass_a, &ctx->ev_pass_b,
-                  &ctx->ev_off_a, &ctx->ev_off_b})
-    for (auto e : *v) cudaEventDestroy(e);
-  if (ctx->ev_step0) cudaEventDestroy(ctx->ev_step0);
-  if (ctx->ev_step1) cudaEventDestroy(ctx->ev_step1);
-  for (auto p : ctx->h_weights) cudaFreeHost(p);
-  for (auto p : ctx->h_grads) cudaFreeHost(p);
-  for (auto p : ctx->h_master) std::free(p);
-  for (auto p : ctx->h_m) std::free(p);
-  for (auto p : ctx->h_v) std::free(p);
-  if (ctx->h_loss) cudaFreeHost(ctx->h_loss);
-  if (ctx->h_tokens) cudaFreeHost(ctx->h_tokens);
-  if (ctx->arena) cudaFree(ctx->arena);
-  if (ctx->keep_pool) cudaFree(ctx->keep_pool);
-  if (ctx->d_opt) cudaFree(ctx->d_opt);
-  if (ctx->d_wstage) cudaFree(ctx->d_wstage);
-  if (ctx->s_comp) cudaStreamDestroy(ctx->s_comp);
-  if (ctx->s_h2d) cudaStreamDestroy(ctx->s_h2d);
-  if (ctx->s_d2h) cudaStreamDestroy(ctx->s_d2h);
-  delete ctx;
+  delete ctx;  // ~mobius_ctx: join the update thread, free HBM / pinned / host state, streams and events
 }

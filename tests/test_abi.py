@@ -208,3 +208,53 @@ def test_package_fails_loudly_without_library(tmp_path):
                        env={**os.environ, "PYTHONPATH": str(tmp_path)})
     assert r.returncode != 0
     assert "libmobius.so not built" in r.stderr
+
+
+def _key(pl):
+    K = pl.n_stages
+    return (pl.makespan_ns, K, tuple(pl.stage_first_layer[j + 1] - pl.stage_first_layer[j] for j in range(K)))
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_plan_above_20_layers_vs_brute_force(mb, seed, monkeypatch):
+    """L' = 21-22 (beyond the enumeration limit): the local search + branch
+    and bound against a brute force over all 2^(L'-1) compositions (the same
+    C++ recurrence, forced with MOBIUS_PLAN_EXHAUSTIVE_MAX).  A certified
+    result (exhaustive = 1) must be the optimum key exactly; an uncertified
+    one must be no worse than the brute force's by the key order."""
+    rng = random.Random(2100 + seed)
+    Lp = 21 + seed % 2
+    layers = _rand_layers(rng, Lp)
+    N, M = 1 + seed % 3, rng.randint(1, 4)
+    G = max(l.mem_bwd for l in layers) + rng.randint(0, 120)
+    topo = mb.make_topology(list(range(N)), 10 ** 9, 10 ** 9)
+    monkeypatch.delenv("MOBIUS_PLAN_EXHAUSTIVE_MAX", raising=False)
+    fast = mb.mobius_plan(layers, N, G, M, topo)
+    monkeypatch.setenv("MOBIUS_PLAN_EXHAUSTIVE_MAX", str(Lp))
+    brute = mb.mobius_plan(layers, N, G, M, topo)
+    assert brute.exhaustive == 1
+    if fast.exhaustive:
+        assert _key(fast) == _key(brute)
+    else:
+        assert fast.makespan_ns >= brute.makespan_ns
+
+
+def test_plan_1p5b_profile_certified_at_n1(mb):
+    """The bench's planning problem (GPT-1.5B, L' = 50, N = 1, M = 4, 1 GiB
+    ring, measured-shape layer times) is solved to proven optimality by the
+    branch and bound (exhaustive = 1) in well under a second."""
+    import time
+    c = synth.GPT_1_5B
+    prof = mb.mobius_layer_sizes(mb.model_cfg(c.n_layers, c.hidden, c.n_heads, c.seq_len, c.vocab, 32))
+    for i, p in enumerate(prof):
+        f = 6_600_000
+        p.t_fwd_ns, p.t_bwd_ns = (200_000, 400_000) if i == 0 else (3 * f, 6 * f) if i == len(prof) - 1 else \
+            (f, int(2.3 * f))
+    t0 = time.time()
+    pl = mb.mobius_plan(prof, 1, 1 << 30, 4, mb.make_topology([0], 55 * 10 ** 9, 0))
+    assert pl.exhaustive == 1
+    assert time.time() - t0 < 5.0
+    assert mb._lib.lib.mobius_plan_search_nodes() > 0
+    # the certificate's partition is no worse than Fig 9's max-stage baseline
+    mx = mb.mobius_plan_partition(prof, 1, 1 << 30, 4, mb.PARTITION_MAX_STAGE, mb.make_topology([0], 55 * 10 ** 9, 0))
+    assert pl.makespan_ns <= mx.makespan_ns

@@ -157,8 +157,10 @@ def test_device_tail_update(dtype, sizes):
         ctx.close()
         runs[flags] = (losses, g, p1, p3, st, st3)
     (lh, gh, p1h, p3h, sth, st3h), (ld, gd, p1d, p3d, std, st3d) = runs[0], runs[FLAG_DEVICE_TAIL_UPDATE]
-    # same first step up to the update (bias-gradient column sums use fp32
-    # atomics, so equal to rounding, not bitwise)
+    # same first step up to the update: bitwise on the fp32 path (fixed-order
+    # reductions); the bf16 flash backward reduces dQ with TMA reduce-adds
+    if dtype == F32:
+        assert np.array_equal(gd, gh) and ld[0] == lh[0]
     assert rel(gd, gh) < 1e-6 and abs(ld[0] - lh[0]) <= 1e-6 * abs(lh[0])
     # step 1 loads every stage from the host; the device-updated first stage
     # never crosses the link again: no gradient / weight D2H, and from step 2
@@ -315,12 +317,14 @@ def test_partial_keep(monkeypatch):
     assert 2 in seen and 0 in seen and 4 in seen, seen
 
 
-@pytest.mark.parametrize("dtype,tol", [(F32, 1e-5), (BF16, 2e-2)])
+@pytest.mark.parametrize("dtype,tol", [(F32, 0.0), (BF16, 2e-2)])
 def test_multistep_mobius_vs_gpipe_mode(dtype, tol):
     """SURVEY f4 / P:L596-602, Fig 13 analog without a dataset: four
     synthetic fine-tuning steps with stages swapped through DRAM (K=3 > N=1)
     follow the same loss curve as the single-resident-stage run (K=N=1,
-    GPipe mode): the synchronous update makes the pipeline invisible."""
+    GPipe mode): the synchronous update makes the pipeline invisible.  On
+    the fp32 debug path the curves are bitwise equal (every reduction runs
+    in a fixed order: no atomics on that path); bf16 within 2e-2."""
     c = synth.TINY
     M = 2
     w = synth.perturb_norm_params(c, synth.gen_params(c), scale=0.1)
@@ -332,5 +336,222 @@ def test_multistep_mobius_vs_gpipe_mode(dtype, tol):
         curves.append([ctx.step(synth.gen_tokens(c, M, seed=100 + i)) for i in range(4)])
         ctx.close()
     a, b = np.array(curves[0]), np.array(curves[1])
-    assert np.all(np.abs(a - b) <= tol * np.abs(a)), (a, b)
+    if tol == 0.0:
+        assert np.array_equal(a, b), (a, b)
+    else:
+        assert np.all(np.abs(a - b) <= tol * np.abs(a)), (a, b)
     assert a[-1] < a[0]
+
+
+def test_token_range_rejected_host_and_device():
+    """Token ids index wte rows and logits columns; an id outside [0, V)
+    is rejected with MOBIUS_EINVAL before anything runs (host tokens:
+    checked on the host; device tokens: a checking copy kernel), and the
+    context stays usable."""
+    from paper_conf_asplos_fengxtwls23_b200 import MobiusError
+    c = synth.TINY
+    M = 2
+    w = synth.round_bf16(synth.gen_params(c))
+    ctx = MobiusContext(mk_cfg(c, BF16), plan_from_sizes((3, 3), 1, M, hbm_cap_bytes=4 * MiB), init_params=w)
+    tok = synth.gen_tokens(c, M)
+    for bad in (c.vocab, -1, 1 << 30):
+        t = tok.copy()
+        t[1, 0, 5] = bad
+        with pytest.raises(MobiusError) as e:
+            ctx.step(t)
+        assert e.value.code == -1
+        with pytest.raises(MobiusError) as e:
+            ctx.step_device(torch.from_numpy(t).to("cuda:0"), M)
+        assert e.value.code == -1
+    l1 = ctx.step(tok)
+    g = ctx.read_grads(c.n_params)
+    ctx.close()
+    ref_loss, ref_g = om.reference_loss_and_grads(c, w, tok)
+    assert abs(l1 - ref_loss) / ref_loss < 2e-2 and rel(g, ref_g) < 2e-2
+
+
+def test_cuda_failure_poisons_context(monkeypatch):
+    """a CUDA failure inside a call poisons the context -
+    that call returns MOBIUS_ECUDA, every later call MOBIUS_ESTATE; destroy
+    still releases everything (MOBIUS_INJECT_CUDA_FAULT makes the step issue
+    one invalid, non-sticky cudaMemcpyAsync)."""
+    from paper_conf_asplos_fengxtwls23_b200 import MobiusError
+    c = synth.TINY
+    M = 2
+    ctx = MobiusContext(mk_cfg(c, BF16), plan_from_sizes((3, 3), 1, M, hbm_cap_bytes=4 * MiB), seed=3)
+    tok = synth.gen_tokens(c, M)
+    ctx.step(tok)
+    monkeypatch.setenv("MOBIUS_INJECT_CUDA_FAULT", "1")
+    with pytest.raises(MobiusError) as e:
+        ctx.step(tok)
+    assert e.value.code == -4
+    monkeypatch.delenv("MOBIUS_INJECT_CUDA_FAULT")
+    for call in (lambda: ctx.step(tok), lambda: ctx.read_grads(c.n_params), lambda: ctx.read_params(c.n_params)):
+        with pytest.raises(MobiusError) as e:
+            call()
+        assert e.value.code == -7
+    ctx.close()
+    # the process' CUDA context is still healthy
+    x = torch.ones(4, device="cuda:0")
+    assert float(x.sum()) == 4.0
+
+
+def test_failed_create_releases_memory():
+    """A create that fails part way (arena larger than HBM -> cudaMalloc
+    fails) releases what it had allocated and leaves no thread running."""
+    from paper_conf_asplos_fengxtwls23_b200 import MobiusError
+    c = synth.TINY
+    torch.cuda.synchronize()
+    free0, _ = torch.cuda.mem_get_info()
+    for _ in range(3):
+        with pytest.raises(MobiusError):
+            MobiusContext(mk_cfg(c, BF16), plan_from_sizes((3, 3), 1, 2, hbm_cap_bytes=1 << 50), seed=1)
+    free1, _ = torch.cuda.mem_get_info()
+    assert free0 - free1 < 64 * MiB, (free0, free1)
+    ctx = MobiusContext(mk_cfg(c, BF16), plan_from_sizes((3, 3), 1, 2, hbm_cap_bytes=4 * MiB), seed=1)
+    assert np.isfinite(ctx.step(synth.gen_tokens(c, 2)))
+    ctx.close()
+
+
+def test_weight_decay_step():
+    """AdamW with weight_decay != 0 (decoupled decay, O-4) through the ABI,
+    host update and device tail update: post-update master parameters equal
+    the oracle's AdamW on the offloaded gradients."""
+    c = synth.TINY
+    M = 2
+    w = synth.round_bf16(synth.perturb_norm_params(c, synth.gen_params(c), scale=0.1))
+    tok = synth.gen_tokens(c, M)
+    cfg = model_cfg(c.n_layers, c.hidden, c.n_heads, c.seq_len, c.vocab, c.micro_batch, dtype=BF16, lr=1e-3,
+                    weight_decay=0.1)
+    for flags in (0, FLAG_DEVICE_TAIL_UPDATE):
+        ctx = MobiusContext(cfg, plan_from_sizes((3, 3), 1, M, hbm_cap_bytes=4 * MiB), init_params=w, flags=flags)
+        ctx.step(tok)
+        g = ctx.read_grads(c.n_params)
+        p1 = ctx.read_params(c.n_params)
+        ctx.close()
+        w1, _, _ = oa.adamw_step(w, np.zeros_like(w), np.zeros_like(w), g, 1, lr=1e-3, wd=0.1)
+        assert np.max(np.abs(p1 - w1)) < 2e-6, flags
+        # the decay term is visible: it differs from the wd = 0 update
+        w1n, _, _ = oa.adamw_step(w, np.zeros_like(w), np.zeros_like(w), g, 1, lr=1e-3, wd=0.0)
+        assert np.max(np.abs(p1 - w1n)) > 1e-5
+
+
+def _arena_plan(c, dtype, sizes, M, ring_extra, flags):
+    """Hand-partitioned plan whose cap is the ring G_eff of a whole-memory
+    cap (MOBIUS_FLAG_ARENA_CAP): the largest backward footprint of the
+    partition (mobius_arena_layer_sizes summed per stage) + ring_extra."""
+    from paper_conf_asplos_fengxtwls23_b200 import mobius_arena_fixed_bytes, mobius_arena_layer_sizes
+    cfg = mk_cfg(c, dtype)
+    prof = mobius_arena_layer_sizes(cfg)
+    b = bounds(sizes)
+    need = max(sum(p.mem_bwd for p in prof[b[j]:b[j + 1]]) for j in range(len(sizes)))
+    ring = need + ring_extra
+    fixed = mobius_arena_fixed_bytes(cfg, M, len(sizes), flags)
+    return cfg, plan_from_sizes(sizes, 1, M, hbm_cap_bytes=ring), ring + fixed
+
+
+@pytest.mark.parametrize("dtype,tol", [(BF16, 2e-2), (F32, 1e-4)])
+@pytest.mark.parametrize("sizes", [(1, 1, 1, 1, 1, 1), (2, 1, 2, 1), (1, 2, 1, 2)])
+@pytest.mark.parametrize("offload", [True, False])
+def test_arena_cap_step_parity(dtype, tol, sizes, offload):
+    """Table 2's G as the whole per-GPU memory (MOBIUS_FLAG_ARENA_CAP): the
+    backward residence holds weights + fp32 dW + staging + recompute
+    workspace, so the ring is exactly the planner's S^b model; with
+    MOBIUS_FLAG_CKPT_OFFLOAD the stage-input checkpoints of stages 2..K-2
+    round-trip through DRAM (A_Mobius).  Two steps (bank slots
+    reused across steps): loss / gradients / post-update params vs the
+    oracle, arena within the cap, checkpoint bytes = (K-3) x M x A each
+    way, weight bytes = O-10."""
+    from paper_conf_asplos_fengxtwls23_b200 import FLAG_ARENA_CAP, FLAG_CKPT_OFFLOAD
+    c = synth.TINY
+    M = 2
+    flags = FLAG_ARENA_CAP | (FLAG_CKPT_OFFLOAD if offload else 0)
+    w = synth.perturb_norm_params(c, synth.gen_params(c), scale=0.1)
+    if dtype == BF16:
+        w = synth.round_bf16(w)
+    cfg, plan, cap = _arena_plan(c, dtype, sizes, M, ring_extra=64 << 10, flags=flags)
+    tok1, tok2 = synth.gen_tokens(c, M, seed=31), synth.gen_tokens(c, M, seed=32)
+    ctx = MobiusContext(cfg, plan, init_params=w, flags=flags)
+    l1 = ctx.step(tok1)
+    g1 = ctx.read_grads(c.n_params)
+    st = ctx.stats()
+    trace = ctx.read_trace()
+    tl = ctx.read_timeline()
+    l2 = ctx.step(tok2)
+    g2 = ctx.read_grads(c.n_params)
+    ctx.close()
+    K = len(sizes)
+    assert st.arena_bytes <= cap, (st.arena_bytes, cap)
+    ref_l1, ref_g1 = om.reference_loss_and_grads(c, w, tok1)
+    assert abs(l1 - ref_l1) / ref_l1 < tol
+    assert max(tensor_errs(c, g1, ref_g1).values()) < tol
+    w1, _, _ = oa.adamw_step(w, np.zeros_like(w), np.zeros_like(w), g1, 1)
+    w1 = synth.round_bf16(w1) if dtype == BF16 else w1
+    ref_l2, ref_g2 = om.reference_loss_and_grads(c, w1, tok2)
+    assert abs(l2 - ref_l2) / ref_l2 < tol and rel(g2, ref_g2) < tol
+    assert trace == osch.per_gpu_ops([0] * K, M)[0]
+    esz = 2 if dtype == BF16 else 4
+    A = c.micro_batch * c.seq_len * c.hidden * esz
+    n_off = max(0, K - 3) if offload else 0
+    assert st.ckpt_d2h_bytes == st.ckpt_h2d_bytes == n_off * M * A
+    prof = mobius_layer_sizes(mk_cfg(c, dtype))
+    layers = [op.LayerProfile(0, 0, p.mem_fwd, p.mem_bwd, p.xfer_fwd, p.xfer_bwd, p.act_out) for p in prof]
+    ss = op.stage_sums(layers, sizes)
+    h2d, d2h, _ = osch.byte_counts(ss, [0] * K, M, [s["Xf"] for s in ss])
+    assert st.h2d_bytes == h2d[0] and st.d2h_bytes == d2h[0]
+    kinds = [x[0] for x in tl]
+    assert kinds.count("ckpt_d2h") == kinds.count("ckpt_h2d") == n_off
+    for k, j, t0, _ in tl:  # every upload starts after its stage's offload finished
+        if k == "ckpt_h2d":
+            off = [x for x in tl if x[0] == "ckpt_d2h" and x[1] == j][0]
+            assert t0 >= off[3] - 1e-3
+
+
+def test_arena_cap_infeasible():
+    """A ring smaller than some stage's backward footprint is rejected
+    (Eq 4 on the whole-memory model)."""
+    from paper_conf_asplos_fengxtwls23_b200 import FLAG_ARENA_CAP, MobiusError
+    c = synth.TINY
+    cfg, plan, _ = _arena_plan(c, BF16, (3, 3), 2, ring_extra=0, flags=FLAG_ARENA_CAP)
+    plan.hbm_cap_bytes -= 1 << 20
+    with pytest.raises(MobiusError) as e:
+        MobiusContext(cfg, plan, seed=1, flags=FLAG_ARENA_CAP)
+    assert e.value.code == -2
+
+
+def test_arena_cap_planner_end_to_end():
+    """mobius_plan on the whole-memory profile with G_eff = G - fixed bytes
+    (SURVEY O-11): the plan's stages fit, the context's arena stays within G,
+    and the step matches the oracle."""
+    from paper_conf_asplos_fengxtwls23_b200 import (FLAG_ARENA_CAP, FLAG_CKPT_OFFLOAD, make_topology,
+                                                    mobius_arena_fixed_bytes, mobius_arena_layer_sizes, mobius_plan)
+    c = synth.TINY
+    M = 2
+    flags = FLAG_ARENA_CAP | FLAG_CKPT_OFFLOAD
+    cfg = mk_cfg(c, BF16)
+    prof = mobius_arena_layer_sizes(cfg)
+    for p in prof:
+        p.t_fwd_ns, p.t_bwd_ns = 100_000, 200_000
+    fixed = mobius_arena_fixed_bytes(cfg, M, 1, flags)
+    G = fixed + 2 * max(p.mem_bwd for p in prof) + (1 << 20)
+    plan = mobius_plan(prof, 1, G - fixed, M, make_topology([0], 25 * 10 ** 9, 0))
+    w = synth.round_bf16(synth.gen_params(c))
+    tok = synth.gen_tokens(c, M)
+    ctx = MobiusContext(cfg, plan, init_params=w, flags=flags)
+    loss = ctx.step(tok)
+    g = ctx.read_grads(c.n_params)
+    st = ctx.stats()
+    ctx.close()
+    assert st.arena_bytes <= G
+    assert plan.n_stages >= 3
+    ref_loss, ref_g = om.reference_loss_and_grads(c, w, tok)
+    assert abs(loss - ref_loss) / ref_loss < 2e-2 and rel(g, ref_g) < 2e-2
+
+
+def test_ckpt_offload_rejects_multi_rank():
+    from paper_conf_asplos_fengxtwls23_b200 import FLAG_CKPT_OFFLOAD, MobiusError
+    c = synth.TINY
+    with pytest.raises(MobiusError) as e:
+        MobiusContext(mk_cfg(c, BF16), plan_from_sizes((2, 2, 2), 2, 2, hbm_cap_bytes=4 * MiB), world=2,
+                      seed=1, flags=FLAG_CKPT_OFFLOAD)
+    assert e.value.code == -1
