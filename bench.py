@@ -64,6 +64,14 @@ def parse():
                     help="Table 2's G as the WHOLE per-GPU memory (ring + checkpoints + workspaces): "
                          "MOBIUS_FLAG_ARENA_CAP, planner fed G_eff = G - fixed bytes (SURVEY O-11), the paper's "
                          "recompute and host update; survey C2 = --micro-batch 8 --arena-cap-gib 2")
+    ap.add_argument("--topology", default="auto", choices=["auto", "probe", "sysfs"],
+                    help="host-link contention groups: measured (probe: concurrent pinned H2D < 0.8 x solo, "
+                         "SURVEY #12) or sysfs root complex; auto = probe when N > 1")
+    ap.add_argument("--mapping", default="cross", choices=["cross", "sequential"],
+                    help="stage->GPU mapping: the planner's cross mapping (Eq 12/13) or sequential (f3 baseline)")
+    ap.add_argument("--no-prefetch-order", action="store_true",
+                    help="N > 1: do not serialise the stage loads of GPUs sharing an uplink by planned stage start "
+                         "(P:L858-863 priority)")
     ap.add_argument("--no-offload", action="store_true",
                     help="with --arena-cap-gib: keep every stage-input checkpoint in HBM (no A_Mobius offload)")
     return ap.parse_args()
@@ -268,7 +276,14 @@ def run_mobius(args, rank, world, local):
         for p, q in zip(prof, mem):
             p.mem_fwd, p.mem_bwd, p.xfer_fwd, p.xfer_bwd = q.mem_fwd, q.mem_bwd, q.xfer_fwd, q.xfer_bwd
     h2d_gbps = measure_h2d_GBps(torch)
-    topo = mobius_discover_topology()
+    topo_src = args.topology if args.topology != "auto" else ("probe" if world > 1 else "sysfs")
+    probe = None
+    if topo_src == "probe" and rank == 0:
+        from paper_conf_asplos_fengxtwls23_b200 import mobius_probe_topology
+        topo, solo, pair = mobius_probe_topology(256 << 20, 0.8)
+        probe = {"solo_GBps": solo, "pair_GBps": pair, "p2p_GBps": topo.p2p_bw_Bps / 1e9}
+    else:
+        topo = mobius_discover_topology()
     groups = [topo.group[i] for i in range(topo.n_gpus)][:world]
     if len(groups) < world:
         groups = list(range(world))
@@ -276,12 +291,12 @@ def run_mobius(args, rank, world, local):
     # profile, link bandwidth and topology are broadcast (measured timings
     # differ slightly per GPU, which would yield different partitions)
     shared = [[(p.t_fwd_ns, p.t_bwd_ns, p.mem_fwd, p.mem_bwd, p.xfer_fwd, p.xfer_bwd, p.act_out) for p in prof],
-              h2d_gbps, groups]
+              h2d_gbps, groups, probe]
     if world > 1:
         dist.broadcast_object_list(shared, src=0)
         from paper_conf_asplos_fengxtwls23_b200._lib import LayerProfile
         prof = [LayerProfile(*x) for x in shared[0]]
-        h2d_gbps, groups = shared[1], shared[2]
+        h2d_gbps, groups, probe = shared[1], shared[2], shared[3]
     t = make_topology(groups, host_bw_Bps=int(h2d_gbps * 1e9), p2p_bw_Bps=int(700e9))
     t0 = time.perf_counter()
     if args.partition == "mip":
@@ -292,6 +307,13 @@ def run_mobius(args, rank, world, local):
         plan = mobius_plan_partition(prof, world, G, M,
                                      PARTITION_MAX_STAGE if args.partition == "max" else PARTITION_MIN_STAGE, t)
     plan_s = time.perf_counter() - t0
+    if args.mapping == "sequential":  # f3 baseline: stage j on GPU (j-1) mod N
+        for g in range(world):
+            plan.gpu_perm[g] = g
+        for j in range(plan.n_stages):
+            plan.stage_gpu[j] = j % world
+    from paper_conf_asplos_fengxtwls23_b200 import mobius_mapping_contention
+    contention = mobius_mapping_contention(plan.n_stages, groups, [plan.gpu_perm[g] for g in range(world)])[0]
     if world > 1:
         from paper_conf_asplos_fengxtwls23_b200 import dist as mdist
         assert mdist.check_same_plan(plan), "ranks derived different plans"
@@ -301,6 +323,9 @@ def run_mobius(args, rank, world, local):
     if arena:  # the paper's regime: everything inside G, recompute, host update
         flags = (FLAG_TIMING if timing else 0) | arena_flags
     ctx = MobiusContext(cfg, plan, rank=rank, world=world, device=local, seed=1234, flags=flags)
+    prefetch_order = world > 1 and not args.no_prefetch_order and len(set(groups)) < world
+    if prefetch_order:  # loads of GPUs sharing an uplink: one at a time, earlier-starting stage first
+        ctx.set_prefetch_groups(groups)
     if world > 1:
         blobs = [None] * world
         dist.all_gather_object(blobs, ctx.dist_export())
@@ -413,6 +438,8 @@ def run_mobius(args, rank, world, local):
                        "n_stages": plan.n_stages, "stage_layers": [plan.stage_first_layer[j + 1] - plan.stage_first_layer[j]
                                                                    for j in range(plan.n_stages)],
                        "gpu_perm": [plan.gpu_perm[g] for g in range(world)], "plan_s": plan_s,
+                       "mapping": args.mapping, "uplink_groups": groups, "topology_source": topo_src,
+                       "mapping_contention": contention, "prefetch_order": prefetch_order, "link_probe": probe,
                        "profile_s": prof_s, "plan_exhaustive": bool(plan.exhaustive),
                        "partition": args.partition, "plan_makespan_ms": plan.makespan_ns / 1e6,
                        "arena_cap_GB": args.arena_cap_gib * GiB / 1e9 if arena else None,

@@ -10,7 +10,9 @@ import ctypes as C
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libmobius.so")
+# MOBIUS_LIB_PATH: an alternative build of the same library (kernel A/B
+# timing tools only); there is no other implementation behind the binding
+LIB_PATH = os.environ.get("MOBIUS_LIB_PATH") or os.path.join(_HERE, "libmobius.so")
 
 MAX_GPUS = 16
 MAX_LAYERS = 256
@@ -98,6 +100,8 @@ SIGNATURES = {
     "mobius_mapping_contention": (I, [I, I, C.POINTER(C.c_int), C.POINTER(C.c_int), C.POINTER(C.c_double),
                                       C.POINTER(I64), C.POINTER(I64)]),
     "mobius_discover_topology": (I, [C.POINTER(Topology)]),
+    "mobius_topology_from_bw": (I, [I, P, P, C.c_double, C.POINTER(Topology)]),
+    "mobius_probe_topology": (I, [I64, C.c_double, C.POINTER(Topology), P, P]),
     "mobius_layer_sizes": (I, [C.POINTER(ModelCfg), C.POINTER(LayerProfile), C.POINTER(C.c_int)]),
     "mobius_profile": (I, [C.POINTER(ModelCfg), I, C.POINTER(LayerProfile), C.POINTER(C.c_int)]),
     "mobius_arena_layer_sizes": (I, [C.POINTER(ModelCfg), C.POINTER(LayerProfile), C.POINTER(C.c_int)]),
@@ -105,6 +109,8 @@ SIGNATURES = {
     "mobius_create": (I, [C.POINTER(ModelCfg), C.POINTER(Plan), C.POINTER(Dist), P, C.c_uint64, C.POINTER(P)]),
     "mobius_dist_export": (I, [P, P, C.c_size_t, C.POINTER(C.c_size_t)]),
     "mobius_dist_connect": (I, [P, P, C.c_size_t]),
+    "mobius_set_prefetch_groups": (I, [P, P, I]),
+    "mobius_read_prefetch_tickets": (I, [P, P, C.c_size_t, C.POINTER(C.c_size_t)]),
     "mobius_step": (I, [P, P, I, C.POINTER(F)]),
     "mobius_step_device": (I, [P, P, I, C.POINTER(F)]),
     "mobius_read_grads": (I, [P, P, C.c_size_t]),

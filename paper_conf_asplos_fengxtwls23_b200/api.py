@@ -13,7 +13,7 @@ from ._lib import (BF16, F32, FLAG_ARENA_CAP, FLAG_CKPT_OFFLOAD, FLAG_DEVICE_TAI
                    FLAG_TIMING, MobiusError, check, lib)
 
 __all__ = ["mobius_plan", "mobius_plan_partition", "PARTITION_MIP", "PARTITION_MAX_STAGE", "PARTITION_MIN_STAGE", "mobius_plan_cost", "mobius_cross_map", "mobius_mapping_contention",
-           "mobius_discover_topology", "mobius_layer_sizes", "mobius_profile", "MobiusContext", "model_cfg",
+           "mobius_discover_topology", "mobius_topology_from_bw", "mobius_probe_topology", "mobius_layer_sizes", "mobius_profile", "MobiusContext", "model_cfg",
            "make_topology", "plan_from_sizes", "kt", "BF16", "F32", "FLAG_TIMING", "FLAG_KEEP_ACTS", "FLAG_DEVICE_TAIL_UPDATE", "FLAG_ARENA_CAP", "FLAG_CKPT_OFFLOAD",
            "mobius_arena_layer_sizes", "mobius_arena_fixed_bytes", "MobiusError",
            "build_info"]
@@ -53,6 +53,26 @@ def mobius_discover_topology() -> L.Topology:
     t = L.Topology()
     check(lib.mobius_discover_topology(C.byref(t)))
     return t
+
+
+def mobius_topology_from_bw(solo: Sequence[float], pair, threshold: float = 0.8) -> L.Topology:
+    """pair: n x n array-like of GB/s (row i: GPU i while column j copies)."""
+    n = len(solo)
+    so = (C.c_double * n)(*solo)
+    pa = (C.c_double * (n * n))(*[float(pair[i][j]) for i in range(n) for j in range(n)])
+    t = L.Topology()
+    check(lib.mobius_topology_from_bw(n, so, pa, threshold, C.byref(t)))
+    return t
+
+
+def mobius_probe_topology(nbytes: int = 256 << 20, threshold: float = 0.8):
+    """(topology, solo GB/s list, pair GB/s n x n list) measured on the visible GPUs."""
+    so = (C.c_double * L.MAX_GPUS)()
+    pa = (C.c_double * (L.MAX_GPUS * L.MAX_GPUS))()
+    t = L.Topology()
+    check(lib.mobius_probe_topology(nbytes, threshold, C.byref(t), so, pa))
+    n = t.n_gpus
+    return t, list(so[:n]), [[pa[i * n + j] for j in range(n)] for i in range(n)]
 
 
 def mobius_plan(layers, n_gpus: int, hbm_cap_bytes: int, n_microbatches: int,
@@ -188,6 +208,16 @@ class MobiusContext:
         ln = max(len(b) for b in blobs)
         flat = b"".join(b.ljust(ln, b"\0") for b in blobs)
         check(lib.mobius_dist_connect(self._ctx, flat, ln))
+
+    def set_prefetch_groups(self, groups: Sequence[int]):
+        g = (C.c_int * len(groups))(*groups)
+        check(lib.mobius_set_prefetch_groups(self._ctx, g, len(groups)))
+
+    def read_prefetch_tickets(self):
+        buf = (C.c_int32 * 1024)()
+        n = C.c_size_t()
+        check(lib.mobius_read_prefetch_tickets(self._ctx, buf, 1024, C.byref(n)))
+        return list(buf[:n.value])
 
     def step(self, tokens: np.ndarray) -> float:
         tok = np.ascontiguousarray(tokens, dtype=np.int32)

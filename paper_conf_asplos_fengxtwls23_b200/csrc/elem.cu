@@ -1052,6 +1052,11 @@ int flag_wait(const volatile int* flag, int value, cudaStream_t st) {
   flag_wait_k<<<1, 1, 0, st>>>(flag, value);
   return check_launch("flag_wait");
 }
+__global__ void ticket_take_k(int* counter, int* out) { *out = atomicAdd_system(counter, 1); }
+int ticket_take(int* counter, int* out, cudaStream_t st) {
+  ticket_take_k<<<1, 1, 0, st>>>(counter, out);
+  return check_launch("ticket_take");
+}
 int flag_set(int* flag, int value, cudaStream_t st) {
   flag_set_k<<<1, 1, 0, st>>>(flag, value);
   return check_launch("flag_set");

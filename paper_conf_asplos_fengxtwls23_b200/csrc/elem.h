@@ -85,5 +85,7 @@ int tokens_check_copy(const int32_t* src, int32_t* dst, int64_t n, int V, int* b
 // device-side flag wait / set (inter-rank arrival flags, release/acquire at system scope)
 int flag_wait(const volatile int* flag, int value, cudaStream_t st);
 int flag_set(int* flag, int value, cudaStream_t st);
+// *out = atomicAdd_system(counter, 1) (prefetch-chain tickets; counter may be peer memory)
+int ticket_take(int* counter, int* out, cudaStream_t st);
 
 }  // namespace mobius

@@ -83,6 +83,37 @@ __device__ __forceinline__ float ex2(float x) {
 
 __device__ __forceinline__ uint32_t pack_bf16x2(float2 v) { return pack_bf16(v.x, v.y); }
 
+// 2^x for a pair on the FMA pipe instead of the MUFU unit (the forward
+// softmax issues one ex2 per score, which makes MUFU its busiest pipe):
+// 2^x = 2^round(x) * q(f), f = x - round(x) in [-1/2, 1/2], q a degree-3
+// fit of 2^f (max relative error 1.8e-4, far below the bf16 rounding of P;
+// coefficients from a relative-error least-squares fit on Chebyshev nodes).
+// round(x) comes from the 1.5 * 2^23 magic-number add, whose low mantissa
+// bits then hold it as an integer that is shifted into the exponent.
+// x is clamped to -125 (2^-125 ~ 0 for softmax weights; no denormals).
+__device__ __forceinline__ float2 ex2_poly2(float2 x) {
+  x.x = fmaxf(x.x, -125.f);
+  x.y = fmaxf(x.y, -125.f);
+  const float2 magic = make_float2(12582912.f, 12582912.f);
+  const float2 j = __fadd2_rn(x, magic);
+  const float2 t = __fadd2_rn(j, make_float2(-12582912.f, -12582912.f));  // round(x)
+  const float2 f = __fadd2_rn(x, make_float2(-t.x, -t.y));
+  float2 q = __ffma2_rn(make_float2(0.053241830319166183f, 0.053241830319166183f), f,
+                        make_float2(0.24228397011756897f, 0.24228397011756897f));
+  q = __ffma2_rn(q, f, make_float2(0.6935495138168335f, 0.6935495138168335f));
+  q = __ffma2_rn(q, f, make_float2(0.9999545216560364f, 0.9999545216560364f));
+  return make_float2(__int_as_float(__float_as_int(q.x) + (__float_as_int(j.x) << 23)),
+                     __int_as_float(__float_as_int(q.y) + (__float_as_int(j.y) << 23)));
+}
+#ifndef MOBIUS_FLASH_POLY_PAIRS
+#define MOBIUS_FLASH_POLY_PAIRS 4  // of every 16 pairs of scores, this many use ex2_poly2 (forward)
+#endif
+// score pair e/2 of a 32-column slab: polynomial or MUFU
+__device__ __forceinline__ float2 ex2_pair(float a, float b, int pair) {
+  if ((pair & 15) < MOBIUS_FLASH_POLY_PAIRS) return ex2_poly2(make_float2(a, b));
+  return make_float2(ex2(a), ex2(b));
+}
+
 // Softmax-gradient math of one 32-query slab of a key row (flash bwd):
 //   P^T[r, q]  = 2^(S^T[r, q] * c - lse_q)          (masked to q >= r on the diagonal tile)
 //   dS^T[r, q] = P^T[r, q] * (dP^T[r, q] - D_q)      (the 1/sqrt(dh) factor is applied to
@@ -450,10 +481,10 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
           uint32_t pk[16];
 #pragma unroll
           for (int e = 0; e < 32; e += 2) {
-            const float p0 = ex2(fmaf(__uint_as_float(v0[e]), sc, -m_new));
-            const float p1 = ex2(fmaf(__uint_as_float(v0[e + 1]), sc, -m_new));
-            rs += p0 + p1;
-            pk[e >> 1] = pack_bf16(p0, p1);
+            const float2 pp = ex2_pair(fmaf(__uint_as_float(v0[e]), sc, -m_new), fmaf(__uint_as_float(v0[e + 1]), sc, -m_new),
+                                       e >> 1);
+            rs += pp.x + pp.y;
+            pk[e >> 1] = pack_bf16(pp.x, pp.y);
           }
           if constexpr (C::P_TMEM) {  // keys hf*64 .. +31 -> packed columns hf*32 .. +15
             ptx::tmem_st16(tmem + 384 + sb * 64 + hf * 32 + lb, pk);
@@ -464,10 +495,10 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
           }
 #pragma unroll
           for (int e = 0; e < 32; e += 2) {
-            const float p0 = ex2(fmaf(__uint_as_float(v1[e]), sc, -m_new));
-            const float p1 = ex2(fmaf(__uint_as_float(v1[e + 1]), sc, -m_new));
-            rs += p0 + p1;
-            pk[e >> 1] = pack_bf16(p0, p1);
+            const float2 pp = ex2_pair(fmaf(__uint_as_float(v1[e]), sc, -m_new), fmaf(__uint_as_float(v1[e + 1]), sc, -m_new),
+                                       (e >> 1) + 8);
+            rs += pp.x + pp.y;
+            pk[e >> 1] = pack_bf16(pp.x, pp.y);
           }
           if constexpr (C::P_TMEM) {
             ptx::tmem_st16(tmem + 384 + sb * 64 + hf * 32 + 16 + lb, pk);

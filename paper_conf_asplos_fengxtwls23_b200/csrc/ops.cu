@@ -184,9 +184,10 @@ int64_t scratch_bytes(const Shape& sh, int e, bool with_head, bool flash) {
   c.take<char>(T * 4);
   c.take<char>(T * 4);
   c.take<char>(T * 4);
-  c.take<char>(T * h * e);      // ra
-  c.take<char>(T * h * e);      // ra2
-  c.take<char>(T * 4 * h * e);  // rg
+  const int64_t kt = sh.no_keep ? 0 : 1;
+  c.take<char>(kt * T * h * e);      // ra
+  c.take<char>(kt * T * h * e);      // ra2
+  c.take<char>(kt * T * 4 * h * e);  // rg
   c.take<char>(red_ws_floats(sh) * 4);
   c.take<char>(RED_WS_COUNTERS * 4);
   return c.off;
@@ -210,9 +211,10 @@ void carve_scratch(const Shape& sh, uint8_t* base, bool with_head, Scratch<T>& s
   sc.loss_rows = c.take<float>(Tn * 4);
   sc.mu = c.take<float>(Tn * 4);
   sc.rs = c.take<float>(Tn * 4);
-  sc.ra = c.take<T>(Tn * h * e);
-  sc.ra2 = c.take<T>(Tn * h * e);
-  sc.rg = c.take<T>(Tn * 4 * h * e);
+  const int64_t kt = sh.no_keep ? 0 : 1;
+  sc.ra = kt ? c.take<T>(Tn * h * e) : nullptr;
+  sc.ra2 = kt ? c.take<T>(Tn * h * e) : nullptr;
+  sc.rg = kt ? c.take<T>(Tn * 4 * h * e) : nullptr;
   sc.red.part = c.take<float>(red_ws_floats(sh) * 4);
   sc.red.cnt = c.take<unsigned>(RED_WS_COUNTERS * 4);
 }

@@ -16,6 +16,7 @@ namespace mobius {
 struct Shape {
   int h, nh, s, mbs, V;
   int head_rows = 0;  // LM head row chunk (multiple of s; 0 = all T rows at once)
+  bool no_keep = false;  // no kept activations: the scratch has no compact-keep recompute targets
   int T() const { return mbs * s; }
   int dh() const { return h / nh; }
   int head_chunk() const { return head_rows > 0 && head_rows < T() ? head_rows : T(); }

@@ -664,3 +664,147 @@ extern "C" int mobius_plan_partition(const mobius_layer_profile* layers, int n_l
                    "unknown partition algorithm %d", algo);
   return plan_impl(layers, n_layers, N, G, M, topo_in, algo, out);
 }
+
+// ---------------------------------------------------------------------------
+// measured contention groups: the "root
+// complex" that matters is the level at which concurrent pinned H2D copies
+// slow each other down; on B200 boxes the PCIe switch / socket layout is not
+// visible from sysfs alone.
+// ---------------------------------------------------------------------------
+extern "C" int mobius_topology_from_bw(int n, const double* solo, const double* pair, double threshold,
+                                       mobius_topology* out) {
+  MOBIUS_CHECK_ARG(n >= 1 && n <= MOBIUS_MAX_GPUS && solo && (pair || n == 1) && out && threshold > 0 &&
+                       threshold <= 1,
+                   "bad arguments");
+  std::vector<int> parent(n);
+  std::iota(parent.begin(), parent.end(), 0);
+  auto find = [&](int x) {
+    while (parent[x] != x) x = parent[x] = parent[parent[x]];
+    return x;
+  };
+  for (int i = 0; i < n; ++i)
+    for (int j = i + 1; j < n; ++j) {
+      MOBIUS_CHECK_ARG(solo[i] > 0 && solo[j] > 0, "solo bandwidth must be positive");
+      const double ri = pair[i * n + j] / solo[i], rj = pair[j * n + i] / solo[j];
+      if (std::min(ri, rj) < threshold) parent[find(i)] = find(j);
+    }
+  std::memset(out, 0, sizeof(*out));
+  out->n_gpus = n;
+  std::map<int, int> ids;  // group ids numbered by first member
+  for (int i = 0; i < n; ++i) {
+    const int r = find(i);
+    auto it = ids.find(r);
+    if (it == ids.end()) it = ids.emplace(r, (int)ids.size()).first;
+    out->group[i] = it->second;
+  }
+  std::vector<double> s(solo, solo + n);
+  std::sort(s.begin(), s.end());
+  out->host_bw_Bps = (int64_t)(s[n / 2] * 1e9);
+  return MOBIUS_OK;
+}
+
+extern "C" int mobius_probe_topology(int64_t bytes, double threshold, mobius_topology* out, double* solo_out,
+                                     double* pair_out) {
+  MOBIUS_CHECK_ARG(out && bytes >= (1 << 20), "bad arguments");
+  int n = 0;
+  if (cudaGetDeviceCount(&n) != cudaSuccess || n <= 0) MOBIUS_FAIL(MOBIUS_ETOPO, "no CUDA devices");
+  n = std::min(n, MOBIUS_MAX_GPUS);
+  int cur = 0;
+  cudaGetDevice(&cur);
+  std::vector<void*> h(n, nullptr), d(n, nullptr);
+  std::vector<cudaStream_t> st(n, nullptr);
+  std::vector<cudaEvent_t> ea(n, nullptr), eb(n, nullptr);
+  int rc = MOBIUS_OK;
+  auto cleanup = [&]() {
+    for (int i = 0; i < n; ++i) {
+      cudaSetDevice(i);
+      if (st[i]) cudaStreamSynchronize(st[i]);
+      if (h[i]) cudaFreeHost(h[i]);
+      if (d[i]) cudaFree(d[i]);
+      if (st[i]) cudaStreamDestroy(st[i]);
+      if (ea[i]) cudaEventDestroy(ea[i]);
+      if (eb[i]) cudaEventDestroy(eb[i]);
+    }
+    cudaSetDevice(cur);
+  };
+  for (int i = 0; i < n && !rc; ++i) {
+    if (cudaSetDevice(i) != cudaSuccess || cudaMalloc(&d[i], bytes) != cudaSuccess ||
+        cudaHostAlloc(&h[i], bytes, cudaHostAllocPortable) != cudaSuccess ||
+        cudaStreamCreateWithFlags(&st[i], cudaStreamNonBlocking) != cudaSuccess ||
+        cudaEventCreate(&ea[i]) != cudaSuccess || cudaEventCreate(&eb[i]) != cudaSuccess)
+      rc = MOBIUS_ENOMEM;
+    else
+      std::memset(h[i], 1, bytes);
+  }
+  if (rc) {
+    cleanup();
+    MOBIUS_FAIL(rc, "probe_topology: allocation");
+  }
+  const int reps = 3;
+  // run the copies of GPUs in `set` concurrently, return per-GPU GB/s
+  auto measure = [&](const std::vector<int>& set, std::vector<double>& gbps) -> int {
+    for (int pass = 0; pass < 2; ++pass) {  // pass 0 warms up
+      for (int i : set) {
+        cudaSetDevice(i);
+        cudaEventRecord(ea[i], st[i]);
+      }
+      for (int k = 0; k < reps; ++k)
+        for (int i : set) {
+          cudaSetDevice(i);
+          cudaMemcpyAsync(d[i], h[i], bytes, cudaMemcpyHostToDevice, st[i]);
+        }
+      for (int i : set) {
+        cudaSetDevice(i);
+        cudaEventRecord(eb[i], st[i]);
+      }
+      for (int i : set) {
+        cudaSetDevice(i);
+        if (cudaStreamSynchronize(st[i]) != cudaSuccess) return MOBIUS_ECUDA;
+      }
+    }
+    gbps.assign(n, 0.0);
+    for (int i : set) {
+      float ms = 0.f;
+      cudaEventElapsedTime(&ms, ea[i], eb[i]);
+      gbps[i] = ms > 0 ? reps * (double)bytes / (ms * 1e-3) / 1e9 : 0.0;
+    }
+    return MOBIUS_OK;
+  };
+  std::vector<double> solo(n), pair((size_t)n * n, 0.0), g;
+  for (int i = 0; i < n && !rc; ++i) {
+    rc = measure({i}, g);
+    solo[i] = g[i];
+  }
+  for (int i = 0; i < n && !rc; ++i)
+    for (int j = i + 1; j < n && !rc; ++j) {
+      rc = measure({i, j}, g);
+      pair[(size_t)i * n + j] = g[i];
+      pair[(size_t)j * n + i] = g[j];
+    }
+  int64_t p2p = 0;
+  if (!rc && n >= 2) {  // GPU0 -> GPU1 over NVLink (peer copy)
+    int can = 0;
+    cudaDeviceCanAccessPeer(&can, 1, 0);
+    if (can) {
+      cudaSetDevice(1);
+      cudaDeviceEnablePeerAccess(0, 0);
+      cudaGetLastError();
+      cudaSetDevice(0);
+      cudaEventRecord(ea[0], st[0]);
+      for (int k = 0; k < reps; ++k) cudaMemcpyPeerAsync(d[1], 1, d[0], 0, bytes, st[0]);
+      cudaEventRecord(eb[0], st[0]);
+      cudaStreamSynchronize(st[0]);
+      float ms = 0.f;
+      cudaEventElapsedTime(&ms, ea[0], eb[0]);
+      if (ms > 0) p2p = (int64_t)(reps * (double)bytes / (ms * 1e-3));
+    }
+  }
+  cleanup();
+  if (rc) MOBIUS_FAIL(rc, "probe_topology: copy failed");
+  rc = mobius_topology_from_bw(n, solo.data(), pair.data(), threshold, out);
+  if (rc) return rc;
+  out->p2p_bw_Bps = p2p;
+  if (solo_out) std::copy(solo.begin(), solo.end(), solo_out);
+  if (pair_out) std::copy(pair.begin(), pair.end(), pair_out);
+  return MOBIUS_OK;
+}

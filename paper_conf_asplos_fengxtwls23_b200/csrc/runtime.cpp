@@ -25,6 +25,7 @@
 #include <algorithm>
 #include <atomic>
 #include <chrono>
+#include <climits>
 #include <cmath>
 #include <condition_variable>
 #include <cstdlib>
@@ -73,6 +74,7 @@ struct PeerInfo {
   cudaIpcMemHandle_t handle;
   int64_t off_ckpt, off_gslot, off_fflag, off_bflag, slot_bytes;
   int n_local, M;
+  int64_t off_pf;  // prefetch-chain region: [ticket counter, load_done[R], tickets[R]] (int32)
 };
 
 struct Load {           // one residence of a stage in the ring
@@ -80,26 +82,42 @@ struct Load {           // one residence of a stage in the ring
   int end;              // 0 bottom, 1 top
   int64_t base;         // byte offset in the ring
   int64_t bytes;        // footprint in the ring (weights; + dW / staging / recompute workspace, arena mode bwd)
-  int64_t copy;         // bytes copied in (the stage weights, at the start of the footprint)
+  int64_t copy;         // bytes copied in (the stage weights)
   bool bwd;             // the residence runs the stage's backward
+  int64_t wofs = 0;     // offset of the weights in the footprint: 0 at the bottom end; at the top end
+                        // the weights sit last (highest addresses), as far as possible from the bottom
+                        // residence, so a top prefetch overlaps the running bottom footprint least
 };
 
-// byte layout of a backward residence in MOBIUS_FLAG_ARENA_CAP mode:
-// [weights | fp32 dW | gradient staging | nb recompute activation sets |
-//  (has_embed + nb) activation buffers]
+// byte layout of a backward residence in MOBIUS_FLAG_ARENA_CAP mode, from
+// the ring's end inwards: [weights | gradient staging | fp32 dW | nb
+// recompute activation sets | (has_embed + nb) activation buffers] at the
+// bottom end, mirrored at the top end.  The weights (prefetched) and the
+// gradient staging (read by the D2H offload after the pass) sit farthest from
+// the other end, where the next residence's workspace would overlap.
 struct BwdFootprint {
   int64_t w, gacc, gst, acts, xs, total;
 };
 inline BwdFootprint bwd_footprint(int64_t np, int esz, int nb, bool has_embed, int64_t acts_bytes,
-                                  int64_t slot_bytes) {
+                                  int64_t slot_bytes, bool top = false) {
   auto al = [](int64_t x) { return (x + 255) & ~int64_t(255); };
+  const int64_t W = al(np * esz), GS = al(np * esz), GA = al(np * 4), AC = nb * acts_bytes,
+                XS = (nb + (has_embed ? 1 : 0)) * slot_bytes;
   BwdFootprint f;
-  f.w = 0;
-  f.gacc = al(np * esz);
-  f.gst = f.gacc + al(np * 4);
-  f.acts = f.gst + al(np * esz);
-  f.xs = f.acts + nb * acts_bytes;
-  f.total = f.xs + (nb + (has_embed ? 1 : 0)) * slot_bytes;
+  f.total = W + GS + GA + AC + XS;
+  if (!top) {
+    f.w = 0;
+    f.gst = W;
+    f.gacc = f.gst + GS;
+    f.acts = f.gacc + GA;
+    f.xs = f.acts + AC;
+  } else {
+    f.xs = 0;
+    f.acts = XS;
+    f.gacc = f.acts + AC;
+    f.gst = f.gacc + GA;
+    f.w = f.gst + GS;
+  }
   return f;
 }
 
@@ -111,7 +129,7 @@ inline BwdFootprint bwd_footprint(int64_t np, int esz, int nb, bool has_embed, i
 // activation set; with checkpoint offload the checkpoint and gradient slots
 // are two banks of M.
 struct FixedLayout {
-  int64_t gacc, gstage, ckpt, gslot, fflag, bflag, xs, scr, tok, loss, bad, acts, end;
+  int64_t gacc, gstage, ckpt, gslot, fflag, bflag, pf, xs, scr, tok, loss, bad, acts, end;
   int xs_slots, slot_sets;
 };
 inline FixedLayout fixed_layout(const Shape& sh, int esz, bool flash, int M, int n, int max_blocks,
@@ -132,6 +150,7 @@ inline FixedLayout fixed_layout(const Shape& sh, int esz, bool flash, int M, int
   f.gslot = take((int64_t)f.slot_sets * M * slot);
   f.fflag = take((int64_t)n * M * 4);
   f.bflag = take((int64_t)n * M * 4);
+  f.pf = take((1 + 2 * (2 * (int64_t)n)) * 4);  // ticket counter, load_done[R], tickets[R]; R = 2n - 1 loads
   f.xs = take(slot * f.xs_slots);
   f.scr = take(scratch_bytes(sh, esz, true, flash));
   f.tok = take((int64_t)M * sh.mbs * (sh.s + 1) * 4);
@@ -142,10 +161,10 @@ inline FixedLayout fixed_layout(const Shape& sh, int esz, bool flash, int M, int
   return f;
 }
 
-// LM head row chunk in arena mode: MOBIUS_HEAD_ROWS (default 2048) rounded
+// LM head row chunk in arena mode: MOBIUS_HEAD_ROWS (default 1024) rounded
 // down to whole sequences
 inline int arena_head_rows(const Shape& sh) {
-  int r = 2048;
+  int r = 1024;
   if (const char* e = getenv("MOBIUS_HEAD_ROWS")) r = atoi(e);
   r = std::max(sh.s, r / sh.s * sh.s);
   return std::min(r, sh.T());
@@ -263,7 +282,13 @@ struct mobius_ctx {
   uint8_t* scratch_base = nullptr;
   uint8_t* tok_dev = nullptr;
   double* loss_dev = nullptr;
-  int64_t off_ckpt = 0, off_gslot = 0, off_fflag = 0, off_bflag = 0;
+  int64_t off_ckpt = 0, off_gslot = 0, off_fflag = 0, off_bflag = 0, off_pf = 0;
+  // cross-GPU prefetch priority chain (mobius_set_prefetch_groups)
+  std::vector<int> pf_group;      // uplink group per rank (empty: no chain)
+  std::vector<int> pf_pred_rank;  // per my load: rank of its predecessor in the group chain (-1: none / mine)
+  std::vector<int> pf_pred_load;  // ... and that rank's load index
+  int pf_leader = -1;             // rank holding the group's ticket counter
+  int* pf_base = nullptr;         // my prefetch-chain region (arena)
   // MOBIUS_FLAG_DEVICE_TAIL_UPDATE: optimizer state of local stage 0 in HBM
   bool dev_tail = false;
   bool tail_resident = false;     // d_wstage holds local stage 0's current weights (after the first update)
@@ -567,7 +592,7 @@ struct StepRunner {
   }
 
   const T* stage_w(int res, const StageDesc& st, int layer) {
-    return tptr<T>(ctx->ring + ctx->loads[res].base) + st.layer_off[layer - st.first];
+    return tptr<T>(ctx->ring + ctx->loads[res].base + ctx->loads[res].wofs) + st.layer_off[layer - st.first];
   }
 
   int issue_part(int r, int64_t b0, int64_t b1) {
@@ -575,7 +600,7 @@ struct StepRunner {
     const Load& L = ctx->loads[r];
     const StageDesc& st = ctx->all[ctx->mine[L.stage_local]];
     (void)st;
-    uint8_t* dst = ctx->ring + L.base + b0;
+    uint8_t* dst = ctx->ring + L.base + L.wofs + b0;
     // device tail update: local stage 0's weights already live in HBM
     const bool d2d = ctx->tail_resident && L.stage_local == 0;
     const uint8_t* src = d2d ? ctx->d_wstage + b0 : (const uint8_t*)ctx->h_weights[L.stage_local] + b0;
@@ -607,8 +632,8 @@ struct StepRunner {
     if (L.end == 0) {  // bottom [0,S) vs top [P.base, G)
       int64_t a = std::min(S, P.base);
       first0 = 0, first1 = a, second0 = a, second1 = S;
-    } else {           // top [L.base, G) vs bottom [0, P.bytes)
-      int64_t ov = std::max<int64_t>(0, std::min(S, P.bytes - L.base));
+    } else {           // top copy [L.base + wofs, +S) vs bottom [0, P.bytes)
+      int64_t ov = std::max<int64_t>(0, std::min(S, P.bytes - (L.base + L.wofs)));
       first0 = ov, first1 = S, second0 = 0, second1 = ov;
     }
     (void)G;
@@ -621,12 +646,39 @@ struct StepRunner {
     if (ctx->arena_mode && P.bwd) CU(cudaStreamWaitEvent(ctx->s_h2d, ctx->ev_d2h[P.stage_local], 0));
     return MOBIUS_OK;
   }
+  // cross-GPU prefetch priority: my load r waits until its predecessor in
+  // the uplink group's chain (a load of another rank serving an earlier
+  // stage) has landed, then takes a ticket from the group counter
+  int* peer_pf(int rank) {
+    if (rank == ctx->dist.rank) return ctx->pf_base;
+    return reinterpret_cast<int*>(ctx->peer_base[rank] + ctx->peers[rank].off_pf);
+  }
+  int chain_enter(int r) {
+    if (ctx->pf_group.empty()) return MOBIUS_OK;
+    const int pr = ctx->pf_pred_rank[r];
+    if (pr >= 0) {
+      RC(flag_wait(peer_pf(pr) + 1 + ctx->pf_pred_load[r], (int)seq, ctx->s_h2d));
+      ++ctx->launches_step;
+    }
+    const int R = (int)ctx->loads.size();
+    RC(ticket_take(peer_pf(ctx->pf_leader), ctx->pf_base + 1 + R + r, ctx->s_h2d));
+    ++ctx->launches_step;
+    return MOBIUS_OK;
+  }
+  int chain_leave(int r) {
+    if (ctx->pf_group.empty()) return MOBIUS_OK;
+    RC(flag_set(ctx->pf_base + 1 + r, (int)seq, ctx->s_h2d));
+    ++ctx->launches_step;
+    return MOBIUS_OK;
+  }
+
   int load_first_part(int r) {  // issued when residence r-1 starts computing
     if (r >= (int)ctx->loads.size()) return MOBIUS_OK;
     if (r >= 2) {
       CU(cudaStreamWaitEvent(ctx->s_h2d, ctx->ev_release[r - 2], 0));
       RC(wait_offload_of(r - 2));
     }
+    RC(chain_enter(r));
     int64_t a0, a1, b0, b1;
     split_of(r, a0, a1, b0, b1);
     return issue_part(r, a0, a1);
@@ -641,6 +693,7 @@ struct StepRunner {
     }
     RC(issue_part(r, b0, b1));
     CU(cudaEventRecord(ctx->ev_loaded[r], ctx->s_h2d));
+    RC(chain_leave(r));
     return MOBIUS_OK;
   }
 
@@ -843,6 +896,25 @@ struct StepRunner {
     return MOBIUS_OK;
   }
 
+  // arena mode: this backward residence's workspace may overlap the other
+  // end's previous residence, whose gradient staging the D2H offload may
+  // still be reading - wait for that offload only when the ranges meet
+  int wait_staging_overlap(int res) {
+    const Load& L = ctx->loads[res];
+    const Load& P = ctx->loads[res - 1];
+    const StageDesc& sl = ctx->all[ctx->mine[L.stage_local]];
+    const StageDesc& sp = ctx->all[ctx->mine[P.stage_local]];
+    const BwdFootprint fl = bwd_footprint(sl.n_params, ctx->esz, sl.n_blocks, sl.has_embed, ctx->acts_bytes,
+                                          ctx->slot_bytes, L.end == 1);
+    const BwdFootprint fp = bwd_footprint(sp.n_params, ctx->esz, sp.n_blocks, sp.has_embed, ctx->acts_bytes,
+                                          ctx->slot_bytes, P.end == 1);
+    // workspace of L: its footprint minus the weights
+    const int64_t w0 = L.base + (L.end == 1 ? 0 : fl.gst), w1 = L.base + (L.end == 1 ? fl.w : fl.total);
+    const int64_t s0 = P.base + fp.gst, s1 = s0 + al256(sp.n_params * ctx->esz);
+    if (w0 < s1 && s0 < w1) CU(cudaStreamWaitEvent(ctx->s_comp, ctx->ev_d2h[P.stage_local], 0));
+    return MOBIUS_OK;
+  }
+
   // backward buffers of local stage ls in residence res: the fixed
   // workspace, or (arena mode) the residence's own dW / staging / recompute
   // region behind the weights
@@ -854,7 +926,7 @@ struct StepRunner {
     }
     const StageDesc& st = ctx->all[ctx->mine[ls]];
     const BwdFootprint f = bwd_footprint(st.n_params, ctx->esz, st.n_blocks, st.has_embed, ctx->acts_bytes,
-                                         ctx->slot_bytes);
+                                         ctx->slot_bytes, ctx->loads[res].end == 1);
     uint8_t* base = ctx->ring + ctx->loads[res].base;
     ctx->grad_acc = reinterpret_cast<float*>(base + f.gacc);
     ctx->grad_stage = base + f.gst;
@@ -917,6 +989,7 @@ struct StepRunner {
       }
       CU(cudaEventRecord(ctx->ev_pass_a[xi], s));
       if (!e.fwd) {
+        if (ctx->arena_mode && e.res >= 1 && ctx->loads[e.res - 1].bwd) RC(wait_staging_overlap(e.res));
         prepare_bwd(e.ls, e.res);
         if (ctx->ck_off[e.ls]) {  // this stage's checkpoints come back from DRAM
           CU(cudaEventRecord(ctx->ev_ckw_a[e.ls], s));
@@ -1090,6 +1163,7 @@ static int arena_shape(const mobius_model_cfg* c, Shape* sh, int* esz, bool* fla
                    "bad model config");
   *sh = Shape{c->hidden, c->n_heads, c->seq_len, c->micro_batch, c->vocab};
   sh->head_rows = arena_head_rows(*sh);
+  sh->no_keep = true;
   *esz = c->dtype == MOBIUS_F32 ? 4 : 2;
   *flash = *esz == 2 && flash_supported(sh->dh(), sh->s);
   return MOBIUS_OK;
@@ -1210,7 +1284,10 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
   MOBIUS_CHECK_ARG(!arena || plan->hbm_cap_bytes > 0, "MOBIUS_FLAG_ARENA_CAP needs a cap");
   ctx->arena_mode = arena;
   ctx->offload = offload;
-  if (arena) ctx->sh.head_rows = arena_head_rows(ctx->sh);
+  if (arena) {
+    ctx->sh.head_rows = arena_head_rows(ctx->sh);
+    ctx->sh.no_keep = true;
+  }
 
   // per-microbatch sizes
   const Shape& sh = ctx->sh;
@@ -1261,6 +1338,10 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
     Load& L = ctx->loads[r];
     L.end = (int)(r % 2);
     L.base = L.end == 0 ? 0 : ((G - L.bytes) & ~int64_t(255));
+    if (arena && L.bwd && L.end == 1) {
+      const StageDesc& st = ctx->all[ctx->mine[L.stage_local]];
+      L.wofs = bwd_footprint(st.n_params, esz, st.n_blocks, st.has_embed, ctx->acts_bytes, ctx->slot_bytes, true).w;
+    }
   }
 
   // arena layout behind the ring
@@ -1273,6 +1354,7 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
   ctx->off_gslot = FL.gslot;
   ctx->off_fflag = FL.fflag;
   ctx->off_bflag = FL.bflag;
+  ctx->off_pf = FL.pf;
   int64_t o_xs = FL.xs;
   int64_t o_scr = FL.scr;
   int64_t o_tok = FL.tok;
@@ -1366,6 +1448,8 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
     ctx->bad_tok_dev = reinterpret_cast<int*>(ctx->arena + o_bad);
     CU(cudaMemset(ctx->fflag, 0, (int64_t)n * M * 4));
     CU(cudaMemset(ctx->bflag, 0, (int64_t)n * M * 4));
+    ctx->pf_base = reinterpret_cast<int*>(ctx->arena + ctx->off_pf);
+    CU(cudaMemset(ctx->pf_base, 0, (1 + 4 * (int64_t)n) * 4));
 
     // streams: H2D prefetch gets the highest priority
     int lo = 0, hi = 0;
@@ -1487,6 +1571,7 @@ struct ExportBlob {
   cudaIpcMemHandle_t handle;
   int64_t off_ckpt, off_gslot, off_fflag, off_bflag, slot_bytes;
   int32_t n_local, M;
+  int64_t off_pf;
 };
 
 static uint64_t plan_digest(const mobius_ctx* ctx) {
@@ -1529,6 +1614,7 @@ extern "C" int mobius_dist_export(mobius_ctx* ctx, void* buf, size_t cap, size_t
   b.off_gslot = ctx->off_gslot;
   b.off_fflag = ctx->off_fflag;
   b.off_bflag = ctx->off_bflag;
+  b.off_pf = ctx->off_pf;
   b.slot_bytes = ctx->slot_bytes;
   b.n_local = (int)ctx->mine.size();
   b.M = ctx->max_M;
@@ -1557,6 +1643,7 @@ extern "C" int mobius_dist_connect(mobius_ctx* ctx, const void* all, size_t blob
     p.off_gslot = b.off_gslot;
     p.off_fflag = b.off_fflag;
     p.off_bflag = b.off_bflag;
+    p.off_pf = b.off_pf;
     p.slot_bytes = b.slot_bytes;
     p.n_local = b.n_local;
     p.M = b.M;
@@ -1567,12 +1654,89 @@ extern "C" int mobius_dist_connect(mobius_ctx* ctx, const void* all, size_t blob
       int a = ctx->all[j].owner, c = ctx->all[j + 1].owner;
       if ((a == ctx->dist.rank && c == r) || (c == ctx->dist.rank && a == r)) neighbour = true;
     }
+    if (!ctx->pf_group.empty() && ctx->pf_group[r] == ctx->pf_group[ctx->dist.rank]) neighbour = true;
     if (!neighbour) continue;
     void* ptr = nullptr;
     CU(cudaIpcOpenMemHandle(&ptr, b.handle, cudaIpcMemLazyEnablePeerAccess));
     ctx->peer_base[r] = (uint8_t*)ptr;
   }
   ctx->connected = true;
+  return MOBIUS_OK;
+}
+
+extern "C" int mobius_set_prefetch_groups(mobius_ctx* ctx, const int* group, int world) {
+  int rc = check_ctx(ctx);
+  if (rc) return rc;
+  MOBIUS_CHECK_ARG(group && world == ctx->dist.world, "group[world] required (world %d)", ctx->dist.world);
+  MOBIUS_CHECK_ARG(ctx->peers.empty(), "call mobius_set_prefetch_groups before mobius_dist_connect");
+  const mobius_plan_t& P = ctx->plan;
+  const int K = P.n_stages, M = ctx->max_M;
+  // unit-time plan schedule (a stage's time = its layer count, free
+  // transfers): the planned start of every stage pass, a linear extension
+  // of the step's dependency graph, so ordering loads by it adds no cycle
+  std::vector<mobius_layer_profile> unit(P.n_layers);
+  for (auto& l : unit) {
+    std::memset(&l, 0, sizeof(l));
+    l.t_fwd_ns = l.t_bwd_ns = 1;
+    l.mem_fwd = l.mem_bwd = 1;
+  }
+  std::vector<int> sizes(K);
+  for (int j = 0; j < K; ++j) sizes[j] = P.stage_first_layer[j + 1] - P.stage_first_layer[j];
+  std::vector<int64_t> tf((size_t)K * M), tb((size_t)K * M);
+  int64_t mk = 0;
+  rc = mobius_plan_cost(unit.data(), P.n_layers, sizes.data(), K, world, INT64_MAX / 4, M, 0, 0, &mk, tf.data(),
+                        tb.data());
+  if (rc) return rc;
+  struct PL {
+    int64_t key;
+    int rank, r;
+  };
+  std::vector<PL> chain;
+  const int me = ctx->dist.rank;
+  int leader = world;
+  for (int g = 0; g < world; ++g) {
+    if (group[g] != group[me]) continue;
+    leader = std::min(leader, g);
+    std::vector<int> st;
+    for (int j = 0; j < K; ++j)
+      if (ctx->all[j].owner == g) st.push_back(j);
+    const int n = (int)st.size();
+    int r = 0;
+    for (int k = 0; k < n; ++k) chain.push_back({tf[(size_t)st[k] * M], g, r++});      // forward loads
+    for (int k = n - 2; k >= 0; --k) chain.push_back({tb[(size_t)st[k] * M], g, r++});  // backward reloads
+  }
+  std::stable_sort(chain.begin(), chain.end(), [](const PL& a, const PL& b) {
+    if (a.key != b.key) return a.key < b.key;
+    if (a.rank != b.rank) return a.rank < b.rank;
+    return a.r < b.r;
+  });
+  const int R = (int)ctx->loads.size();
+  ctx->pf_pred_rank.assign(R, -1);
+  ctx->pf_pred_load.assign(R, -1);
+  for (size_t i = 0; i < chain.size(); ++i) {
+    if (chain[i].rank != me) continue;
+    MOBIUS_CHECK_ARG(chain[i].r < R, "prefetch chain: load count mismatch");
+    if (i > 0 && chain[i - 1].rank != me) {
+      ctx->pf_pred_rank[chain[i].r] = chain[i - 1].rank;
+      ctx->pf_pred_load[chain[i].r] = chain[i - 1].r;
+    }
+  }
+  ctx->pf_group.assign(group, group + world);
+  ctx->pf_leader = leader;
+  return MOBIUS_OK;
+}
+
+extern "C" int mobius_read_prefetch_tickets(mobius_ctx* ctx, int32_t* out, size_t cap, size_t* n) {
+  int rc = check_ctx(ctx);
+  if (rc) return rc;
+  MOBIUS_CHECK_ARG(out && n, "null argument");
+  const int R = (int)ctx->loads.size();
+  *n = R;
+  if (ctx->pf_group.empty()) MOBIUS_FAIL(MOBIUS_ESTATE, "no prefetch chain (mobius_set_prefetch_groups)");
+  CU(cudaSetDevice(ctx->dist.device));
+  std::vector<int32_t> t(R);
+  CU(cudaMemcpy(t.data(), ctx->pf_base + 1 + R, R * 4, cudaMemcpyDeviceToHost));
+  std::memcpy(out, t.data(), std::min(cap, (size_t)R) * 4);
   return MOBIUS_OK;
 }
 

@@ -258,3 +258,44 @@ def test_plan_1p5b_profile_certified_at_n1(mb):
     # the certificate's partition is no worse than Fig 9's max-stage baseline
     mx = mb.mobius_plan_partition(prof, 1, 1 << 30, 4, mb.PARTITION_MAX_STAGE, mb.make_topology([0], 55 * 10 ** 9, 0))
     assert pl.makespan_ns <= mx.makespan_ns
+
+
+def _pair_from(solo, groups, share=0.5, noise=0.0):
+    """Synthetic concurrent bandwidths: GPUs of one uplink group halve each
+    other's bandwidth, others do not interfere."""
+    n = len(solo)
+    return [[(solo[i] * (share if groups[i] == groups[j] else 1.0 - noise)) if i != j else 0.0 for j in range(n)]
+            for i in range(n)]
+
+
+@pytest.mark.parametrize("groups", [[0, 0, 1, 1], [0, 1, 1, 1], [0, 0, 0, 0], [0, 1, 2, 3],
+                                    [0, 0, 0, 0, 1, 1, 1, 1], [0, 1, 0, 1, 2, 2, 3, 3]])
+def test_topology_from_measured_bandwidth(mb, groups):
+    """GPUs whose concurrent pinned H2D falls below 0.8 x
+    solo share an uplink group (Topo 2+2, 1+3, 4, and 8-GPU layouts); group
+    ids are numbered by first member; host W = median solo."""
+    n = len(groups)
+    solo = [55.0 + i for i in range(n)]
+    t = mb.mobius_topology_from_bw(solo, _pair_from(solo, groups, noise=0.05), 0.8)
+    got = [t.group[i] for i in range(n)]
+    canon, ids = [], {}
+    for g in groups:
+        ids.setdefault(g, len(ids))
+        canon.append(ids[g])
+    assert got == canon
+    assert t.host_bw_Bps == int(sorted(solo)[n // 2] * 1e9)
+    # the measured groups feed the cross mapping: adjacent stages avoid sharing
+    if 1 < len(set(groups)) < n and n <= 8:
+        perm, c, _, _ = mb.mobius_cross_map(2 * n, got)
+        seq, _, _ = mb.mobius_mapping_contention(2 * n, got, list(range(n)))
+        assert c <= seq
+
+
+def test_topology_from_bw_threshold_edge(mb):
+    """Exactly at the threshold the pair is not contended (strict <);
+    contention is judged on the worse of the two directions."""
+    solo = [50.0, 50.0]
+    t = mb.mobius_topology_from_bw(solo, [[0, 40.0], [40.0, 0]], 0.8)
+    assert [t.group[0], t.group[1]] == [0, 1]
+    t = mb.mobius_topology_from_bw(solo, [[0, 50.0], [39.0, 0]], 0.8)
+    assert [t.group[0], t.group[1]] == [0, 0]

@@ -64,8 +64,10 @@ def from_dev(t):
     return t.float().cpu().numpy()
 
 
-@pytest.mark.parametrize("name", ["1.5b", "13b"])
+@pytest.mark.parametrize("name", ["1.5b", "13b", "70b"])
 def test_block_full_size(name):
+    """One block fwd+bwd at configs[1..3] widths (70B: h = 8192, 64 heads of
+    dh 128, s = 2048) vs the oracle."""
     base = synth.CONFIGS[name]
     cfg = synth.GPTConfig(n_layers=base.n_layers, hidden=base.hidden, n_heads=base.n_heads, seq_len=base.seq_len,
                           vocab=64, micro_batch=1)

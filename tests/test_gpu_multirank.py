@@ -25,7 +25,7 @@ def _free_port():
     return p
 
 
-def _rank_main(rank, world, port, sizes, perm, dtype, M, q, steps=1, devices=None):
+def _rank_main(rank, world, port, sizes, perm, dtype, M, q, steps=1, devices=None, groups=None):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     import torch.distributed as dist
@@ -43,6 +43,8 @@ def _rank_main(rank, world, port, sizes, perm, dtype, M, q, steps=1, devices=Non
         plan = plan_from_sizes(sizes, world, M, perm=perm, hbm_cap_bytes=(4 << 20) * (2 if dtype else 1))
         dev = devices[rank] if devices else 0
         ctx = MobiusContext(cfg, plan, rank=rank, world=world, device=dev, init_params=w)
+        if groups is not None:
+            ctx.set_prefetch_groups(groups)
         mdist.connect(ctx)
         losses = [ctx.step(tok)]
         g = ctx.read_grads(c.n_params)
@@ -51,10 +53,11 @@ def _rank_main(rank, world, port, sizes, perm, dtype, M, q, steps=1, devices=Non
         losses += [ctx.step(synth.gen_tokens(c, M, seed=40 + i)) for i in range(steps - 1)]
         tr = ctx.read_trace()
         st = ctx.stats()
+        tickets = ctx.read_prefetch_tickets() if groups is not None else None
         ctx.close()
-        q.put((rank, losses, g, tr, st.h2d_bytes))
+        q.put((rank, losses, g, tr, st.h2d_bytes, tickets))
     except Exception as e:  # pragma: no cover
-        q.put((rank, "ERR", repr(e), None, None))
+        q.put((rank, "ERR", repr(e), None, None, None))
     finally:
         dist.destroy_process_group()
 
@@ -96,11 +99,11 @@ def test_two_ranks_one_gpu(dtype, tol, sizes, perm):
         assert res[r][3] == queues[r]
 
 
-def _run_ranks(world, sizes, perm, dtype, M, steps, devices=None):
+def _run_ranks(world, sizes, perm, dtype, M, steps, devices=None, groups=None):
     port = _free_port()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_rank_main, args=(r, world, port, sizes, perm, dtype, M, q, steps, devices))
+    procs = [ctx.Process(target=_rank_main, args=(r, world, port, sizes, perm, dtype, M, q, steps, devices, groups))
              for r in range(world)]
     for p in procs:
         p.start()
@@ -171,3 +174,64 @@ def test_two_ranks_two_gpus(dtype):
     assert abs(curve[0] - ref_loss) / ref_loss < tol
     ref = _single_rank_curve(sizes, dtype, M, steps)
     assert np.all(np.abs(curve - ref) <= tol * np.abs(ref)), (curve, ref)
+
+
+def _expected_chain(sizes, perm, world, M):
+    """Oracle of the A4 prefetch order: every rank's loads
+    (forward loads of its stages ascending, backward reloads descending
+    except its last stage) keyed by the planned start of the stage pass they
+    serve in the unit-time Eq 3-11 schedule (oracle planner.stage_cost,
+    stage time = its layer count, free transfers); ties by (rank, load)."""
+    from oracle import planner as op
+    layers = op.uniform_profile(sum(sizes), 1, 1, 1, 0)
+    _, tf, tb = op.stage_cost(layers, sizes, world, M, 10 ** 15, None, None)
+    sg = [perm[j % world] for j in range(len(sizes))]
+    chain = []
+    for g in range(world):
+        st = [j for j in range(len(sizes)) if sg[j] == g]
+        loads = [(tf[j + 1][1], j + 1, "F") for j in st] + [(tb[j + 1][1], j + 1, "B") for j in st[:-1][::-1]]
+        chain += [(key, g, r, stage, kind) for r, (key, stage, kind) in enumerate(loads)]
+    return sorted(chain)
+
+
+@pytest.mark.parametrize("sizes,perm", [((1, 1, 1, 1, 1, 1), [0, 1]), ((2, 1, 1, 2), [1, 0])])
+def test_prefetch_priority_chain_shared_uplink(sizes, perm):
+    """SURVEY row a1 / R3 (Fig 4b: "if the prefetching of Stage 5
+    and Stage 7 execute simultaneously, Stage 5 has a higher priority"): two
+    ranks whose GPUs share one host-link group (fake topology [0, 0]; here two
+    processes on one GPU) issue their stage loads one at a time in the
+    oracle's order of planned stage starts - the tickets taken from the
+    group counter reproduce that order exactly, so a stage that starts
+    earlier always gets the link first - and the step still matches the
+    oracle."""
+    import synth
+    from oracle import model as om
+    world, M, steps = 2, 2, 2
+    res = _run_ranks(world, sizes, perm, 0, M, steps, groups=[0, 0])
+    chain = _expected_chain(sizes, perm, world, M)
+    tick = {(r[0], i): t for r in res for i, t in enumerate(r[5])}
+    got = sorted(chain, key=lambda e: tick[(e[1], e[2])])
+    assert [(e[1], e[2]) for e in got] == [(e[1], e[2]) for e in chain]
+    assert len(set(tick.values())) == len(tick)  # one load at a time
+    # R3 directly: of two loads on different GPUs, the earlier-starting stage's goes first
+    for a in chain:
+        for b in chain:
+            if a[1] != b[1] and a[0] < b[0]:
+                assert tick[(a[1], a[2])] < tick[(b[1], b[2])], (a, b)
+    c = synth.TINY
+    w = synth.round_bf16(synth.perturb_norm_params(c, synth.gen_params(c), scale=0.1))
+    ref_loss, ref_g = om.reference_loss_and_grads(c, w, synth.gen_tokens(c, M))
+    g = np.where(np.isnan(res[0][2]), res[1][2], res[0][2])
+    assert np.linalg.norm(g - ref_g) / np.linalg.norm(ref_g) < 2e-2
+    last = res[perm[(len(sizes) - 1) % world]][1]
+    assert abs(last[0] - ref_loss) / ref_loss < 2e-2
+
+
+def test_prefetch_chain_separate_groups_no_cross_wait():
+    """GPUs in different uplink groups (fake topology [0, 1]) never wait for
+    each other: each rank's tickets come from its own counter and are its
+    own load order."""
+    res = _run_ranks(2, (1, 1, 1, 1, 1, 1), [0, 1], 0, 2, 1, groups=[0, 1])
+    for r in res:
+        t = r[5]
+        assert t == sorted(t) and t[-1] - t[0] == len(t) - 1

@@ -555,3 +555,25 @@ def test_ckpt_offload_rejects_multi_rank():
         MobiusContext(mk_cfg(c, BF16), plan_from_sizes((2, 2, 2), 2, 2, hbm_cap_bytes=4 * MiB), world=2,
                       seed=1, flags=FLAG_CKPT_OFFLOAD)
     assert e.value.code == -1
+
+
+@pytest.mark.parametrize("sizes", [(1, 2, 1, 2), (1, 1, 1, 1, 1, 1)])
+def test_arena_cap_repeated_steps_tight_ring(sizes):
+    """Tight whole-memory ring (every backward residence overlaps the other
+    end's): the gradient staging of a finished stage is read by the D2H
+    offload while the next stage's workspace is being set up - five contexts
+    x two steps on the same inputs must give the oracle's gradients every
+    time (a race would zero or corrupt a stage's offloaded gradient)."""
+    from paper_conf_asplos_fengxtwls23_b200 import FLAG_ARENA_CAP
+    c = synth.TINY
+    M = 2
+    w = synth.round_bf16(synth.perturb_norm_params(c, synth.gen_params(c), scale=0.1))
+    tok = synth.gen_tokens(c, M, seed=31)
+    ref_l, ref_g = om.reference_loss_and_grads(c, w, tok)
+    cfg, plan, _ = _arena_plan(c, BF16, sizes, M, ring_extra=0, flags=FLAG_ARENA_CAP)
+    for _ in range(5):
+        ctx = MobiusContext(cfg, plan, init_params=w, flags=FLAG_ARENA_CAP)
+        ctx.step(tok)
+        g = ctx.read_grads(c.n_params)
+        ctx.close()
+        assert max(tensor_errs(c, g, ref_g).values()) < 2e-2
