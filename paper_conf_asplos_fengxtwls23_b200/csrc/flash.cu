@@ -106,7 +106,7 @@ __device__ __forceinline__ float2 ex2_poly2(float2 x) {
                      __int_as_float(__float_as_int(q.y) + (__float_as_int(j.y) << 23)));
 }
 #ifndef MOBIUS_FLASH_POLY_PAIRS
-#define MOBIUS_FLASH_POLY_PAIRS 4  // of every 16 pairs of scores, this many use ex2_poly2 (forward)
+#define MOBIUS_FLASH_POLY_PAIRS 2  // of every 16 pairs of scores, this many use ex2_poly2 (forward)
 #endif
 // score pair e/2 of a 32-column slab: polynomial or MUFU
 __device__ __forceinline__ float2 ex2_pair(float a, float b, int pair) {

@@ -471,7 +471,7 @@ void update_worker(mobius_ctx* ctx) {
   }
 }
 
-void fill_seeded(float* dst, int64_t n, uint64_t seed, int64_t stream_off, float std_) {
+void fill_seeded_serial(float* dst, int64_t n, uint64_t seed, int64_t stream_off, float std_) {
   // counter-based N(0, std^2): splitmix64 -> Box-Muller (deterministic per element index)
   for (int64_t i = 0; i < n; ++i) {
     uint64_t z = seed * 0x9E3779B97F4A7C15ull + (uint64_t)(stream_off + i) * 0xBF58476D1CE4E5B9ull;
@@ -482,6 +482,19 @@ void fill_seeded(float* dst, int64_t n, uint64_t seed, int64_t stream_off, float
     double u2 = ((z & 0x7FF) + 0.5) / 2048.0;
     dst[i] = (float)(std::sqrt(-2.0 * std::log(u1)) * std::cos(6.283185307179586 * u2) * std_);
   }
+}
+
+// the same values from the host thread pool (element-indexed: any split gives
+// identical numbers); the 13B-width stages hold billions of parameters
+thread_local ThreadPool* g_init_pool = nullptr;
+void fill_seeded(float* dst, int64_t n, uint64_t seed, int64_t stream_off, float std_) {
+  const int64_t chunk = 1 << 20;
+  const int tasks = (int)((n + chunk - 1) / chunk);
+  if (!g_init_pool || tasks <= 1) return fill_seeded_serial(dst, n, seed, stream_off, std_);
+  g_init_pool->parallel_for(tasks, [&](int t) {
+    const int64_t b = (int64_t)t * chunk, e = std::min(n, b + chunk);
+    fill_seeded_serial(dst + b, e - b, seed, stream_off + b, std_);
+  });
 }
 
 // initialise the fp32 master of one local stage (oracle init recipe O-1 when
@@ -1535,7 +1548,11 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
         std::memset(mm + b, 0, (e - b) * 4);
         std::memset(vv + b, 0, (e - b) * 4);
       });
-      if (!init_params) seeded_stage_init(c, st, mst, seed);
+      if (!init_params) {
+        g_init_pool = ctx->pool.get();
+        seeded_stage_init(c, st, mst, seed);
+        g_init_pool = nullptr;
+      }
       ctx->pool->parallel_for(tasks, [&](int t) {
         int64_t b = (int64_t)t * chunk, e = std::min(np, b + chunk);
         if (esz == 2) {
