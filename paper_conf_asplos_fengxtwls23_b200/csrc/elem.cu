@@ -742,6 +742,12 @@ __global__ void cast_k(const float* src, T* dst, int64_t n) {
   }
 }
 
+template <typename T>
+__global__ void fill_ones_col_k(T* p, int64_t n) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    p[i] = from_f<T>((i & 63) == 0 ? 1.f : 0.f);
+}
+
 __global__ void tokens_check_k(const int32_t* __restrict__ src, int32_t* __restrict__ dst, int64_t n, int V,
                                int* bad) {
   int cnt = 0;
@@ -1041,6 +1047,13 @@ int gelu_fwd_bf16(const __nv_bfloat16* u, __nv_bfloat16* g, int64_t n, cudaStrea
   return check_launch("gelu_fwd");
 }
 
+template <typename T>
+int fill_ones_col(T* p, int rows, cudaStream_t st) {
+  const int64_t n = (int64_t)rows * 64;
+  fill_ones_col_k<T><<<(unsigned)std::min<int64_t>(148 * 8, (n + 255) / 256), 256, 0, st>>>(p, n);
+  return check_launch("fill_ones_col");
+}
+
 int tokens_check_copy(const int32_t* src, int32_t* dst, int64_t n, int V, int* bad_dev, cudaStream_t st) {
   if (cudaMemsetAsync(bad_dev, 0, sizeof(int), st) != cudaSuccess) MOBIUS_FAIL(MOBIUS_ECUDA, "tokens_check: memset");
   const int grid = (int)std::min<int64_t>(148 * 2, (n + 255) / 256);
@@ -1073,6 +1086,7 @@ int flag_set(int* flag, int value, cudaStream_t st) {
   template int cross_entropy_fwd_bwd<T>(T*, const int32_t*, float*, int, int, int, float, cudaStream_t);        \
   template int colsum_accum<T>(const T*, int64_t, int, int, float*, const RedWs&, cudaStream_t);               \
   template int cast_from_f32<T>(const float*, T*, int64_t, cudaStream_t);                                       \
+  template int fill_ones_col<T>(T*, int, cudaStream_t);                                                          \
   template int adamw_device<T>(float*, float*, float*, const T*, T*, int64_t, float, float, float, float, float,   \
                                float, float, cudaStream_t);
 INST(float)

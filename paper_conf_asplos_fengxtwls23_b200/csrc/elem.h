@@ -79,6 +79,11 @@ template <typename T>
 int adamw_device(float* w, float* m, float* v, const T* g, T* w_out, int64_t n, float lr, float b1, float b2,
                  float eps, float wd, float bc1, float bc2, cudaStream_t st);
 
+// p[r][0..63] = (1, 0, ..., 0) for r < rows: the ones block the weight-
+// gradient GEMM loads as the extra A row that yields the bias gradient
+template <typename T>
+int fill_ones_col(T* p, int rows, cudaStream_t st);
+
 // dst = src (n token ids) and *bad_dev (device int) = number of ids outside [0, V)
 int tokens_check_copy(const int32_t* src, int32_t* dst, int64_t n, int V, int* bad_dev, cudaStream_t st);
 

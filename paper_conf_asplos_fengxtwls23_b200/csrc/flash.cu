@@ -173,7 +173,25 @@ struct FwdParams {
   float* lse;        // [mbs, nh, s], log2 domain
   int s, nh, h, mbs;
   float scale_log2;  // log2(e) / sqrt(dh)
+  int group;         // (batch, head) pairs per item chunk (see chunked_item)
 };
+
+// Item order of the persistent kernels: the (batch, head) pairs are taken
+// `group` at a time and each chunk's items are listed heaviest tile first.
+// All tiles of a pair then run within a few waves of each other, so the
+// pair's fp32 dQ accumulator (backward) stays in L2 between its key tiles;
+// ordering the whole list heaviest first (one tile level for every pair,
+// then the next; group = all pairs, still the forward's order) re-reads it
+// from DRAM (ncu: flash bwd moved 3.1 GB per call at mbs 32, five times its
+// algorithmic bytes).
+// Returns the tile level (0 = heaviest) and the pair index.
+__device__ __forceinline__ void chunked_item(int i, int n_t, int nbh, int group, int& level, int& pair) {
+  const int per = group * n_t;
+  const int c = i / per, idx = i - c * per;
+  const int gc = min(group, nbh - c * group);  // pairs in this (possibly partial) chunk
+  level = idx / gc;
+  pair = c * group + idx % gc;
+}
 
 // Persistent item order: pass k visits CTAs left-to-right for even k and
 // right-to-left for odd k over a list sorted heaviest first, so per-CTA
@@ -184,8 +202,9 @@ __device__ __forceinline__ int snake_item(int pass, int ncta, int cta) {
 
 __device__ __forceinline__ void fwd_item(const FwdParams& p, int i, int& qt, int& hd, int& b) {
   const int n_qt = p.s / BQ, nb = p.nh * p.mbs;
-  qt = n_qt - 1 - i / nb;  // heaviest (most kv tiles) first
-  const int r = i % nb;
+  int level, r;
+  chunked_item(i, n_qt, nb, p.group, level, r);
+  qt = n_qt - 1 - level;  // heaviest (most kv tiles) first within a chunk
   hd = r % p.nh;
   b = r / p.nh;
 }
@@ -568,6 +587,7 @@ struct BwdParams {
   float* dQacc;         // [mbs*s, h] fp32 (head view), accumulated by TMA reduce-add
   int s, nh, h, mbs;
   float scale_log2, scale;
+  int group;            // (batch, head) pairs per item chunk (chunked_item)
 };
 
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
@@ -628,8 +648,8 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
   // item index -> (key tile, head, batch); the list is sorted heaviest
   // first: every (b, head) with key tile 0 (n_t query tiles) before key tile 1 ...
   auto decode = [&](int item, int& kt, int& hd, int& b) {
-    kt = item / nbh;
-    const int r = item % nbh;
+    int r;
+    chunked_item(item, n_t, nbh, p.group, kt, r);  // key tile 0 (most query tiles) first within a chunk
     hd = r % p.nh;
     b = r / p.nh;
   };
@@ -734,7 +754,9 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
       for (int pass = 0; pass * ncta < n_items; ++pass) {
         const int item = snake_item(pass, ncta, cta);
         if (item >= n_items) continue;
-        const int nq = n_t - item / nbh;
+        int kt_, hd_, b_;
+        decode(item, kt_, hd_, b_);
+        const int nq = n_t - kt_;
         ptx::mbar_wait(kv_full, n & 1);
         // S^T / dP^T TMEM must have been read (dh 64; dh 128: issue_st waits dq_empty)
         if (C::DQ_OWN && g >= 1) ptx::mbar_wait(st_empty, (g - 1) & 1);
@@ -1050,6 +1072,24 @@ __global__ void flash_dq_cast_kernel(const float* dQacc, __nv_bfloat16* dq, int6
   o[1] = __floats2bfloat162_rn(v.z * scale, v.w * scale);
 }
 
+// (batch, head) pairs per item chunk of the backward: MOBIUS_FLASH_GROUP
+// (0 or >= the pair count = one chunk, the global heaviest-first order).
+// Default 64 at dh 64 (1.5B, mbs 32: bwd 701 -> 663 us; 16 / 32 / 128:
+// 667 / 686 / 672 us) and one chunk at dh 128, where a chunk that keeps the
+// fp32 dQ of its pairs in L2 (<= ~40 pairs of 1 MB) has too few items to
+// balance 148 CTAs (13B shape, mbs 2: 402 us ungrouped, 419-488 grouped).
+// The forward stays ungrouped (K / V re-reads measured cheaper than the lost
+// balance: 261 us ungrouped, 266-274 grouped).
+static int flash_group(int nbh, int dh) {
+  static int g = -2;
+  if (g == -2) {
+    const char* e = getenv("MOBIUS_FLASH_GROUP");
+    g = e ? atoi(e) : -1;
+  }
+  const int v = g == -1 ? (dh == 64 ? 64 : 0) : g;
+  return (v <= 0 || v > nbh) ? nbh : v;
+}
+
 typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
@@ -1126,6 +1166,7 @@ int flash_attn_fwd(const __nv_bfloat16* qkv, __nv_bfloat16* o, float* lse, int m
   p.h = h;
   p.mbs = mbs;
   p.scale_log2 = 1.4426950408889634f / sqrtf((float)dh);
+  p.group = nh * mbs;  // one chunk: global heaviest-first order
   int n_items = (s / BQ) * nh * mbs;
   int sms = 148;
   {
@@ -1179,6 +1220,7 @@ int flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* o, const __nv_
   p.scale_log2 = 1.4426950408889634f / sqrtf((float)dh);
   p.scale = 1.0f / sqrtf((float)dh);
   p.mbs = mbs;
+  p.group = flash_group(nh * mbs, dh);
   const int n_items = (s / 128) * nh * mbs;
   int sms = 148;
   {

@@ -50,7 +50,19 @@ struct GemmDesc {
   MatView AUX;                // EPI_BIAS_GELU: pre-activation output (path type)
   int causal = CAUSAL_NONE;
   bool accumulate = false;    // EPI_ACCUM
+  // Bias gradient in the weight-gradient GEMM (a_mn, EPI_ACCUM): logical row
+  // M-1 of A is all ones (A holds only rows 0..M-2), so row M-1 of C gets
+  // sum_k B[n, k] - the column sums of dY - next to dW (the packed block
+  // layout stores each bias right after its weight).  bf16: `ones` is a
+  // [>= K][64] buffer whose column 0 is 1 (row M-1 is loaded from it; M-1 a
+  // multiple of 64); fp32 debug path: the kernel synthesises the row.
+  bool ones_row = false;
+  const void* ones = nullptr;
 };
+
+// true when gemm_bf16 / gemm_f32 run d with ones_row (else the caller sums
+// the bias gradient itself)
+bool gemm_ones_row_supported(const GemmDesc& d, bool f32);
 
 // tcgen05/TMEM/TMA kernel (bf16 operands, fp32 accumulate).  Returns a
 // mobius_status.

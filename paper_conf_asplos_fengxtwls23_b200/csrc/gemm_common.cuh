@@ -62,6 +62,9 @@ struct Params {
   int64_t sk_units;
   float* sk_ws;
   int* sk_cnt;
+  // ones row (2-CTA kernel, A_MN): the 64-row A box starting at M row
+  // ones_m0p1 - 1 is loaded from the ones map (tmX) instead of A (0 = off)
+  int ones_m0p1;
 };
 
 __device__ __forceinline__ float tanh_fast(float x) {

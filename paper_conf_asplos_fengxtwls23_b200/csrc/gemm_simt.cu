@@ -16,6 +16,7 @@ struct SParams {
   const float *A, *B;
   int64_t lda, abs1, abs2, ldb, bbs1, bbs2;
   int a_mn, b_mn;
+  int ones_row;  // A row M-1 is all ones (bias gradient next to dW)
   float* C;
   int64_t ldc, cbs1, cbs2;
   int epi, causal, accumulate;
@@ -57,7 +58,8 @@ __global__ void __launch_bounds__(256) gemm_simt_kernel(const SParams p) {
       if (p.a_mn) { kk = i / TM; mm = i % TM; } else { mm = i / TK; kk = i % TK; }
       int gm = m0 + mm, gk = k0 + kk;
       float v = 0.f;
-      if (gm < p.M && gk < k_end) v = p.a_mn ? A[(int64_t)gk * p.lda + gm] : A[(int64_t)gm * p.lda + gk];
+      if (gm < p.M && gk < k_end)
+        v = (p.ones_row && gm == p.M - 1) ? 1.f : p.a_mn ? A[(int64_t)gk * p.lda + gm] : A[(int64_t)gm * p.lda + gk];
       As[kk][mm] = v;
     }
     for (int i = threadIdx.x; i < TK * TN; i += 256) {
@@ -112,6 +114,7 @@ int gemm_f32(const GemmDesc& d, cudaStream_t s) {
   p.M = d.M; p.N = d.N; p.K = d.K; p.nb2 = d.nb2;
   p.A = (const float*)d.A.ptr; p.lda = d.A.ld; p.abs1 = d.A.bs1; p.abs2 = d.A.bs2; p.a_mn = d.a_mn;
   p.B = (const float*)d.B.ptr; p.ldb = d.B.ld; p.bbs1 = d.B.bs1; p.bbs2 = d.B.bs2; p.b_mn = d.b_mn;
+  p.ones_row = d.ones_row ? 1 : 0;
   p.C = (float*)d.C.ptr; p.ldc = d.C.ld; p.cbs1 = d.C.bs1; p.cbs2 = d.C.bs2;
   p.epi = d.epi; p.causal = d.causal; p.accumulate = d.accumulate; p.alpha = d.alpha;
   p.bias = (const float*)d.bias;

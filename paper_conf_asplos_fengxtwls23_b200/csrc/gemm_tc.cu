@@ -275,14 +275,24 @@ void gemm_set_config(int two_cta, int stream_k) {
   gemm_2cta_set_stream_k(stream_k);
 }
 
-int gemm_bf16(const GemmDesc& d, cudaStream_t s) {
+static bool use_2cta(const GemmDesc& d) {
   if (g_gemm_mode < 0) {
     const char* e = getenv("MOBIUS_GEMM_2CTA");
     g_gemm_mode = (e && e[0] == '0') ? 0 : 1;
   }
-  if (g_gemm_mode == 1 && d.causal == CAUSAL_NONE && d.nb1 == 1 && d.nb2 == 1 && d.N >= 256 && d.M >= 256 &&
-      d.K >= 64)
-    return gemm_bf16_2cta(d, s);
+  return g_gemm_mode == 1 && d.causal == CAUSAL_NONE && d.nb1 == 1 && d.nb2 == 1 && d.N >= 256 && d.M >= 256 &&
+         d.K >= 64;
+}
+
+bool gemm_ones_row_supported(const GemmDesc& d, bool f32) {
+  if (f32) return true;  // the SIMT kernel synthesises the row
+  const int r = d.M - 1;
+  return use_2cta(d) && d.a_mn && d.epi == EPI_ACCUM && r % 64 == 0 && r % 256 != 0;
+}
+
+int gemm_bf16(const GemmDesc& d, cudaStream_t s) {
+  if (use_2cta(d)) return gemm_bf16_2cta(d, s);
+  MOBIUS_CHECK_ARG(!d.ones_row, "gemm: the ones row needs the 2-CTA kernel");
   MOBIUS_CHECK_ARG(d.M > 0 && d.N > 0 && d.K > 0, "gemm: empty shape %d x %d x %d", d.M, d.N, d.K);
   MOBIUS_CHECK_ARG(d.N % 8 == 0 || !true, "gemm: N must be a multiple of 8");
   int BN = d.N >= 256 ? 256 : (d.N > 64 ? 128 : 64);

@@ -401,7 +401,13 @@ __global__ void __launch_bounds__(NUM_THREADS2, 1)
           if (NP == 1) {
             if (A_MN) {
 #pragma unroll
-              for (int i = 0; i < 2; ++i) ptx::tma_load_4d_2sm(a + i * 8192, &tmA, &full[stage], m0 + 64 * i, k0, 0, 0);
+              for (int i = 0; i < 2; ++i) {
+                const int mm = m0 + 64 * i;
+                if (p.ones_m0p1 && mm == p.ones_m0p1 - 1)  // bias-gradient row: [1, 0 .. 0] per k
+                  ptx::tma_load_4d_2sm(a + i * 8192, &tmX, &full[stage], 0, k0, 0, 0);
+                else
+                  ptx::tma_load_4d_2sm(a + i * 8192, &tmA, &full[stage], mm, k0, 0, 0);
+              }
             } else {
               ptx::tma_load_4d_2sm(a, &tmA, &full[stage], k0, m0, 0, 0);
             }
@@ -816,8 +822,12 @@ template <int BN>
 static int gemm_bf16_2cta_bn(const GemmDesc& d, cudaStream_t s) {
   CUtensorMap ta, tb, tc, tr, tx;
   int rc;
+  const bool ones = d.ones_row;
+  if (ones)
+    MOBIUS_CHECK_ARG(d.a_mn && d.epi == EPI_ACCUM && d.ones && (d.M - 1) % 64 == 0 && (d.M - 1) % 256 != 0,
+                     "gemm: ones row needs a_mn, EPI_ACCUM, a ones buffer and M-1 a multiple of 64 inside a tile");
   if (d.a_mn)
-    rc = make_map(&ta, d.A, d.M, d.K, d.nb1, d.nb2, BK);
+    rc = make_map(&ta, d.A, ones ? d.M - 1 : d.M, d.K, d.nb1, d.nb2, BK);
   else
     rc = make_map(&ta, d.A, d.K, d.M, d.nb1, d.nb2, 128);
   if (rc) return rc;
@@ -837,6 +847,11 @@ static int gemm_bf16_2cta_bn(const GemmDesc& d, cudaStream_t s) {
   }
   if (d.epi == EPI_BIAS_GELU || (d.epi == EPI_GELU_BWD && d.AUX.ptr)) {
     if ((rc = make_map_2d(&tx, d.AUX.ptr, false, d.AUX.ld, d.N, d.M, 64, 32))) return rc;
+  } else if (ones) {  // EPI_ACCUM reads no AUX: the slot carries the ones map ([K][64], column 0 = 1)
+    MatView ov;
+    ov.ptr = d.ones;
+    ov.ld = 64;
+    if ((rc = make_map(&tx, ov, 64, d.K, 1, 1, BK))) return rc;
   } else {
     tx = tc;
   }
@@ -852,6 +867,7 @@ static int gemm_bf16_2cta_bn(const GemmDesc& d, cudaStream_t s) {
   p.bias = (const __nv_bfloat16*)d.bias;
   p.R = (const __nv_bfloat16*)d.R.ptr; p.ldr = d.R.ld;
   p.AUX = (__nv_bfloat16*)d.AUX.ptr; p.ldx = d.AUX.ld;
+  p.ones_m0p1 = ones ? d.M : 0;  // (M - 1) + 1
   plan_stream_k(p, num_sms() / 2);
   if (p.sk_tiles) {
     const size_t ws = (size_t)p.sk_tiles * p.sk_maxseg * 16 * 32 * (BN / 2) * sizeof(float);

@@ -82,7 +82,8 @@ MatView mv(const void* p, int64_t ld, int64_t bs1 = 0, int64_t bs2 = 0) {
 template <typename T>
 int run_gemm(GemmDesc& d, cudaStream_t st, int cls) {
   KernelTimer* t = g_timer;
-  int64_t flops = 2LL * d.M * d.N * d.K * d.nb1 * d.nb2;
+  // algorithmic GEMM work: a ones row (the fused bias gradient) is not counted
+  int64_t flops = 2LL * (d.ones_row ? d.M - 1 : d.M) * d.N * d.K * d.nb1 * d.nb2;
   if (d.causal != CAUSAL_NONE) flops /= 2;  // algorithmic work of a causal product
   if (t) t->begin(cls, st);
   int rc = gemm<T>(d, st);
@@ -100,16 +101,38 @@ int run_gemm(GemmDesc& d, cudaStream_t st, int cls) {
 struct ElemScope {
   cudaStream_t st;
   int n;
+  bool open = true;
   ElemScope(cudaStream_t s, int n_) : st(s), n(n_) {
     if (g_timer) g_timer->begin(KCLS_ELEM, st);
   }
-  ~ElemScope() {
+  void timed_end() {  // close the timing bracket early (work that follows belongs to another class)
+    if (!open) return;
+    open = false;
     if (g_timer) g_timer->end(KCLS_ELEM, st, 0);
     g_kernel_launches += n;
   }
+  ~ElemScope() { timed_end(); }
 };
 
 }  // namespace
+
+// The weight-gradient GEMM d (C += A^T B, A = X^T MN-major) also produces
+// the bias gradient sum_rows B as the row after the weight's last row (where
+// the packed layout keeps the bias) when the GEMM kernel supports a ones row
+// there; returns whether it does (else the caller runs a column sum).
+template <typename T>
+bool with_bias_row(GemmDesc& d, const Scratch<T>& sc) {
+  static const bool off = getenv("MOBIUS_NO_BIAS_ROW") != nullptr;  // A/B: separate column sums
+  if (off) return false;
+  GemmDesc t = d;
+  t.M = d.M + 1;
+  t.ones_row = true;
+  t.ones = sc.ones;
+  const bool f32 = sizeof(T) == 4;
+  if ((!f32 && !sc.ones) || !gemm_ones_row_supported(t, f32)) return false;
+  d = t;
+  return true;
+}
 
 template <>
 bool use_flash<float>(const Shape&) {
@@ -190,6 +213,7 @@ int64_t scratch_bytes(const Shape& sh, int e, bool with_head, bool flash) {
   c.take<char>(kt * T * 4 * h * e);  // rg
   c.take<char>(red_ws_floats(sh) * 4);
   c.take<char>(RED_WS_COUNTERS * 4);
+  c.take<char>(e == 2 ? T * 64 * 2 : 0);  // ones column block of the fused bias gradients
   return c.off;
 }
 
@@ -217,12 +241,15 @@ void carve_scratch(const Shape& sh, uint8_t* base, bool with_head, Scratch<T>& s
   sc.rg = kt ? c.take<T>(Tn * 4 * h * e) : nullptr;
   sc.red.part = c.take<float>(red_ws_floats(sh) * 4);
   sc.red.cnt = c.take<unsigned>(RED_WS_COUNTERS * 4);
+  sc.ones = sizeof(T) == 2 ? c.take<T>(Tn * 64 * 2) : nullptr;
+  sc.ones_rows = Tn;
 }
 
 template <typename T>
 int scratch_zero(const Scratch<T>& sc, cudaStream_t st) {
   if (cudaMemsetAsync(sc.red.cnt, 0, RED_WS_COUNTERS * 4, st) != cudaSuccess)
     MOBIUS_FAIL(MOBIUS_ECUDA, "scratch_zero");
+  if (sc.ones) return fill_ones_col(sc.ones, sc.ones_rows, st);
   return MOBIUS_OK;
 }
 
@@ -425,18 +452,18 @@ int block_bwd(const Shape& sh, const T* w, const BlockActs<T>& A_in, const T* dy
     d.epi = EPI_ACCUM; d.accumulate = true;
     RC(run_gemm<T>(d, st, KCLS_GEMM));
   }
-  {
-    ElemScope es(st, 2);
-    RC(colsum_accum<T>(dy, h, Tn, h, G + L.b_2, sc.red, st));
-    RC(colsum_accum<T>(du, 4 * h, Tn, 4 * h, G + L.b_1, sc.red, st));
-  }
-  {  // dW1 += a2^T du
+  {  // dW1 += a2^T du, and db1 += sum du as its ones row (b_1 follows w_1 in the layout)
     GemmDesc d;
     d.M = h; d.N = 4 * h; d.K = Tn;
     d.A = mv(A.a2, h); d.a_mn = true;
     d.B = mv(du, 4 * h); d.b_mn = true;
     d.C = mv(G + L.w_1, 4 * h); d.c_f32 = true;
     d.epi = EPI_ACCUM; d.accumulate = true;
+    const bool fused = with_bias_row<T>(d, sc);
+    ElemScope es(st, fused ? 1 : 2);
+    RC(colsum_accum<T>(dy, h, Tn, h, G + L.b_2, sc.red, st));
+    if (!fused) RC(colsum_accum<T>(du, 4 * h, Tn, 4 * h, G + L.b_1, sc.red, st));
+    es.timed_end();
     RC(run_gemm<T>(d, st, KCLS_GEMM));
   }
   {  // da2 = du W1^T
@@ -452,18 +479,19 @@ int block_bwd(const Shape& sh, const T* w, const BlockActs<T>& A_in, const T* dy
     ElemScope es(st, 2);
     RC(layernorm_bwd<T>(sc.t1, A.x1, w + L.ln2_g, A.mu2, A.rs2, dy, dx1, G + L.ln2_g, G + L.ln2_b, Tn, h, sc.red, st));
   }
-  {  // dWo += o^T dx1
+  {  // dWo += o^T dx1, db_o += sum dx1 as its ones row
     GemmDesc d;
     d.M = h; d.N = h; d.K = Tn;
     d.A = mv(A.o, h); d.a_mn = true;
     d.B = mv(dx1, h); d.b_mn = true;
     d.C = mv(G + L.w_o, h); d.c_f32 = true;
     d.epi = EPI_ACCUM; d.accumulate = true;
+    const bool fused = with_bias_row<T>(d, sc);
     RC(run_gemm<T>(d, st, KCLS_GEMM));
-  }
-  {
-    ElemScope es(st, 1);
-    RC(colsum_accum<T>(dx1, h, Tn, h, G + L.b_o, sc.red, st));
+    if (!fused) {
+      ElemScope es(st, 1);
+      RC(colsum_accum<T>(dx1, h, Tn, h, G + L.b_o, sc.red, st));
+    }
   }
   T* dO = sc.t3;
   {  // do = dx1 Wo^T
@@ -476,18 +504,19 @@ int block_bwd(const Shape& sh, const T* w, const BlockActs<T>& A_in, const T* dy
   }
   T* dqkv = sc.qkv_g;
   RC(attention_bwd<T>(sh, A.qkv, A.o, A.P, A.lse, dO, dqkv, sc, st));
-  {  // dWqkv += a^T dqkv
+  {  // dWqkv += a^T dqkv, db_qkv += sum dqkv as its ones row
     GemmDesc d;
     d.M = h; d.N = 3 * h; d.K = Tn;
     d.A = mv(A.a, h); d.a_mn = true;
     d.B = mv(dqkv, 3 * h); d.b_mn = true;
     d.C = mv(G + L.w_qkv, 3 * h); d.c_f32 = true;
     d.epi = EPI_ACCUM; d.accumulate = true;
+    const bool fused = with_bias_row<T>(d, sc);
     RC(run_gemm<T>(d, st, KCLS_GEMM));
-  }
-  {
-    ElemScope es(st, 1);
-    RC(colsum_accum<T>(dqkv, 3 * h, Tn, 3 * h, G + L.b_qkv, sc.red, st));
+    if (!fused) {
+      ElemScope es(st, 1);
+      RC(colsum_accum<T>(dqkv, 3 * h, Tn, 3 * h, G + L.b_qkv, sc.red, st));
+    }
   }
   {  // da = dqkv Wqkv^T
     GemmDesc d;

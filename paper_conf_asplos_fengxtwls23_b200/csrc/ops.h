@@ -69,6 +69,8 @@ struct Scratch {
   float *mu, *rs;  // [T] (head LN)
   T *ra, *ra2, *rg;  // recompute targets of a compact BlockActs: [T, h], [T, h], [T, 4h]
   RedWs red;       // deterministic column-reduction workspace (counters zeroed by scratch_zero)
+  T* ones = nullptr;   // bf16 path: [T][64], column 0 = 1 (ones row of the fused bias gradients; scratch_zero fills it)
+  int ones_rows = 0;
 };
 // zero the reduction counters of a freshly carved Scratch (once per arena)
 template <typename T>

@@ -183,6 +183,7 @@ def test_bench_launch_config_step_properties():
     from paper_conf_asplos_fengxtwls23_b200 import FLAG_DEVICE_TAIL_UPDATE, FLAG_KEEP_ACTS
     c = dataclasses.replace(synth.GPT_1_5B, micro_batch=32)
     M = 4
+    torch.cuda.empty_cache()  # the keep pool sizes itself from the free HBM: release earlier tests' cached blocks
     cfg = model_cfg(c.n_layers, c.hidden, c.n_heads, c.seq_len, c.vocab, c.micro_batch, dtype=BF16)
     prof = mobius_profile(cfg, 0)
     plan = mobius_plan(prof, 1, 1 << 30, M, make_topology([0], 55 * 10 ** 9, 0))

@@ -54,9 +54,18 @@ def main():
     if world > 1:
         import torch.distributed as dist
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    from paper_conf_asplos_fengxtwls23_b200 import mobius_cross_map, mobius_discover_topology
-    topo = mobius_discover_topology()
-    groups = [topo.group[i] for i in range(topo.n_gpus)][:max(world, 1)]
+    from paper_conf_asplos_fengxtwls23_b200 import (mobius_cross_map, mobius_mapping_contention,
+                                                    mobius_probe_topology)
+    probe = None
+    if rank == 0:  # measured contention groups (SURVEY #12): concurrent pinned H2D < 0.8 x solo
+        topo, solo, pair = mobius_probe_topology(256 << 20, 0.8)
+        probe = {"solo_GBps": solo, "pair_GBps": pair, "p2p_GBps": topo.p2p_bw_Bps / 1e9,
+                 "groups": [topo.group[i] for i in range(topo.n_gpus)]}
+    if world > 1:
+        obj = [probe]
+        dist.broadcast_object_list(obj, src=0)
+        probe = obj[0]
+    groups = probe["groups"][:max(world, 1)]
     hi = torch.cuda.Stream(priority=-1)
     lo = torch.cuda.Stream(priority=0)
     comp = torch.cuda.Stream(priority=0)
@@ -101,8 +110,11 @@ def main():
         del host, dev, dev2, host2
     if rank == 0:
         perm, cont, num, den = mobius_cross_map(2 * max(world, 1), groups)
-        summary = {"summary": True, "groups": groups, "cross_map": list(perm), "cross_contention": cont,
-                   "note": "N=1: no host-link contention between GPUs; cross vs sequential differs only for N>1"}
+        seq = mobius_mapping_contention(2 * max(world, 1), groups, list(range(len(groups))))[0]
+        summary = {"summary": True, "groups": groups, "probe": probe, "cross_map": list(perm),
+                   "cross_contention": cont, "sequential_contention": seq,
+                   "note": "N=1: no host-link contention between GPUs; cross vs sequential differs only for N>1 "
+                           "(end-to-end comparison: bench.py --mapping cross|sequential --topology probe)"}
         print(json.dumps(summary))
         if args.out:
             with open(args.out, "w") as f:
