@@ -90,10 +90,11 @@ __device__ __forceinline__ uint32_t pack_bf16x2(float2 v) { return pack_bf16(v.x
 // coefficients from a relative-error least-squares fit on Chebyshev nodes).
 // round(x) comes from the 1.5 * 2^23 magic-number add, whose low mantissa
 // bits then hold it as an integer that is shifted into the exponent.
-// x is clamped to -125 (2^-125 ~ 0 for softmax weights; no denormals).
-__device__ __forceinline__ float2 ex2_poly2(float2 x) {
-  x.x = fmaxf(x.x, -125.f);
-  x.y = fmaxf(x.y, -125.f);
+// Arguments below -125 (masked scores: -inf) give exactly 0, like ex2.approx.ftz.
+__device__ __forceinline__ float2 ex2_poly2(float2 x0) {
+  float2 x;
+  x.x = fmaxf(x0.x, -125.f);
+  x.y = fmaxf(x0.y, -125.f);
   const float2 magic = make_float2(12582912.f, 12582912.f);
   const float2 j = __fadd2_rn(x, magic);
   const float2 t = __fadd2_rn(j, make_float2(-12582912.f, -12582912.f));  // round(x)
@@ -102,8 +103,8 @@ __device__ __forceinline__ float2 ex2_poly2(float2 x) {
                         make_float2(0.24228397011756897f, 0.24228397011756897f));
   q = __ffma2_rn(q, f, make_float2(0.6935495138168335f, 0.6935495138168335f));
   q = __ffma2_rn(q, f, make_float2(0.9999545216560364f, 0.9999545216560364f));
-  return make_float2(__int_as_float(__float_as_int(q.x) + (__float_as_int(j.x) << 23)),
-                     __int_as_float(__float_as_int(q.y) + (__float_as_int(j.y) << 23)));
+  return make_float2(x0.x < -125.f ? 0.f : __int_as_float(__float_as_int(q.x) + (__float_as_int(j.x) << 23)),
+                     x0.y < -125.f ? 0.f : __int_as_float(__float_as_int(q.y) + (__float_as_int(j.y) << 23)));
 }
 #ifndef MOBIUS_FLASH_POLY_PAIRS
 #define MOBIUS_FLASH_POLY_PAIRS 2  // of every 16 pairs of scores, this many use ex2_poly2 (forward)
