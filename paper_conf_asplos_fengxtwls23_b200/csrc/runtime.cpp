@@ -297,6 +297,10 @@ struct mobius_ctx {
   uint8_t* d_wstage = nullptr;    // new stage-0 weights (transfer precision) for the D2H
 
   // peers
+  std::vector<char> p2p_copy;       // per rank: activations to it go through a local slot + copy engine
+  uint8_t* send_stage = nullptr;    // 2 local slots (microbatch parity) staging those sends
+  cudaStream_t s_p2p = nullptr;
+  cudaEvent_t ev_send[2] = {nullptr, nullptr}, ev_sprod = nullptr;
   std::vector<uint8_t*> peer_base;  // opened IPC bases (nullptr for me)
   std::vector<PeerInfo> peers;
   bool connected = false;
@@ -367,6 +371,14 @@ void mobius_ctx::teardown() {
     if (p) cudaIpcCloseMemHandle(p);
   peer_base.clear();
   if (s_ckup) cudaStreamSynchronize(s_ckup);
+  if (s_p2p) cudaStreamSynchronize(s_p2p);
+  for (cudaEvent_t* e : {&ev_send[0], &ev_send[1], &ev_sprod})
+    if (*e) {
+      cudaEventDestroy(*e);
+      *e = nullptr;
+    }
+  if (send_stage) cudaFree(send_stage);
+  send_stage = nullptr;
   for (auto* v : {&ev_release, &ev_loaded, &ev_part_a, &ev_part_b, &ev_gready, &ev_d2h, &ev_wait_a, &ev_wait_b,
                   &ev_pass_a, &ev_pass_b, &ev_off_a, &ev_off_b, &ev_ckoff, &ev_ckprod, &ev_ckup, &ev_ck_a,
                   &ev_ck_b, &ev_ckw_a, &ev_ckw_b}) {
@@ -412,7 +424,8 @@ void mobius_ctx::teardown() {
   if (s_h2d) cudaStreamDestroy(s_h2d);
   if (s_d2h) cudaStreamDestroy(s_d2h);
   if (s_ckup) cudaStreamDestroy(s_ckup);
-  s_comp = s_h2d = s_d2h = s_ckup = nullptr;
+  if (s_p2p) cudaStreamDestroy(s_p2p);
+  s_comp = s_h2d = s_d2h = s_ckup = s_p2p = nullptr;
   cudaGetLastError();  // a failed create must not leave a stale error for the caller's next CUDA call
 }
 
@@ -575,6 +588,38 @@ struct StepRunner {
     *flag = reinterpret_cast<int*>(b + pi.off_fflag) + (int64_t)nx.ord * pi.M + m;
     return tptr<T>(b + pi.off_ckpt + ((int64_t)nx.ord * pi.M + m) * pi.slot_bytes);
   }
+  // Destination of stage j's forward output for microbatch m.  A peer on
+  // another GPU gets it through a local staging slot and a copy-engine
+  // transfer over NVLink (send_staged) - the producing GEMM's TMA stores stay
+  // local - unless MOBIUS_P2P_DIRECT=1 (the epilogue stores straight into
+  // the peer's slot, as it does for a peer sharing this GPU).
+  T* fwd_target(int j, int m, int** flag, T** remote) {
+    T* d = fwd_dest(j, m, flag);
+    *remote = nullptr;
+    if (!*flag || !ctx->p2p_copy[ctx->all[j + 1].owner]) return d;
+    *remote = d;
+    cudaStreamWaitEvent(ctx->s_comp, ctx->ev_send[m % 2], 0);  // the slot's previous send has left
+    return tptr<T>(ctx->send_stage + (int64_t)(m % 2) * ctx->slot_bytes);
+  }
+  int send_staged(const T* local, T* remote, int* flag, int m) {
+    CU(cudaEventRecord(ctx->ev_sprod, ctx->s_comp));
+    CU(cudaStreamWaitEvent(ctx->s_p2p, ctx->ev_sprod, 0));
+    CU(cudaMemcpyAsync(remote, local, (int64_t)ctx->sh.T() * ctx->sh.h * sizeof(T), cudaMemcpyDeviceToDevice,
+                       ctx->s_p2p));
+    RC(flag_set(flag, (int)seq, ctx->s_p2p));  // after the copy (stream order): release to the consumer
+    ++ctx->launches_step;
+    CU(cudaEventRecord(ctx->ev_send[m % 2], ctx->s_p2p));
+    return MOBIUS_OK;
+  }
+  // flag after a local producer wrote the output: direct -> set on the compute stream
+  int deliver(const T* y, T* remote, int* flag, int m) {
+    if (!flag) return MOBIUS_OK;
+    if (remote) return send_staged(y, remote, flag, m);
+    RC(flag_set(flag, (int)seq, ctx->s_comp));
+    ++ctx->launches_step;
+    return MOBIUS_OK;
+  }
+
   T* bwd_dest(int j, int m, int** flag) {
     const StageDesc& pv = ctx->all[j - 1];
     int r = pv.owner;
@@ -734,12 +779,13 @@ struct StepRunner {
     if (st.has_embed) {
       T* out;
       int* flag = nullptr;
+      T* remote = nullptr;
       if (st.n_blocks == 0 && !last_stage)
-        out = fwd_dest(st.j, m, &flag);
+        out = fwd_target(st.j, m, &flag, &remote);
       else
         out = (kept(ls) && kf(ls) == 0) ? keep_x(ls, m, 0) : xbuf(0);
       RC(embed_layer_fwd<T>(sh, stage_w(res, st, 0), tok(m), out, s));
-      if (flag) { RC(flag_set(flag, (int)seq, s)); ++ctx->launches_step; }
+      RC(deliver(out, remote, flag, m));
       x = out;
     } else {
       if (ctx->all[st.j - 1].owner != ctx->dist.rank)
@@ -752,21 +798,22 @@ struct StepRunner {
       if (li == 0) continue;
       const bool last_block = (bi == st.n_blocks - 1);
       int* flag = nullptr;
+      T* remote = nullptr;
       if (kept(ls) && bi >= kf(ls)) {  // keep this block's activations for its backward (no recompute)
-        T* y = last_block ? fwd_dest(st.j, m, &flag) : keep_x(ls, m, bi + 1);
+        T* y = last_block ? fwd_target(st.j, m, &flag, &remote) : keep_x(ls, m, bi + 1);
         BlockActs<T> ka = keep_acts(ls, m, bi);
         ka.x = x;
         RC(block_fwd<T>(sh, stage_w(res, st, li), ka, y, sc, s));
-        if (flag) { RC(flag_set(flag, (int)seq, s)); ++ctx->launches_step; }
+        RC(deliver(y, remote, flag, m));
         x = y;
         ++bi;
         continue;
       }
-      T* y = last_block ? fwd_dest(st.j, m, &flag)
+      T* y = last_block ? fwd_target(st.j, m, &flag, &remote)
                         : (kept(ls) && bi + 1 == kf(ls)) ? keep_x(ls, m, bi + 1) : xbuf(1 + (bi % 2));
       acts[0].x = x;
       RC(block_fwd<T>(sh, stage_w(res, st, li), acts[0], y, sc, s));
-      if (flag) { RC(flag_set(flag, (int)seq, s)); ++ctx->launches_step; }
+      RC(deliver(y, remote, flag, m));
       x = y;
       ++bi;
     }
@@ -1084,6 +1131,7 @@ int do_step(mobius_ctx* ctx, const int32_t* tok_dev, int M, float* loss_out) {
   CU(cudaStreamSynchronize(ctx->s_comp));
   CU(cudaStreamSynchronize(ctx->s_h2d));
   CU(cudaStreamSynchronize(ctx->s_d2h));
+  if (ctx->s_p2p) CU(cudaStreamSynchronize(ctx->s_p2p));
   int64_t t_gpu_done = now_ns();
   {  // synchronous update: every stage's AdamW has landed
     std::unique_lock<std::mutex> lk(ctx->upd_mu);
@@ -1646,6 +1694,7 @@ extern "C" int mobius_dist_connect(mobius_ctx* ctx, const void* all, size_t blob
   MOBIUS_CHECK_ARG(all && blob_len >= sizeof(ExportBlob), "bad blobs");
   const int W = ctx->dist.world;
   ctx->peers.resize(W);
+  ctx->p2p_copy.assign(W, 0);
   CU(cudaSetDevice(ctx->dist.device));
   for (int r = 0; r < W; ++r) {
     ExportBlob b;
@@ -1676,6 +1725,20 @@ extern "C" int mobius_dist_connect(mobius_ctx* ctx, const void* all, size_t blob
     void* ptr = nullptr;
     CU(cudaIpcOpenMemHandle(&ptr, b.handle, cudaIpcMemLazyEnablePeerAccess));
     ctx->peer_base[r] = (uint8_t*)ptr;
+    cudaPointerAttributes pa;
+    CU(cudaPointerGetAttributes(&pa, ptr));
+    const char* direct = getenv("MOBIUS_P2P_DIRECT");
+    const char* copy = getenv("MOBIUS_P2P_COPY");
+    ctx->p2p_copy[r] = (copy && copy[0] == '1') || (pa.device != ctx->dist.device && !(direct && direct[0] == '1'));
+  }
+  bool any_copy = false;
+  for (char c : ctx->p2p_copy) any_copy |= c != 0;
+  if (any_copy && !ctx->send_stage) {
+    CU(cudaMalloc(&ctx->send_stage, 2 * ctx->slot_bytes));
+    CU(cudaStreamCreateWithFlags(&ctx->s_p2p, cudaStreamNonBlocking));
+    for (auto* e : {&ctx->ev_send[0], &ctx->ev_send[1], &ctx->ev_sprod}) CU(cudaEventCreateWithFlags(e, cudaEventDisableTiming));
+    CU(cudaEventRecord(ctx->ev_send[0], ctx->s_p2p));
+    CU(cudaEventRecord(ctx->ev_send[1], ctx->s_p2p));
   }
   ctx->connected = true;
   return MOBIUS_OK;

@@ -235,3 +235,31 @@ def test_prefetch_chain_separate_groups_no_cross_wait():
     for r in res:
         t = r[5]
         assert t == sorted(t) and t[-1] - t[0] == len(t) - 1
+
+
+@pytest.mark.parametrize("dtype", [0, 1])
+def test_two_ranks_copy_engine_transport(dtype, monkeypatch):
+    """The transport used for peers on other GPUs: the producing kernel
+    writes a local staging slot and a copy-engine transfer (its own stream,
+    then the release flag) moves it to the peer's checkpoint slot
+    (MOBIUS_P2P_COPY=1 forces it for ranks sharing this GPU).  Gradients vs
+    the oracle, three-step loss curve vs one rank (bitwise on fp32)."""
+    import synth
+    from oracle import model as om
+    monkeypatch.setenv("MOBIUS_P2P_COPY", "1")
+    sizes, perm, world, M, steps = (1, 2, 2, 1), [0, 1], 2, 2, 3
+    res = _run_ranks(world, sizes, perm, dtype, M, steps)
+    c = synth.TINY
+    w = synth.perturb_norm_params(c, synth.gen_params(c), scale=0.1)
+    if dtype == 0:
+        w = synth.round_bf16(w)
+    ref_loss, ref_g = om.reference_loss_and_grads(c, w, synth.gen_tokens(c, M))
+    tol = 2e-2 if dtype == 0 else 1e-4
+    g = np.where(np.isnan(res[0][2]), res[1][2], res[0][2])
+    assert np.linalg.norm(g - ref_g) / np.linalg.norm(ref_g) < tol
+    curve = np.array(res[perm[(len(sizes) - 1) % world]][1])
+    ref = _single_rank_curve(sizes, dtype, M, steps)
+    if dtype == 1:
+        assert np.array_equal(curve, ref), (curve, ref)
+    else:
+        assert np.all(np.abs(curve - ref) <= tol * np.abs(ref)), (curve, ref)
