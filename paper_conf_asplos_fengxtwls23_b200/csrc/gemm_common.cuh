@@ -65,6 +65,10 @@ struct Params {
   // ones row (2-CTA kernel, A_MN): the 64-row A box starting at M row
   // ones_m0p1 - 1 is loaded from the ones map (tmX) instead of A (0 = off)
   int ones_m0p1;
+  // split-K with reduce-add (2-CTA kernel, EPI_ACCUM + accumulate): the
+  // sk_tiles * sk_slices units of the k-aligned schedule cover every tile
+  // and each unit reduce-adds its partial straight into C (no workspace).
+  int splitk_reduce;
 };
 
 __device__ __forceinline__ float tanh_fast(float x) {

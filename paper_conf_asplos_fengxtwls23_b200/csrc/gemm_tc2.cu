@@ -283,8 +283,8 @@ struct Sched {
       w.t = (int)(g % p.sk_tiles);
       w.k0 = sl * kbs;
       w.k1 = min(p.num_kb, w.k0 + kbs);
-      w.seg = sl;
-      w.nseg = p.sk_slices;
+      w.seg = p.splitk_reduce ? 0 : sl;
+      w.nseg = p.splitk_reduce ? 1 : p.sk_slices;  // split-K: each unit reduce-adds into C itself
       g += ncl;
       return true;
     }
@@ -752,6 +752,7 @@ static void plan_stream_k(Params& p, int P) {
   p.sk_units = 0;
   p.sk_maxseg = 0;
   p.sk_slices = 0;
+  p.splitk_reduce = 0;
   if (g_gemm_sk < 0) {
     const char* e = getenv("MOBIUS_GEMM_SK");
     g_gemm_sk = (e && e[0] == '0') ? 0 : 1;
@@ -762,6 +763,37 @@ static void plan_stream_k(Params& p, int P) {
     g_gemm_skmode = e ? atoi(e) : 0;
   }
   const int T = p.tiles_m * p.tiles_n, nkb = p.num_kb;
+  // fp32-accumulating long-K GEMMs (the weight gradients, C += A^T B with
+  // TMA reduce-add epilogues): split every tile's K range into S slices dealt
+  // slice-major over the clusters, each slice reduce-adding its partial into
+  // C - the sum order across slices then varies in the last bits (the bf16
+  // path is not bitwise reproducible anyway).  S minimises
+  // ceil(T S / P) / S waves plus 0.02 per extra slice (its reduce traffic);
+  // MOBIUS_GEMM_SPLITK=0 keeps the Stream-K tail below.
+  static int splitk = -1;
+  if (splitk < 0) {
+    const char* e = getenv("MOBIUS_GEMM_SPLITK");
+    splitk = e ? atoi(e) : 1;
+  }
+  if (splitk && p.epi == EPI_ACCUM && p.accumulate && p.c_f32 && nkb >= 64) {
+    int best_s = 1;
+    double best = (double)((T + P - 1) / P);
+    for (int S = 2; S <= 8 && nkb / S >= 16; ++S) {
+      const double c = (double)((T * S + P - 1) / P) / S + 0.02 * (S - 1);
+      if (c < best - 1e-9) {
+        best = c;
+        best_s = S;
+      }
+    }
+    if (best_s > 1) {
+      p.sk_tiles = T;
+      p.sk_slices = best_s;
+      p.sk_maxseg = 1;
+      p.sk_units = (int64_t)T * best_s;
+      p.splitk_reduce = 1;
+      return;
+    }
+  }
   if (T % P == 0) return;
   static int min_slice = -1;  // k-blocks per slice (MOBIUS_GEMM_SKSLICE, default 16)
   if (min_slice < 0) {
@@ -869,7 +901,7 @@ static int gemm_bf16_2cta_bn(const GemmDesc& d, cudaStream_t s) {
   p.AUX = (__nv_bfloat16*)d.AUX.ptr; p.ldx = d.AUX.ld;
   p.ones_m0p1 = ones ? d.M : 0;  // (M - 1) + 1
   plan_stream_k(p, num_sms() / 2);
-  if (p.sk_tiles) {
+  if (p.sk_tiles && !p.splitk_reduce) {
     const size_t ws = (size_t)p.sk_tiles * p.sk_maxseg * 16 * 32 * (BN / 2) * sizeof(float);
     int rc2 = sk_workspace(s, ws, (size_t)p.sk_tiles * 16, &p.sk_ws, &p.sk_cnt);
     if (rc2) return rc2;
