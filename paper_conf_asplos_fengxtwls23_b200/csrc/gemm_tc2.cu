@@ -768,12 +768,15 @@ static void plan_stream_k(Params& p, int P) {
   // slice-major over the clusters, each slice reduce-adding its partial into
   // C - the sum order across slices then varies in the last bits (the bf16
   // path is not bitwise reproducible anyway).  S minimises
-  // ceil(T S / P) / S waves plus 0.02 per extra slice (its reduce traffic);
-  // MOBIUS_GEMM_SPLITK=0 keeps the Stream-K tail below.
+  // ceil(T S / P) / S waves plus 0.02 per extra slice (its reduce traffic).
+  // Opt-in (MOBIUS_GEMM_SPLITK=1): faster in isolation (dW GEMMs 1806 ->
+  // 1704 us per block at T = 32768) but neutral inside the step (A/B on one
+  // box: 91.4k vs 91.2-91.4k tokens/s), so the deterministic Stream-K tail
+  // below stays the default.
   static int splitk = -1;
   if (splitk < 0) {
     const char* e = getenv("MOBIUS_GEMM_SPLITK");
-    splitk = e ? atoi(e) : 1;
+    splitk = e ? atoi(e) : 0;
   }
   if (splitk && p.epi == EPI_ACCUM && p.accumulate && p.c_f32 && nkb >= 64) {
     int best_s = 1;
