@@ -166,7 +166,7 @@ struct FwdCfg {
   // dh 64: O leaves through a staging tile (4 KB per 32-row quadrant) and
   // TMA stores; dh 128 has no smem left for it and stores row per thread
   static constexpr int O_STG = DH == 64 ? 128 * 128 : 0;
-  static constexpr int SMEM = 1024 + 2 * Q_BYTES + 2 * KVS * KV_BYTES + 2 * P_BYTES + O_STG + 4096;
+  static constexpr int SMEM = 1024 + 2 * Q_BYTES + 2 * KVS * KV_BYTES + 2 * P_BYTES + O_STG + 8192;  // + sMax/sSum (<= 6 KB at CP 4), barriers
 };
 
 struct FwdParams {
@@ -217,10 +217,12 @@ __device__ __forceinline__ void fwd_item(const FwdParams& p, int i, int& qt, int
 // TMEM with lazy rescaling.  Each query row is handled by two softmax warps
 // (column halves) that exchange only the row max.  All barrier phases run on
 // global step counters across items.
-template <int DH>
-__global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_constant__ CUtensorMap tm,
-                                                              const __grid_constant__ CUtensorMap tmo, const FwdParams p) {
+template <int DH, int CP>
+__global__ void __launch_bounds__((2 + 4 * CP) * 32, 1)
+    flash_fwd_kernel(const __grid_constant__ CUtensorMap tm, const __grid_constant__ CUtensorMap tmo,
+                     const FwdParams p) {
   using C = FwdCfg<DH>;
+  constexpr int NSW = 4 * CP;  // softmax warps
   constexpr int KVS = C::KVS;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -229,9 +231,9 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
   uint8_t* sV = sK + KVS * C::KV_BYTES;   // [KVS]
   uint8_t* sP = sV + KVS * C::KV_BYTES;   // [2]
   uint8_t* sO = sP + 2 * C::P_BYTES;      // O staging (dh 64)
-  float* sMax = reinterpret_cast<float*>(sO + C::O_STG);  // [2 iters][2 halves][128]
-  float* sSum = sMax + 512;                                       // [2 halves][128]
-  uint64_t* bars = reinterpret_cast<uint64_t*>(sSum + 256);
+  float* sMax = reinterpret_cast<float*>(sO + C::O_STG);  // [2 iters][CP parts][128]
+  float* sSum = sMax + 2 * CP * 128;                              // [CP parts][128]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sSum + CP * 128);
   uint64_t* q_full = bars;                  // [2]
   uint64_t* q_empty = bars + 2;             // [2]
   uint64_t* s_full = bars + 4;              // [2]
@@ -261,11 +263,11 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
       ptx::mbar_init(&q_full[i], 1);
       ptx::mbar_init(&q_empty[i], 1);
       ptx::mbar_init(&s_full[i], 1);
-      ptx::mbar_init(&s_empty[i], 8);
-      ptx::mbar_init(&p_full[i], 8);
+      ptx::mbar_init(&s_empty[i], NSW);
+      ptx::mbar_init(&p_full[i], NSW);
       ptx::mbar_init(&pv_done[i], 1);
       ptx::mbar_init(&o_ready[i], 1);
-      ptx::mbar_init(&o_empty[i], 8);
+      ptx::mbar_init(&o_empty[i], NSW);
     }
     ptx::fence_mbar_init();
   }
@@ -369,8 +371,12 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
     }
   } else {
     // ------------------------------------------------ softmax warps
-    const int q4 = warp & 3;          // TMEM lane quadrant
-    const int hf = (warp - 2) >> 2;   // column half of S (and of O)
+    // 4 * CP warps: (TMEM lane quadrant q4) x (column part cq of CP); a
+    // thread owns row `row` of S, columns [cq SC, cq SC + SC), and OC
+    // columns of O
+    constexpr int SC = 128 / CP, NG = SC / 32, OC = DH / CP;
+    const int q4 = warp & 3;           // TMEM lane quadrant
+    const int cq = (warp - 2) >> 2;    // column part of S (and of O)
     const int row = q4 * 32 + lane;
     const uint32_t lb = (uint32_t)(q4 * 32) << 16;
     const float sc = p.scale_log2;
@@ -383,8 +389,50 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
     __nv_bfloat16* pd_orow = nullptr;
     float* pd_lse = nullptr;
     int pd_qt = 0, pd_hd = 0, pd_b = 0;
-    const bool o_issuer = hf == 0 && lane == 0;  // issues this quadrant's O TMA stores (dh 64)
+    const bool o_issuer = cq == 0 && lane == 0;  // issues this quadrant's O TMA stores (dh 64)
     const uint32_t o_slab = ptx::smem_u32(sO) + q4 * 4096;
+    // OC columns of O in TMEM (oc0: first column of this part) <-> registers
+    auto o_pack_store = [&](uint32_t base, float inv_l) {
+      // base: TMEM address of this part's O columns; writes bf16(O * inv_l)
+      if constexpr (OC == 16) {
+        uint32_t v[16];
+        __syncwarp();
+        ptx::tmem_ld16(base, v);
+        ptx::tmem_ld_wait();
+        uint32_t pk[8];
+#pragma unroll
+        for (int e = 0; e < 16; e += 2)
+          pk[e / 2] = pack_bf16(__uint_as_float(v[e]) * inv_l, __uint_as_float(v[e + 1]) * inv_l);
+        static_assert(DH == 64, "OC 16 only at dh 64");
+#pragma unroll
+        for (int k = 0; k < 2; ++k)
+          st_shared_v4(o_slab + lane * 128 + (((cq * 2 + k) ^ (lane & 7)) << 4), pk[4 * k], pk[4 * k + 1],
+                       pk[4 * k + 2], pk[4 * k + 3]);
+      } else {
+#pragma unroll
+        for (int c = 0; c < OC / 32; ++c) {
+          uint32_t v[32];
+          __syncwarp();
+          ptx::tmem_ld32(base + c * 32, v);
+          ptx::tmem_ld_wait();
+          uint32_t pk[16];
+#pragma unroll
+          for (int e = 0; e < 32; e += 2)
+            pk[e / 2] = pack_bf16(__uint_as_float(v[e]) * inv_l, __uint_as_float(v[e + 1]) * inv_l);
+          if constexpr (DH == 64) {  // row `lane` of the quadrant's 32-row slab, 16-byte chunks, SW128
+#pragma unroll
+            for (int k = 0; k < 4; ++k)
+              st_shared_v4(o_slab + lane * 128 + (((cq * (OC / 8) + c * 4 + k) ^ (lane & 7)) << 4), pk[4 * k],
+                           pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
+          } else {
+#pragma unroll
+            for (int k = 0; k < 4; ++k)
+              *reinterpret_cast<uint4*>(pd_orow + c * 32 + k * 8) =
+                  make_uint4(pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
+          }
+        }
+      }
+    };
     auto store_o = [&]() {
       if (!pend) return;
       pend = false;
@@ -393,33 +441,12 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
       const float inv_l = 1.f / pd_l;
       if constexpr (DH == 64) {
         if (o_issuer) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // previous store read the slab
-        named_bar(2 + q4, 64);
+        named_bar(2 + q4, 32 * CP);
       }
-#pragma unroll
-      for (int c = 0; c < DH / 64; ++c) {
-        uint32_t v[32];
-        __syncwarp();
-        ptx::tmem_ld32(tmem + 256 + pd_ob * DH + hf * (DH / 2) + c * 32 + lb, v);
-        ptx::tmem_ld_wait();
-        uint32_t pk[16];
-#pragma unroll
-        for (int e = 0; e < 32; e += 2)
-          pk[e / 2] = pack_bf16(__uint_as_float(v[e]) * inv_l, __uint_as_float(v[e + 1]) * inv_l);
-        if constexpr (DH == 64) {  // row `lane` of the quadrant's 32-row slab, 16-byte chunks hf*4.., SW128
-#pragma unroll
-          for (int k = 0; k < 4; ++k)
-            st_shared_v4(o_slab + lane * 128 + (((hf * 4 + k) ^ (lane & 7)) << 4), pk[4 * k], pk[4 * k + 1],
-                         pk[4 * k + 2], pk[4 * k + 3]);
-        } else {
-#pragma unroll
-          for (int k = 0; k < 4; ++k)
-            *reinterpret_cast<uint4*>(pd_orow + c * 32 + k * 8) =
-                make_uint4(pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
-        }
-      }
+      o_pack_store(tmem + 256 + pd_ob * DH + cq * OC + lb, inv_l);
       if constexpr (DH == 64) {
         ptx::fence_proxy_async();
-        named_bar(2 + q4, 64);
+        named_bar(2 + q4, 32 * CP);
         if (o_issuer) {
           asm volatile("cp.async.bulk.tensor.4d.global.shared::cta.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
                            reinterpret_cast<uint64_t>(&tmo)),
@@ -428,7 +455,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
           asm volatile("cp.async.bulk.commit_group;" ::: "memory");
         }
       }
-      if (hf == 0) *pd_lse = pd_m + __log2f(pd_l);
+      if (cq == 0) *pd_lse = pd_m + __log2f(pd_l);
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(&o_empty[pd_ob]);
@@ -444,91 +471,92 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
       for (int j = 0; j < nkv; ++j, ++g) {
         const int sb = g & 1;
         const bool diag = (j == qt);
-        const uint32_t TS = tmem + sb * 128 + hf * 64 + lb;
+        const uint32_t TS = tmem + sb * 128 + cq * SC + lb;
         ptx::mbar_wait(&s_full[sb], (g >> 1) & 1);
         ptx::tc_fence_after();
-        uint32_t v0[32], v1[32];
+        uint32_t v[NG][32];
         __syncwarp();
-        ptx::tmem_ld32(TS, v0);
-        ptx::tmem_ld32(TS + 32, v1);
+#pragma unroll
+        for (int gi = 0; gi < NG; ++gi) ptx::tmem_ld32(TS + gi * 32, v[gi]);
         ptx::tmem_ld_wait();
         ptx::tc_fence_before();
         __syncwarp();
         if (lane == 0) ptx::mbar_arrive(&s_empty[sb]);  // S values are in registers
-        const int cbase = hf * 64;  // first key column of this half
+        const int cbase = cq * SC;  // first key column of this part
         if (diag) {  // mask keys > query (only on the diagonal tile)
 #pragma unroll
-          for (int e = 0; e < 32; ++e) {
-            if (cbase + e > row) v0[e] = __float_as_uint(-INFINITY);
-            if (cbase + 32 + e > row) v1[e] = __float_as_uint(-INFINITY);
-          }
+          for (int gi = 0; gi < NG; ++gi)
+#pragma unroll
+            for (int e = 0; e < 32; ++e)
+              if (cbase + gi * 32 + e > row) v[gi][e] = __float_as_uint(-INFINITY);
         }
-        // pass A: half-row max of raw scores, combined across the warp pair
+        // pass A: part-row max of raw scores, combined across the CP warps of the row
         float mx = -INFINITY;
 #pragma unroll
-        for (int e = 0; e < 32; e += 2) mx = fmaxf(mx, fmaxf(__uint_as_float(v0[e]), __uint_as_float(v0[e + 1])));
+        for (int gi = 0; gi < NG; ++gi)
 #pragma unroll
-        for (int e = 0; e < 32; e += 2) mx = fmaxf(mx, fmaxf(__uint_as_float(v1[e]), __uint_as_float(v1[e + 1])));
-        sts_f32(ptx::smem_u32(sMax + (g & 1) * 256 + hf * 128 + row), mx);
-        named_bar(2 + q4, 64);
-        mx = fmaxf(mx, lds_f32(ptx::smem_u32(sMax + (g & 1) * 256 + (1 - hf) * 128 + row)));
+          for (int e = 0; e < 32; e += 2)
+            mx = fmaxf(mx, fmaxf(__uint_as_float(v[gi][e]), __uint_as_float(v[gi][e + 1])));
+        float* smx = sMax + (g & 1) * (CP * 128);
+        sts_f32(ptx::smem_u32(smx + cq * 128 + row), mx);
+        named_bar(2 + q4, 32 * CP);
+#pragma unroll
+        for (int c = 0; c < CP; ++c)
+          if (c != cq) mx = fmaxf(mx, lds_f32(ptx::smem_u32(smx + c * 128 + row)));
         // lazy rescaling: keep the running max unless it grows by > 8 (log2)
         const float m_cand = fmaxf(m_run, mx * sc);
         const bool grow = m_cand > m_run + 8.f;
         const float m_new = grow ? m_cand : m_run;
         const float alpha = ex2(m_run - m_new);  // 1 when not growing; 0 at j = 0
-        if (j >= 1 && __any_sync(0xffffffffu, grow)) {  // rescale this half of O (PV of step g-1 done)
+        if (j >= 1 && __any_sync(0xffffffffu, grow)) {  // rescale this part of O (PV of step g-1 done)
           ptx::mbar_wait(&pv_done[(g - 1) & 1], ((g - 1) >> 1) & 1);
           ptx::tc_fence_after();
-#pragma unroll
-          for (int c = 0; c < DH / 64; ++c) {
-            uint32_t o[32];
-            const uint32_t TO = tmem + 256 + ob * DH + hf * (DH / 2) + c * 32 + lb;
-            ptx::tmem_ld32(TO, o);
+          const uint32_t TO = tmem + 256 + ob * DH + cq * OC + lb;
+          if constexpr (OC == 16) {
+            uint32_t o[16];
+            ptx::tmem_ld16(TO, o);
             ptx::tmem_ld_wait();
 #pragma unroll
-            for (int e = 0; e < 32; ++e) o[e] = __float_as_uint(__uint_as_float(o[e]) * alpha);
-            ptx::tmem_st32(TO, o);
+            for (int e = 0; e < 16; ++e) o[e] = __float_as_uint(__uint_as_float(o[e]) * alpha);
+            ptx::tmem_st16(TO, o);
+          } else {
+#pragma unroll
+            for (int c = 0; c < OC / 32; ++c) {
+              uint32_t o[32];
+              ptx::tmem_ld32(TO + c * 32, o);
+              ptx::tmem_ld_wait();
+#pragma unroll
+              for (int e = 0; e < 32; ++e) o[e] = __float_as_uint(__uint_as_float(o[e]) * alpha);
+              ptx::tmem_st32(TO + c * 32, o);
+            }
           }
           ptx::tmem_st_wait();
         }
         // P buffer sb is free once the PV of global step g-2 completed
         if (g >= 2) ptx::mbar_wait(&pv_done[sb], ((g - 2) >> 1) & 1);
-        // pass B: P = 2^(x*sc - m_new) -> smem (bf16), half-row sum
+        // pass B: P = 2^(x*sc - m_new) -> TMEM / smem (bf16), part-row sum
         const uint32_t sp = ptx::smem_u32(sP + sb * C::P_BYTES);
         float rs = 0.f;
-        {
+#pragma unroll
+        for (int gi = 0; gi < NG; ++gi) {
           uint32_t pk[16];
 #pragma unroll
           for (int e = 0; e < 32; e += 2) {
-            const float2 pp = ex2_pair(fmaf(__uint_as_float(v0[e]), sc, -m_new), fmaf(__uint_as_float(v0[e + 1]), sc, -m_new),
-                                       e >> 1);
+            const float2 pp = ex2_pair(fmaf(__uint_as_float(v[gi][e]), sc, -m_new),
+                                       fmaf(__uint_as_float(v[gi][e + 1]), sc, -m_new), (e >> 1) + gi * 8);
             rs += pp.x + pp.y;
             pk[e >> 1] = pack_bf16(pp.x, pp.y);
           }
-          if constexpr (C::P_TMEM) {  // keys hf*64 .. +31 -> packed columns hf*32 .. +15
-            ptx::tmem_st16(tmem + 384 + sb * 64 + hf * 32 + lb, pk);
+          if constexpr (C::P_TMEM) {  // keys cq*SC + gi*32 .. -> packed columns cq*SC/2 + gi*16 ..
+            ptx::tmem_st16(tmem + 384 + sb * 64 + cq * (SC / 2) + gi * 16 + lb, pk);
           } else {
 #pragma unroll
             for (int k = 0; k < 4; ++k)
-              st_shared_v4(sp + sw128_off(row, hf * 8 + k), pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
-          }
-#pragma unroll
-          for (int e = 0; e < 32; e += 2) {
-            const float2 pp = ex2_pair(fmaf(__uint_as_float(v1[e]), sc, -m_new), fmaf(__uint_as_float(v1[e + 1]), sc, -m_new),
-                                       (e >> 1) + 8);
-            rs += pp.x + pp.y;
-            pk[e >> 1] = pack_bf16(pp.x, pp.y);
-          }
-          if constexpr (C::P_TMEM) {
-            ptx::tmem_st16(tmem + 384 + sb * 64 + hf * 32 + 16 + lb, pk);
-            ptx::tmem_st_wait();
-          } else {
-#pragma unroll
-            for (int k = 0; k < 4; ++k)
-              st_shared_v4(sp + sw128_off(row, hf * 8 + 4 + k), pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
+              st_shared_v4(sp + sw128_off(row, cq * (SC / 8) + gi * 4 + k), pk[4 * k], pk[4 * k + 1], pk[4 * k + 2],
+                           pk[4 * k + 3]);
           }
         }
+        if constexpr (C::P_TMEM) ptx::tmem_st_wait();
         l_run = l_run * alpha + rs;
         m_run = m_new;
         ptx::tc_fence_before();
@@ -537,19 +565,21 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_fwd_kernel(const __grid_const
         if (lane == 0) ptx::mbar_arrive(&p_full[sb]);
         if (j == 0) store_o();  // previous item's O while this tile's PV runs
       }
-      // output: O / l  (l = sum of both halves).  The O read-out waits for
+      // output: O / l  (l = sum over the CP parts).  The O read-out waits for
       // the item's last PV, so it is deferred until the next item's first P
       // tile is handed to the tensor core (O is double-buffered in TMEM)
-      sts_f32(ptx::smem_u32(sSum + hf * 128 + row), l_run);
-      named_bar(2 + q4, 64);
-      const float l_tot = l_run + lds_f32(ptx::smem_u32(sSum + (1 - hf) * 128 + row));
-      named_bar(2 + q4, 64);  // partner read sSum before the next item overwrites it
+      sts_f32(ptx::smem_u32(sSum + cq * 128 + row), l_run);
+      named_bar(2 + q4, 32 * CP);
+      float l_tot = 0.f;
+#pragma unroll
+      for (int c = 0; c < CP; ++c) l_tot += lds_f32(ptx::smem_u32(sSum + c * 128 + row));
+      named_bar(2 + q4, 32 * CP);  // partners read sSum before the next item overwrites it
       pend = true;
       pd_ob = ob;
       pd_ph = (it >> 1) & 1;
       pd_l = l_tot;
       pd_m = m_run;
-      pd_orow = p.O + ((int64_t)b * p.s + qrow) * p.h + hd * DH + hf * (DH / 2);
+      pd_orow = p.O + ((int64_t)b * p.s + qrow) * p.h + hd * DH + cq * OC;
       pd_lse = p.lse + ((int64_t)b * p.nh + hd) * p.s + qrow;
       pd_qt = qt;
       pd_hd = hd;
@@ -1178,12 +1208,24 @@ int flash_attn_fwd(const __nv_bfloat16* qkv, __nv_bfloat16* o, float* lse, int m
   dim3 grid(n_items < sms ? n_items : sms);
   if (dh == 64) {
     static bool once = false;
-    if (!once) { rc = set_smem(flash_fwd_kernel<64>, FwdCfg<64>::SMEM); if (rc) return rc; once = true; }
-    flash_fwd_kernel<64><<<grid, NT_FWD, FwdCfg<64>::SMEM, st>>>(tm, tmo, p);
+    // MOBIUS_FLASH_FWD_CP: softmax warps per S row (2: 8 warps of half rows, 4: 16 warps of quarter rows)
+    static int cp = -1;
+    if (cp < 0) {
+      const char* e = getenv("MOBIUS_FLASH_FWD_CP");
+      cp = (e && atoi(e) == 4) ? 4 : 2;
+    }
+    if (cp == 4) {
+      static bool once4 = false;
+      if (!once4) { rc = set_smem(flash_fwd_kernel<64, 4>, FwdCfg<64>::SMEM); if (rc) return rc; once4 = true; }
+      flash_fwd_kernel<64, 4><<<grid, (2 + 16) * 32, FwdCfg<64>::SMEM, st>>>(tm, tmo, p);
+    } else {
+      if (!once) { rc = set_smem(flash_fwd_kernel<64, 2>, FwdCfg<64>::SMEM); if (rc) return rc; once = true; }
+      flash_fwd_kernel<64, 2><<<grid, NT_FWD, FwdCfg<64>::SMEM, st>>>(tm, tmo, p);
+    }
   } else {
     static bool once = false;
-    if (!once) { rc = set_smem(flash_fwd_kernel<128>, FwdCfg<128>::SMEM); if (rc) return rc; once = true; }
-    flash_fwd_kernel<128><<<grid, NT_FWD, FwdCfg<128>::SMEM, st>>>(tm, tm, p);
+    if (!once) { rc = set_smem(flash_fwd_kernel<128, 2>, FwdCfg<128>::SMEM); if (rc) return rc; once = true; }
+    flash_fwd_kernel<128, 2><<<grid, NT_FWD, FwdCfg<128>::SMEM, st>>>(tm, tm, p);
   }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) MOBIUS_FAIL(MOBIUS_ECUDA, "flash_fwd launch: %s", cudaGetErrorString(e));

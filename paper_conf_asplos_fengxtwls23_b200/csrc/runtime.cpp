@@ -324,8 +324,11 @@ struct mobius_ctx {
   std::thread upd_thread;
   std::mutex upd_mu;
   std::condition_variable upd_cv, upd_done_cv;
-  std::deque<int> upd_queue;
+  std::deque<std::pair<int, int64_t>> upd_queue;  // (local stage, AdamW step number)
   int upd_pending = 0;
+  std::vector<int64_t> upd_done;  // per local stage: AdamW step of its last finished host update
+  int64_t upd_wait_ns = 0;        // host time the issue path spent waiting for updates this step
+  bool sync_update = false;       // MOBIUS_SYNC_UPDATE at create: wait for every update inside the step
   bool upd_stop = false;
   int64_t upd_ns = 0;
   int64_t last_bwd_host_ns = 0, last_update_end_ns = 0;
@@ -459,18 +462,19 @@ int64_t layer_numel(const mobius_model_cfg& c, int i) {
 void update_worker(mobius_ctx* ctx) {
   for (;;) {
     int ls;
+    int64_t step;
     {
       std::unique_lock<std::mutex> lk(ctx->upd_mu);
       ctx->upd_cv.wait(lk, [&] { return ctx->upd_stop || !ctx->upd_queue.empty(); });
       if (ctx->upd_stop && ctx->upd_queue.empty()) return;
-      ls = ctx->upd_queue.front();
+      ls = ctx->upd_queue.front().first;
+      step = ctx->upd_queue.front().second;
       ctx->upd_queue.pop_front();
     }
     cudaEventSynchronize(ctx->ev_d2h[ls]);
     int64_t t0 = now_ns();
     const StageDesc& st = ctx->all[ctx->mine[ls]];
-    AdamWArgs a{ctx->cfg.lr, ctx->cfg.beta1, ctx->cfg.beta2, ctx->cfg.eps, ctx->cfg.weight_decay,
-                ctx->step_count + 1};
+    AdamWArgs a{ctx->cfg.lr, ctx->cfg.beta1, ctx->cfg.beta2, ctx->cfg.eps, ctx->cfg.weight_decay, step};
     const int kind = ctx->cfg.dtype == MOBIUS_F32 ? 1 : 0;
     adamw_update(ctx->h_master[ls], ctx->h_m[ls], ctx->h_v[ls], ctx->h_grads[ls], kind, ctx->h_weights[ls], kind,
                  st.n_params, a, *ctx->pool);
@@ -479,9 +483,30 @@ void update_worker(mobius_ctx* ctx) {
       std::lock_guard<std::mutex> g(ctx->upd_mu);
       ctx->upd_ns += t1 - t0;
       ctx->last_update_end_ns = t1;
-      if (--ctx->upd_pending == 0) ctx->upd_done_cv.notify_all();
+      ctx->upd_done[ls] = step;
+      --ctx->upd_pending;
     }
+    ctx->upd_done_cv.notify_all();
   }
+}
+
+// Synchronous update across steps: stage ls's host AdamW of
+// step `need` must have finished before its weights are swapped in again or
+// its gradient landing buffer is overwritten.  Blocks the issuing thread
+// only; the GPU keeps running what was issued before.
+void wait_update(mobius_ctx* ctx, int ls, int64_t need) {
+  if (need <= 0) return;
+  std::unique_lock<std::mutex> lk(ctx->upd_mu);
+  if (ctx->upd_done[ls] >= need) return;
+  const int64_t t0 = now_ns();
+  ctx->upd_done_cv.wait(lk, [&] { return ctx->upd_done[ls] >= need || ctx->upd_stop; });
+  ctx->upd_wait_ns += now_ns() - t0;
+}
+
+// every queued host update finished (the readers and destroy see them)
+void drain_updates(mobius_ctx* ctx) {
+  std::unique_lock<std::mutex> lk(ctx->upd_mu);
+  ctx->upd_done_cv.wait(lk, [&] { return ctx->upd_pending == 0; });
 }
 
 void fill_seeded_serial(float* dst, int64_t n, uint64_t seed, int64_t stream_off, float std_) {
@@ -661,6 +686,7 @@ struct StepRunner {
     uint8_t* dst = ctx->ring + L.base + L.wofs + b0;
     // device tail update: local stage 0's weights already live in HBM
     const bool d2d = ctx->tail_resident && L.stage_local == 0;
+    if (!d2d) wait_update(ctx, L.stage_local, ctx->step_count);  // the previous step's update of this stage landed
     const uint8_t* src = d2d ? ctx->d_wstage + b0 : (const uint8_t*)ctx->h_weights[L.stage_local] + b0;
     cudaEvent_t a = ctx->ev_part_a[n_parts], b = ctx->ev_part_b[n_parts];
     CU(cudaEventRecord(a, ctx->s_h2d));
@@ -940,6 +966,7 @@ struct StepRunner {
     CU(cudaStreamWaitEvent(ctx->s_d2h, ctx->ev_gready[ls], 0));
     CU(cudaEventRecord(ctx->ev_off_a[ls], ctx->s_d2h));
     if (!dev_upd) {  // the device-updated stage's weights stay in HBM (d_wstage): nothing crosses the link
+      wait_update(ctx, ls, ctx->step_count);  // the previous step's update has read h_grads[ls]
       CU(cudaMemcpyAsync(ctx->h_grads[ls], ctx->grad_stage, st.n_params * sizeof(T), cudaMemcpyDeviceToHost,
                          ctx->s_d2h));
       ctx->stats.d2h_bytes += st.n_params * sizeof(T);
@@ -949,7 +976,7 @@ struct StepRunner {
     if (dev_upd) return MOBIUS_OK;
     {
       std::lock_guard<std::mutex> g(ctx->upd_mu);
-      ctx->upd_queue.push_back(ls);
+      ctx->upd_queue.push_back({ls, ctx->step_count + 1});
       ++ctx->upd_pending;
     }
     ctx->upd_cv.notify_one();
@@ -1133,10 +1160,12 @@ int do_step(mobius_ctx* ctx, const int32_t* tok_dev, int M, float* loss_out) {
   CU(cudaStreamSynchronize(ctx->s_d2h));
   if (ctx->s_p2p) CU(cudaStreamSynchronize(ctx->s_p2p));
   int64_t t_gpu_done = now_ns();
-  {  // synchronous update: every stage's AdamW has landed
-    std::unique_lock<std::mutex> lk(ctx->upd_mu);
-    ctx->upd_done_cv.wait(lk, [&] { return ctx->upd_pending == 0; });
-  }
+  // The host updates of the stages still in the queue finish while the next
+  // step's earlier stages run: every consumer of a stage's new weights (its
+  // next swap-in, read_params, destroy) waits for that stage's update, so
+  // each step still sees the previous step's parameters.
+  // MOBIUS_SYNC_UPDATE=1: wait for all of them here (round-1 behaviour).
+  if (ctx->sync_update) drain_updates(ctx);
   int64_t t1 = now_ns();
   const bool has_last = ctx->all.back().owner == ctx->dist.rank;
   *loss_out = has_last ? (float)(*ctx->h_loss * R.inv_ntok) : NAN;
@@ -1204,7 +1233,8 @@ int do_step(mobius_ctx* ctx, const int32_t* tok_dev, int M, float* loss_out) {
   }
   S.pinned_bytes = pinned;
   S.host_update_ns = ctx->upd_ns;
-  S.update_tail_ns = t1 - t_gpu_done;
+  S.update_tail_ns = t1 - t_gpu_done + ctx->upd_wait_ns;  // exposed waiting for host updates (here or at issue)
+  ctx->upd_wait_ns = 0;
   S.n_local_stages = (int)ctx->mine.size();
   S.recompute = 0;
   for (int ls = 0; ls < (int)ctx->mine.size(); ++ls)
@@ -1569,6 +1599,8 @@ extern "C" int mobius_create(const mobius_model_cfg* cfg, const mobius_plan_t* p
     ctx->pool.reset(new ThreadPool(nthreads));
     ctx->h_weights.resize(n);
     ctx->h_grads.resize(n);
+    ctx->upd_done.assign(n, 0);
+    ctx->sync_update = getenv("MOBIUS_SYNC_UPDATE") != nullptr;
     ctx->h_master.resize(n);
     ctx->h_m.resize(n);
     ctx->h_v.resize(n);
@@ -1865,6 +1897,7 @@ extern "C" int mobius_step_device(mobius_ctx* ctx, const int32_t* tokens_dev, in
 extern "C" int mobius_read_grads(mobius_ctx* ctx, float* out, size_t n) {
   int rc = check_ctx(ctx);
   if (rc) return rc;
+  drain_updates(ctx);  // the landing buffers are stable once their updates have read them
   MOBIUS_CHECK_ARG(out, "null out");
   for (int ls = 0; ls < (int)ctx->mine.size(); ++ls) {
     const StageDesc& st = ctx->all[ctx->mine[ls]];
@@ -1890,6 +1923,7 @@ extern "C" int mobius_read_grads(mobius_ctx* ctx, float* out, size_t n) {
 extern "C" int mobius_read_params(mobius_ctx* ctx, float* out, size_t n) {
   int rc = check_ctx(ctx);
   if (rc) return rc;
+  drain_updates(ctx);
   MOBIUS_CHECK_ARG(out, "null out");
   for (int ls = 0; ls < (int)ctx->mine.size(); ++ls) {
     const StageDesc& st = ctx->all[ctx->mine[ls]];

@@ -577,3 +577,38 @@ def test_arena_cap_repeated_steps_tight_ring(sizes):
         g = ctx.read_grads(c.n_params)
         ctx.close()
         assert max(tensor_errs(c, g, ref_g).values()) < 2e-2
+
+
+@pytest.mark.parametrize("dtype", [F32, BF16])
+@pytest.mark.parametrize("flags_name", ["host", "device_tail"])
+def test_deferred_host_update_matches_synchronous(dtype, flags_name, monkeypatch):
+    """mobius_step returns when its GPU work is done and the remaining host
+    AdamW updates overlap the next step's first stages; each stage's next
+    swap-in waits for its own update (P:L596-602 synchronous update).  Four
+    steps give the same loss curve and parameters as waiting for every
+    update inside the step (MOBIUS_SYNC_UPDATE=1) - bitwise on fp32."""
+    c = synth.TINY
+    M = 2
+    flags = FLAG_DEVICE_TAIL_UPDATE if flags_name == "device_tail" else 0
+    w = synth.perturb_norm_params(c, synth.gen_params(c), scale=0.1)
+    if dtype == BF16:
+        w = synth.round_bf16(w)
+    cap = 4 * MiB if dtype == BF16 else 8 * MiB
+    toks = [synth.gen_tokens(c, M, seed=60 + i) for i in range(4)]
+    runs = []
+    for sync in (False, True):
+        if sync:
+            monkeypatch.setenv("MOBIUS_SYNC_UPDATE", "1")
+        else:
+            monkeypatch.delenv("MOBIUS_SYNC_UPDATE", raising=False)
+        ctx = MobiusContext(mk_cfg(c, dtype), plan_from_sizes((1, 2, 1, 2), 1, M, hbm_cap_bytes=cap), init_params=w,
+                            flags=flags)
+        losses = [ctx.step(t) for t in toks]
+        p = ctx.read_params(c.n_params)
+        ctx.close()
+        runs.append((np.array(losses), p))
+    (la, pa), (lb, pb) = runs
+    if dtype == F32:
+        assert np.array_equal(la, lb) and np.array_equal(pa, pb)
+    else:
+        assert np.all(np.abs(la - lb) <= 1e-3 * np.abs(lb)) and rel(pa - w, pb - w) < 1e-2
