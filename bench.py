@@ -139,6 +139,34 @@ def model_flops_per_token(c: synth.GPTConfig) -> float:
 
 
 # --------------------------------------------------------------- reference
+def host_cpu_info():
+    """CPU model and the BLAS numpy links (printed with the oracle timing)."""
+    model = "unknown"
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    blas = "unknown"
+    try:
+        import io
+        import contextlib
+        buf = io.StringIO()
+        with contextlib.redirect_stdout(buf):
+            np.show_config()
+        txt = buf.getvalue().lower()
+        for name in ("openblas", "mkl", "blis", "accelerate"):
+            if name in txt:
+                blas = name
+                break
+    except Exception:
+        pass
+    return model, blas
+
+
 def cpu_oracle_sample(c: synth.GPTConfig, tokens_per_step: int, budget_s: float = 20.0):
     """Time the oracle (numpy fp32) on one block fwd+bwd and the head at
     mbs=1, extrapolate to tokens/s:  T_step ~ (L t_block + t_head + t_embed)
@@ -170,7 +198,9 @@ def cpu_oracle_sample(c: synth.GPTConfig, tokens_per_step: int, budget_s: float 
             break
     t_block, t_head = float(np.median(tb)), float(np.median(th))
     t_step = (c.n_layers * t_block + t_head) * tokens_per_step / s
+    cpu_model, blas = host_cpu_info()
     return {"value": tokens_per_step / t_step, "unit": "tokens/s", "cores": cores, "kind": "oracle",
+            "cpu_model": cpu_model, "blas": blas,
             "sample": f"numpy fp32 oracle: {len(tb)} x (1 block fwd+bwd, median {t_block:.2f}s + LM head fwd+bwd, "
                       f"median {t_head:.2f}s) at mbs=1 s={s} h={h} V={V} (~{budget_s:.0f}s of CPU work), "
                       f"extrapolated x{c.n_layers} blocks to the step's {tokens_per_step} tokens "
@@ -417,6 +447,8 @@ def run_mobius(args, rank, world, local):
         traffic = float(np.mean([t["dram_bytes"] for t in tr]))
         traffic_alg = float(np.mean([t["algorithmic_bytes"] for t in tr]))
         tr_n = len(tr)
+    # model GEMM FLOPs per step (no recompute): L (72 h^2) per token fwd+bwd + the LM head 6 h V
+    model_gemm_flop_step = (c.n_layers * 72 * c.hidden ** 2 + 6 * c.hidden * c.vocab) * tokens_per_step / world
     # step roofline (north_star): max(FLOP / P_tc, H2D bytes / host link), per GPU
     flop_step = model_flops_per_token(c) * tokens_per_step / world
     t_tc = flop_step / (peak_tf * 1e12)
@@ -455,7 +487,11 @@ def run_mobius(args, rank, world, local):
                          "traffic_source": f"profiles/{tr_name}: dram__bytes_read+write per launch, mean over the "
                                            f"{tr_n} captured 1.5B block GEMM shapes at T={c.micro_batch * c.seq_len} "
                                            "(ncu --set full, cold L2; tools/gemm_prof.py + tools/gemm_traffic.py)",
-                         "peak_source": f"MEASURED_PEAKS.json bf16_tflops_sustained ({peak_src})"},
+                         "peak_source": f"MEASURED_PEAKS.json bf16_tflops_sustained ({peak_src})",
+                         "flops_counted": "2MNK of every sampled GEMM launch, including the launches of the "
+                                          "recomputed blocks (launches of the same kernel)",
+                         "frac_model_flops": (model_gemm_flop_step / (avg("gemm_ns") * 1e-9) / 1e12 / peak_tf
+                                              if avg("gemm_ns") and peak_tf else None)},
             "step_roofline": {"t_tensor_ms": t_tc * 1e3, "t_link_ms": t_link * 1e3, "t_roofline_ms": t_roof * 1e3,
                               "frac": t_roof / (ms * 1e-3), "h2d_GBps_link": h2d_gbps,
                               "note": "north_star step roofline = max(algorithmic FLOPs / tensor peak, stage bytes / "
