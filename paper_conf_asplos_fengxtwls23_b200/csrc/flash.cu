@@ -638,8 +638,8 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
 // dQ(i), then [S^T, dP^T](i+1) right away (the softmax-gradient warps are
 // done with S^T(i)), so the next scores overlap the dQ read-out.
 
-template <int DH>
-__global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_constant__ CUtensorMap tm,
+template <int DH, int CP>
+__global__ void __launch_bounds__((2 + 4 * CP) * 32, 1) flash_bwd_kernel(const __grid_constant__ CUtensorMap tm,
                                                               const __grid_constant__ CUtensorMap tdo,
                                                               const __grid_constant__ CUtensorMap tdq,
                                                               const __grid_constant__ CUtensorMap tdkv, const BwdParams p) {
@@ -696,13 +696,13 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
       ptx::mbar_init(&q_empty[i], 1);
     }
     ptx::mbar_init(s_full, 1);
-    ptx::mbar_init(p_full, 8);
+    ptx::mbar_init(p_full, 4 * CP);
     ptx::mbar_init(mm_done, 1);
-    ptx::mbar_init(dq_empty, 8);
-    ptx::mbar_init(st_empty, 8);
+    ptx::mbar_init(dq_empty, 4 * CP);
+    ptx::mbar_init(st_empty, 4 * CP);
     ptx::mbar_init(pt_free, 1);
     ptx::mbar_init(kv_empty, 1);
-    ptx::mbar_init(acc_empty, 8);
+    ptx::mbar_init(acc_empty, 4 * CP);
     ptx::fence_mbar_init();
   }
   if (warp == 1) ptx::tmem_alloc<512>(tmem_slot);
@@ -857,10 +857,12 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
     }
   } else {
     // ---------------------------------------- softmax-gradient warps
-    // 8 warps: (lane quadrant q4, column half hf); thread = key row r,
-    // query columns [64 hf, 64 hf + 64)
+    // 4 CP warps: (lane quadrant q4, column part cq); thread = key row r,
+    // query columns [QC cq, QC cq + QC); dQ columns [DC cq, DC cq + DC)
+    constexpr int NSW = 4 * CP, QC = 128 / CP, NG = QC / 32, DC = DH / CP;
+    static_assert(CP == 2 || (DH == 64 && CP == 4), "CP 4 only at dh 64");
     const int q4 = warp & 3;
-    const int hf = (warp - 2) >> 2;
+    const int cq = (warp - 2) >> 2;
     const int r = q4 * 32 + lane;  // key row of this thread (TMEM lane)
     const uint32_t lane_base = (uint32_t)(q4 * 32) << 16;
     const uint32_t spt = ptx::smem_u32(sPT);
@@ -872,13 +874,28 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
     // the bulk copy has long finished reading it - so no warp stalls on it.
     auto stage_free = [&]() {
       if (warp == 2 && lane == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
-      named_bar(1, 256);
+      named_bar(1, 32 * NSW);
     };
     auto dq_drain = [&](int qiq, int hd, int b, uint32_t stg) {
-      uint32_t v[DH / 64][32];
+      if constexpr (DC == 16) {  // a quarter of a 32-column slab: chunks (cq % 2) * 4 .. +3 of slab cq / 2
+        uint32_t v[16];
+        __syncwarp();
+        ptx::tmem_ld16(T_DQ + cq * 16 + lane_base, v);
+        ptx::tmem_ld_wait();
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(dq_empty);  // dQ TMEM may be overwritten
+        stage_free();
+        const int c = cq >> 1;
 #pragma unroll
-      for (int cc = 0; cc < DH / 64; ++cc) {
-        const int c = hf * (DH / 64) + cc;  // 32-column slab
+        for (int k = 0; k < 4; ++k)
+          st_shared_v4(stg + c * 16384 + r * 128 + ((((cq & 1) * 4 + k) ^ (r & 7)) << 4), v[4 * k], v[4 * k + 1],
+                       v[4 * k + 2], v[4 * k + 3]);
+      } else {
+      uint32_t v[DC / 32][32];
+#pragma unroll
+      for (int cc = 0; cc < DC / 32; ++cc) {
+        const int c = cq * (DC / 32) + cc;  // 32-column slab
         __syncwarp();
         ptx::tmem_ld32(T_DQ + c * 32 + lane_base, v[cc]);
       }
@@ -888,15 +905,16 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
       if (lane == 0) ptx::mbar_arrive(dq_empty);  // dQ TMEM may be overwritten
       if (C::DQ_OWN) stage_free();                 // dh 128: done before the P^T / dS^T writes
 #pragma unroll
-      for (int cc = 0; cc < DH / 64; ++cc) {
-        const int c = hf * (DH / 64) + cc;
+      for (int cc = 0; cc < DC / 32; ++cc) {
+        const int c = cq * (DC / 32) + cc;
 #pragma unroll
         for (int k = 0; k < 8; ++k)
           st_shared_v4(stg + c * 16384 + r * 128 + ((k ^ (r & 7)) << 4), v[cc][4 * k], v[cc][4 * k + 1],
                        v[cc][4 * k + 2], v[cc][4 * k + 3]);
       }
+      }
       ptx::fence_proxy_async();
-      named_bar(1, 256);
+      named_bar(1, 32 * NSW);
       if (warp == 2 && lane == 0) {
 #pragma unroll
         for (int c = 0; c < DH / 32; ++c)
@@ -922,12 +940,13 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
         ptx::mbar_wait(&q_full[st], (gg / QS) & 1);  // lse / D of this query tile in smem
         ptx::mbar_wait(s_full, gg & 1);
         ptx::tc_fence_after();
-        uint32_t vs[2][32], vd[2][32];
+        uint32_t vs[NG][32], vd[NG][32];
         __syncwarp();
-        ptx::tmem_ld32(T_S + hf * 64 + lane_base, vs[0]);
-        ptx::tmem_ld32(T_S + hf * 64 + 32 + lane_base, vs[1]);
-        ptx::tmem_ld32(T_DP + hf * 64 + lane_base, vd[0]);
-        ptx::tmem_ld32(T_DP + hf * 64 + 32 + lane_base, vd[1]);
+#pragma unroll
+        for (int cc = 0; cc < NG; ++cc) {
+          ptx::tmem_ld32(T_S + cq * QC + cc * 32 + lane_base, vs[cc]);
+          ptx::tmem_ld32(T_DP + cq * QC + cc * 32 + lane_base, vd[cc]);
+        }
         ptx::tmem_ld_wait();
         ptx::tc_fence_before();
         __syncwarp();
@@ -950,8 +969,8 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
         if (C::DQ_OWN && it == 0 && gg >= 1) stage_free();  // previous item's dV/dK stores read the P^T / dS^T tiles
         const uint32_t sds = ptx::smem_u32(sdS_buf[C::PT_TMEM ? (gg & 1) : 0]);
 #pragma unroll
-        for (int cc = 0; cc < 2; ++cc) {
-          const int c = hf * 2 + cc;
+        for (int cc = 0; cc < NG; ++cc) {
+          const int c = cq * NG + cc;  // 32-query slab
           uint32_t ppk[16], dpk[16];
           const uint32_t aL = ptx::smem_u32(sLD + st * 256 + c * 32);
           if (diag)
@@ -1004,20 +1023,25 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
       // TMA stores per tensor atom (row-per-thread global stores are 64 B
       // pieces 3h apart); the next item's first P^T / dS^T write waits for
       // the stores' smem reads (stage_free)
-      const uint32_t stg = ptx::smem_u32(sPT) + hf * (DH / 64) * 16384;
+      // warp (q4, cq): tensor tv = cq / (CP/2) (0 dV, 1 dK), its 32-column chunks
+      // [(cq % (CP/2)) * NCH, + NCH) of the DH / 32
+      constexpr int HP = CP / 2, NCH = DH / 32 / HP;
+      const int tv = cq / HP, ch0 = (cq % HP) * NCH;
+      const uint32_t stg = ptx::smem_u32(sPT) + tv * (DH / 64) * 16384;
 #pragma unroll
-      for (int c = 0; c < DH / 32; ++c) {
+      for (int ci = 0; ci < NCH; ++ci) {
+        const int c = ch0 + ci;
         uint32_t v[32];
         __syncwarp();
-        ptx::tmem_ld32(T_DV + hf * DH + c * 32 + lane_base, v);
+        ptx::tmem_ld32(T_DV + tv * DH + c * 32 + lane_base, v);
         ptx::tmem_ld_wait();
-        if (c == DH / 32 - 1) {  // last TMEM read of this item's accumulators
+        if (ci == NCH - 1) {  // last TMEM read of this item's accumulators by this warp
           ptx::tc_fence_before();
           __syncwarp();
           if (lane == 0) ptx::mbar_arrive(acc_empty);
         }
         uint32_t pk[16];
-        const float f = hf == 0 ? 1.f : p.scale;  // dK = scale * sum dS^T Q (dS^T was stored unscaled)
+        const float f = tv == 0 ? 1.f : p.scale;  // dK = scale * sum dS^T Q (dS^T was stored unscaled)
 #pragma unroll
         for (int e = 0; e < 32; e += 2)
           pk[e / 2] = pack_bf16x2(__fmul2_rn(make_float2(__uint_as_float(v[e]), __uint_as_float(v[e + 1])), make_float2(f, f)));
@@ -1026,7 +1050,7 @@ __global__ void __launch_bounds__(NT_FWD, 1) flash_bwd_kernel(const __grid_const
           st_shared_v4(stg + sw128_off(r, c * 4 + k), pk[4 * k], pk[4 * k + 1], pk[4 * k + 2], pk[4 * k + 3]);
       }
       ptx::fence_proxy_async();
-      named_bar(1, 256);
+      named_bar(1, 32 * NSW);
       if (warp == 2 && lane == 0) {
 #pragma unroll
         for (int t = 0; t < 2; ++t)
@@ -1274,12 +1298,24 @@ int flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* o, const __nv_
   dim3 grid(n_items < sms ? n_items : sms);  // persistent
   if (dh == 64) {
     static bool once = false;
-    if (!once) { rc = set_smem(flash_bwd_kernel<64>, BwdCfg<64>::SMEM); if (rc) return rc; once = true; }
-    flash_bwd_kernel<64><<<grid, NT_FWD, BwdCfg<64>::SMEM, st>>>(tm, tdo, tdq, tdkv, p);
+    // MOBIUS_FLASH_BWD_CP: softmax-gradient warps per key row (2: 8 warps of 64 queries, 4: 16 of 32)
+    static int cp = -1;
+    if (cp < 0) {
+      const char* e = getenv("MOBIUS_FLASH_BWD_CP");
+      cp = (e && atoi(e) == 4) ? 4 : 2;
+    }
+    if (cp == 4) {
+      static bool once4 = false;
+      if (!once4) { rc = set_smem(flash_bwd_kernel<64, 4>, BwdCfg<64>::SMEM); if (rc) return rc; once4 = true; }
+      flash_bwd_kernel<64, 4><<<grid, (2 + 16) * 32, BwdCfg<64>::SMEM, st>>>(tm, tdo, tdq, tdkv, p);
+    } else {
+      if (!once) { rc = set_smem(flash_bwd_kernel<64, 2>, BwdCfg<64>::SMEM); if (rc) return rc; once = true; }
+      flash_bwd_kernel<64, 2><<<grid, NT_FWD, BwdCfg<64>::SMEM, st>>>(tm, tdo, tdq, tdkv, p);
+    }
   } else {
     static bool once = false;
-    if (!once) { rc = set_smem(flash_bwd_kernel<128>, BwdCfg<128>::SMEM); if (rc) return rc; once = true; }
-    flash_bwd_kernel<128><<<grid, NT_FWD, BwdCfg<128>::SMEM, st>>>(tm, tdo, tdq, tdkv, p);
+    if (!once) { rc = set_smem(flash_bwd_kernel<128, 2>, BwdCfg<128>::SMEM); if (rc) return rc; once = true; }
+    flash_bwd_kernel<128, 2><<<grid, NT_FWD, BwdCfg<128>::SMEM, st>>>(tm, tdo, tdq, tdkv, p);
   }
   {
     const int64_t n = rows * h / 4;
