@@ -491,12 +491,17 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1)
               if (cbase + gi * 32 + e > row) v[gi][e] = __float_as_uint(-INFINITY);
         }
         // pass A: part-row max of raw scores, combined across the CP warps of the row
-        float mx = -INFINITY;
+        float mx;
+        {  // four independent max chains (one serial chain was 32 dependent FMNMX3)
+          float m4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
 #pragma unroll
-        for (int gi = 0; gi < NG; ++gi)
+          for (int gi = 0; gi < NG; ++gi)
 #pragma unroll
-          for (int e = 0; e < 32; e += 2)
-            mx = fmaxf(mx, fmaxf(__uint_as_float(v[gi][e]), __uint_as_float(v[gi][e + 1])));
+            for (int e = 0; e < 32; e += 2)
+              m4[(e >> 1) & 3] =
+                  fmaxf(m4[(e >> 1) & 3], fmaxf(__uint_as_float(v[gi][e]), __uint_as_float(v[gi][e + 1])));
+          mx = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3]));
+        }
         float* smx = sMax + (g & 1) * (CP * 128);
         sts_f32(ptx::smem_u32(smx + cq * 128 + row), mx);
         named_bar(2 + q4, 32 * CP);
@@ -536,15 +541,22 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1)
         if (g >= 2) ptx::mbar_wait(&pv_done[sb], ((g - 2) >> 1) & 1);
         // pass B: P = 2^(x*sc - m_new) -> TMEM / smem (bf16), part-row sum
         const uint32_t sp = ptx::smem_u32(sP + sb * C::P_BYTES);
-        float rs = 0.f;
+        // packed f32x2 scale-subtract and two interleaved f32x2 row-sum
+        // accumulators (a scalar sum was one 64-long dependent FADD chain)
+        float2 rsa = make_float2(0.f, 0.f), rsb = make_float2(0.f, 0.f);
+        const float2 sc2 = make_float2(sc, sc), nm2 = make_float2(-m_new, -m_new);
 #pragma unroll
         for (int gi = 0; gi < NG; ++gi) {
           uint32_t pk[16];
 #pragma unroll
           for (int e = 0; e < 32; e += 2) {
-            const float2 pp = ex2_pair(fmaf(__uint_as_float(v[gi][e]), sc, -m_new),
-                                       fmaf(__uint_as_float(v[gi][e + 1]), sc, -m_new), (e >> 1) + gi * 8);
-            rs += pp.x + pp.y;
+            const float2 xx =
+                __ffma2_rn(make_float2(__uint_as_float(v[gi][e]), __uint_as_float(v[gi][e + 1])), sc2, nm2);
+            const float2 pp = ex2_pair(xx.x, xx.y, (e >> 1) + gi * 8);
+            if ((e >> 1) & 1)
+              rsb = __fadd2_rn(rsb, pp);
+            else
+              rsa = __fadd2_rn(rsa, pp);
             pk[e >> 1] = pack_bf16(pp.x, pp.y);
           }
           if constexpr (C::P_TMEM) {  // keys cq*SC + gi*32 .. -> packed columns cq*SC/2 + gi*16 ..
@@ -557,10 +569,11 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1)
           }
         }
         if constexpr (C::P_TMEM) ptx::tmem_st_wait();
+        const float rs = (rsa.x + rsa.y) + (rsb.x + rsb.y);
         l_run = l_run * alpha + rs;
         m_run = m_new;
         ptx::tc_fence_before();
-        ptx::fence_proxy_async();
+        if constexpr (!C::P_TMEM) ptx::fence_proxy_async();  // P in smem feeds the PV MMA
         __syncwarp();
         if (lane == 0) ptx::mbar_arrive(&p_full[sb]);
         if (j == 0) store_o();  // previous item's O while this tile's PV runs

@@ -37,6 +37,18 @@ __device__ __forceinline__ void tma_store_2d(const CUtensorMap* m, uint32_t src,
                "r"(src), "r"(c0), "r"(c1), "r"(0), "r"(0)
                : "memory");
 }
+// TMA store with an L2 evict-first policy: for outputs not read again soon
+// (the GeLU pre-activation u is read only by the backward), so they do not
+// push this GEMM's operand tiles out of L2 (fc1 fwd: 526 -> 521 us at T = 32768)
+__device__ __forceinline__ void tma_store_2d_evict_first(const CUtensorMap* m, uint32_t src, int c0, int c1) {
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+  asm volatile(
+      "cp.async.bulk.tensor.4d.global.shared::cta.bulk_group.L2::cache_hint [%0, {%2, %3, %4, %5}], [%1], %6;" ::"l"(
+          reinterpret_cast<uint64_t>(m)),
+      "r"(src), "r"(c0), "r"(c1), "r"(0), "r"(0), "l"(pol)
+      : "memory");
+}
 __device__ __forceinline__ void tma_reduce_add_2d(const CUtensorMap* m, uint32_t src, int c0, int c1) {
   asm volatile(
       "cp.reduce.async.bulk.tensor.4d.global.shared::cta.add.tile.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
@@ -199,7 +211,7 @@ __device__ __forceinline__ void epi_tma(const Params& p, const EpiMaps& mp, uint
         ptx::fence_proxy_async();
         __syncwarp();
         if (lane == 0) {
-          tma_store_2d(mp.X, stg, n0, m0w);
+          tma_store_2d_evict_first(mp.X, stg, n0, m0w);
           tma_store_2d(mp.C, stg + 4096, n0, m0w);
           bulk_commit();
         }

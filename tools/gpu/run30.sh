@@ -1,0 +1,6 @@
+export MOBIUS_KT_NOSYNC=1
+for i in 1 2; do
+python tools/gemm_epi_ab.py 32768 6400 1600 0 2 4
+python tools/gemm_epi_ab.py 32768 1600 1600 3
+for v in MOBIUS_EPI_HINT1 MOBIUS_EPI_HINT2; do echo $v; MOBIUS_LIB_PATH=tools/gpu/var/libmobius_$v.so python tools/gemm_epi_ab.py 32768 6400 1600 0 2 4; MOBIUS_LIB_PATH=tools/gpu/var/libmobius_$v.so python tools/gemm_epi_ab.py 32768 1600 1600 3; done
+done
