@@ -106,6 +106,15 @@ __device__ __forceinline__ float2 ex2_poly2(float2 x0) {
   return make_float2(x0.x < -125.f ? 0.f : __int_as_float(__float_as_int(q.x) + (__float_as_int(j.x) << 23)),
                      x0.y < -125.f ? 0.f : __int_as_float(__float_as_int(q.y) + (__float_as_int(j.y) << 23)));
 }
+#ifdef MOBIUS_BWD_PROF  // debug: per-phase clock64 totals of one CTA's MMA / softmax-gradient warps (printf)
+#define BPROF_DECL long long bprof[8] = {0, 0, 0, 0, 0, 0, 0, 0}; long long bprof_t0 = clock64();
+#define BPROF(k, ...) do { long long t0_ = clock64(); __VA_ARGS__; bprof[k] += clock64() - t0_; } while (0)
+#define BPROF_DUMP(tag) if ((blockIdx.x == 0 || blockIdx.x == 77) && lane == 0) printf("%s blk %d warp %d total %lld: %lld %lld %lld %lld %lld %lld %lld %lld\n", tag, blockIdx.x, warp, clock64() - bprof_t0, bprof[0], bprof[1], bprof[2], bprof[3], bprof[4], bprof[5], bprof[6], bprof[7]);
+#else
+#define BPROF_DECL
+#define BPROF(k, ...) __VA_ARGS__
+#define BPROF_DUMP(tag)
+#endif
 #ifndef MOBIUS_FLASH_POLY_PAIRS
 #define MOBIUS_FLASH_POLY_PAIRS 2  // of every 16 pairs of scores, this many use ex2_poly2 (forward)
 #endif
@@ -115,6 +124,8 @@ __device__ __forceinline__ float2 ex2_pair(float a, float b, int pair) {
   return make_float2(ex2(a), ex2(b));
 }
 
+// (Polynomial exp2 for part of the backward's P^T was measured slower: 2 / 4 /
+// 6 of 16 pairs: 672 / 740 / 734 us against 665 us at mbs 32, dh 64.)
 // Softmax-gradient math of one 32-query slab of a key row (flash bwd):
 //   P^T[r, q]  = 2^(S^T[r, q] * c - lse_q)          (masked to q >= r on the diagonal tile)
 //   dS^T[r, q] = P^T[r, q] * (dP^T[r, q] - D_q)      (the 1/sqrt(dh) factor is applied to
@@ -775,10 +786,11 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1) flash_bwd_kernel(const _
       constexpr uint32_t ID_DQ = ptx::idesc_bf16(128, DH, 1, 1);   // dQ
       const uint32_t ak = ptx::smem_u32(sK), av = ptx::smem_u32(sV);
       const uint32_t apt = ptx::smem_u32(sPT), adst = ptx::smem_u32(sdST);
+      BPROF_DECL
       auto issue_st = [&](int gg) {
         const int st = gg % QS, ph = (gg / QS) & 1;
         const uint32_t aq = ptx::smem_u32(sQ + st * C::T_BYTES), ado = ptx::smem_u32(sdO + st * C::T_BYTES);
-        ptx::mbar_wait(&q_full[st], ph);
+        BPROF(5, ptx::mbar_wait(&q_full[st], ph));
         if (!C::DQ_OWN && gg >= 1) ptx::mbar_wait(dq_empty, (gg - 1) & 1);  // S^T region holds dQ(gg-1)
         ptx::tc_fence_after();
 #pragma unroll
@@ -801,7 +813,7 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1) flash_bwd_kernel(const _
         int kt_, hd_, b_;
         decode(item, kt_, hd_, b_);
         const int nq = n_t - kt_;
-        ptx::mbar_wait(kv_full, n & 1);
+        BPROF(0, ptx::mbar_wait(kv_full, n & 1));
         // S^T / dP^T TMEM must have been read (dh 64; dh 128: issue_st waits dq_empty)
         if (C::DQ_OWN && g >= 1) ptx::mbar_wait(st_empty, (g - 1) & 1);
         issue_st(g);
@@ -813,7 +825,7 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1) flash_bwd_kernel(const _
           // (blocking on the load here would stall the whole chain)
           bool st_next = false;
           if (C::DQ_OWN && it + 1 < nq) {
-            ptx::mbar_wait(st_empty, gg & 1);
+            BPROF(1, ptx::mbar_wait(st_empty, gg & 1));
             const int sn = (gg + 1) % QS;
             const bool landed = __shfl_sync(0xffffffffu, (int)ptx::mbar_test(&q_full[sn], ((gg + 1) / QS) & 1), 0);
             if (landed) {  // warp-uniform decision
@@ -821,8 +833,8 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1) flash_bwd_kernel(const _
               st_next = true;
             }
           }
-          ptx::mbar_wait(p_full, gg & 1);
-          if (it == 0 && n >= 1) ptx::mbar_wait(acc_empty, (n - 1) & 1);  // previous item's dV/dK read out
+          BPROF(2, ptx::mbar_wait(p_full, gg & 1));
+          if (it == 0 && n >= 1) BPROF(3, ptx::mbar_wait(acc_empty, (n - 1) & 1));  // previous item's dV/dK read out
           ptx::tc_fence_after();
           if (C::PT_TMEM) {
             const uint32_t ads = ptx::smem_u32(sdS_buf[gg & 1]);
@@ -838,7 +850,7 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1) flash_bwd_kernel(const _
                             ID_DV, (it > 0 || t > 0) ? 1u : 0u);
             }
             ptx::mma_commit_w(&q_empty[st]);  // last reads of Q / dO (dQ needs only dS and K): refill the slot now
-            if (gg >= 1) ptx::mbar_wait(dq_empty, (gg - 1) & 1);  // dQ(gg-1) read out
+            if (gg >= 1) BPROF(4, ptx::mbar_wait(dq_empty, (gg - 1) & 1));  // dQ(gg-1) read out
 #pragma unroll
             for (int t = 0; t < 128 / 16; ++t)  // K = 128 keys: dQ = dS K
               ptx::mma_bf16_w(T_DQ, ptx::sdesc_sw128(ads + t * 2048, 16384, 1024),
@@ -867,6 +879,7 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1) flash_bwd_kernel(const _
         g += nq;
         ++n;
       }
+      BPROF_DUMP("bmma")
     }
   } else {
     // ---------------------------------------- softmax-gradient warps
@@ -940,6 +953,7 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1) flash_bwd_kernel(const _
       }
     };
     int g = 0, n = 0;
+    BPROF_DECL
     for (int pass = 0; pass * ncta < n_items; ++pass) {
       const int item = snake_item(pass, ncta, cta);
       if (item >= n_items) continue;
@@ -947,12 +961,18 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1) flash_bwd_kernel(const _
       decode(item, kt, hd, b);
       const int nq = n_t - kt;
       for (int it = 0; it < nq; ++it) {
+#ifdef MOBIUS_BWD_PROF
+        long long tb = clock64();
+#endif
         const int gg = g + it, st = gg % QS;
         const int qi = kt + it;
         const bool diag = (it == 0);
         ptx::mbar_wait(&q_full[st], (gg / QS) & 1);  // lse / D of this query tile in smem
         ptx::mbar_wait(s_full, gg & 1);
         ptx::tc_fence_after();
+#ifdef MOBIUS_BWD_PROF
+        bprof[0] += clock64() - tb; tb = clock64();
+#endif
         uint32_t vs[NG][32], vd[NG][32];
         __syncwarp();
 #pragma unroll
@@ -964,6 +984,9 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1) flash_bwd_kernel(const _
         ptx::tc_fence_before();
         __syncwarp();
         if (lane == 0) ptx::mbar_arrive(st_empty);  // S^T / dP^T TMEM may be overwritten
+#ifdef MOBIUS_BWD_PROF
+        bprof[1] += clock64() - tb; tb = clock64();
+#endif
         // P^T / dS^T smem must be free: dh 128 - the previous tile's dQ drain
         // (staged there) completed; dh 64 - the previous tile's MMAs completed
         if (C::PT_TMEM) {
@@ -980,6 +1003,9 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1) flash_bwd_kernel(const _
         }
         if (!C::DQ_OWN && gg >= 1) stage_free();  // dQ(gg-1) staged in P^T / dS^T: reduce must have read it
         if (C::DQ_OWN && it == 0 && gg >= 1) stage_free();  // previous item's dV/dK stores read the P^T / dS^T tiles
+#ifdef MOBIUS_BWD_PROF
+        bprof[2] += clock64() - tb; tb = clock64();
+#endif
         const uint32_t sds = ptx::smem_u32(sdS_buf[C::PT_TMEM ? (gg & 1) : 0]);
 #pragma unroll
         for (int cc = 0; cc < NG; ++cc) {
@@ -1009,6 +1035,9 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1) flash_bwd_kernel(const _
         ptx::fence_proxy_async();
         __syncwarp();
         if (lane == 0) ptx::mbar_arrive(p_full);
+#ifdef MOBIUS_BWD_PROF
+        bprof[3] += clock64() - tb; tb = clock64();
+#endif
         if (C::DQ_OWN) {
           // drain dQ of the previous query tile of this item while this tile's MMAs run
           if (it >= 1) {
@@ -1023,7 +1052,13 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1) flash_bwd_kernel(const _
           ptx::tc_fence_after();
           dq_drain(qi, hd, b, spt);  // staged in the (now free) P^T / dS^T tiles
         }
+#ifdef MOBIUS_BWD_PROF
+        bprof[4] += clock64() - tb;
+#endif
       }
+#ifdef MOBIUS_BWD_PROF
+      long long tb2 = clock64();
+#endif
       const int glast = g + nq - 1;
       ptx::mbar_wait(mm_done, glast & 1);
       ptx::tc_fence_after();
@@ -1076,9 +1111,13 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1) flash_bwd_kernel(const _
                          : "memory");
         asm volatile("cp.async.bulk.commit_group;" ::: "memory");
       }
+#ifdef MOBIUS_BWD_PROF
+      bprof[5] += clock64() - tb2;
+#endif
       g += nq;
       ++n;
     }
+    BPROF_DUMP("bsmx")
     if (warp == 2 && lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");  // last dQ reduce
     ptx::tc_fence_before();
   }
