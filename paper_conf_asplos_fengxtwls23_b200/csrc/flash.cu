@@ -640,6 +640,7 @@ struct BwdParams {
   const float* lse;     // [mbs, nh, s] log2 domain
   const float* Dsum;    // [mbs, nh, s] -rowsum(dO * O) (negated)
   float* dQacc;         // [mbs*s, h] fp32 (head view), accumulated by TMA reduce-add
+  __nv_bfloat16* dqkv;  // [mbs*s, 3h] (dh 64 kernel: dK / dV rows stored by the drain warpgroup)
   int s, nh, h, mbs;
   float scale_log2, scale;
   int group;            // (batch, head) pairs per item chunk (chunked_item)
@@ -1128,6 +1129,437 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1) flash_bwd_kernel(const _
   }
 }
 
+// ---------------------------------------------------------------- bwd, dh 64
+// Warp-specialised backward for dh 64 (the 1.5B shape), 16 warps:
+//   warp 0      TMA: K / V of an item into one of two slots (the next
+//               item's K / V land while the current item runs), Q / dO /
+//               lse / -D of each query tile through a 3-deep ring
+//   warp 1      MMA: S^T = K Q^T and dP^T = V dO^T (TMEM), dV += P^T dO
+//               (TS: P^T from TMEM), dK += dS^T Q, dQ = dS K (TMEM); the
+//               scores of the next query tile - also across an item boundary
+//               - are issued as soon as the softmax-gradient warps hold the
+//               current ones in registers
+//   warps 2, 3  idle
+//   warps 4-11  softmax-gradient: thread = key row, 64 query columns;
+//               P^T -> TMEM (hands dV its operand at once), dS^T kept in
+//               registers and written to the single smem dS^T tile once the
+//               previous tile's dK / dQ MMAs have read it
+//   warps 12-15 drain: dQ of each tile (TMEM -> swizzled fp32 staging ->
+//               TMA reduce-add) and dV / dK of each item (TMEM -> bf16 ->
+//               staging -> TMA store), off the softmax warps' path
+// setmaxnreg re-splits the register file per warpgroup: 56 / 176 / 176 / 104.
+struct Bwd64Cfg {
+  static constexpr int T_BYTES = 128 * 64 * 2;  // one K / V / Q / dO tile (16 KB)
+  static constexpr int QS = 3;                  // Q / dO ring depth
+  static constexpr int DS_BYTES = 128 * 128 * 2;
+  static constexpr int NSTG = 3;                  // drain staging ring of 8 KB slots: an fp32 16-column dQ
+  static constexpr int STG_BYTES = NSTG * 8192;   // slab or 64 rows of a bf16 dV / dK tile
+  static constexpr int SMEM = 1024 + 4 * T_BYTES + QS * 2 * T_BYTES + DS_BYTES + STG_BYTES + QS * 1024 + 256;
+};
+
+__global__ void __launch_bounds__(512, 1) flash_bwd64_kernel(const __grid_constant__ CUtensorMap tm,
+                                                          const __grid_constant__ CUtensorMap tdo,
+                                                          const __grid_constant__ CUtensorMap tdq,
+                                                          const __grid_constant__ CUtensorMap tdkv, const BwdParams p) {
+  using C = Bwd64Cfg;
+  constexpr int QS = C::QS, DH = 64;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sK = smem;                         // [2]
+  uint8_t* sV = sK + 2 * C::T_BYTES;          // [2]
+  uint8_t* sQ = sV + 2 * C::T_BYTES;          // [QS]
+  uint8_t* sdO = sQ + QS * C::T_BYTES;        // [QS]
+  uint8_t* sdS = sdO + QS * C::T_BYTES;       // dS^T (keys x queries, K-major SW128 atoms)
+  uint8_t* sSTG = sdS + C::DS_BYTES;          // drain staging
+  float* sLD = reinterpret_cast<float*>(sSTG + C::STG_BYTES);  // [QS][lse 128 | -D 128]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sLD + QS * 256);
+  uint64_t* kv_full = bars;             // [2]
+  uint64_t* kv_empty = bars + 2;        // [2] every MMA of the slot's item done
+  uint64_t* q_full = bars + 4;          // [QS] Q, dO, lse, -D
+  uint64_t* q_empty = bars + 4 + QS;    // [QS]
+  uint64_t* s_full = bars + 4 + 2 * QS;  // S^T and dP^T in TMEM
+  uint64_t* st_empty = s_full + 1;       // S^T / dP^T in registers (count 8)
+  uint64_t* pt_full = s_full + 2;        // P^T in TMEM (count 8)
+  uint64_t* ds_full = s_full + 3;        // dS^T in smem (count 8)
+  uint64_t* pt_free = s_full + 4;        // dV MMAs done: P^T TMEM may be overwritten
+  uint64_t* mm_done = s_full + 5;        // [2] dV/dK/dQ of tile g done ([g & 1])
+  uint64_t* dq_empty = s_full + 7;       // dQ read out of TMEM (count 4)
+  uint64_t* acc_empty = s_full + 8;      // dV / dK of an item read out of TMEM (count 4)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(s_full + 9);
+  auto mm_wait = [&](int t) { ptx::mbar_wait(&mm_done[t & 1], (t >> 1) & 1); };
+
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int n_t = p.s / 128;
+  const int nbh = p.nh * p.mbs;
+  const int n_items = n_t * nbh;
+  const int ncta = (int)gridDim.x, cta = (int)blockIdx.x;
+  auto decode = [&](int item, int& kt, int& hd, int& b) {
+    int r;
+    chunked_item(item, n_t, nbh, p.group, kt, r);
+    hd = r % p.nh;
+    b = r / p.nh;
+  };
+
+  if (threadIdx.x == 0) {
+    ptx::tma_prefetch_desc(&tm);
+    ptx::tma_prefetch_desc(&tdo);
+    ptx::tma_prefetch_desc(&tdq);
+    ptx::tma_prefetch_desc(&tdkv);
+    for (int i = 0; i < 2; ++i) {
+      ptx::mbar_init(&kv_full[i], 1);
+      ptx::mbar_init(&kv_empty[i], 1);
+      ptx::mbar_init(&mm_done[i], 1);
+    }
+    for (int i = 0; i < QS; ++i) {
+      ptx::mbar_init(&q_full[i], 1);
+      ptx::mbar_init(&q_empty[i], 1);
+    }
+    ptx::mbar_init(s_full, 1);
+    ptx::mbar_init(st_empty, 8);
+    ptx::mbar_init(pt_full, 8);
+    ptx::mbar_init(ds_full, 8);
+    ptx::mbar_init(pt_free, 1);
+    ptx::mbar_init(dq_empty, 4);
+    ptx::mbar_init(acc_empty, 4);
+    ptx::fence_mbar_init();
+  }
+  if (warp == 1) ptx::tmem_alloc<512>(tmem_slot);
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  // TMEM: S^T 0..127, dP^T 128..255, dV 256..319, dK 320..383, dQ 384..447, P^T 448..511 (packed bf16)
+
+  if (warp == 0) {
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");
+    if (lane == 0) {
+      int g = 0, n = 0;
+      for (int pass = 0; pass * ncta < n_items; ++pass) {
+        const int item = snake_item(pass, ncta, cta);
+        if (item >= n_items) continue;
+        int kt, hd, b;
+        decode(item, kt, hd, b);
+        const int nq = n_t - kt;
+        const int64_t ld_base = ((int64_t)b * p.nh + hd) * p.s;
+        auto load_q = [&](int it) {
+          const int gg = g + it, st = gg % QS, ph = (gg / QS) & 1, qi = kt + it;
+          ptx::mbar_wait(&q_empty[st], ph ^ 1);
+          ptx::mbar_arrive_expect_tx(&q_full[st], 2 * C::T_BYTES + 1024);
+          ptx::tma_load_4d(sQ + st * C::T_BYTES, &tm, &q_full[st], 0, qi * 128, hd, b);
+          ptx::tma_load_4d(sdO + st * C::T_BYTES, &tdo, &q_full[st], 0, qi * 128, hd, b);
+          bulk_g2s(sLD + st * 256, p.lse + ld_base + qi * 128, 512, &q_full[st]);
+          bulk_g2s(sLD + st * 256 + 128, p.Dsum + ld_base + qi * 128, 512, &q_full[st]);
+        };
+        load_q(0);
+        const int kvs = n & 1;
+        ptx::mbar_wait(&kv_empty[kvs], ((n >> 1) & 1) ^ 1);  // item n - 2 done with the slot
+        ptx::mbar_arrive_expect_tx(&kv_full[kvs], 2 * C::T_BYTES);
+        ptx::tma_load_4d(sK + kvs * C::T_BYTES, &tm, &kv_full[kvs], 0, kt * 128, p.nh + hd, b);
+        ptx::tma_load_4d(sV + kvs * C::T_BYTES, &tm, &kv_full[kvs], 0, kt * 128, 2 * p.nh + hd, b);
+        for (int it = 1; it < nq; ++it) load_q(it);
+        g += nq;
+        ++n;
+      }
+    }
+  } else if (warp == 1) {
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");
+    const uint32_t T_S = __shfl_sync(0xffffffffu, tmem, 0), T_DP = T_S + 128, T_DV = T_S + 256;
+    const uint32_t T_DK = T_S + 320, T_DQ = T_S + 384, T_PT = T_S + 448;
+    constexpr uint32_t ID_ST = ptx::idesc_bf16(128, 128, 0, 0);  // S^T, dP^T
+    constexpr uint32_t ID_DV = ptx::idesc_bf16(128, DH, 0, 1);   // dV, dK
+    constexpr uint32_t ID_DQ = ptx::idesc_bf16(128, DH, 1, 1);   // dQ
+    const uint32_t ads = ptx::smem_u32(sdS);
+    BPROF_DECL
+    auto issue_st = [&](int gg, int kvs) {
+      const int st = gg % QS;
+      const uint32_t aq = ptx::smem_u32(sQ + st * C::T_BYTES), ado = ptx::smem_u32(sdO + st * C::T_BYTES);
+      const uint32_t ak = ptx::smem_u32(sK + kvs * C::T_BYTES), av = ptx::smem_u32(sV + kvs * C::T_BYTES);
+      ptx::tc_fence_after();
+#pragma unroll
+      for (int t = 0; t < DH / 16; ++t)
+        ptx::mma_bf16_w(T_S, ptx::sdesc_sw128(ak + t * 32, 16, 1024), ptx::sdesc_sw128(aq + t * 32, 16, 1024), ID_ST, t > 0);
+#pragma unroll
+      for (int t = 0; t < DH / 16; ++t)
+        ptx::mma_bf16_w(T_DP, ptx::sdesc_sw128(av + t * 32, 16, 1024), ptx::sdesc_sw128(ado + t * 32, 16, 1024), ID_ST,
+                        t > 0);
+      ptx::mma_commit_w(s_full);
+    };
+    auto landed = [&](uint64_t* bar, uint32_t ph) {  // warp-uniform non-blocking test
+      return __shfl_sync(0xffffffffu, (int)ptx::mbar_test(bar, ph), 0) != 0;
+    };
+    int g = 0, n = 0;
+    bool pre = false;  // the current item's first scores were issued during the previous item
+    for (int pass = 0; pass * ncta < n_items; ++pass) {
+      const int item = snake_item(pass, ncta, cta);
+      if (item >= n_items) continue;
+      int kt_, hd_, b_;
+      decode(item, kt_, hd_, b_);
+      const int nq = n_t - kt_, kvs = n & 1;
+      const bool has_next = snake_item(pass + 1, ncta, cta) < n_items;
+      const uint32_t ak = ptx::smem_u32(sK + kvs * C::T_BYTES);
+      if (!pre) {
+        BPROF(0, ptx::mbar_wait(&kv_full[kvs], (n >> 1) & 1));
+        BPROF(5, ptx::mbar_wait(&q_full[g % QS], (g / QS) & 1));
+        if (g >= 1) ptx::mbar_wait(st_empty, (g - 1) & 1);
+        issue_st(g, kvs);
+      }
+      pre = false;
+      for (int it = 0; it < nq; ++it) {
+        const int gg = g + it, st = gg % QS;
+        const uint32_t aq = ptx::smem_u32(sQ + st * C::T_BYTES), ado = ptx::smem_u32(sdO + st * C::T_BYTES);
+        // scores of the next query tile (of this item, or the next item's
+        // first) overlap this tile's softmax gradient if their operands landed
+        BPROF(1, ptx::mbar_wait(st_empty, gg & 1));
+        const int sn = (gg + 1) % QS;
+        const uint32_t qph = ((gg + 1) / QS) & 1;
+        bool next_done = false;
+        if (it + 1 < nq) {
+          if (landed(&q_full[sn], qph)) {
+            issue_st(gg + 1, kvs);
+            next_done = true;
+          }
+        } else if (has_next) {
+          if (landed(&kv_full[kvs ^ 1], ((n + 1) >> 1) & 1) && landed(&q_full[sn], qph)) {
+            issue_st(gg + 1, kvs ^ 1);
+            pre = true;
+          }
+        }
+        BPROF(2, ptx::mbar_wait(pt_full, gg & 1));
+        if (it == 0 && n >= 1) BPROF(3, ptx::mbar_wait(acc_empty, (n - 1) & 1));  // previous item's dV/dK read out
+        ptx::tc_fence_after();
+#pragma unroll
+        for (int t = 0; t < 128 / 16; ++t)  // dV += P^T dO, P^T from TMEM (8 columns per 16 queries)
+          ptx::mma_bf16_ts_w(T_DV, T_PT + 8 * t, ptx::sdesc_sw128(ado + t * 2048, 16384, 1024), ID_DV,
+                             (it > 0 || t > 0) ? 1u : 0u);
+        ptx::mma_commit_w(pt_free);
+        BPROF(6, ptx::mbar_wait(ds_full, gg & 1));
+        ptx::tc_fence_after();
+#pragma unroll
+        for (int t = 0; t < 128 / 16; ++t) {  // dK += dS^T Q
+          const uint32_t offa = (t >> 2) * 16384 + (t & 3) * 32;
+          ptx::mma_bf16_w(T_DK, ptx::sdesc_sw128(ads + offa, 16, 1024), ptx::sdesc_sw128(aq + t * 2048, 16384, 1024),
+                          ID_DV, (it > 0 || t > 0) ? 1u : 0u);
+        }
+        ptx::mma_commit_w(&q_empty[st]);  // last reads of Q / dO / lse / -D
+        if (gg >= 1) BPROF(4, ptx::mbar_wait(dq_empty, (gg - 1) & 1));  // dQ(gg-1) read out
+        ptx::tc_fence_after();
+#pragma unroll
+        for (int t = 0; t < 128 / 16; ++t)  // dQ = dS K (K = 128 keys)
+          ptx::mma_bf16_w(T_DQ, ptx::sdesc_sw128(ads + t * 2048, 16384, 1024), ptx::sdesc_sw128(ak + t * 2048, 16384, 1024),
+                          ID_DQ, t > 0);
+        ptx::mma_commit_w(&mm_done[gg & 1]);
+        if (it + 1 < nq && !next_done) {
+          BPROF(5, ptx::mbar_wait(&q_full[sn], qph));
+          issue_st(gg + 1, kvs);
+        }
+      }
+      ptx::mma_commit_w(&kv_empty[kvs]);
+      g += nq;
+      ++n;
+    }
+    BPROF_DUMP("bmma")
+  } else if (warp < 4) {
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");  // idle
+  } else if (warp < 12) {
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 176;");
+    // ---------------------------------------- softmax-gradient warps
+    // (lane quadrant q4, column half cq); thread = key row r, queries [64 cq, 64 cq + 64)
+    const int q4 = warp & 3, cq = (warp - 4) >> 2;
+    const int r = q4 * 32 + lane;
+    const uint32_t lane_base = (uint32_t)(q4 * 32) << 16;
+    const uint32_t T_S = tmem + lane_base, T_DP = T_S + 128, T_PT = T_S + 448;
+    const uint32_t sds = ptx::smem_u32(sdS);
+    int g = 0;
+    BPROF_DECL
+    for (int pass = 0; pass * ncta < n_items; ++pass) {
+      const int item = snake_item(pass, ncta, cta);
+      if (item >= n_items) continue;
+      int kt, hd, b;
+      decode(item, kt, hd, b);
+      const int nq = n_t - kt;
+      for (int it = 0; it < nq; ++it) {
+        const int gg = g + it, st = gg % QS;
+        BPROF(0, ptx::mbar_wait(&q_full[st], (gg / QS) & 1); ptx::mbar_wait(s_full, gg & 1));
+        ptx::tc_fence_after();
+        uint32_t vs[2][32], vd[2][32];
+        __syncwarp();
+#pragma unroll
+        for (int cc = 0; cc < 2; ++cc) {
+          ptx::tmem_ld32(T_S + cq * 64 + cc * 32, vs[cc]);
+          ptx::tmem_ld32(T_DP + cq * 64 + cc * 32, vd[cc]);
+        }
+        ptx::tmem_ld_wait();
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(st_empty);  // S^T / dP^T TMEM may be overwritten
+        if (gg >= 1) BPROF(1, ptx::mbar_wait(pt_free, (gg - 1) & 1));  // dV(gg-1) read P^T
+        ptx::tc_fence_after();
+        uint32_t dpk[2][16];
+#ifdef MOBIUS_BWD_PROF
+        long long tm0 = clock64();
+#endif
+#pragma unroll
+          for (int cc = 0; cc < 2; ++cc) {
+            const int c = cq * 2 + cc;  // 32-query slab
+            uint32_t ppk[16];
+            const uint32_t aL = ptx::smem_u32(sLD + st * 256 + c * 32);
+            if (it == 0)
+              bwd_slab_math<true>(vs[cc], vd[cc], aL, c * 32, r, p.scale_log2, ppk, dpk[cc]);
+            else
+              bwd_slab_math<false>(vs[cc], vd[cc], aL, c * 32, r, p.scale_log2, ppk, dpk[cc]);
+            ptx::tmem_st16(T_PT + c * 16, ppk);  // P^T row r, queries c*32.. (2 bf16 per column)
+          }
+          ptx::tmem_st_wait();
+#ifdef MOBIUS_BWD_PROF
+        bprof[2] += clock64() - tm0;
+#endif
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(pt_full);
+        // the single dS^T tile is free once dK / dQ of the previous tile completed
+        if (gg >= 1) BPROF(3, mm_wait(gg - 1));
+        ptx::tc_fence_after();
+#pragma unroll
+        for (int cc = 0; cc < 2; ++cc)
+#pragma unroll
+          for (int k = 0; k < 4; ++k)
+            st_shared_v4(sds + sw128_off(r, (cq * 2 + cc) * 4 + k), dpk[cc][4 * k], dpk[cc][4 * k + 1], dpk[cc][4 * k + 2],
+                         dpk[cc][4 * k + 3]);
+        ptx::fence_proxy_async();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(ds_full);
+      }
+      g += nq;
+    }
+    BPROF_DUMP("bsmx")
+  } else {
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 104;");
+    // ---------------------------------------- drain warpgroup
+    // thread = TMEM lane r: dQ row r of each query tile as soon as its MMAs
+    // complete -> four fp32 16-column slabs [128 rows][64 B], 16-byte chunks
+    // XOR-swizzled (TMA SWIZZLE_64B) -> TMA reduce-add into the dQ
+    // accumulator; at an item's last tile, before its dQ, dV / dK (rows =
+    // keys) -> bf16 -> 64-row halves (SWIZZLE_128B) -> TMA stores.  Every
+    // slab goes through a ring of NSTG 8 KB staging slots, one bulk group
+    // each: a slot is rewritten once at most NSTG - 1 later groups are
+    // still reading (the TMA engine reads a 16 KB reduce slab in ~700
+    // cycles, so waiting for the previous one serialised the drain).
+    const int q4 = warp & 3;
+    const int r = q4 * 32 + lane;
+    const uint32_t lane_base = (uint32_t)(q4 * 32) << 16;
+    const uint32_t T_DV = tmem + lane_base + 256, T_DQ = tmem + lane_base + 384;
+    const bool leader = warp == 12 && lane == 0;
+    const uint32_t stg0 = ptx::smem_u32(sSTG);
+    int ks = 0;  // staged slabs so far
+    auto slot_acquire = [&]() -> uint32_t {
+      if (leader) asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(C::NSTG - 1) : "memory");
+      named_bar(1, 128);
+      return stg0 + (ks % C::NSTG) * 8192;
+    };
+    auto slot_done = [&]() {  // staging written: hand it to the async proxy
+      ptx::fence_proxy_async();
+      named_bar(1, 128);
+      ++ks;
+    };
+    int g = 0;
+    BPROF_DECL
+    for (int pass = 0; pass * ncta < n_items; ++pass) {
+      const int item = snake_item(pass, ncta, cta);
+      if (item >= n_items) continue;
+      int kt, hd, b;
+      decode(item, kt, hd, b);
+      const int nq = n_t - kt;
+      for (int it = 0; it < nq; ++it) {
+        const int gg = g + it;
+        BPROF(0, mm_wait(gg));
+        ptx::tc_fence_after();
+        if (it == nq - 1) {
+          // the item's dV / dK accumulators are final: read them out of TMEM
+          // first (the next item's first dV MMA waits for acc_empty), keep
+          // them packed bf16 (64 registers), then stage and TMA-store them
+          uint32_t pk[2][32];
+#pragma unroll
+          for (int tv = 0; tv < 2; ++tv) {
+            const float f = tv == 0 ? 1.f : p.scale;  // dK = scale * sum dS^T Q (dS^T was stored unscaled)
+#pragma unroll
+            for (int c = 0; c < 2; ++c) {
+              uint32_t v[32];
+              __syncwarp();
+              ptx::tmem_ld32(T_DV + tv * DH + c * 32, v);
+              ptx::tmem_ld_wait();
+#pragma unroll
+              for (int e = 0; e < 32; e += 2)
+                pk[tv][c * 16 + e / 2] = pack_bf16x2(
+                    __fmul2_rn(make_float2(__uint_as_float(v[e]), __uint_as_float(v[e + 1])), make_float2(f, f)));
+            }
+          }
+          ptx::tc_fence_before();
+          __syncwarp();
+          if (lane == 0) ptx::mbar_arrive(acc_empty);
+#pragma unroll
+          for (int tv = 0; tv < 2; ++tv) {
+#pragma unroll
+            for (int hf = 0; hf < 2; ++hf) {  // rows [64 hf, 64 hf + 64): lane quadrants 2 hf, 2 hf + 1
+              uint32_t stg;
+              BPROF(2, stg = slot_acquire());
+              if ((q4 >> 1) == hf) {
+#pragma unroll
+                for (int k = 0; k < 8; ++k)
+                  st_shared_v4(stg + sw128_off(r - 64 * hf, k), pk[tv][4 * k], pk[tv][4 * k + 1], pk[tv][4 * k + 2],
+                               pk[tv][4 * k + 3]);
+              }
+              slot_done();
+              if (leader) {
+                asm volatile("cp.async.bulk.tensor.4d.global.shared::cta.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
+                                 reinterpret_cast<uint64_t>(&tdkv)),
+                             "r"(stg), "r"(0), "r"(kt * 128 + 64 * hf), "r"((tv == 0 ? 2 * p.nh : p.nh) + hd), "r"(b)
+                             : "memory");
+                asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+              }
+            }
+          }
+        }
+        uint32_t v[2][32];
+        __syncwarp();
+        ptx::tmem_ld32(T_DQ, v[0]);
+        ptx::tmem_ld32(T_DQ + 32, v[1]);
+        ptx::tmem_ld_wait();
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(dq_empty);  // dQ TMEM may be overwritten
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {  // 16-column slabs
+          uint32_t stg;
+          BPROF(1, stg = slot_acquire());
+#pragma unroll
+          for (int k = 0; k < 4; ++k)
+            st_shared_v4(stg + r * 64 + ((k ^ ((r >> 1) & 3)) << 4), v[c >> 1][(c & 1) * 16 + 4 * k],
+                         v[c >> 1][(c & 1) * 16 + 4 * k + 1], v[c >> 1][(c & 1) * 16 + 4 * k + 2],
+                         v[c >> 1][(c & 1) * 16 + 4 * k + 3]);
+          slot_done();
+          if (leader) {
+            asm volatile(
+                "cp.reduce.async.bulk.tensor.4d.global.shared::cta.add.tile.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
+                    reinterpret_cast<uint64_t>(&tdq)),
+                "r"(stg), "r"(c * 16), "r"((kt + it) * 128), "r"(hd), "r"(b)
+                : "memory");
+            asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+          }
+        }
+      }
+      g += nq;
+    }
+    BPROF_DUMP("bdrn")
+    if (leader) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");  // last stores / reduces complete
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc<512>(tmem);
+  }
+}
+
 // Pre-pass of the flash backward, one warp per token row: negD[b, head, q] =
 // -sum_d dO[q, d] O[q, d] (stored negated so the softmax-gradient loop adds
 // it with FADD2), and the row's fp32 dQ accumulator zeroed (the kernel
@@ -1229,16 +1661,17 @@ int head_map(CUtensorMap* m, const void* base, int64_t ld, int dh, int s, int n_
   return MOBIUS_OK;
 }
 
-// fp32 {d, token, head, batch} map over the dQ accumulator [mbs*s, h]; box {32, 128, 1, 1}, 128B swizzle
-int dq_map(CUtensorMap* m, const float* base, int h, int dh, int s, int nh, int mbs) {
+// fp32 {d, token, head, batch} map over the dQ accumulator [mbs*s, h]; box
+// {32, 128, 1, 1} with 128B swizzle, or (cols 16) {16, 128, 1, 1} with 64B swizzle
+int dq_map(CUtensorMap* m, const float* base, int h, int dh, int s, int nh, int mbs, int cols = 32) {
   EncodeTiledFn enc = encode_fn();
   if (!enc) MOBIUS_FAIL(MOBIUS_ECUDA, "cuTensorMapEncodeTiled unavailable");
   cuuint64_t dims[4] = {(cuuint64_t)dh, (cuuint64_t)s, (cuuint64_t)nh, (cuuint64_t)mbs};
   cuuint64_t strides[3] = {(cuuint64_t)h * 4, (cuuint64_t)dh * 4, (cuuint64_t)s * h * 4};
-  cuuint32_t box[4] = {32, 128, 1, 1};
+  cuuint32_t box[4] = {(cuuint32_t)cols, 128, 1, 1};
   cuuint32_t es[4] = {1, 1, 1, 1};
   CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, const_cast<float*>(base), dims, strides, box, es,
-                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, cols == 16 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) MOBIUS_FAIL(MOBIUS_ECUDA, "flash dQ tensor map (%d)", (int)r);
   return MOBIUS_OK;
@@ -1319,10 +1752,11 @@ int flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* o, const __nv_
   if (rc) return rc;
   rc = head_map(&tdo, dout, h, dh, s, nh, mbs);
   if (rc) return rc;
-  rc = dq_map(&tdq, dq_ws, h, dh, s, nh, mbs);
+  // dh 64 kernel: 16-column dQ slabs and 64-row dV / dK halves (8 KB staging slots)
+  rc = dq_map(&tdq, dq_ws, h, dh, s, nh, mbs, dh == 64 ? 16 : 32);
   if (rc) return rc;
   CUtensorMap tdkv;  // TMA-store view of dqkv (dK / dV head slots)
-  rc = head_map(&tdkv, dqkv, 3 * h, dh, s, 3 * nh, mbs);
+  rc = head_map(&tdkv, dqkv, 3 * h, dh, s, 3 * nh, mbs, dh == 64 ? 64 : 128);
   if (rc) return rc;
   if (dh == 64)
     flash_dsum_kernel<64><<<(unsigned)((rows + 7) / 8), 256, 0, st>>>(dout, o, dsum_ws, dq_ws, (int)rows, nh, s);
@@ -1333,6 +1767,7 @@ int flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* o, const __nv_
   p.lse = lse;
   p.Dsum = dsum_ws;
   p.dQacc = dq_ws;
+  p.dqkv = dqkv;
   p.s = s;
   p.nh = nh;
   p.h = h;
@@ -1350,19 +1785,19 @@ int flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* o, const __nv_
   dim3 grid(n_items < sms ? n_items : sms);  // persistent
   if (dh == 64) {
     static bool once = false;
-    // MOBIUS_FLASH_BWD_CP: softmax-gradient warps per key row (2: 8 warps of 64 queries, 4: 16 of 32)
-    static int cp = -1;
-    if (cp < 0) {
-      const char* e = getenv("MOBIUS_FLASH_BWD_CP");
-      cp = (e && atoi(e) == 4) ? 4 : 2;
+    // MOBIUS_FLASH_BWD_V1=1: the round-2 10-warp kernel (softmax-gradient warps drain dQ themselves)
+    static int v1 = -1;
+    if (v1 < 0) {
+      const char* e = getenv("MOBIUS_FLASH_BWD_V1");
+      v1 = (e && atoi(e) == 1) ? 1 : 0;
     }
-    if (cp == 4) {
-      static bool once4 = false;
-      if (!once4) { rc = set_smem(flash_bwd_kernel<64, 4>, BwdCfg<64>::SMEM); if (rc) return rc; once4 = true; }
-      flash_bwd_kernel<64, 4><<<grid, (2 + 16) * 32, BwdCfg<64>::SMEM, st>>>(tm, tdo, tdq, tdkv, p);
-    } else {
+    if (v1) {
       if (!once) { rc = set_smem(flash_bwd_kernel<64, 2>, BwdCfg<64>::SMEM); if (rc) return rc; once = true; }
       flash_bwd_kernel<64, 2><<<grid, NT_FWD, BwdCfg<64>::SMEM, st>>>(tm, tdo, tdq, tdkv, p);
+    } else {
+      static bool once64 = false;
+      if (!once64) { rc = set_smem(flash_bwd64_kernel, Bwd64Cfg::SMEM); if (rc) return rc; once64 = true; }
+      flash_bwd64_kernel<<<grid, 512, Bwd64Cfg::SMEM, st>>>(tm, tdo, tdq, tdkv, p);
     }
   } else {
     static bool once = false;

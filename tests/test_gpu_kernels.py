@@ -460,7 +460,8 @@ def test_block_fwd_bwd(dtype, tol, wscale, h, nh, s, mbs):
 
 
 @pytest.mark.parametrize("dtype", [BF16, F32])
-@pytest.mark.parametrize("mbs,s,nh,dh", [(2, 128, 2, 64), (1, 384, 3, 64), (2, 256, 2, 128), (1, 1024, 2, 64)])
+@pytest.mark.parametrize("mbs,s,nh,dh", [(2, 128, 2, 64), (1, 384, 3, 64), (2, 256, 2, 128), (1, 1024, 2, 64),
+                                         (4, 1024, 25, 64), (2, 1024, 12, 128)])
 def test_attention_core(dtype, mbs, s, nh, dh):
     """Causal attention fwd+bwd (fused tcgen05 flash kernels on the bf16 path)
     vs the oracle's attention_fwd / attention_bwd in fp64."""

@@ -1,4 +1,4 @@
-MOBIUS_LIB_PATH=tools/gpu/var/libmobius_MOBIUS_BWD_PROF1.so python - <<'PY' 2>&1 | grep "blk 0" | sort
+MOBIUS_LIB_PATH=tools/gpu/var/libmobius_MOBIUS_BWD_PROF1.so python - <<'PY' 2>&1 | grep "blk 0 " | sort
 import os, sys
 sys.path.insert(0, '.')
 import torch
