@@ -161,6 +161,53 @@ __device__ __forceinline__ void bwd_slab_math(const uint32_t (&vs)[32], const ui
   }
 }
 
+// The same math for the dh 64 kernel, software-pipelined: the lse / -D
+// values of the next 4 queries (two broadcast LDS.128) are requested before
+// the current 4 are computed, so the shared-memory latency overlaps the MUFU
+// work instead of stalling the FFMA that consumes them (ncu: short-scoreboard
+// stalls on exactly those FFMAs were the largest stall in the slab math); the
+// scale-subtract runs as packed FFMA2 (computing -x, negated for free in the
+// MUFU operand).
+template <bool DIAG>
+__device__ __forceinline__ void bwd_slab_math_pl(const uint32_t (&vs)[32], const uint32_t (&vd)[32], uint32_t sLDq,
+                                                 int q0, int r, float sl2, uint32_t (&ppk)[16], uint32_t (&dpk)[16]) {
+  float4 L = lds_f32x4(sLDq), nD = lds_f32x4(sLDq + 512);
+  const float2 nsl = make_float2(-sl2, -sl2);
+#pragma unroll
+  for (int e = 0; e < 32; e += 4) {
+    float4 Ln = L, nDn = nD;
+    if (e + 4 < 32) {
+      Ln = lds_f32x4(sLDq + (e + 4) * 4);
+      nDn = lds_f32x4(sLDq + 512 + (e + 4) * 4);
+    }
+    // -x = L - s sl2 (FFMA2), P = 2^x with the negation folded into MUFU.EX2's operand
+    const float2 y01 = __ffma2_rn(make_float2(__uint_as_float(vs[e]), __uint_as_float(vs[e + 1])), nsl, make_float2(L.x, L.y));
+    const float2 y23 =
+        __ffma2_rn(make_float2(__uint_as_float(vs[e + 2]), __uint_as_float(vs[e + 3])), nsl, make_float2(L.z, L.w));
+    float p0 = ex2(-y01.x), p1 = ex2(-y01.y), p2 = ex2(-y23.x), p3 = ex2(-y23.y);
+    if (DIAG) {  // key r attends only from queries >= r
+      const int q = q0 + e;
+      if (q < r) p0 = 0.f;
+      if (q + 1 < r) p1 = 0.f;
+      if (q + 2 < r) p2 = 0.f;
+      if (q + 3 < r) p3 = 0.f;
+    }
+    const float2 P01 = make_float2(p0, p1), P23 = make_float2(p2, p3);
+    const float2 t01 = __fadd2_rn(make_float2(__uint_as_float(vd[e]), __uint_as_float(vd[e + 1])), make_float2(nD.x, nD.y));
+    const float2 t23 =
+        __fadd2_rn(make_float2(__uint_as_float(vd[e + 2]), __uint_as_float(vd[e + 3])), make_float2(nD.z, nD.w));
+    ppk[e >> 1] = pack_bf16x2(P01);
+    ppk[(e >> 1) + 1] = pack_bf16x2(P23);
+    dpk[e >> 1] = pack_bf16x2(__fmul2_rn(P01, t01));
+    dpk[(e >> 1) + 1] = pack_bf16x2(__fmul2_rn(P23, t23));
+    L = Ln;
+    nD = nDn;
+  }
+}
+#ifndef MOBIUS_BWD_MATH
+#define MOBIUS_BWD_MATH 1  // dh 64 kernel: 1 = bwd_slab_math_pl, 0 = bwd_slab_math
+#endif
+
 constexpr int NT_FWD = 320;  // 10 warps: TMA, MMA, 8 softmax warps (4 lane quadrants x 2 column halves)
 
 template <int DH>
@@ -1403,10 +1450,17 @@ __global__ void __launch_bounds__(512, 1) flash_bwd64_kernel(const __grid_consta
             const int c = cq * 2 + cc;  // 32-query slab
             uint32_t ppk[16];
             const uint32_t aL = ptx::smem_u32(sLD + st * 256 + c * 32);
+#if MOBIUS_BWD_MATH
+            if (it == 0)
+              bwd_slab_math_pl<true>(vs[cc], vd[cc], aL, c * 32, r, p.scale_log2, ppk, dpk[cc]);
+            else
+              bwd_slab_math_pl<false>(vs[cc], vd[cc], aL, c * 32, r, p.scale_log2, ppk, dpk[cc]);
+#else
             if (it == 0)
               bwd_slab_math<true>(vs[cc], vd[cc], aL, c * 32, r, p.scale_log2, ppk, dpk[cc]);
             else
               bwd_slab_math<false>(vs[cc], vd[cc], aL, c * 32, r, p.scale_log2, ppk, dpk[cc]);
+#endif
             ptx::tmem_st16(T_PT + c * 16, ppk);  // P^T row r, queries c*32.. (2 bf16 per column)
           }
           ptx::tmem_st_wait();
