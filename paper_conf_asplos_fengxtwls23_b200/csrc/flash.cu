@@ -667,6 +667,388 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1)
   }
 }
 
+// ---------------------------------------------------------------- fwd, dh 64
+// Ping-pong forward for dh 64 (the 1.5B shape): two query tiles in flight per
+// CTA, one per stream, so one softmax warpgroup's row max / exponentials
+// overlap the other's and the tensor core interleaves both tiles' MMAs.
+// 16 warps:
+//   warps 0, 2  TMA of stream A / B: Q of the stream's items (double
+//               buffered, the next item's Q prefetched at the current item's
+//               last S), K / V tiles through the stream's 4-deep ring
+//   warps 1, 3  MMA of stream A / B: S(r) = Q K_r^T as soon as the softmax
+//               warps hold S(r-1) in registers, then O += P(r-1) V_{r-1};
+//               each issuer commits its own MMAs, so neither stream's
+//               issue order waits on the other's softmax
+//   warps 4-7   softmax, stream A; warps 8-11 softmax, stream B: thread =
+//               query row, all 128 key columns of the tile (no cross-warp
+//               max / sum exchange); P (bf16) -> TMEM, feeds PV as a TS-MMA
+//   warps 12-15 epilogue: O / l of a finished item -> bf16 -> 32-row smem
+//               slab per warp -> TMA store; lse
+// The CTA's persistent item list (heaviest first, snake order) is dealt
+// alternately to the two streams.  setmaxnreg: 56 / 192 / 192 / 72.
+// TMEM per stream X: S at 256 X (128 cols), P at 256 X + 128 (64 packed
+// cols), O at 256 X + 192 (64 cols).
+struct Fwd64Cfg {
+  static constexpr int T_BYTES = 128 * 64 * 2;  // Q / K / V tile
+  static constexpr int KVR = 4;                 // K / V ring per stream (16 KB entries)
+  static constexpr int SMEM = 1024 + 4 * T_BYTES + 2 * KVR * T_BYTES + 4 * 4096 + 2 * 2 * 2 * 128 * 4 + 512;
+};
+
+// per-stream walk over the CTA's items (stream X takes local items X, X+2, ...)
+struct FwdStream {
+  int k;              // items of this stream started so far - 1
+  int nkv, qt, hd, b;
+  int r;              // round within the item: S(r) if r < nkv, PV(r-1) if r >= 1
+  bool act;
+};
+
+__global__ void __launch_bounds__(512, 1) flash_fwd64_kernel(const __grid_constant__ CUtensorMap tm,
+                                                          const __grid_constant__ CUtensorMap tmo, const FwdParams p) {
+  using C = Fwd64Cfg;
+  constexpr int DH = 64, KVR = C::KVR;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sQ = smem;                         // [stream][buf]
+  uint8_t* sKV = sQ + 4 * C::T_BYTES;         // [stream][KVR]
+  uint8_t* sO = sKV + 2 * KVR * C::T_BYTES;   // [4 warps] 32-row O staging slabs (4 KB)
+  float* sLM = reinterpret_cast<float*>(sO + 4 * 4096);  // [stream][item parity][l | m][128]
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sLM + 2 * 2 * 2 * 128);
+  uint64_t* q_full = bars;         // [stream * 2 + buf]
+  uint64_t* q_empty = bars + 4;    // [stream * 2 + buf]
+  uint64_t* kv_full = bars + 8;    // [stream * KVR + e]
+  uint64_t* kv_empty = bars + 8 + 2 * KVR;
+  uint64_t* s_full = bars + 8 + 4 * KVR;  // [stream]
+  uint64_t* s_free = s_full + 2;          // [stream] (count 4)
+  uint64_t* p_full = s_full + 4;          // [stream] (count 4)
+  uint64_t* pv_done = s_full + 6;         // [stream]
+  uint64_t* o_ready = s_full + 8;         // [stream]
+  uint64_t* o_empty = s_full + 10;        // [stream] (count 4)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(s_full + 12);
+
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int n_items = (p.s / BQ) * p.nh * p.mbs;
+  const int ncta = (int)gridDim.x, cta = (int)blockIdx.x;
+  // stream-local item k of stream X -> (qt, hd, b); false past the CTA's list
+  auto item_of = [&](int X, int k, FwdStream& x) {
+    const int li = 2 * k + X;
+    const int i = snake_item(li, ncta, cta);
+    x.act = i < n_items;
+    if (x.act) {
+      fwd_item(p, i, x.qt, x.hd, x.b);
+      x.nkv = x.qt + 1;
+    }
+  };
+  auto stream_init = [&](int X, FwdStream& x) {
+    x.k = 0;
+    x.r = 0;
+    item_of(X, 0, x);
+  };
+  auto stream_advance = [&](int X, FwdStream& x) {  // after a round
+    if (++x.r > x.nkv) {
+      ++x.k;
+      x.r = 0;
+      item_of(X, x.k, x);
+    }
+  };
+
+  if (threadIdx.x == 0) {
+    ptx::tma_prefetch_desc(&tm);
+    ptx::tma_prefetch_desc(&tmo);
+    for (int i = 0; i < 4; ++i) {
+      ptx::mbar_init(&q_full[i], 1);
+      ptx::mbar_init(&q_empty[i], 1);
+    }
+    for (int i = 0; i < 2 * KVR; ++i) {
+      ptx::mbar_init(&kv_full[i], 1);
+      ptx::mbar_init(&kv_empty[i], 1);
+    }
+    for (int x = 0; x < 2; ++x) {
+      ptx::mbar_init(&s_full[x], 1);
+      ptx::mbar_init(&s_free[x], 4);
+      ptx::mbar_init(&p_full[x], 4);
+      ptx::mbar_init(&pv_done[x], 1);
+      ptx::mbar_init(&o_ready[x], 1);
+      ptx::mbar_init(&o_empty[x], 4);
+    }
+    ptx::fence_mbar_init();
+  }
+  if (warp == 1) ptx::tmem_alloc<512>(tmem_slot);
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0 || warp == 2) {
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");
+    const int X = warp >> 1;
+    if (lane == 0) {
+      FwdStream x;
+      stream_init(X, x);
+      int op = 0;  // ring entries issued
+      uint64_t* kvf = kv_full + X * KVR;
+      uint64_t* kve = kv_empty + X * KVR;
+      uint8_t* ring = sKV + X * KVR * C::T_BYTES;
+      auto load_q = [&](int k, int qt, int hd, int b) {
+        const int qb = X * 2 + (k & 1);
+        ptx::mbar_wait(&q_empty[qb], ((k >> 1) & 1) ^ 1);
+        ptx::mbar_arrive_expect_tx(&q_full[qb], C::T_BYTES);
+        ptx::tma_load_4d(sQ + qb * C::T_BYTES, &tm, &q_full[qb], 0, qt * BQ, hd, b);
+      };
+      auto load_kv = [&](int slot_nh, int j, int hd, int b) {  // slot_nh: nh (K) or 2 nh (V)
+        const int e = op % KVR;
+        ptx::mbar_wait(&kve[e], ((op / KVR) & 1) ^ 1);
+        ptx::mbar_arrive_expect_tx(&kvf[e], C::T_BYTES);
+        ptx::tma_load_4d(ring + e * C::T_BYTES, &tm, &kvf[e], 0, j * BKV, slot_nh + hd, b);
+        ++op;
+      };
+      if (x.act) load_q(0, x.qt, x.hd, x.b);
+      while (x.act) {
+        if (x.r < x.nkv) {
+          load_kv(p.nh, x.r, x.hd, x.b);
+          if (x.r == x.nkv - 1) {  // last S of the item: prefetch the stream's next Q
+            FwdStream nx;
+            item_of(X, x.k + 1, nx);
+            if (nx.act) load_q(x.k + 1, nx.qt, nx.hd, nx.b);
+          }
+        }
+        if (x.r >= 1) load_kv(2 * p.nh, x.r - 1, x.hd, x.b);
+        stream_advance(X, x);
+      }
+    }
+  } else if (warp == 1 || warp == 3) {
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");
+    const int X = warp >> 1;
+    const uint32_t tm0 = __shfl_sync(0xffffffffu, tmem, 0) + X * 256;  // warp-uniform TMEM base of the stream
+    constexpr uint32_t ID_S = ptx::idesc_bf16(BQ, BKV, 0, 0);
+    constexpr uint32_t ID_O = ptx::idesc_bf16(BQ, DH, 0, 1);
+    uint64_t* kvf = kv_full + X * KVR;
+    uint64_t* kve = kv_empty + X * KVR;
+    const uint32_t ring = ptx::smem_u32(sKV + X * KVR * C::T_BYTES);
+    FwdStream x;
+    stream_init(X, x);
+    int op = 0, gs = 0, gp = 0;
+    BPROF_DECL
+    while (x.act) {
+      if (x.r < x.nkv) {  // S(r) = Q K_r^T
+        const int e = op % KVR, qb = X * 2 + (x.k & 1);
+        if (x.r == 0) BPROF(0, ptx::mbar_wait(&q_full[qb], (x.k >> 1) & 1));
+        BPROF(1, ptx::mbar_wait(&kvf[e], (op / KVR) & 1));
+        if (gs >= 1) BPROF(2, ptx::mbar_wait(&s_free[X], (gs - 1) & 1));  // softmax holds the previous S
+        ptx::tc_fence_after();
+        const uint32_t aq = ptx::smem_u32(sQ + qb * C::T_BYTES), ak = ring + e * C::T_BYTES;
+#pragma unroll
+        for (int t = 0; t < DH / 16; ++t)
+          ptx::mma_bf16_w(tm0, ptx::sdesc_sw128(aq + t * 32, 16, 1024), ptx::sdesc_sw128(ak + t * 32, 16, 1024), ID_S,
+                          t > 0);
+        ptx::mma_commit_w(&s_full[X]);
+        ptx::mma_commit_w(&kve[e]);
+        if (x.r == x.nkv - 1) ptx::mma_commit_w(&q_empty[qb]);
+        ++op;
+        ++gs;
+      }
+      if (x.r >= 1) {  // O += P(r-1) V_{r-1}
+        const int j = x.r - 1, e = op % KVR;
+        BPROF(3, ptx::mbar_wait(&p_full[X], gp & 1));
+        BPROF(4, ptx::mbar_wait(&kvf[e], (op / KVR) & 1));
+        if (j == 0 && x.k >= 1) BPROF(5, ptx::mbar_wait(&o_empty[X], (x.k - 1) & 1));  // previous item's O read out
+        ptx::tc_fence_after();
+        const uint32_t av = ring + e * C::T_BYTES;
+#pragma unroll
+        for (int t = 0; t < BKV / 16; ++t)  // 16 keys = 8 packed TMEM columns of P
+          ptx::mma_bf16_ts_w(tm0 + 192, tm0 + 128 + 8 * t, ptx::sdesc_sw128(av + t * 2048, 16384, 1024), ID_O,
+                             (j > 0 || t > 0) ? 1u : 0u);
+        ptx::mma_commit_w(&pv_done[X]);
+        ptx::mma_commit_w(&kve[e]);
+        if (j == x.nkv - 1) ptx::mma_commit_w(&o_ready[X]);
+        ++op;
+        ++gp;
+      }
+      stream_advance(X, x);
+    }
+    BPROF_DUMP("fmma")
+  } else if (warp < 12) {
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 192;");
+    // ------------------------------------------------ softmax, stream X
+    const int X = (warp - 4) >> 2, q4 = warp & 3;
+    const int row = q4 * 32 + lane;
+    const uint32_t lb = (uint32_t)(q4 * 32) << 16;
+    const uint32_t TS = tmem + lb + X * 256, TP = TS + 128, TO = TS + 192;
+    const float sc = p.scale_log2;
+    int g = 0;  // tiles of this stream so far (S and PV counters)
+    FwdStream x;
+    stream_init(X, x);
+    BPROF_DECL
+#ifdef MOBIUS_BWD_PROF
+    long long tb;
+#define FP_MARK(k) { long long t_ = clock64(); bprof[k] += t_ - tb; tb = t_; }
+#else
+#define FP_MARK(k)
+#endif
+    while (x.act) {
+      const int nkv = x.nkv;
+      float m_run = -INFINITY, l_run = 0.f;
+      for (int j = 0; j < nkv; ++j, ++g) {
+#ifdef MOBIUS_BWD_PROF
+        tb = clock64();
+#endif
+        ptx::mbar_wait(&s_full[X], g & 1);
+        FP_MARK(0)
+        ptx::tc_fence_after();
+        uint32_t v[4][32];
+        __syncwarp();
+#pragma unroll
+        for (int gi = 0; gi < 4; ++gi) ptx::tmem_ld32(TS + gi * 32, v[gi]);
+        ptx::tmem_ld_wait();
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(&s_free[X]);  // S values are in registers
+        FP_MARK(1)
+        if (j == x.qt) {  // diagonal tile: mask keys > query
+#pragma unroll
+          for (int gi = 0; gi < 4; ++gi)
+#pragma unroll
+            for (int e = 0; e < 32; ++e)
+              if (gi * 32 + e > row) v[gi][e] = __float_as_uint(-INFINITY);
+        }
+        float mx;
+        {  // four independent max chains
+          float m4[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
+#pragma unroll
+          for (int gi = 0; gi < 4; ++gi)
+#pragma unroll
+            for (int e = 0; e < 32; e += 2)
+              m4[(e >> 1) & 3] = fmaxf(m4[(e >> 1) & 3], fmaxf(__uint_as_float(v[gi][e]), __uint_as_float(v[gi][e + 1])));
+          mx = fmaxf(fmaxf(m4[0], m4[1]), fmaxf(m4[2], m4[3]));
+        }
+        // lazy rescaling: keep the running max unless it grows by > 8 (log2)
+        const float m_cand = fmaxf(m_run, mx * sc);
+        const bool grow = m_cand > m_run + 8.f;
+        const float m_new = grow ? m_cand : m_run;
+        const float alpha = ex2(m_run - m_new);  // 1 when not growing; 0 at j = 0
+        // P = 2^(x sc - m_new) packed bf16, row sum (two f32x2 accumulators)
+        uint32_t pk[4][16];
+        float2 rsa = make_float2(0.f, 0.f), rsb = make_float2(0.f, 0.f);
+        const float2 sc2 = make_float2(sc, sc), nm2 = make_float2(-m_new, -m_new);
+#pragma unroll
+        for (int gi = 0; gi < 4; ++gi) {
+#pragma unroll
+          for (int e = 0; e < 32; e += 2) {
+            const float2 xx = __ffma2_rn(make_float2(__uint_as_float(v[gi][e]), __uint_as_float(v[gi][e + 1])), sc2, nm2);
+            // all on MUFU: a polynomial share (2 / 4 / 6 / 8 of 16 pairs) measured
+            // 232 / 246 / 258 / 281 us against 227 us at mbs 32
+            const float2 pp = make_float2(ex2(xx.x), ex2(xx.y));
+            if ((e >> 1) & 1)
+              rsb = __fadd2_rn(rsb, pp);
+            else
+              rsa = __fadd2_rn(rsa, pp);
+            pk[gi][e >> 1] = pack_bf16(pp.x, pp.y);
+          }
+        }
+        const float rs = (rsa.x + rsa.y) + (rsb.x + rsb.y);
+        l_run = l_run * alpha + rs;
+        m_run = m_new;
+        FP_MARK(2)
+        // P and O of this stream are free once its previous PV completed
+        if (g >= 1) {
+          ptx::mbar_wait(&pv_done[X], (g - 1) & 1);
+          ptx::tc_fence_after();
+        }
+        FP_MARK(3)
+        if (j >= 1 && __any_sync(0xffffffffu, grow)) {  // rescale O (the item's PVs so far are done)
+          uint32_t o[32];
+#pragma unroll
+          for (int c = 0; c < 2; ++c) {
+            ptx::tmem_ld32(TO + c * 32, o);
+            ptx::tmem_ld_wait();
+#pragma unroll
+            for (int e = 0; e < 32; ++e) o[e] = __float_as_uint(__uint_as_float(o[e]) * alpha);
+            ptx::tmem_st32(TO + c * 32, o);
+          }
+        }
+#pragma unroll
+        for (int gi = 0; gi < 4; ++gi) ptx::tmem_st16(TP + gi * 16, pk[gi]);
+        ptx::tmem_st_wait();
+        if (j == nkv - 1) {  // l / m of the item for the epilogue (double-buffered by item parity)
+          float* lm = sLM + (X * 2 + (x.k & 1)) * 256;
+          lm[row] = l_run;
+          lm[128 + row] = m_run;
+        }
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(&p_full[X]);
+        FP_MARK(4)
+      }
+      ++x.k;
+      item_of(X, x.k, x);
+    }
+    BPROF_DUMP("fsmx")
+  } else {
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 72;");
+    // ------------------------------------------------ epilogue
+    // whichever stream's item finishes next: O / l -> bf16 -> this warp's
+    // 32-row SW128 slab -> TMA store (one per warp); lse = m + log2 l
+    const int q4 = warp & 3, row = q4 * 32 + lane;
+    const uint32_t lb = (uint32_t)(q4 * 32) << 16;
+    const uint32_t slab = ptx::smem_u32(sO) + q4 * 4096;
+    FwdStream st[2];
+    stream_init(0, st[0]);
+    stream_init(1, st[1]);
+    while (st[0].act || st[1].act) {
+      int X = -1;
+      while (X < 0) {  // poll: the streams finish items in an order set by the MMA interleave
+        for (int c = 0; c < 2 && X < 0; ++c)
+          if (st[c].act && ptx::mbar_test(&o_ready[c], st[c].k & 1)) X = c;
+        X = __shfl_sync(0xffffffffu, X, 0);
+      }
+      FwdStream& x = st[X];
+      ptx::tc_fence_after();
+      const float* lm = sLM + (X * 2 + (x.k & 1)) * 256;
+      const float l = lm[row], m = lm[128 + row];
+      uint32_t v[2][32];
+      __syncwarp();
+      ptx::tmem_ld32(tmem + lb + X * 256 + 192, v[0]);
+      ptx::tmem_ld32(tmem + lb + X * 256 + 224, v[1]);
+      ptx::tmem_ld_wait();
+      ptx::tc_fence_before();
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(&o_empty[X]);  // O of this stream may be overwritten
+      const float inv_l = 1.f / l;
+      if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // previous store read the slab
+      __syncwarp();
+#pragma unroll
+      for (int c = 0; c < 2; ++c) {
+        uint32_t pk[16];
+#pragma unroll
+        for (int e = 0; e < 32; e += 2)
+          pk[e / 2] = pack_bf16(__uint_as_float(v[c][e]) * inv_l, __uint_as_float(v[c][e + 1]) * inv_l);
+#pragma unroll
+        for (int k = 0; k < 4; ++k)
+          st_shared_v4(slab + lane * 128 + (((c * 4 + k) ^ (lane & 7)) << 4), pk[4 * k], pk[4 * k + 1], pk[4 * k + 2],
+                       pk[4 * k + 3]);
+      }
+      ptx::fence_proxy_async();
+      __syncwarp();
+      if (lane == 0) {
+        asm volatile("cp.async.bulk.tensor.4d.global.shared::cta.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
+                         reinterpret_cast<uint64_t>(&tmo)),
+                     "r"(slab), "r"(0), "r"(x.qt * BQ + q4 * 32), "r"(x.hd), "r"(x.b)
+                     : "memory");
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+      }
+      p.lse[((int64_t)x.b * p.nh + x.hd) * p.s + x.qt * BQ + row] = m + __log2f(l);
+      ++x.k;
+      item_of(X, x.k, x);
+    }
+    if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc<512>(tmem);
+  }
+}
+
 // ====================================================================== bwd
 template <int DH>
 struct BwdCfg {
@@ -1777,7 +2159,17 @@ int flash_attn_fwd(const __nv_bfloat16* qkv, __nv_bfloat16* o, float* lse, int m
       const char* e = getenv("MOBIUS_FLASH_FWD_CP");
       cp = (e && atoi(e) == 4) ? 4 : 2;
     }
-    if (cp == 4) {
+    // MOBIUS_FLASH_FWD_V1=1: the round-2 10-warp kernel (one query tile at a time)
+    static int v1 = -1;
+    if (v1 < 0) {
+      const char* e = getenv("MOBIUS_FLASH_FWD_V1");
+      v1 = (e && atoi(e) == 1) ? 1 : 0;
+    }
+    if (!v1) {
+      static bool once64 = false;
+      if (!once64) { rc = set_smem(flash_fwd64_kernel, Fwd64Cfg::SMEM); if (rc) return rc; once64 = true; }
+      flash_fwd64_kernel<<<grid, 512, Fwd64Cfg::SMEM, st>>>(tm, tmo, p);
+    } else if (cp == 4) {
       static bool once4 = false;
       if (!once4) { rc = set_smem(flash_fwd_kernel<64, 4>, FwdCfg<64>::SMEM); if (rc) return rc; once4 = true; }
       flash_fwd_kernel<64, 4><<<grid, (2 + 16) * 32, FwdCfg<64>::SMEM, st>>>(tm, tmo, p);
