@@ -62,6 +62,26 @@ __global__ void __launch_bounds__(512, 1) probe(int n_iter, long long* out, floa
           acc[i + 1] = v.y;
         }
       }
+    } else if (MODE == 5) {  // ex2.approx.f16x2: two exponentials per lane per instruction
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          uint32_t h = __float_as_uint(acc[i]), o;
+          asm volatile("ex2.approx.f16x2 %0, %1;" : "=r"(o) : "r"(h));
+          acc[i] = __uint_as_float(o ^ 0x80008000u);
+        }
+      }
+    } else if (MODE == 6) {  // ex2.approx.ftz.bf16x2
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          uint32_t h = __float_as_uint(acc[i]), o;
+          asm volatile("ex2.approx.ftz.bf16x2 %0, %1;" : "=r"(o) : "r"(h));
+          acc[i] = __uint_as_float(o ^ 0x80008000u);
+        }
+      }
     } else if (MODE == 4) {  // four tcgen05.ld x32 in flight, one wait (a 128-column row chunk)
       uint32_t r2[32], r3[32], r4[32];
       ptx::tmem_ld32(tmem + lb + 0, r);
@@ -108,6 +128,8 @@ void run(const char* name, int warps, double units_per_iter_per_warp, const char
 
 int main() {
   for (int w : {4, 8, 16}) run<0>("MUFU ex2", w, 64 * 32, "ex2");
+  for (int w : {4, 8, 16}) run<5>("MUFU ex2 f16x2", w, 64 * 32 * 2, "ex2");
+  for (int w : {4, 8, 16}) run<6>("MUFU ex2 bf16x2", w, 64 * 32 * 2, "ex2");
   for (int w : {4, 8, 16}) run<3>("FFMA2", w, 32 * 32 * 2, "flop-lanes");
   for (int w : {4, 8, 16}) run<1>("tcgen05.ld 32x32b.x32", w, 32 * 32 * 4, "bytes");
   for (int w : {4, 8, 16}) run<4>("tcgen05.ld 4 x x32 in flight", w, 4 * 32 * 32 * 4, "bytes");
