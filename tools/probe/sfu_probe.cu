@@ -82,6 +82,26 @@ __global__ void __launch_bounds__(512, 1) probe(int n_iter, long long* out, floa
           acc[i] = __uint_as_float(o ^ 0x80008000u);
         }
       }
+    } else if (MODE == 7) {  // tanh.approx.f32
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          float y;
+          asm volatile("tanh.approx.f32 %0, %1;" : "=f"(y) : "f"(acc[i]));
+          acc[i] = y * 1.5f;
+        }
+      }
+    } else if (MODE == 8) {  // rcp.approx.ftz.f32
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          float y;
+          asm volatile("rcp.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(acc[i]));
+          acc[i] = y + 0.5f;
+        }
+      }
     } else if (MODE == 4) {  // four tcgen05.ld x32 in flight, one wait (a 128-column row chunk)
       uint32_t r2[32], r3[32], r4[32];
       ptx::tmem_ld32(tmem + lb + 0, r);
@@ -128,6 +148,8 @@ void run(const char* name, int warps, double units_per_iter_per_warp, const char
 
 int main() {
   for (int w : {4, 8, 16}) run<0>("MUFU ex2", w, 64 * 32, "ex2");
+  for (int w : {4, 8, 16}) run<7>("MUFU tanh", w, 64 * 32, "tanh");
+  for (int w : {4, 8, 16}) run<8>("MUFU rcp", w, 64 * 32, "rcp");
   for (int w : {4, 8, 16}) run<5>("MUFU ex2 f16x2", w, 64 * 32 * 2, "ex2");
   for (int w : {4, 8, 16}) run<6>("MUFU ex2 bf16x2", w, 64 * 32 * 2, "ex2");
   for (int w : {4, 8, 16}) run<3>("FFMA2", w, 32 * 32 * 2, "flop-lanes");
