@@ -69,6 +69,9 @@ struct Params {
   // sk_tiles * sk_slices units of the k-aligned schedule cover every tile
   // and each unit reduce-adds its partial straight into C (no workspace).
   int splitk_reduce;
+  // 2-CTA kernel: M tiles per rasterisation group (tiles of a group share
+  // their B panels in L2); chosen on the host from the shape
+  int group_m;
 };
 
 __device__ __forceinline__ float tanh_fast(float x) {

@@ -388,7 +388,7 @@ __global__ void __launch_bounds__(NUM_THREADS2, 1)
   const int total = p.tiles_m * tiles_n2;
 
   auto tile_of = [&](int t, int& mt, int& nt) {  // grouped along M for L2 reuse
-    constexpr int GROUP = 8;
+    const int GROUP = p.group_m;
     const int span = GROUP * tiles_n2;
     const int g = t / span, first_m = g * GROUP;
     const int gm = min(GROUP, p.tiles_m - first_m);
@@ -923,6 +923,20 @@ static int gemm_bf16_2cta_bn(const GemmDesc& d, cudaStream_t s) {
   p.R = (const __nv_bfloat16*)d.R.ptr; p.ldr = d.R.ld;
   p.AUX = (__nv_bfloat16*)d.AUX.ptr; p.ldx = d.AUX.ld;
   p.ones_m0p1 = ones ? d.M : 0;  // (M - 1) + 1
+  // rasterisation group: 4 M tiles for the activation-major GEMMs (forward,
+  // dX), 8 for the weight-gradient ones (A MN-major, long K).  Measured under
+  // the power cap (tools/gemm_sustained.py, T = 32768): group 4 / 8 / 16 / 32
+  // give fc2 fwd 559 / 585 / 610 / 661 us, fc1 dX 546 / 576 / 592 / 639 us,
+  // qkv dX 409 / 422 / 433 / 464 us (the larger groups run at lower clocks),
+  // K = 1600 shapes within 1%; qkv dW 489 / 472 us with 4 / 8
+  {
+    static int g_env = -2;
+    if (g_env == -2) {
+      const char* e = getenv("MOBIUS_GEMM_GROUP");
+      g_env = e ? atoi(e) : -1;
+    }
+    p.group_m = g_env > 0 ? g_env : (d.a_mn ? 8 : 4);
+  }
   plan_stream_k(p, num_sms() / 2);
   if (p.sk_tiles && !p.splitk_reduce) {
     const size_t ws = (size_t)p.sk_tiles * p.sk_maxseg * 16 * 32 * (BN / 2) * sizeof(float);
