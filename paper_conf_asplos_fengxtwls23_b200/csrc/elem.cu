@@ -604,6 +604,185 @@ __global__ void __launch_bounds__(256) ln_bwd_dx_k(const T* __restrict__ dy, con
   }
 }
 
+// ------------------------------------- LayerNorm backward, fused (bf16)
+// One pass over dy / x (/ dres): a persistent CTA per SM walks blocks of R
+// rows; each block's dy, x (and dres) rows arrive in shared memory by bulk
+// copies through a ring of LNF_NBUF buffers (the next LNF_NBUF - 1 blocks'
+// rows are in flight while one is computed), then
+//   phase A (warp per row): s1 = mean(dy g), s2 = mean(dy g xhat)
+//   phase B (thread per 8-column vector, all R rows): dx = rstd (dy g - s1 -
+//           xhat s2) (+ dres), and the thread's dgamma / dbeta partials
+//           (sum of dy xhat, dy) over every row the CTA handles
+// Each CTA writes its partial rows to part[cta] (fixed row order inside the
+// CTA); ln_param_reduce_k adds the G partial rows in CTA order into dg / db:
+// deterministic, dy and x read from DRAM once (the two-kernel version read
+// them twice: 158 us at 32768 x 1600).
+constexpr int LNF_THREADS = 256;
+constexpr int LNF_MAXV = 4;  // column vectors per thread (h <= 256 * 8 * 4 = 8192)
+constexpr int LNF_MAX_GRID = 512;
+#ifndef MOBIUS_LNF_NBUF
+#define MOBIUS_LNF_NBUF 2
+#endif
+constexpr int LNF_NBUF = MOBIUS_LNF_NBUF;  // row-block buffers in flight (ring)
+
+__device__ __forceinline__ void lnf_bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+               "l"(reinterpret_cast<uint64_t>(src)), "r"(bytes), "r"(bar)
+               : "memory");
+}
+__device__ __forceinline__ uint32_t lnf_smem(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+#ifndef MOBIUS_LNF_CTAS
+#define MOBIUS_LNF_CTAS 2  // CTAs per SM (shared-memory budget split between them)
+#endif
+template <int MAXV>  // column vectors per thread: ceil(h / 8 / LNF_THREADS)
+__global__ void __launch_bounds__(LNF_THREADS, MOBIUS_LNF_CTAS)
+    ln_bwd_fused_k(const __nv_bfloat16* __restrict__ dy, const __nv_bfloat16* __restrict__ x,
+                   const __nv_bfloat16* __restrict__ g, const float* __restrict__ mu, const float* __restrict__ rstd,
+                   const __nv_bfloat16* __restrict__ dres, __nv_bfloat16* __restrict__ dx, float* __restrict__ part,
+                   int rows, int h, int R) {
+  extern __shared__ __align__(128) uint8_t lnf_smem_raw[];
+  // [LNF_NBUF buffers][dy | x (| dres)][R rows][h] bf16 (a block's rows are
+  // contiguous in each tensor: one bulk copy per tensor), then R floats each
+  // of mu, rstd, s1, s2, then LNF_NBUF mbarriers
+  const int NT = dres ? 3 : 2;  // tensors per row
+  __nv_bfloat16* buf = reinterpret_cast<__nv_bfloat16*>(lnf_smem_raw);
+  float* st = reinterpret_cast<float*>(buf + (size_t)LNF_NBUF * R * NT * h);  // [4][R]
+  uint64_t* bar = reinterpret_cast<uint64_t*>(st + 4 * R + 2);
+  bar = reinterpret_cast<uint64_t*>((reinterpret_cast<uintptr_t>(bar) + 7) & ~uintptr_t(7));
+  const int tid = threadIdx.x, warp = tid / 32, lane = tid % 32;
+  const int nvec = h / 8;
+  const int nblk = (rows + R - 1) / R;
+  if (tid == 0) {
+    for (int i = 0; i < LNF_NBUF; ++i)
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(lnf_smem(&bar[i])) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  auto issue = [&](int blk, int b) {  // one thread: rows of block blk -> buffer b
+    const int r0 = blk * R, nr = min(R, rows - r0);
+    const uint32_t bytes = (uint32_t)nr * NT * h * 2;
+    const uint32_t bb = lnf_smem(&bar[b]);
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bb), "r"(bytes) : "memory");
+    __nv_bfloat16* base = buf + (size_t)b * R * NT * h;
+    const uint32_t tb = (uint32_t)nr * h * 2;
+    lnf_bulk_g2s(lnf_smem(base), dy + (int64_t)r0 * h, tb, bb);
+    lnf_bulk_g2s(lnf_smem(base + (size_t)R * h), x + (int64_t)r0 * h, tb, bb);
+    if (dres) lnf_bulk_g2s(lnf_smem(base + (size_t)2 * R * h), dres + (int64_t)r0 * h, tb, bb);
+  };
+  // this thread's column vectors and their gamma
+  float gv[MAXV][8], adg[MAXV][8], adb[MAXV][8];
+#pragma unroll
+  for (int k = 0; k < MAXV; ++k) {
+    const int v = tid + k * LNF_THREADS;
+#pragma unroll
+    for (int e = 0; e < 8; ++e) adg[k][e] = adb[k][e] = 0.f;
+    if (v < nvec) Vec<__nv_bfloat16>::load(g + v * 8, gv[k]);
+  }
+  const float inv_h = 1.f / (float)h;
+  int it = 0;
+  if (tid == 0)
+    for (int k = 0; k < LNF_NBUF - 1; ++k)
+      if ((int)blockIdx.x + k * (int)gridDim.x < nblk) issue(blockIdx.x + k * gridDim.x, k);
+  for (int blk = blockIdx.x; blk < nblk; blk += gridDim.x, ++it) {
+    const int b = it % LNF_NBUF;
+    const int r0 = blk * R, nr = min(R, rows - r0);
+    // buffer (it - 1) % LNF_NBUF was released by the __syncthreads that ended the previous block
+    const int ahead = blk + (LNF_NBUF - 1) * (int)gridDim.x;
+    if (tid == 0 && ahead < nblk) issue(ahead, (it + LNF_NBUF - 1) % LNF_NBUF);
+    {
+      const uint32_t bb = lnf_smem(&bar[b]), ph = (uint32_t)(it / LNF_NBUF) & 1u;
+      asm volatile(
+          "{\n\t.reg .pred P1;\n\tLNF_WAIT:\n\t"
+          "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1, 10000000;\n\t"
+          "@P1 bra LNF_DONE;\n\tbra LNF_WAIT;\n\tLNF_DONE:\n\t}\n" ::"r"(bb),
+          "r"(ph)
+          : "memory");
+    }
+    const __nv_bfloat16* bs = buf + (size_t)b * R * NT * h;
+    float* sm = st;  // mu | rstd | s1 | s2 of this block
+    // phase A: row statistics, warp per row
+    for (int r = warp; r < nr; r += LNF_THREADS / 32) {
+      const float m = mu[r0 + r], rs = rstd[r0 + r];
+      const __nv_bfloat16* dr = bs + (size_t)r * h;
+      float s1 = 0.f, s2 = 0.f;
+      for (int v = lane; v < nvec; v += 32) {
+        float dv[8], xv[8], gg[8];
+        Vec<__nv_bfloat16>::load(dr + v * 8, dv);
+        Vec<__nv_bfloat16>::load(dr + (size_t)R * h + v * 8, xv);
+        Vec<__nv_bfloat16>::load(g + v * 8, gg);
+#pragma unroll
+        for (int e = 0; e < 8; ++e) {
+          const float dh = dv[e] * gg[e];
+          s1 += dh;
+          s2 += dh * (xv[e] - m) * rs;
+        }
+      }
+      s1 = warp_sum(s1);
+      s2 = warp_sum(s2);
+      if (lane == 0) {
+        sm[r] = m;
+        sm[R + r] = rs;
+        sm[2 * R + r] = s1 * inv_h;
+        sm[3 * R + r] = s2 * inv_h;
+      }
+    }
+    __syncthreads();
+    // phase B: dx and the parameter-gradient partials, thread per column vector
+#pragma unroll
+    for (int k = 0; k < MAXV; ++k) {
+      const int v = tid + k * LNF_THREADS;
+      if (v >= nvec) continue;
+      for (int r = 0; r < nr; ++r) {
+        const float m = sm[r], rs = sm[R + r], s1 = sm[2 * R + r], s2 = sm[3 * R + r];
+        const __nv_bfloat16* dr = bs + (size_t)r * h;
+        float dv[8], xv[8], ov[8];
+        Vec<__nv_bfloat16>::load(dr + v * 8, dv);
+        Vec<__nv_bfloat16>::load(dr + (size_t)R * h + v * 8, xv);
+        const int64_t off = (int64_t)(r0 + r) * h + v * 8;
+        if (dres) Vec<__nv_bfloat16>::load(dr + (size_t)2 * R * h + v * 8, ov);
+#pragma unroll
+        for (int e = 0; e < 8; ++e) {
+          const float xh = (xv[e] - m) * rs;
+          const float val = rs * (dv[e] * gv[k][e] - s1 - (xv[e] - m) * rs * s2);
+          ov[e] = dres ? ov[e] + val : val;
+          adg[k][e] += dv[e] * xh;
+          adb[k][e] += dv[e];
+        }
+        Vec<__nv_bfloat16>::store(dx + off, ov);
+      }
+    }
+    __syncthreads();  // buffer b and the row statistics are free again
+  }
+  // partial rows: part[cta][0][c] = dgamma, part[cta][1][c] = dbeta
+  float* pr = part + (size_t)blockIdx.x * 2 * h;
+#pragma unroll
+  for (int k = 0; k < MAXV; ++k) {
+    const int v = tid + k * LNF_THREADS;
+    if (v >= nvec) continue;
+#pragma unroll
+    for (int e = 0; e < 8; e += 4) {
+      *reinterpret_cast<float4*>(pr + v * 8 + e) = make_float4(adg[k][e], adg[k][e + 1], adg[k][e + 2], adg[k][e + 3]);
+      *reinterpret_cast<float4*>(pr + h + v * 8 + e) =
+          make_float4(adb[k][e], adb[k][e + 1], adb[k][e + 2], adb[k][e + 3]);
+    }
+  }
+}
+
+// dg[c] += sum_{cta} part[cta][0][c], db[c] += sum_{cta} part[cta][1][c], in CTA order
+__global__ void ln_param_reduce_k(const float* __restrict__ part, int G, int h, float* dg, float* db) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= 2 * h) return;
+  float s = 0.f;
+  for (int c = 0; c < G; ++c) s += part[(size_t)c * 2 * h + i];
+  if (i < h)
+    dg[i] += s;
+  else
+    db[i - h] += s;
+}
+
 // Column reductions over `rows` rows, 16-byte vectors per thread, partial
 // sums in registers, CTA-level smem reduction.  mode 0: out0[c] += sum_r
 // X[r,c].  mode 1 (LayerNorm parameters): out0[c] += sum_r X[r,c] *
@@ -871,10 +1050,70 @@ int layernorm_fwd(const T* x, const T* g, const T* b, T* y, float* mu, float* rs
     LN_DISPATCH(ln_fwd_k, rows, x, g, b, y, mu, rstd, h);
   return check_launch("layernorm_fwd");
 }
+// rows per block of the fused bf16 LN backward (LNF_NBUF buffers of R rows
+// of nt tensors in <= 200 KB of shared memory), 0 when it does not apply
+static int lnf_rows(int h, int nt) {
+  if (h % 8 || h > 256 * 8 * LNF_MAXV) return 0;
+  const int r = std::min((200 * 1024 / MOBIUS_LNF_CTAS) / (LNF_NBUF * nt * h * 2), 16);
+  return r >= 1 ? r : 0;
+}
+static int lnf_smem_bytes(int h, int R, int nt) { return LNF_NBUF * R * nt * h * 2 + 4 * R * 4 + 8 * LNF_NBUF + 64; }
+static int lnf_grid() {
+  static int g = 0;
+  if (!g) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&g, cudaDevAttrMultiProcessorCount, dev);
+    g = std::min(g * MOBIUS_LNF_CTAS, LNF_MAX_GRID);
+  }
+  return g;
+}
+
+template <int MV>
+static int lnf_launch(int G, int smem, cudaStream_t st, const __nv_bfloat16* dy, const __nv_bfloat16* x,
+                      const __nv_bfloat16* g, const float* mu, const float* rstd, const __nv_bfloat16* dres,
+                      __nv_bfloat16* dx, float* part, int rows, int h, int R) {
+  static int smem_set = 0;  // per instantiation
+  if (smem > smem_set) {
+    if (cudaFuncSetAttribute(ln_bwd_fused_k<MV>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
+      MOBIUS_FAIL(MOBIUS_ECUDA, "layernorm_bwd: smem attribute");
+    smem_set = smem;
+  }
+  ln_bwd_fused_k<MV><<<G, LNF_THREADS, smem, st>>>(dy, x, g, mu, rstd, dres, dx, part, rows, h, R);
+  return MOBIUS_OK;
+}
+
 template <typename T>
 int layernorm_bwd(const T* dy, const T* x, const T* g, const float* mu, const float* rstd, const T* dres, T* dx,
                   float* dg, float* db, int rows, int h, const RedWs& ws, cudaStream_t st) {
   MOBIUS_CHECK_ARG(h % Vec<T>::N == 0, "layernorm: unsupported h=%d", h);
+  if constexpr (sizeof(T) == 2) {
+    static int fused = -1;
+    if (fused < 0) {
+      const char* e = getenv("MOBIUS_LN_BWD_FUSED");
+      fused = e ? atoi(e) : 1;
+    }
+    const int nt = dres ? 3 : 2;
+    const int R = lnf_rows(h, nt);
+    if (fused && R && aligned16(dy) && aligned16(x) && aligned16(dx) && (!dres || aligned16(dres))) {
+      MOBIUS_CHECK_ARG(ws.part, "layernorm_bwd: reduction workspace");
+      const int G = std::min(lnf_grid(), (rows + R - 1) / R);
+      const int smem = lnf_smem_bytes(h, R, nt);
+      const int mv = (h / 8 + LNF_THREADS - 1) / LNF_THREADS;
+      const auto* a = (const __nv_bfloat16*)dy;
+      int rc = mv == 1   ? lnf_launch<1>(G, smem, st, a, (const __nv_bfloat16*)x, (const __nv_bfloat16*)g, mu, rstd,
+                                         (const __nv_bfloat16*)dres, (__nv_bfloat16*)dx, ws.part, rows, h, R)
+               : mv == 2 ? lnf_launch<2>(G, smem, st, a, (const __nv_bfloat16*)x, (const __nv_bfloat16*)g, mu, rstd,
+                                         (const __nv_bfloat16*)dres, (__nv_bfloat16*)dx, ws.part, rows, h, R)
+                         : lnf_launch<4>(G, smem, st, a, (const __nv_bfloat16*)x, (const __nv_bfloat16*)g, mu, rstd,
+                                         (const __nv_bfloat16*)dres, (__nv_bfloat16*)dx, ws.part, rows, h, R);
+      if (rc) return rc;
+      rc = check_launch("layernorm_bwd_fused");
+      if (rc) return rc;
+      ln_param_reduce_k<<<(2 * h + 255) / 256, 256, 0, st>>>(ws.part, G, h, dg, db);
+      return check_launch("layernorm_param_reduce");
+    }
+  }
   // dx, then gamma / beta grads by a column-reduction pass.  Caching the
   // row's x and dy in registers for the second pass (one read each instead
   // of a re-read that hits L1/L2 anyway) was measured slower at 32768 x
@@ -927,8 +1166,9 @@ int loss_accumulate(const float* loss_rows, int rows, double* acc, cudaStream_t 
 }
 
 int64_t colsum_ws_floats(int rows, int n, int planes) {
-  // the bf16 grid (8-wide vectors) has fewer column CTAs, hence more row CTAs
-  int64_t best = 0;
+  // the bf16 grid (8-wide vectors) has fewer column CTAs, hence more row CTAs;
+  // the fused LN backward (planes 2) needs one partial row pair per CTA
+  int64_t best = planes == 2 ? (int64_t)LNF_MAX_GRID * n * 2 : 0;
   for (int vw : {4, 8}) {
     int gx, gy, rpc;
     colsum_grid(rows, n, vw, &gx, &gy, &rpc);

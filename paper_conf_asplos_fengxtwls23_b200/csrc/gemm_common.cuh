@@ -88,33 +88,6 @@ __device__ __forceinline__ float gelu_f(float u) {
   const float hu = 0.5f * u;
   return fmaf(hu, t, hu);
 }
-// gelu_f on a pair in packed f32x2 arithmetic (FMUL2 / FFMA2): the same
-// operations in the same order, so bit-identical to gelu_f per lane, with
-// about half the FP32 instructions (the fused GEMM epilogues are issue-bound
-// under the power cap: bias+GeLU fc1 forward 511 -> 612 us sustained)
-__device__ __forceinline__ float2 gelu2_f(float2 u) {
-  const float2 c = make_float2(0.7978845608028654f, 0.7978845608028654f);
-  const float2 ca = make_float2(0.7978845608028654f * 0.044715f, 0.7978845608028654f * 0.044715f);
-  const float2 y = __fmul2_rn(u, __ffma2_rn(ca, __fmul2_rn(u, u), c));
-  const float2 t = make_float2(tanh_fast(y.x), tanh_fast(y.y));
-  const float2 hu = __fmul2_rn(make_float2(0.5f, 0.5f), u);
-  return __ffma2_rn(hu, t, hu);
-}
-// gelu'(u) on a pair in packed f32x2 arithmetic:
-// 0.5 (1 + t) + 0.5 u (1 - t^2) (c + 3 c a u^2), t = tanh(u (c + c a u^2))
-__device__ __forceinline__ float2 gelu_grad2_f(float2 u) {
-  const float2 c = make_float2(0.7978845608028654f, 0.7978845608028654f);
-  const float2 ca = make_float2(0.7978845608028654f * 0.044715f, 0.7978845608028654f * 0.044715f);
-  const float2 ca3 = make_float2(3.f * 0.7978845608028654f * 0.044715f, 3.f * 0.7978845608028654f * 0.044715f);
-  const float2 h = make_float2(0.5f, 0.5f);
-  const float2 u2 = __fmul2_rn(u, u);
-  const float2 y = __fmul2_rn(u, __ffma2_rn(ca, u2, c));
-  const float2 t = make_float2(tanh_fast(y.x), tanh_fast(y.y));
-  const float2 s = __ffma2_rn(make_float2(-t.x, -t.y), t, make_float2(1.f, 1.f));  // 1 - t^2
-  const float2 d = __ffma2_rn(ca3, u2, c);
-  const float2 q = __fmul2_rn(__fmul2_rn(h, u), s);
-  return __ffma2_rn(q, d, __ffma2_rn(t, h, h));
-}
 __device__ __forceinline__ float gelu_grad_f(float u) {
   const float c = 0.7978845608028654f, a = 0.044715f;
   float t = tanh_fast(c * (u + a * u * u * u));

@@ -133,15 +133,10 @@ __device__ __forceinline__ void epi_tma(const Params& p, const EpiMaps& mp, uint
       if (j == NCH - 1) release();
       if (n0 >= p.N) continue;
       float v[64];
-      const float2 al2 = make_float2(p.alpha, p.alpha);
 #pragma unroll
-      for (int i = 0; i < 32; i += 2) {  // packed: FMUL2 (and FADD2 below), same rounding as the scalar ops
-        const float2 a2 = __fmul2_rn(make_float2(__uint_as_float(ra[i]), __uint_as_float(ra[i + 1])), al2);
-        const float2 b2 = __fmul2_rn(make_float2(__uint_as_float(rb[i]), __uint_as_float(rb[i + 1])), al2);
-        v[i] = a2.x;
-        v[i + 1] = a2.y;
-        v[32 + i] = b2.x;
-        v[32 + i + 1] = b2.y;
+      for (int i = 0; i < 32; ++i) {
+        v[i] = __uint_as_float(ra[i]) * p.alpha;
+        v[32 + i] = __uint_as_float(rb[i]) * p.alpha;
       }
       if constexpr (has_bias) {
         if (n0 + 64 <= p.N) {
@@ -151,9 +146,9 @@ __device__ __forceinline__ void epi_tma(const Params& p, const EpiMaps& mp, uint
             const __nv_bfloat162* h2 = reinterpret_cast<const __nv_bfloat162*>(&pk);
 #pragma unroll
             for (int k = 0; k < 4; ++k) {
-              const float2 x = __fadd2_rn(make_float2(v[8 * i + 2 * k], v[8 * i + 2 * k + 1]), __bfloat1622float2(h2[k]));
-              v[8 * i + 2 * k] = x.x;
-              v[8 * i + 2 * k + 1] = x.y;
+              const float2 x = __bfloat1622float2(h2[k]);
+              v[8 * i + 2 * k] += x.x;
+              v[8 * i + 2 * k + 1] += x.y;
             }
           }
         } else {
@@ -177,18 +172,15 @@ __device__ __forceinline__ void epi_tma(const Params& p, const EpiMaps& mp, uint
           for (int k = 0; k < 4; ++k) {
             const float2 x = __bfloat1622float2(h2[k]);
             if constexpr (EPI == EPI_BIAS_RESID) {
-              const float2 y = __fadd2_rn(make_float2(v[8 * c + 2 * k], v[8 * c + 2 * k + 1]), x);
-              v[8 * c + 2 * k] = y.x;
-              v[8 * c + 2 * k + 1] = y.y;
+              v[8 * c + 2 * k] += x.x;
+              v[8 * c + 2 * k + 1] += x.y;
             } else {
               if (p.AUX) {  // g = gelu(u), bf16, as the forward epilogue computed it
-                const float2 gf = gelu2_f(x);
-                const __nv_bfloat162 g2 = __floats2bfloat162_rn(gf.x, gf.y);
+                const __nv_bfloat162 g2 = __floats2bfloat162_rn(gelu_f(x.x), gelu_f(x.y));
                 gk[c][k] = *reinterpret_cast<const uint32_t*>(&g2);
               }
-              const float2 gg = __fmul2_rn(make_float2(v[8 * c + 2 * k], v[8 * c + 2 * k + 1]), gelu_grad2_f(x));
-              v[8 * c + 2 * k] = gg.x;
-              v[8 * c + 2 * k + 1] = gg.y;
+              v[8 * c + 2 * k] *= gelu_grad_f(x.x);
+              v[8 * c + 2 * k + 1] *= gelu_grad_f(x.y);
             }
           }
         }
@@ -204,8 +196,8 @@ __device__ __forceinline__ void epi_tma(const Params& p, const EpiMaps& mp, uint
 #pragma unroll
           for (int k = 0; k < 4; ++k) {
             const __nv_bfloat162 u2 = __floats2bfloat162_rn(v[8 * c + 2 * k], v[8 * c + 2 * k + 1]);
-            const float2 gf = gelu2_f(__bfloat1622float2(u2));
-            const __nv_bfloat162 g2 = __floats2bfloat162_rn(gf.x, gf.y);
+            const float2 uf = __bfloat1622float2(u2);
+            const __nv_bfloat162 g2 = __floats2bfloat162_rn(gelu_f(uf.x), gelu_f(uf.y));
             pu[k] = *reinterpret_cast<const uint32_t*>(&u2);
             pg[k] = *reinterpret_cast<const uint32_t*>(&g2);
           }

@@ -275,6 +275,40 @@ def test_layernorm(dtype, h):
     assert rel(from_dev(db), db_ref) < 1e-5
 
 
+@pytest.mark.parametrize("with_res", [True, False])
+def test_layernorm_bwd_many_blocks(with_res):
+    """Fused bf16 LN backward with several row blocks per CTA, a ragged last
+    block, with and without the residual gradient, parameter gradients
+    accumulated onto non-zero buffers (+=), against the oracle in fp64."""
+    rows, h = 4100, 1600
+    x = rnd(BF16, randn(rows, h) * 2 + 0.5)
+    g = rnd(BF16, 1 + 0.1 * randn(h))
+    b = rnd(BF16, 0.1 * randn(h))
+    dy = rnd(BF16, randn(rows, h))
+    dres = rnd(BF16, randn(rows, h))
+    _, cache = om.layernorm_fwd(x.astype(np.float64), g.astype(np.float64), b.astype(np.float64))
+    dx_ref, dg_ref, db_ref = om.layernorm_bwd(dy.astype(np.float64), g.astype(np.float64), cache)
+    tx, tg, tb_ = to_dev(x, BF16), to_dev(g, BF16), to_dev(b, BF16)
+    ty = torch.empty_like(tx)
+    mu = torch.empty(rows, device=DEV)
+    rs = torch.empty(rows, device=DEV)
+    kt.layernorm_fwd(BF16, tx, tg, tb_, ty, mu, rs, rows, h)
+    tdy, tdres = to_dev(dy, BF16), to_dev(dres, BF16)
+    tdx = torch.full_like(tx, float("nan"))
+    dg0, db0 = randn(h), randn(h)
+    dg = torch.from_numpy(dg0.astype(np.float32)).to(DEV)
+    db = torch.from_numpy(db0.astype(np.float32)).to(DEV)
+    kt.layernorm_bwd(BF16, tdy, tx, tg, mu, rs, tdres if with_res else None, tdx, dg, db, rows, h)
+    torch.cuda.synchronize()
+    got = from_dev(tdx)
+    want = dx_ref + dres if with_res else dx_ref
+    assert np.isfinite(got).all()
+    assert rel(got, want) < 1e-2
+    assert np.max(np.abs(got - want)) <= 0.05 * np.max(np.abs(want))
+    assert rel(from_dev(dg) - dg0, dg_ref) < 1e-4
+    assert rel(from_dev(db) - db0, db_ref) < 1e-5
+
+
 @pytest.mark.parametrize("dtype", [BF16, F32])
 @pytest.mark.parametrize("s", [128, 384])
 def test_softmax_causal(dtype, s):
