@@ -437,7 +437,7 @@ def run_mobius(args, rank, world, local):
     peak_tf = peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops"))
     traffic = traffic_alg = None
     # ncu --set full capture of the block GEMM shapes (per launch) at this T
-    tr_name = {32768: "r1_gemm_traffic_v6.json", 16384: "r1_gemm_traffic_v5.json",
+    tr_name = {32768: "r2_gemm_traffic_v7.json", 16384: "r1_gemm_traffic_v5.json",
                8192: "r1_gemm_traffic_v3.json"}.get(c.micro_batch * c.seq_len)
     tr_path = os.path.join(ROOT, "profiles", tr_name) if tr_name else ""
     tr_n = 0
