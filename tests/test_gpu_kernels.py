@@ -276,11 +276,12 @@ def test_layernorm(dtype, h):
 
 
 @pytest.mark.parametrize("with_res", [True, False])
-def test_layernorm_bwd_many_blocks(with_res):
+@pytest.mark.parametrize("rows,h", [(4100, 1600), (301, 8192)])
+def test_layernorm_bwd_many_blocks(with_res, rows, h):
     """Fused bf16 LN backward with several row blocks per CTA, a ragged last
     block, with and without the residual gradient, parameter gradients
-    accumulated onto non-zero buffers (+=), against the oracle in fp64."""
-    rows, h = 4100, 1600
+    accumulated onto non-zero buffers (+=), against the oracle in fp64
+    (h 8192: one row per block, four column vectors per thread)."""
     x = rnd(BF16, randn(rows, h) * 2 + 0.5)
     g = rnd(BF16, 1 + 0.1 * randn(h))
     b = rnd(BF16, 0.1 * randn(h))
@@ -495,7 +496,7 @@ def test_block_fwd_bwd(dtype, tol, wscale, h, nh, s, mbs):
 
 @pytest.mark.parametrize("dtype", [BF16, F32])
 @pytest.mark.parametrize("mbs,s,nh,dh", [(2, 128, 2, 64), (1, 384, 3, 64), (2, 256, 2, 128), (1, 1024, 2, 64),
-                                         (4, 1024, 25, 64), (2, 1024, 12, 128)])
+                                         (4, 1024, 25, 64), (2, 1024, 12, 128), (1, 2048, 3, 64)])
 def test_attention_core(dtype, mbs, s, nh, dh):
     """Causal attention fwd+bwd (fused tcgen05 flash kernels on the bf16 path)
     vs the oracle's attention_fwd / attention_bwd in fp64."""
