@@ -688,6 +688,20 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1)
 // alternately to the two streams.  setmaxnreg: 56 / 192 / 192 / 72.
 // TMEM per stream X: S at 256 X (128 cols), P at 256 X + 128 (64 packed
 // cols), O at 256 X + 192 (64 cols).
+#ifndef MOBIUS_FWD_MMA_BATCH
+#define MOBIUS_FWD_MMA_BATCH 1
+#endif
+// register split of the dh-64 forward (per thread; 4 warpgroups, sum 512)
+#ifndef MOBIUS_FWD_REG_WG0
+#define MOBIUS_FWD_REG_WG0 56
+#endif
+#ifndef MOBIUS_FWD_REG_SMX
+#define MOBIUS_FWD_REG_SMX 192
+#endif
+#ifndef MOBIUS_FWD_REG_EPI
+#define MOBIUS_FWD_REG_EPI 72
+#endif
+static_assert(MOBIUS_FWD_REG_WG0 + 2 * MOBIUS_FWD_REG_SMX + MOBIUS_FWD_REG_EPI <= 512, "fwd64 register split");
 struct Fwd64Cfg {
   static constexpr int T_BYTES = 128 * 64 * 2;  // Q / K / V tile
   static constexpr int KVR = 4;                 // K / V ring per stream (16 KB entries)
@@ -779,7 +793,7 @@ __global__ void __launch_bounds__(512, 1) flash_fwd64_kernel(const __grid_consta
   const uint32_t tmem = *tmem_slot;
 
   if (warp == 0 || warp == 2) {
-    asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(MOBIUS_FWD_REG_WG0));
     const int X = warp >> 1;
     if (lane == 0) {
       FwdStream x;
@@ -816,7 +830,7 @@ __global__ void __launch_bounds__(512, 1) flash_fwd64_kernel(const __grid_consta
       }
     }
   } else if (warp == 1 || warp == 3) {
-    asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(MOBIUS_FWD_REG_WG0));
     const int X = warp >> 1;
     const uint32_t tm0 = __shfl_sync(0xffffffffu, tmem, 0) + X * 256;  // warp-uniform TMEM base of the stream
     constexpr uint32_t ID_S = ptx::idesc_bf16(BQ, BKV, 0, 0);
@@ -836,10 +850,14 @@ __global__ void __launch_bounds__(512, 1) flash_fwd64_kernel(const __grid_consta
         if (gs >= 1) BPROF(2, ptx::mbar_wait(&s_free[X], (gs - 1) & 1));  // softmax holds the previous S
         ptx::tc_fence_after();
         const uint32_t aq = ptx::smem_u32(sQ + qb * C::T_BYTES), ak = ring + e * C::T_BYTES;
+#if MOBIUS_FWD_MMA_BATCH  // 4 MMAs (K = 64) in one issue block, descriptors advanced by 32 bytes
+        ptx::mma_bf16_ss4_w(tm0, ptx::sdesc_sw128(aq, 16, 1024), ptx::sdesc_sw128(ak, 16, 1024), ID_S, 0u, 2ull);
+#else
 #pragma unroll
         for (int t = 0; t < DH / 16; ++t)
           ptx::mma_bf16_w(tm0, ptx::sdesc_sw128(aq + t * 32, 16, 1024), ptx::sdesc_sw128(ak + t * 32, 16, 1024), ID_S,
                           t > 0);
+#endif
         ptx::mma_commit_w(&s_full[X]);
         ptx::mma_commit_w(&kve[e]);
         if (x.r == x.nkv - 1) ptx::mma_commit_w(&q_empty[qb]);
@@ -853,10 +871,14 @@ __global__ void __launch_bounds__(512, 1) flash_fwd64_kernel(const __grid_consta
         if (j == 0 && x.k >= 1) BPROF(5, ptx::mbar_wait(&o_empty[X], (x.k - 1) & 1));  // previous item's O read out
         ptx::tc_fence_after();
         const uint32_t av = ring + e * C::T_BYTES;
+#if MOBIUS_FWD_MMA_BATCH  // 8 TS MMAs (K = 128 keys) in one issue block; V rows advance 2048 bytes per 16 keys
+        ptx::mma_bf16_ts8_w(tm0 + 192, tm0 + 128, ptx::sdesc_sw128(av, 16384, 1024), ID_O, j > 0 ? 1u : 0u, 128ull);
+#else
 #pragma unroll
         for (int t = 0; t < BKV / 16; ++t)  // 16 keys = 8 packed TMEM columns of P
           ptx::mma_bf16_ts_w(tm0 + 192, tm0 + 128 + 8 * t, ptx::sdesc_sw128(av + t * 2048, 16384, 1024), ID_O,
                              (j > 0 || t > 0) ? 1u : 0u);
+#endif
         ptx::mma_commit_w(&pv_done[X]);
         ptx::mma_commit_w(&kve[e]);
         if (j == x.nkv - 1) ptx::mma_commit_w(&o_ready[X]);
@@ -867,7 +889,7 @@ __global__ void __launch_bounds__(512, 1) flash_fwd64_kernel(const __grid_consta
     }
     BPROF_DUMP("fmma")
   } else if (warp < 12) {
-    asm volatile("setmaxnreg.inc.sync.aligned.u32 192;");
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(MOBIUS_FWD_REG_SMX));
     // ------------------------------------------------ softmax, stream X
     const int X = (warp - 4) >> 2, q4 = warp & 3;
     const int row = q4 * 32 + lane;
@@ -983,7 +1005,7 @@ __global__ void __launch_bounds__(512, 1) flash_fwd64_kernel(const __grid_consta
     }
     BPROF_DUMP("fsmx")
   } else {
-    asm volatile("setmaxnreg.dec.sync.aligned.u32 72;");
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(MOBIUS_FWD_REG_EPI));
     // ------------------------------------------------ epilogue
     // whichever stream's item finishes next: O / l -> bf16 -> this warp's
     // 32-row SW128 slab -> TMA store (one per warp); lse = m + log2 l
