@@ -642,7 +642,7 @@ __global__ void __launch_bounds__(LNF_THREADS, MOBIUS_LNF_CTAS)
     ln_bwd_fused_k(const __nv_bfloat16* __restrict__ dy, const __nv_bfloat16* __restrict__ x,
                    const __nv_bfloat16* __restrict__ g, const float* __restrict__ mu, const float* __restrict__ rstd,
                    const __nv_bfloat16* __restrict__ dres, __nv_bfloat16* __restrict__ dx, float* __restrict__ part,
-                   int rows, int h, int R) {
+                   int rows, int h, int R, int planes) {
   extern __shared__ __align__(128) uint8_t lnf_smem_raw[];
   // [LNF_NBUF buffers][dy | x (| dres)][R rows][h] bf16 (a block's rows are
   // contiguous in each tensor: one bulk copy per tensor), then R floats each
@@ -673,12 +673,12 @@ __global__ void __launch_bounds__(LNF_THREADS, MOBIUS_LNF_CTAS)
     if (dres) lnf_bulk_g2s(lnf_smem(base + (size_t)2 * R * h), dres + (int64_t)r0 * h, tb, bb);
   };
   // this thread's column vectors and their gamma
-  float gv[MAXV][8], adg[MAXV][8], adb[MAXV][8];
+  float gv[MAXV][8], adg[MAXV][8], adb[MAXV][8], adr[MAXV][8];  // adr: column sums of dres (planes == 3)
 #pragma unroll
   for (int k = 0; k < MAXV; ++k) {
     const int v = tid + k * LNF_THREADS;
 #pragma unroll
-    for (int e = 0; e < 8; ++e) adg[k][e] = adb[k][e] = 0.f;
+    for (int e = 0; e < 8; ++e) adg[k][e] = adb[k][e] = adr[k][e] = 0.f;
     if (v < nvec) Vec<__nv_bfloat16>::load(g + v * 8, gv[k]);
   }
   const float inv_h = 1.f / (float)h;
@@ -742,7 +742,11 @@ __global__ void __launch_bounds__(LNF_THREADS, MOBIUS_LNF_CTAS)
         Vec<__nv_bfloat16>::load(dr + v * 8, dv);
         Vec<__nv_bfloat16>::load(dr + (size_t)R * h + v * 8, xv);
         const int64_t off = (int64_t)(r0 + r) * h + v * 8;
-        if (dres) Vec<__nv_bfloat16>::load(dr + (size_t)2 * R * h + v * 8, ov);
+        if (dres) {
+          Vec<__nv_bfloat16>::load(dr + (size_t)2 * R * h + v * 8, ov);
+#pragma unroll
+          for (int e = 0; e < 8; ++e) adr[k][e] += ov[e];
+        }
 #pragma unroll
         for (int e = 0; e < 8; ++e) {
           const float xh = (xv[e] - m) * rs;
@@ -756,8 +760,8 @@ __global__ void __launch_bounds__(LNF_THREADS, MOBIUS_LNF_CTAS)
     }
     __syncthreads();  // buffer b and the row statistics are free again
   }
-  // partial rows: part[cta][0][c] = dgamma, part[cta][1][c] = dbeta
-  float* pr = part + (size_t)blockIdx.x * 2 * h;
+  // partial rows: part[cta][0][c] = dgamma, part[cta][1][c] = dbeta (, part[cta][2][c] = sum dres)
+  float* pr = part + (size_t)blockIdx.x * planes * h;
 #pragma unroll
   for (int k = 0; k < MAXV; ++k) {
     const int v = tid + k * LNF_THREADS;
@@ -767,6 +771,9 @@ __global__ void __launch_bounds__(LNF_THREADS, MOBIUS_LNF_CTAS)
       *reinterpret_cast<float4*>(pr + v * 8 + e) = make_float4(adg[k][e], adg[k][e + 1], adg[k][e + 2], adg[k][e + 3]);
       *reinterpret_cast<float4*>(pr + h + v * 8 + e) =
           make_float4(adb[k][e], adb[k][e + 1], adb[k][e + 2], adb[k][e + 3]);
+      if (planes == 3)
+        *reinterpret_cast<float4*>(pr + 2 * h + v * 8 + e) =
+            make_float4(adr[k][e], adr[k][e + 1], adr[k][e + 2], adr[k][e + 3]);
     }
   }
 }
@@ -778,25 +785,27 @@ __global__ void __launch_bounds__(LNF_THREADS, MOBIUS_LNF_CTAS)
 // partials serially took 21 us at h 1600, G 296.)
 constexpr int LNR_WARPS = 32;
 __global__ void __launch_bounds__(32 * LNR_WARPS) ln_param_reduce_k(const float* __restrict__ part, int G, int h,
-                                                                    float* dg, float* db) {
+                                                                    int planes, float* dg, float* db, float* dr) {
   __shared__ float red[LNR_WARPS][32];
   const int lane = threadIdx.x % 32, w = threadIdx.x / 32;
   const int i = blockIdx.x * 32 + lane;
   float s = 0.f;
-  if (i < 2 * h) {
+  if (i < planes * h) {
 #pragma unroll 4
-    for (int c = w; c < G; c += LNR_WARPS) s += part[(size_t)c * 2 * h + i];
+    for (int c = w; c < G; c += LNR_WARPS) s += part[(size_t)c * planes * h + i];
   }
   red[w][lane] = s;
   __syncthreads();
-  if (w == 0 && i < 2 * h) {
+  if (w == 0 && i < planes * h) {
     float t = 0.f;
 #pragma unroll
     for (int k = 0; k < LNR_WARPS; ++k) t += red[k][lane];
     if (i < h)
       dg[i] += t;
-    else
+    else if (i < 2 * h)
       db[i - h] += t;
+    else
+      dr[i - 2 * h] += t;
   }
 }
 
@@ -1089,45 +1098,57 @@ static int lnf_grid() {
 template <int MV>
 static int lnf_launch(int G, int smem, cudaStream_t st, const __nv_bfloat16* dy, const __nv_bfloat16* x,
                       const __nv_bfloat16* g, const float* mu, const float* rstd, const __nv_bfloat16* dres,
-                      __nv_bfloat16* dx, float* part, int rows, int h, int R) {
+                      __nv_bfloat16* dx, float* part, int rows, int h, int R, int planes) {
   static int smem_set = 0;  // per instantiation
   if (smem > smem_set) {
     if (cudaFuncSetAttribute(ln_bwd_fused_k<MV>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
       MOBIUS_FAIL(MOBIUS_ECUDA, "layernorm_bwd: smem attribute");
     smem_set = smem;
   }
-  ln_bwd_fused_k<MV><<<G, LNF_THREADS, smem, st>>>(dy, x, g, mu, rstd, dres, dx, part, rows, h, R);
+  ln_bwd_fused_k<MV><<<G, LNF_THREADS, smem, st>>>(dy, x, g, mu, rstd, dres, dx, part, rows, h, R, planes);
   return MOBIUS_OK;
+}
+
+static bool lnf_enabled() {
+  static int fused = -1;
+  if (fused < 0) {
+    const char* e = getenv("MOBIUS_LN_BWD_FUSED");
+    fused = e ? atoi(e) : 1;
+  }
+  return fused != 0;
+}
+
+template <typename T>
+int layernorm_bwd_launches(int h, bool dres, bool dres_sum) {
+  if (sizeof(T) == 2 && lnf_enabled() && lnf_rows(h, dres ? 3 : 2)) return 2;
+  return dres_sum ? 3 : 2;
 }
 
 template <typename T>
 int layernorm_bwd(const T* dy, const T* x, const T* g, const float* mu, const float* rstd, const T* dres, T* dx,
-                  float* dg, float* db, int rows, int h, const RedWs& ws, cudaStream_t st) {
+                  float* dg, float* db, int rows, int h, const RedWs& ws, cudaStream_t st, float* dres_sum) {
   MOBIUS_CHECK_ARG(h % Vec<T>::N == 0, "layernorm: unsupported h=%d", h);
+  MOBIUS_CHECK_ARG(!dres_sum || dres, "layernorm_bwd: dres_sum needs dres");
   if constexpr (sizeof(T) == 2) {
-    static int fused = -1;
-    if (fused < 0) {
-      const char* e = getenv("MOBIUS_LN_BWD_FUSED");
-      fused = e ? atoi(e) : 1;
-    }
     const int nt = dres ? 3 : 2;
     const int R = lnf_rows(h, nt);
-    if (fused && R && aligned16(dy) && aligned16(x) && aligned16(dx) && (!dres || aligned16(dres))) {
+    if (lnf_enabled() && R && aligned16(dy) && aligned16(x) && aligned16(dx) && (!dres || aligned16(dres))) {
       MOBIUS_CHECK_ARG(ws.part, "layernorm_bwd: reduction workspace");
       const int G = std::min(lnf_grid(), (rows + R - 1) / R);
       const int smem = lnf_smem_bytes(h, R, nt);
       const int mv = (h / 8 + LNF_THREADS - 1) / LNF_THREADS;
+      const int planes = dres_sum ? 3 : 2;
       const auto* a = (const __nv_bfloat16*)dy;
       int rc = mv == 1   ? lnf_launch<1>(G, smem, st, a, (const __nv_bfloat16*)x, (const __nv_bfloat16*)g, mu, rstd,
-                                         (const __nv_bfloat16*)dres, (__nv_bfloat16*)dx, ws.part, rows, h, R)
+                                         (const __nv_bfloat16*)dres, (__nv_bfloat16*)dx, ws.part, rows, h, R, planes)
                : mv == 2 ? lnf_launch<2>(G, smem, st, a, (const __nv_bfloat16*)x, (const __nv_bfloat16*)g, mu, rstd,
-                                         (const __nv_bfloat16*)dres, (__nv_bfloat16*)dx, ws.part, rows, h, R)
+                                         (const __nv_bfloat16*)dres, (__nv_bfloat16*)dx, ws.part, rows, h, R, planes)
                          : lnf_launch<4>(G, smem, st, a, (const __nv_bfloat16*)x, (const __nv_bfloat16*)g, mu, rstd,
-                                         (const __nv_bfloat16*)dres, (__nv_bfloat16*)dx, ws.part, rows, h, R);
+                                         (const __nv_bfloat16*)dres, (__nv_bfloat16*)dx, ws.part, rows, h, R, planes);
       if (rc) return rc;
       rc = check_launch("layernorm_bwd_fused");
       if (rc) return rc;
-      ln_param_reduce_k<<<(2 * h + 31) / 32, 32 * LNR_WARPS, 0, st>>>(ws.part, G, h, dg, db);
+      ln_param_reduce_k<<<(planes * h + 31) / 32, 32 * LNR_WARPS, 0, st>>>(ws.part, G, h, planes, dg, db, dres_sum);
       return check_launch("layernorm_param_reduce");
     }
   }
@@ -1153,7 +1174,9 @@ int layernorm_bwd(const T* dy, const T* x, const T* g, const float* mu, const fl
     MOBIUS_CHECK_ARG(ws.part && ws.cnt && gx <= RED_WS_COUNTERS, "layernorm_bwd: reduction workspace");
     colsum2_k<T, 1><<<dim3(gx, gy), CS_THREADS, 0, st>>>(dy, h, x, mu, rstd, rows, h, dg, db, rpc, ws.part, ws.cnt);
   }
-  return check_launch("layernorm_param_grad");
+  int rc2 = check_launch("layernorm_param_grad");
+  if (rc2 || !dres_sum) return rc2;
+  return colsum_accum<T>(dres, h, rows, h, dres_sum, ws, st);
 }
 
 template <typename T>
@@ -1185,7 +1208,7 @@ int loss_accumulate(const float* loss_rows, int rows, double* acc, cudaStream_t 
 int64_t colsum_ws_floats(int rows, int n, int planes) {
   // the bf16 grid (8-wide vectors) has fewer column CTAs, hence more row CTAs;
   // the fused LN backward (planes 2) needs one partial row pair per CTA
-  int64_t best = planes == 2 ? (int64_t)LNF_MAX_GRID * n * 2 : 0;
+  int64_t best = planes == 2 ? (int64_t)LNF_MAX_GRID * n * 3 : 0;  // (+ the dres column sums)
   for (int vw : {4, 8}) {
     int gx, gy, rpc;
     colsum_grid(rows, n, vw, &gx, &gy, &rpc);
@@ -1342,7 +1365,8 @@ int flag_set(int* flag, int value, cudaStream_t st) {
   template int embed_bwd<T>(const int32_t*, const T*, float*, float*, int, int, int, int, cudaStream_t);        \
   template int layernorm_fwd<T>(const T*, const T*, const T*, T*, float*, float*, int, int, cudaStream_t);      \
   template int layernorm_bwd<T>(const T*, const T*, const T*, const float*, const float*, const T*, T*, float*, \
-                                float*, int, int, const RedWs&, cudaStream_t);                                  \
+                                float*, int, int, const RedWs&, cudaStream_t, float*);                          \
+  template int layernorm_bwd_launches<T>(int, bool, bool);                                                      \
   template int softmax_causal_fwd<T>(const float*, T*, int, int, float, cudaStream_t);                          \
   template int softmax_causal_bwd<T>(const T*, const float*, T*, int, int, float, cudaStream_t);                \
   template int cross_entropy_fwd_bwd<T>(T*, const int32_t*, float*, int, int, int, float, cudaStream_t);        \

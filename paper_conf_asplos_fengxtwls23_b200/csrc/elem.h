@@ -36,11 +36,16 @@ int embed_bwd(const int32_t* tok, const T* dx, float* dwte, float* dwpe, int mbs
 // y = g (x - mu) rstd + b over rows of length h; saves mu, rstd (fp32)
 template <typename T>
 int layernorm_fwd(const T* x, const T* g, const T* b, T* y, float* mu, float* rstd, int rows, int h, cudaStream_t st);
-// dx = rstd (g dy - mean(g dy) - xhat mean(g dy xhat)) [+ dres];  dg += sum dy xhat; db += sum dy
-// (the parameter sums in a fixed order: bitwise reproducible)
+// dx = rstd (g dy - mean(g dy) - xhat mean(g dy xhat)) [+ dres];  dg += sum dy xhat; db += sum dy;
+// and, if dres_sum is given, dres_sum += sum over rows of dres (the column
+// sum of the residual gradient, e.g. the bias gradient of the layer whose
+// output it is) - all sums in a fixed order: bitwise reproducible
 template <typename T>
 int layernorm_bwd(const T* dy, const T* x, const T* g, const float* mu, const float* rstd, const T* dres, T* dx,
-                  float* dg, float* db, int rows, int h, const RedWs& ws, cudaStream_t st);
+                  float* dg, float* db, int rows, int h, const RedWs& ws, cudaStream_t st, float* dres_sum = nullptr);
+// kernels one layernorm_bwd call launches
+template <typename T>
+int layernorm_bwd_launches(int h, bool dres, bool dres_sum);
 
 // Causal row softmax of S (fp32, [B][s][s], row stride s) scaled by `scale`:
 // P[i, j] = softmax_j<=i(scale S[i, :]) and 0 for i < j < roundup(i+1, 128).

@@ -460,10 +460,11 @@ int block_bwd(const Shape& sh, const T* w, const BlockActs<T>& A_in, const T* dy
     d.C = mv(G + L.w_1, 4 * h); d.c_f32 = true;
     d.epi = EPI_ACCUM; d.accumulate = true;
     const bool fused = with_bias_row<T>(d, sc);
-    ElemScope es(st, fused ? 1 : 2);
-    RC(colsum_accum<T>(dy, h, Tn, h, G + L.b_2, sc.red, st));
-    if (!fused) RC(colsum_accum<T>(du, 4 * h, Tn, 4 * h, G + L.b_1, sc.red, st));
-    es.timed_end();
+    if (!fused) {
+      ElemScope es(st, 1);
+      RC(colsum_accum<T>(du, 4 * h, Tn, 4 * h, G + L.b_1, sc.red, st));
+      es.timed_end();
+    }
     RC(run_gemm<T>(d, st, KCLS_GEMM));
   }
   {  // da2 = du W1^T
@@ -476,8 +477,10 @@ int block_bwd(const Shape& sh, const T* w, const BlockActs<T>& A_in, const T* dy
   }
   T* dx1 = sc.t2;
   {
-    ElemScope es(st, 2);
-    RC(layernorm_bwd<T>(sc.t1, A.x1, w + L.ln2_g, A.mu2, A.rs2, dy, dx1, G + L.ln2_g, G + L.ln2_b, Tn, h, sc.red, st));
+    ElemScope es(st, layernorm_bwd_launches<T>(h, true, true));
+    // db2 += sum dy rides along: dy is this LN's residual gradient
+    RC(layernorm_bwd<T>(sc.t1, A.x1, w + L.ln2_g, A.mu2, A.rs2, dy, dx1, G + L.ln2_g, G + L.ln2_b, Tn, h, sc.red, st,
+                        G + L.b_2));
   }
   {  // dWo += o^T dx1, db_o += sum dx1 as its ones row
     GemmDesc d;
