@@ -1,10 +1,16 @@
 // Fused causal attention (flash-style) on tcgen05 for sm_100a (SURVEY
 // §8(f) f1; replaces the materialised S / P of K3/K4).
 //
-// Both kernels are persistent (one CTA per SM walking a heaviest-first item
+// All kernels are persistent (one CTA per SM walking a heaviest-first item
 // list in snake order) with warp-specialised roles and mbarrier hand-offs.
+// At dh 64 (the 1.5B shape) two 16-warp kernels written for it run by default
+// (flash_fwd64_kernel: two query tiles in flight per CTA, per-stream TMA /
+// MMA issuers, an epilogue warpgroup; flash_bwd64_kernel: a drain warpgroup
+// for dQ / dV / dK, K / V double-buffered, next-item score prefetch - see
+// their headers); the generic kernels below serve dh 128 (and dh 64 with
+// MOBIUS_FLASH_FWD_V1 / MOBIUS_FLASH_BWD_V1 = 1).
 //
-// Forward, item = (batch, head, 128-query tile):
+// Generic forward, item = (batch, head, 128-query tile):
 //   warp 0     TMA producer: Q (double buffered across items), K_j / V_j
 //              tiles through a 4-deep ring (dh 64)
 //   warp 1     MMA issuer:   S_j = Q K_j^T -> TMEM (double buffered);
@@ -16,7 +22,7 @@
 //                            O / l read-out of an item is deferred until the
 //                            next item's first P tile is issued and leaves
 //                            through smem + TMA stores (dh 64); writes lse.
-// Backward, item = (batch, head, 128-key tile kt), query tiles i >= kt:
+// Generic backward, item = (batch, head, 128-key tile kt), query tiles i >= kt:
 //   S^T = K Q_i^T, dP^T = V dO_i^T (TMEM); thread = key row computes
 //   P^T = 2^(S^T*c - lse_q) (-> TMEM, dh 64) and dS^T = P^T (dP^T - D_q)
 //   (-> smem); then dV += P^T dO_i, dK += dS^T Q_i (TMEM accumulators),
@@ -1595,9 +1601,10 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1) flash_bwd_kernel(const _
 //               P^T -> TMEM (hands dV its operand at once), dS^T kept in
 //               registers and written to the single smem dS^T tile once the
 //               previous tile's dK / dQ MMAs have read it
-//   warps 12-15 drain: dQ of each tile (TMEM -> swizzled fp32 staging ->
-//               TMA reduce-add) and dV / dK of each item (TMEM -> bf16 ->
-//               staging -> TMA store), off the softmax warps' path
+//   warps 12-15 drain: dQ of each tile (TMEM -> 16-column fp32 slabs,
+//               SWIZZLE_64B, through a 3-slot 8 KB staging ring -> TMA
+//               reduce-add) and dV / dK of each item (TMEM -> bf16 -> 64-row
+//               halves -> TMA store), off the softmax warps' path
 // setmaxnreg re-splits the register file per warpgroup: 56 / 176 / 176 / 104.
 struct Bwd64Cfg {
   static constexpr int T_BYTES = 128 * 64 * 2;  // one K / V / Q / dO tile (16 KB)
