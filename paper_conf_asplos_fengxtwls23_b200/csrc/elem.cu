@@ -1078,10 +1078,13 @@ int layernorm_fwd(const T* x, const T* g, const T* b, T* y, float* mu, float* rs
 }
 // rows per block of the fused bf16 LN backward (LNF_NBUF buffers of R rows
 // of nt tensors in <= 200 KB of shared memory), 0 when it does not apply
+// (at least 4 rows: with fewer, phase A leaves most warps idle and the
+// per-block barriers dominate - h 5120 with 1-2 rows per block was slower
+// than the two-kernel path)
 static int lnf_rows(int h, int nt) {
   if (h % 8 || h > 256 * 8 * LNF_MAXV) return 0;
   const int r = std::min((200 * 1024 / MOBIUS_LNF_CTAS) / (LNF_NBUF * nt * h * 2), 16);
-  return r >= 1 ? r : 0;
+  return r >= 4 ? r : 0;
 }
 static int lnf_smem_bytes(int h, int R, int nt) { return LNF_NBUF * R * nt * h * 2 + 4 * R * 4 + 8 * LNF_NBUF + 64; }
 static int lnf_grid() {

@@ -915,20 +915,21 @@ static int gemm_bf16_2cta_bn(const GemmDesc& d, cudaStream_t s) {
   p.R = (const __nv_bfloat16*)d.R.ptr; p.ldr = d.R.ld;
   p.AUX = (__nv_bfloat16*)d.AUX.ptr; p.ldx = d.AUX.ld;
   p.ones_m0p1 = ones ? d.M : 0;  // (M - 1) + 1
-  // rasterisation group: 4 M tiles, 8 for the weight-gradient GEMMs (A
-  // MN-major, long K) with fewer than 16 M tiles.  Measured under
-  // the power cap (tools/gemm_sustained.py, T = 32768): group 4 / 8 / 16 / 32
-  // give fc2 fwd 559 / 585 / 610 / 661 us, fc1 dX 546 / 576 / 592 / 639 us,
-  // qkv dX 409 / 422 / 433 / 464 us (the larger groups run at lower clocks),
-  // K = 1600 shapes within 1%; the dW GEMMs with few M tiles prefer 8 (qkv dW
-  // 489 / 472 us with 4 / 8, fc1 dW 639 / 630), fc2 dW (25 M tiles) 4 (625 / 640)
+  // rasterisation group: 4 M tiles when the output is narrow (<= 8 column
+  // tiles: a group of 8 x 7 tiles spans less than a wave of 74 clusters),
+  // else 8.  Measured under the power cap (tools/gemm_sustained.py, 1.5B
+  // shapes at T = 32768, N = 1600): group 4 / 8 / 16 / 32 give fc2 fwd 559 /
+  // 585 / 610 / 661 us, fc1 dX 546 / 576 / 592 / 639, qkv dX 409 / 422 / 433 /
+  // 464 (the larger groups run at lower clocks), fc2 dW 625 / 640; the wide
+  // outputs are within 1% or prefer 8 (qkv dW 489 / 472, fc1 dW 639 / 630);
+  // 4 for every activation-major GEMM cost 6% on the 13B-width shapes
   {
     static int g_env = -2;
     if (g_env == -2) {
       const char* e = getenv("MOBIUS_GEMM_GROUP");
       g_env = e ? atoi(e) : -1;
     }
-    p.group_m = g_env > 0 ? g_env : ((d.a_mn && p.tiles_m < 16) ? 8 : 4);
+    p.group_m = g_env > 0 ? g_env : (p.tiles_n <= 8 ? 4 : 8);
   }
   plan_stream_k(p, num_sms() / 2);
   if (p.sk_tiles && !p.splitk_reduce) {
