@@ -1606,12 +1606,21 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1) flash_bwd_kernel(const _
 //               reduce-add) and dV / dK of each item (TMEM -> bf16 -> 64-row
 //               halves -> TMA store), off the softmax warps' path
 // setmaxnreg re-splits the register file per warpgroup: 56 / 176 / 176 / 104.
+#ifndef MOBIUS_BWD_QS
+#define MOBIUS_BWD_QS 3
+#endif
+#ifndef MOBIUS_BWD_SLAB32
+#define MOBIUS_BWD_SLAB32 0
+#endif
 struct Bwd64Cfg {
   static constexpr int T_BYTES = 128 * 64 * 2;  // one K / V / Q / dO tile (16 KB)
-  static constexpr int QS = 3;                  // Q / dO ring depth
+  static constexpr int QS = MOBIUS_BWD_QS;      // Q / dO ring depth
   static constexpr int DS_BYTES = 128 * 128 * 2;
-  static constexpr int NSTG = 3;                  // drain staging ring of 8 KB slots: an fp32 16-column dQ
-  static constexpr int STG_BYTES = NSTG * 8192;   // slab or 64 rows of a bf16 dV / dK tile
+  // drain staging ring: 8 KB slots (an fp32 16-column dQ slab or 64 rows of
+  // a bf16 dV / dK tile), or with MOBIUS_BWD_SLAB32 16 KB slots of 32-column slabs
+  static constexpr int SLOT = MOBIUS_BWD_SLAB32 ? 16384 : 8192;
+  static constexpr int NSTG = MOBIUS_BWD_SLAB32 ? 2 : 3;
+  static constexpr int STG_BYTES = NSTG * SLOT;
   static constexpr int SMEM = 1024 + 4 * T_BYTES + QS * 2 * T_BYTES + DS_BYTES + STG_BYTES + QS * 1024 + 256;
 };
 
@@ -1919,7 +1928,7 @@ __global__ void __launch_bounds__(512, 1) flash_bwd64_kernel(const __grid_consta
     auto slot_acquire = [&]() -> uint32_t {
       if (leader) asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(C::NSTG - 1) : "memory");
       named_bar(1, 128);
-      return stg0 + (ks % C::NSTG) * 8192;
+      return stg0 + (ks % C::NSTG) * C::SLOT;
     };
     auto slot_done = [&]() {  // staging written: hand it to the async proxy
       ptx::fence_proxy_async();
@@ -1992,21 +2001,29 @@ __global__ void __launch_bounds__(512, 1) flash_bwd64_kernel(const __grid_consta
         ptx::tc_fence_before();
         __syncwarp();
         if (lane == 0) ptx::mbar_arrive(dq_empty);  // dQ TMEM may be overwritten
+        constexpr int NSL = MOBIUS_BWD_SLAB32 ? 2 : 4, SW = 64 / NSL;  // slabs of SW columns
 #pragma unroll
-        for (int c = 0; c < 4; ++c) {  // 16-column slabs
+        for (int c = 0; c < NSL; ++c) {
           uint32_t stg;
           BPROF(1, stg = slot_acquire());
+          if (MOBIUS_BWD_SLAB32) {  // 128-byte rows, SWIZZLE_128B
 #pragma unroll
-          for (int k = 0; k < 4; ++k)
-            st_shared_v4(stg + r * 64 + ((k ^ ((r >> 1) & 3)) << 4), v[c >> 1][(c & 1) * 16 + 4 * k],
-                         v[c >> 1][(c & 1) * 16 + 4 * k + 1], v[c >> 1][(c & 1) * 16 + 4 * k + 2],
-                         v[c >> 1][(c & 1) * 16 + 4 * k + 3]);
+            for (int k = 0; k < 8; ++k)
+              st_shared_v4(stg + r * 128 + ((k ^ (r & 7)) << 4), v[c & 1][4 * k], v[c & 1][4 * k + 1],
+                           v[c & 1][4 * k + 2], v[c & 1][4 * k + 3]);
+          } else {  // 64-byte rows, SWIZZLE_64B
+#pragma unroll
+            for (int k = 0; k < 4; ++k)
+              st_shared_v4(stg + r * 64 + ((k ^ ((r >> 1) & 3)) << 4), v[c >> 1][(c & 1) * 16 + 4 * k],
+                           v[c >> 1][(c & 1) * 16 + 4 * k + 1], v[c >> 1][(c & 1) * 16 + 4 * k + 2],
+                           v[c >> 1][(c & 1) * 16 + 4 * k + 3]);
+          }
           slot_done();
           if (leader) {
             asm volatile(
                 "cp.reduce.async.bulk.tensor.4d.global.shared::cta.add.tile.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
                     reinterpret_cast<uint64_t>(&tdq)),
-                "r"(stg), "r"(c * 16), "r"((kt + it) * 128), "r"(hd), "r"(b)
+                "r"(stg), "r"(c * SW), "r"((kt + it) * 128), "r"(hd), "r"(b)
                 : "memory");
             asm volatile("cp.async.bulk.commit_group;" ::: "memory");
           }
@@ -2222,16 +2239,23 @@ int flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* o, const __nv_
   MOBIUS_CHECK_ARG(flash_supported(dh, s), "flash: dh %d / s %d unsupported", dh, s);
   const int h = nh * dh;
   const int64_t rows = (int64_t)mbs * s;
+  // MOBIUS_FLASH_BWD_V1=1: the round-2 10-warp kernel at dh 64 (softmax-gradient warps drain dQ themselves)
+  static int v1 = -1;
+  if (v1 < 0) {
+    const char* e = getenv("MOBIUS_FLASH_BWD_V1");
+    v1 = (e && atoi(e) == 1) ? 1 : 0;
+  }
+  const bool k64 = dh == 64 && !v1;  // flash_bwd64_kernel
   CUtensorMap tm, tdo, tdq;
   int rc = head_map(&tm, qkv, 3 * h, dh, s, 3 * nh, mbs);
   if (rc) return rc;
   rc = head_map(&tdo, dout, h, dh, s, nh, mbs);
   if (rc) return rc;
   // dh 64 kernel: 16-column dQ slabs and 64-row dV / dK halves (8 KB staging slots)
-  rc = dq_map(&tdq, dq_ws, h, dh, s, nh, mbs, dh == 64 ? 16 : 32);
+  rc = dq_map(&tdq, dq_ws, h, dh, s, nh, mbs, (k64 && !MOBIUS_BWD_SLAB32) ? 16 : 32);
   if (rc) return rc;
   CUtensorMap tdkv;  // TMA-store view of dqkv (dK / dV head slots)
-  rc = head_map(&tdkv, dqkv, 3 * h, dh, s, 3 * nh, mbs, dh == 64 ? 64 : 128);
+  rc = head_map(&tdkv, dqkv, 3 * h, dh, s, 3 * nh, mbs, k64 ? 64 : 128);
   if (rc) return rc;
   if (dh == 64)
     flash_dsum_kernel<64><<<(unsigned)((rows + 7) / 8), 256, 0, st>>>(dout, o, dsum_ws, dq_ws, (int)rows, nh, s);
@@ -2260,12 +2284,6 @@ int flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* o, const __nv_
   dim3 grid(n_items < sms ? n_items : sms);  // persistent
   if (dh == 64) {
     static bool once = false;
-    // MOBIUS_FLASH_BWD_V1=1: the round-2 10-warp kernel (softmax-gradient warps drain dQ themselves)
-    static int v1 = -1;
-    if (v1 < 0) {
-      const char* e = getenv("MOBIUS_FLASH_BWD_V1");
-      v1 = (e && atoi(e) == 1) ? 1 : 0;
-    }
     if (v1) {
       if (!once) { rc = set_smem(flash_bwd_kernel<64, 2>, BwdCfg<64>::SMEM); if (rc) return rc; once = true; }
       flash_bwd_kernel<64, 2><<<grid, NT_FWD, BwdCfg<64>::SMEM, st>>>(tm, tdo, tdq, tdkv, p);
