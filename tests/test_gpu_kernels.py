@@ -275,6 +275,21 @@ def test_layernorm(dtype, h):
     assert rel(from_dev(db), db_ref) < 1e-5
 
 
+@pytest.mark.parametrize("env", ["MOBIUS_FLASH_FWD_V1", "MOBIUS_FLASH_BWD_V1"])
+def test_attention_v1_fallback(env):
+    """The generic (round-2 first session) flash kernels stay selectable at
+    dh 64 through MOBIUS_FLASH_FWD_V1 / MOBIUS_FLASH_BWD_V1 = 1 (read once per
+    process, so the parity cases run in a child pytest with the variable set)."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", os.path.join(root, "tests", "test_gpu_kernels.py"),
+                        "-k", "attention_core and 64"], cwd=root, env={**os.environ, env: "1"},
+                       capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
+
+
 @pytest.mark.parametrize("with_res", [True, False])
 @pytest.mark.parametrize("rows,h", [(4100, 1600), (301, 8192)])
 def test_layernorm_bwd_many_blocks(with_res, rows, h):
