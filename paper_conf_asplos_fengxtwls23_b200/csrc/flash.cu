@@ -2170,6 +2170,16 @@ int set_smem(K k, int bytes) {
 
 int flash_supported(int dh, int s) { return (dh == 64 || dh == 128) && s % 128 == 0; }
 
+// MOBIUS_FLASH_FWD_V1=1: the round-2 10-warp forward (one query tile at a time) at dh 64
+static bool flash_fwd_v1() {
+  static int v1 = -1;
+  if (v1 < 0) {
+    const char* e = getenv("MOBIUS_FLASH_FWD_V1");
+    v1 = (e && atoi(e) == 1) ? 1 : 0;
+  }
+  return v1 == 1;
+}
+
 int flash_attn_fwd(const __nv_bfloat16* qkv, __nv_bfloat16* o, float* lse, int mbs, int s, int nh, int dh,
                    cudaStream_t st) {
   MOBIUS_CHECK_ARG(flash_supported(dh, s), "flash: dh %d / s %d unsupported", dh, s);
@@ -2189,6 +2199,18 @@ int flash_attn_fwd(const __nv_bfloat16* qkv, __nv_bfloat16* o, float* lse, int m
   p.mbs = mbs;
   p.scale_log2 = 1.4426950408889634f / sqrtf((float)dh);
   p.group = nh * mbs;  // one chunk: global heaviest-first order
+  {  // (batch, head) pairs per item chunk: MOBIUS_FLASH_FWD_GROUP, default 128
+     // for the dh-64 ping-pong kernel (mbs 32: one chunk 212 us, 32 / 64 / 128 /
+     // 256 pairs 212 / 206 / 206 / 211 us - a chunk's K / V stay in L2), one
+     // chunk for the generic kernel (grouping cost it balance: 261 vs 266-274 us)
+    static int fg = -2;
+    if (fg == -2) {
+      const char* e = getenv("MOBIUS_FLASH_FWD_GROUP");
+      fg = e ? atoi(e) : -1;
+    }
+    const int want = fg >= 0 ? fg : (dh == 64 && !flash_fwd_v1() ? 128 : 0);
+    if (want > 0 && want < p.group) p.group = want;
+  }
   int n_items = (s / BQ) * nh * mbs;
   int sms = 148;
   {
@@ -2205,13 +2227,7 @@ int flash_attn_fwd(const __nv_bfloat16* qkv, __nv_bfloat16* o, float* lse, int m
       const char* e = getenv("MOBIUS_FLASH_FWD_CP");
       cp = (e && atoi(e) == 4) ? 4 : 2;
     }
-    // MOBIUS_FLASH_FWD_V1=1: the round-2 10-warp kernel (one query tile at a time)
-    static int v1 = -1;
-    if (v1 < 0) {
-      const char* e = getenv("MOBIUS_FLASH_FWD_V1");
-      v1 = (e && atoi(e) == 1) ? 1 : 0;
-    }
-    if (!v1) {
+    if (!flash_fwd_v1()) {
       static bool once64 = false;
       if (!once64) { rc = set_smem(flash_fwd64_kernel, Fwd64Cfg::SMEM); if (rc) return rc; once64 = true; }
       flash_fwd64_kernel<<<grid, 512, Fwd64Cfg::SMEM, st>>>(tm, tmo, p);
