@@ -694,6 +694,9 @@ __global__ void __launch_bounds__((2 + 4 * CP) * 32, 1)
 // alternately to the two streams.  setmaxnreg: 56 / 192 / 192 / 72.
 // TMEM per stream X: S at 256 X (128 cols), P at 256 X + 128 (64 packed
 // cols), O at 256 X + 192 (64 cols).
+#ifndef MOBIUS_FWD_POLL_NS
+#define MOBIUS_FWD_POLL_NS 256  // epilogue warps' back-off between o_ready polls (ns, 0 = spin)
+#endif
 #ifndef MOBIUS_FWD_MMA_BATCH
 #define MOBIUS_FWD_MMA_BATCH 1
 #endif
@@ -1027,6 +1030,9 @@ __global__ void __launch_bounds__(512, 1) flash_fwd64_kernel(const __grid_consta
         for (int c = 0; c < 2 && X < 0; ++c)
           if (st[c].act && ptx::mbar_test(&o_ready[c], st[c].k & 1)) X = c;
         X = __shfl_sync(0xffffffffu, X, 0);
+        // back off between polls: a spinning warp takes issue slots from the
+        // softmax warps on its SMSP (items finish every few thousand cycles)
+        if (X < 0 && MOBIUS_FWD_POLL_NS) __nanosleep(MOBIUS_FWD_POLL_NS);
       }
       FwdStream& x = st[X];
       ptx::tc_fence_after();
