@@ -2088,15 +2088,21 @@ __global__ void __launch_bounds__(256) flash_dsum_kernel(const __nv_bfloat16* __
 }
 
 // dqkv q-part (bf16, row stride 3h) = scale * dQacc (fp32, row stride h)
+// 8 elements per thread: two streaming 16-byte loads (the accumulator is not
+// read again before the next call zeroes it), one 16-byte store (h % 8 == 0)
 __global__ void flash_dq_cast_kernel(const float* dQacc, __nv_bfloat16* dq, int64_t rows, int h, int64_t ldd,
                                      float scale) {
-  const int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 4;
+  const int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * 8;
   if (i >= rows * h) return;
   const int64_t r = i / h, c = i % h;
-  float4 v = *reinterpret_cast<const float4*>(dQacc + i);
-  __nv_bfloat162* o = reinterpret_cast<__nv_bfloat162*>(dq + r * ldd + c);
-  o[0] = __floats2bfloat162_rn(v.x * scale, v.y * scale);
-  o[1] = __floats2bfloat162_rn(v.z * scale, v.w * scale);
+  const float4 v0 = __ldcs(reinterpret_cast<const float4*>(dQacc + i));
+  const float4 v1 = __ldcs(reinterpret_cast<const float4*>(dQacc + i) + 1);
+  uint4 o;
+  o.x = pack_bf16(v0.x * scale, v0.y * scale);
+  o.y = pack_bf16(v0.z * scale, v0.w * scale);
+  o.z = pack_bf16(v1.x * scale, v1.y * scale);
+  o.w = pack_bf16(v1.z * scale, v1.w * scale);
+  *reinterpret_cast<uint4*>(dq + r * ldd + c) = o;
 }
 
 // (batch, head) pairs per item chunk of the backward: MOBIUS_FLASH_GROUP
@@ -2320,7 +2326,7 @@ int flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* o, const __nv_
     flash_bwd_kernel<128, 2><<<grid, NT_FWD, BwdCfg<128>::SMEM, st>>>(tm, tdo, tdq, tdkv, p);
   }
   {
-    const int64_t n = rows * h / 4;
+    const int64_t n = rows * h / 8;
     flash_dq_cast_kernel<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(dq_ws, dqkv, rows, h, 3 * h, p.scale);
   }
   e = cudaGetLastError();
