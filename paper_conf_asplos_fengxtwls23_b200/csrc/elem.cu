@@ -508,16 +508,21 @@ __global__ void __launch_bounds__(CE_NT) ce_k(T* z, const int32_t* tok, float* l
   const int b = r / s, i = r % s;
   const int t = tok[(int64_t)b * (s + 1) + i + 1];
   T* zr = z + (int64_t)r * V;
+  // online max / sum, rescaled once per vector (VW + 1 exponentials per VW
+  // logits instead of 2 VW: the pass is MUFU-bound, not HBM-bound)
   float m = -INFINITY, l = 0.f;
   for (int c = threadIdx.x * VW; c < V; c += CE_NT * VW) {
     float f[VW];
     Vec<T>::load(zr + c, f);
+    float vm = f[0];
 #pragma unroll
-    for (int e = 0; e < VW; ++e) {
-      float nm = fmaxf(m, f[e]);
-      l = l * __expf(m - nm) + __expf(f[e] - nm);
-      m = nm;
-    }
+    for (int e = 1; e < VW; ++e) vm = fmaxf(vm, f[e]);
+    const float nm = fmaxf(m, vm);
+    float sv = 0.f;
+#pragma unroll
+    for (int e = 0; e < VW; ++e) sv += __expf(f[e] - nm);
+    l = l * __expf(m - nm) + sv;
+    m = nm;
   }
   const float gm = block_max<CE_NT>(m, red);
   l = (m == -INFINITY) ? 0.f : l * __expf(m - gm);
